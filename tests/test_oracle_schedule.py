@@ -1,0 +1,123 @@
+"""Pins for the oracle's replay of Algorithms 1-3 (§IV-B/§IV-C)."""
+import json
+import os
+
+import numpy as np
+import pytest
+
+from oracle import qasm as oq
+from oracle import schedule as os_
+from oracle import statevector as osv
+from workloads import circuits as wc
+
+GOLDEN = os.path.join(os.path.dirname(__file__), "golden")
+
+
+def _gs5():
+    g = json.load(open(os.path.join(GOLDEN, "gs5_walkthrough.json")))
+    gates = [tuple(t) + tuple(c) for t, c in g["gates"]]
+    return g, gates
+
+
+def test_get_chunk_size_paper_example():
+    g = json.load(open(os.path.join(GOLDEN, "alg1_examples.json")))
+    for ex in g["getChunkSize"]:
+        assert os_.get_chunk_size(int(ex["involvement"], 2)) == ex["chunkSize"]
+
+
+def test_chunk_count_paper_example():
+    """34 qubits, 2^21-amplitude chunks -> 8192 chunks; 16 B per amplitude."""
+    g = json.load(open(os.path.join(GOLDEN, "alg1_examples.json")))["chunk_count"]
+    assert 1 << (g["n"] - g["chunk_amplitudes_log2"]) == g["n_chunks"]
+    assert len(os_.chunk_bitmap((1 << 34) - 1, 34, 21)) == 8192
+    # 496 chunks of 2^21 * 16 B = 32 MiB = 15.5 GiB fit in a 16 GiB P100
+    assert 496 * (1 << 21) * g["bytes_per_amplitude"] <= 16 * 2**30
+
+
+@pytest.mark.parametrize("inv,cs,chunks", [
+    (0b00000011, 2, [0]),
+    (0b00100111, 3, [0, 4]),
+    (0b10110111, 3, [0, 2, 4, 6, 16, 18, 20, 22]),
+    (0b00000000, 0, [0]),
+    (0b11111111, 8, [0]),
+])
+def test_alg1_hand_values(inv, cs, chunks):
+    got_cs, got = os_.alg1_chunks(inv, 8)
+    assert (got_cs, got) == (cs, chunks)
+
+
+def test_alg1_processes_exactly_the_nonzero_support():
+    """with m uninvolved qubits exactly 2^(n-m) amplitudes may be non-zero; Alg.1's
+    processed chunks cover exactly {i : i & ~involvement == 0} (brute force, all 8-bit I)."""
+    n = 8
+    for inv in range(1 << n):
+        cs, ch = os_.alg1_chunks(inv, n)
+        covered = {(j << cs) + k for j in ch for k in range(1 << cs)}
+        support = {i for i in range(1 << n) if i & ~inv == 0}
+        assert covered == support
+        assert len(covered) == 1 << bin(inv).count("1")
+
+
+def test_bitmap_definition_vs_bruteforce():
+    n, c = 9, 3
+    for inv in [0, 1, 0b101, 0b110010111, (1 << n) - 1, 0b100000000]:
+        bm = os_.chunk_bitmap(inv, n, c)
+        for j in range(1 << (n - c)):
+            may = any(((i & ~inv) == 0) for i in range(j << c, (j + 1) << c))
+            assert bm[j] == int(may)
+
+
+def test_gs5_original_greedy_forward():
+    """P:239 baseline 1,2,3,4,5,5,5,5,5; P:286 greedy 1,2,3,4,4,4,5,5,5 (paper's random picks
+    g1,g3,g5,g2); P:336 forward-looking 1,2,2,3,3,4,4,4,5."""
+    g, gates = _gs5()
+    cnt = lambda order: [bin(i).count("1") for i in os_.involvement_trace(gates, order)]
+    assert cnt(None) == g["original_involved_counts"]
+    gr = os_.reorder_greedy(gates, forced=g["greedy_forced_picks"])
+    assert cnt(gr) == g["greedy_involved_counts"]
+    fw = os_.reorder_forward(gates)
+    assert cnt(fw) == g["forward_involved_counts"]
+    for o in (gr, fw):
+        assert os_.is_topological(gates, o)
+
+
+@pytest.mark.parametrize("seed", range(6))
+def test_reorder_is_topological_and_exact(seed):
+    """reorder obeys dependencies and does not change results."""
+    c = wc.random_circuit(7, 60, seed=seed)
+    n, gates = oq.parse(c.qasm())
+    ref = osv.simulate_gates(n, gates)
+    for mode in (1, 2):
+        order = os_.reorder(gates, mode)
+        assert os_.is_topological(gates, order)
+        psi = osv.simulate_gates(n, gates, order=order)
+        assert np.abs(psi - ref).max() < 1e-12
+
+
+@pytest.mark.parametrize("fam", ["qft", "gs", "hlf", "random"])
+def test_pruning_soundness(fam):
+    """after every step of a schedule, every bitmap-0 chunk is exactly zero in the
+    unpruned state evolved along the same schedule."""
+    c = {"qft": lambda: wc.qft(9), "gs": lambda: wc.gs(3, 3), "hlf": lambda: wc.hlf(3, 3, 2),
+         "random": lambda: wc.random_circuit(9, 40, seed=2)}[fam]()
+    n, gates = oq.parse(c.qasm())
+    for mode in (0, 2):
+        order = os_.reorder(gates, mode)
+        psi = osv.zero_state(n)
+        inv = 0
+        for i in order:
+            g = gates[i]
+            osv.apply_gate(psi, n, g.U, g.targets, g.controls)
+            inv = os_.update_involvement(inv, g.qubits)
+            for cb in (0, 2, 4):
+                bm = np.array(os_.chunk_bitmap(inv, n, cb), dtype=bool)
+                z = osv.zero_map(psi, n, cb)
+                assert np.all(z[~bm])
+
+
+def test_forward_reorder_delays_involvement_on_qft():
+    """Fig.9: forward-looking reordering delays involvement on qft."""
+    n, gates = oq.parse(wc.qft(12).qasm())
+    base = os_.ops_before_full_involvement(gates, n)
+    fw = os_.ops_before_full_involvement(gates, n, os_.reorder_forward(gates))
+    assert fw > base
