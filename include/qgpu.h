@@ -1,0 +1,212 @@
+/* qgpu.h -- C ABI of the B200-native Q-GPU hot path (libqgpu.so).
+ *
+ * Implements the data-parallel hot path of Q-GPU (Zhao et al., "Q-GPU: A Recipe of
+ * Optimizations for Quantum Circuit Simulation Using GPUs", HPCA 2022; cited as P:<line> of
+ * /root/reference/PAPER.md): applying 1- and 2-qubit, optionally controlled, gates to a 2^n
+ * complex128 state vector (Eq.8), with zero-amplitude pruning driven by the
+ * per-qubit `involvement` flags (Algorithm 1), dependency-aware reordering that
+ * delays qubit involvement (Algorithms 2/3), and -- B200-specific, not in the
+ * paper -- a resident-in-HBM state whose live part is a contiguous prefix (first-touch qubit
+ * placement), fused multi-gate HBM passes, and global-local qubit swaps across GPUs.
+ *
+ * Conventions (readings listed in DESIGN.md):
+ *  - Qubit q is bit q of the amplitude index (little-endian, Eq.8).
+ *  - Amplitudes are complex128 stored as interleaved (re, im) doubles.
+ *  - A gate matrix U is 2^t x 2^t, row-major, as (re, im) pairs; bit j of the row/column
+ *    index refers to targets[j]. Controls fire on |1> only. Targets and controls are
+ *    distinct and in [0, n).
+ *  - All status codes are returned; a human-readable detail is in qgpu_last_error().
+ *    No C++ exception or abort() crosses the ABI. On an argument error the state is left
+ *    unchanged.
+ *  - Apply calls are asynchronous on the state's stream; readout calls synchronise it. An
+ *    asynchronous CUDA failure surfaces at the next synchronising call as QGPU_ERR_CUDA and
+ *    marks the state QGPU_ERR_STATE.
+ *  - Sharded mode (world_size > 1): every call is a collective, made by all ranks in the
+ *    same order (SPMD); readout results are valid on every rank.
+ *  - Thread safety: a state must not be used from two threads at once.
+ */
+#ifndef QGPU_H
+#define QGPU_H
+
+#include <stddef.h>
+#include <stdint.h>
+
+#ifdef __cplusplus
+extern "C" {
+#endif
+
+#define QGPU_ABI_VERSION 1
+
+typedef enum {
+  QGPU_OK = 0,
+  QGPU_ERR_INVALID_ARG = 1,    /* bad argument; nothing was changed                         */
+  QGPU_ERR_OUT_OF_MEMORY = 2,  /* device allocation failed or buffer too small              */
+  QGPU_ERR_UNSUPPORTED = 3,    /* valid request outside the supported subset                */
+  QGPU_ERR_PARSE = 4,          /* QASM syntax error; detail has line:col                    */
+  QGPU_ERR_CUDA = 5,           /* CUDA runtime error                                        */
+  QGPU_ERR_NCCL = 6,           /* NCCL error (sharded mode)                                 */
+  QGPU_ERR_STATE = 7           /* state poisoned by an earlier asynchronous failure         */
+} qgpu_status;
+
+typedef struct qgpu_state qgpu_state;       /* opaque; owned by the library */
+typedef struct qgpu_circuit qgpu_circuit;   /* opaque; owned by the library */
+
+typedef struct {
+  uint32_t struct_size;       /* = sizeof(qgpu_config); ABI guard                           */
+  int device;                 /* CUDA device ordinal                                       */
+  void* stream;               /* cudaStream_t to enqueue on; NULL = library-owned stream   */
+  void* state_buffer;         /* optional caller-owned device memory (e.g. a torch tensor) */
+  uint64_t state_buffer_bytes;/* its size; must be >= 16 * 2^(n - log2 world_size)          */
+  int rank, world_size;       /* world_size = 2^g GPUs; 1 = single GPU                     */
+  const void* nccl_unique_id; /* 128-byte ncclUniqueId (world_size > 1), same on all ranks */
+  int chunk_bits;             /* c: bitmap/pruning unit 2^c amplitudes;
+                                 default 21, clamped to [0, n]                             */
+  int prune;                  /* 1 (default): pruning + delayed involvement;
+                                 0: every pass over the full local range (ablation)        */
+  int reorder;                /* qgpu_apply_circuit order: 0 program, 1 greedy (Alg.2),
+                                 2 forward-looking (Alg.3, default)            */
+  int fuse_bits;              /* b: tile qubits per fused HBM pass (default 12);
+                                 0 = one kernel per gate (pair/quad/diag kernels)          */
+  int timing;                 /* 1: time every launch with CUDA events into qgpu_stats     */
+  uint64_t swap_slab_bytes;   /* staging bytes per all-to-all slab (sharded mode)          */
+} qgpu_config;
+
+typedef struct {
+  uint64_t gates_applied;      /* gates executed (SWAPs handled as relabels included)        */
+  uint64_t passes;             /* HBM passes (kernel launches over the state)                */
+  uint64_t kernels_launched;   /* every kernel launched by the library                       */
+  uint64_t relabels;           /* SWAP gates executed as qubit-map relabels (no data moved)  */
+  uint64_t amps_processed;     /* sum over passes of live local amplitudes written           */
+  uint64_t amps_full;          /* sum over passes of 2^(n-g) (what an unpruned pass touches) */
+  uint64_t chunks_processed;   /* sum over passes of live chunks (2^c granularity)           */
+  uint64_t chunks_skipped;     /* sum over passes of all-zero chunks skipped         */
+  uint64_t algo_bytes;         /* algorithmic HBM bytes: reads of live input + writes        */
+  uint64_t unfused_bytes;      /* bytes the same gates would move one gate per pass          */
+  uint64_t swaps;              /* global-local swaps (sharded mode)                          */
+  uint64_t swap_bytes;         /* bytes sent by this rank in swaps                           */
+  int64_t ops_before_full_involvement; /* Table II statistic, -1 if never    */
+  double kernel_ms;            /* timing=1: summed CUDA-event time of pass kernels           */
+  double tile_kernel_ms;       /* timing=1: time of fused tile kernels only                  */
+  uint64_t tile_kernel_launches;
+  uint64_t tile_algo_bytes;    /* algorithmic bytes of fused tile kernels only               */
+  double swap_ms;              /* timing=1: time in swaps                                    */
+} qgpu_stats;
+
+/* ---- configuration and state ---------------------------------------------------------- */
+
+/* Fill *cfg with defaults (device 0, own stream, prune=1, reorder=2, chunk_bits=21,
+ * fuse_bits=12, world_size=1). Returns INVALID_ARG if cfg is NULL. */
+qgpu_status qgpu_config_init(qgpu_config* cfg);
+
+/* Create an n-qubit state |0...0> (all qubits start in |0>). cfg may be NULL
+ * (defaults). The device buffer is cudaMalloc'ed unless cfg->state_buffer is given, in which
+ * case it stays caller-owned and must outlive the state. No memset of the full buffer is done:
+ * the live part grows by first-touch expansion, which writes the new half explicitly.
+ * Errors: INVALID_ARG (n < 1, n > 40, bad world size), OUT_OF_MEMORY, CUDA, NCCL.
+ * *out receives an owned handle; release it with qgpu_state_destroy. */
+qgpu_status qgpu_state_create(int n_qubits, const qgpu_config* cfg, qgpu_state** out);
+
+/* Destroy a state (synchronises its stream, frees library-owned memory). NULL is a no-op. */
+qgpu_status qgpu_state_destroy(qgpu_state* st);
+
+/* Return the state to |0...0> and clear involvement, qubit map, schedule trace and stats.
+ * O(1) device work (one 16-byte write), asynchronous. */
+qgpu_status qgpu_state_reset(qgpu_state* st);
+
+/* Overwrite the full logical state from host memory: amps = 2 * 2^n doubles (re, im) in
+ * logical index order. Marks every qubit involved (nothing left to prune). Synchronises.
+ * Single-GPU only (UNSUPPORTED when sharded). */
+qgpu_status qgpu_set_amplitudes(qgpu_state* st, const double* amps);
+
+/* Block until all work enqueued on the state's stream is done; reports async errors. */
+qgpu_status qgpu_synchronize(qgpu_state* st);
+
+/* Number of qubits, local qubits (n - log2 world) and device pointer of the local buffer. */
+qgpu_status qgpu_state_info(const qgpu_state* st, int* n_qubits, int* n_local, void** dev_ptr);
+
+/* ---- gate application (the hot path) --------------------------------------------------- */
+
+/* Apply one gate (Eq.8): U is (2^t x 2^t) row-major complex128 as 2*4^t
+ * doubles (copied on call), t = n_targets in {1, 2}; targets[j] <-> bit j of U's index;
+ * controls (n_controls >= 0, may be NULL when 0) must all be |1>. Updates `involvement`
+ * with targets and controls (P:229 l.11), places first-touched qubits, and launches one pair
+ * (t=1), quad (t=2) or diagonal kernel over the live prefix only (pruning).
+ * Errors: INVALID_ARG (range, duplicates, NULL), STATE. Asynchronous. */
+qgpu_status qgpu_apply_gate(qgpu_state* st, const double* U, int n_targets, const int* targets,
+                            int n_controls, const int* controls);
+
+/* Apply a parsed circuit: reorder (cfg.reorder: Alg.2/Alg.3), update involvement and qubit
+ * placement per gate, cut the order into consecutive fused passes (cfg.fuse_bits), execute
+ * SWAP gates as qubit relabels, and launch. The result equals program-order application up to
+ * floating-point rounding. The circuit must have n_qubits <= the state's n.
+ * Errors: INVALID_ARG, STATE, CUDA, NCCL. Asynchronous. */
+qgpu_status qgpu_apply_circuit(qgpu_state* st, const qgpu_circuit* c);
+
+/* ---- readout (synchronising) ------------------------------------------------------------ */
+
+/* Copy amplitudes [start, start+count) of the LOGICAL index space to host out[2*count]
+ * (re, im). Handles the qubit map; never-involved qubits read as |0>. */
+qgpu_status qgpu_get_amplitudes(qgpu_state* st, uint64_t start, uint64_t count, double* out);
+
+/* Same into caller-owned DEVICE memory dev_out[2*count] (no host copy). Asynchronous. */
+qgpu_status qgpu_get_amplitudes_device(qgpu_state* st, uint64_t start, uint64_t count,
+                                       double* dev_out);
+
+/* Marginal probabilities (Eq.1): out[y] = sum_{i: bits_Q(i)=y} |psi_i|^2, with
+ * qubits[0] <-> bit 0 of y; 0 <= m <= 30; out has 2^m doubles (host). m = 0 gives the norm. */
+qgpu_status qgpu_probabilities(qgpu_state* st, int m, const int* qubits, double* out);
+
+/* ---- circuits ---------------------------------------------------------------------------- */
+
+/* Parse an OpenQASM-2 subset. Errors: PARSE (with line:col),
+ * UNSUPPORTED (gate definitions, reset, if, unknown gates), INVALID_ARG. *out is owned by
+ * the caller; release with qgpu_circuit_destroy. */
+qgpu_status qgpu_circuit_from_qasm(const char* text, size_t len, qgpu_circuit** out);
+qgpu_status qgpu_circuit_info(const qgpu_circuit* c, int* n_qubits, uint64_t* n_gates);
+qgpu_status qgpu_circuit_destroy(qgpu_circuit* c);
+
+/* Host-only (no GPU needed): the execution order chosen by `mode` (0 program, 1 greedy
+ * Alg.2, 2 forward-looking Alg.3) as gate indices into order[cap]. *n = number of gates. */
+qgpu_status qgpu_circuit_reorder(const qgpu_circuit* c, int mode, uint64_t* order, uint64_t cap,
+                                 uint64_t* n);
+
+/* Host-only pass plan summary for diagnostics/tests: for each pass p (up to cap),
+ * info[8p..8p+7] = {first gate position, gate count, kind, log2 L_in, log2 L_out, tile bits,
+ * tile position mask (low 32 bits), high 32 bits of the mask}. kind: 0 tile, 1 pair, 2 quad,
+ * 3 diag, 4 relabel, 5 swap. */
+qgpu_status qgpu_circuit_plan(const qgpu_circuit* c, int n_qubits, int world_size, int reorder,
+                              int fuse_bits, int64_t* info, uint64_t cap, uint64_t* n_passes);
+
+/* ---- scheduler state (tests / diagnostics) ---------------------------------------------- */
+
+/* Current `involvement` flags, bit q = logical qubit q has been acted on. */
+qgpu_status qgpu_get_involvement(qgpu_state* st, uint64_t* mask);
+
+/* Logical chunk bitmap for chunk size 2^chunk_bits: bit j (word j/64, bit j%64) = 1 iff
+ * chunk j may hold a non-zero amplitude, i.e. ((j << c) & ~involvement) == 0.
+ * n_words must be >= ceil(2^(n-c) / 64). */
+qgpu_status qgpu_get_chunk_bitmap(qgpu_state* st, int chunk_bits, uint64_t* words,
+                                  uint64_t n_words);
+
+/* Execution trace since the last reset: order[k] = program index (within its circuit, or a
+ * running gate counter for qgpu_apply_gate) of the k-th executed gate and
+ * involvement_after[k] the flags after it. Either output may be NULL. *n = trace length. */
+qgpu_status qgpu_get_schedule(qgpu_state* st, uint64_t* order, uint64_t* involvement_after,
+                              uint64_t cap, uint64_t* n);
+
+/* Physical position of each logical qubit (-1 = never involved), pos[n_qubits]. */
+qgpu_status qgpu_get_qubit_map(qgpu_state* st, int* pos);
+
+qgpu_status qgpu_get_stats(qgpu_state* st, qgpu_stats* out);
+qgpu_status qgpu_reset_stats(qgpu_state* st);
+
+/* Thread-local detail of the last error on this thread (valid until the next call). */
+const char* qgpu_last_error(void);
+
+/* Library version / build string (ABI version, arch). */
+const char* qgpu_version(void);
+
+#ifdef __cplusplus
+}
+#endif
+#endif /* QGPU_H */

@@ -1,0 +1,780 @@
+// C ABI of libqgpu (include/qgpu.h): state management, execution of the planned passes,
+// readout, statistics. No exception crosses the ABI; every CUDA error is mapped to a status.
+#include <cuda_runtime.h>
+
+#include <algorithm>
+#include <bit>
+#include <cstdarg>
+#include <cstdio>
+#include <cstring>
+#include <exception>
+#include <string>
+#include <vector>
+
+#include "comm.h"
+#include "kernels.h"
+#include "qgpu_internal.h"
+
+using namespace qgpu;
+
+struct qgpu_circuit {
+  Circuit c;
+};
+
+namespace {
+
+thread_local std::string g_err;
+
+qgpu_status fail(qgpu_status s, const char* fmt, ...) {
+  char buf[1024];
+  va_list ap;
+  va_start(ap, fmt);
+  vsnprintf(buf, sizeof(buf), fmt, ap);
+  va_end(ap);
+  g_err = buf;
+  return s;
+}
+
+struct TimedLaunch {
+  cudaEvent_t a, b;
+  int kind;
+  uint64_t bytes;
+};
+
+}  // namespace
+
+struct qgpu_state {
+  qgpu_config cfg;
+  int n = 0, g = 0, m = 0;
+  cudaStream_t stream = nullptr;
+  bool own_stream = false;
+  double2* psi = nullptr;
+  bool own_buf = false;
+  uint64_t cap_amps = 0;
+  QubitMap map;
+  std::vector<uint64_t> trace_order, trace_inv;
+  uint64_t gate_counter = 0;
+  qgpu_stats stats;
+  bool poisoned = false;
+  // device op arena (fused tile passes read their ops from here)
+  DevOp* d_ops = nullptr;
+  DevOp* h_ops = nullptr;
+  size_t ops_cap = 0;
+  cudaEvent_t ops_evt = nullptr;
+  // readout scratch
+  double* d_scratch = nullptr;
+  size_t scratch_cap = 0;  // doubles
+  // timing
+  std::vector<TimedLaunch> pending;
+  std::vector<cudaEvent_t> event_pool;
+  Comm* comm = nullptr;
+};
+
+namespace {
+
+#define CK(expr)                                                                        \
+  do {                                                                                  \
+    cudaError_t _e = (expr);                                                            \
+    if (_e != cudaSuccess) {                                                            \
+      st->poisoned = true;                                                              \
+      return fail(QGPU_ERR_CUDA, "%s: %s (%s:%d)", #expr, cudaGetErrorString(_e), __FILE__, \
+                  __LINE__);                                                            \
+    }                                                                                   \
+  } while (0)
+
+#define CK0(expr)                                                                        \
+  do {                                                                                   \
+    cudaError_t _e = (expr);                                                             \
+    if (_e != cudaSuccess)                                                               \
+      return fail(QGPU_ERR_CUDA, "%s: %s", #expr, cudaGetErrorString(_e));               \
+  } while (0)
+
+cudaEvent_t get_event(qgpu_state* st) {
+  if (!st->event_pool.empty()) {
+    cudaEvent_t e = st->event_pool.back();
+    st->event_pool.pop_back();
+    return e;
+  }
+  cudaEvent_t e = nullptr;
+  cudaEventCreate(&e);
+  return e;
+}
+
+qgpu_status drain_timing(qgpu_state* st) {
+  for (auto& t : st->pending) {
+    CK(cudaEventSynchronize(t.b));
+    float ms = 0;
+    CK(cudaEventElapsedTime(&ms, t.a, t.b));
+    if (t.kind == PK_SWAP) {
+      st->stats.swap_ms += ms;
+    } else {
+      st->stats.kernel_ms += ms;
+      if (t.kind == PK_TILE) {
+        st->stats.tile_kernel_ms += ms;
+        st->stats.tile_kernel_launches++;
+        st->stats.tile_algo_bytes += t.bytes;
+      }
+    }
+    st->event_pool.push_back(t.a);
+    st->event_pool.push_back(t.b);
+  }
+  st->pending.clear();
+  return QGPU_OK;
+}
+
+inline uint64_t live(const qgpu_state* st, int k) {
+  return st->cfg.prune ? (1ull << k) : (1ull << st->m);
+}
+
+void account(qgpu_state* st, uint64_t L_out, uint64_t bytes) {
+  qgpu_stats& s = st->stats;
+  s.passes++;
+  s.amps_processed += L_out;
+  s.amps_full += 1ull << st->m;
+  const int c = std::min(std::max(st->cfg.chunk_bits, 0), st->m);
+  const uint64_t chunk = 1ull << c;
+  const uint64_t proc = (L_out + chunk - 1) / chunk;
+  s.chunks_processed += proc;
+  s.chunks_skipped += (1ull << (st->m - c)) - proc;
+  s.algo_bytes += bytes;
+}
+
+void sorted_positions(uint64_t mask, int* out, int* n) {
+  *n = 0;
+  for (; mask; mask &= mask - 1) out[(*n)++] = std::countr_zero(mask);
+}
+
+qgpu_status zero_fill(qgpu_state* st, uint64_t from, uint64_t to) {
+  if (to > from) CK(cudaMemsetAsync(st->psi + from, 0, (to - from) * sizeof(double2), st->stream));
+  return QGPU_OK;
+}
+
+// Execute one planned pass on this rank's local buffer.
+qgpu_status exec_pass(qgpu_state* st, const Pass& p, const DevOp* d_ops) {
+  const int m = st->m;
+  const uint64_t lmask = (m >= 64) ? ~0ull : ((1ull << m) - 1);
+  const int kin = st->cfg.prune ? p.k_in : m, kout = st->cfg.prune ? p.k_out : m;
+  const uint64_t L_in = 1ull << kin, L_out = 1ull << kout;
+  const bool timing = st->cfg.timing != 0;
+  TimedLaunch tl{};
+  uint64_t bytes = 0;
+  if (p.kind == PK_RELABEL) {
+    if (kout > kin) {
+      qgpu_status s = zero_fill(st, L_in, L_out);
+      if (s) return s;
+      st->stats.kernels_launched++;
+      account(st, L_out, 16 * (L_out - L_in));
+    }
+    return QGPU_OK;
+  }
+  if (timing) {
+    tl.a = get_event(st);
+    tl.b = get_event(st);
+    tl.kind = p.kind;
+    CK(cudaEventRecord(tl.a, st->stream));
+  }
+  const uint64_t rank = uint64_t(st->cfg.rank);
+  if (p.kind == PK_TILE) {
+    TileArgs a{};
+    a.psi = st->psi;
+    a.ops = d_ops;
+    a.nops = int(p.ops.size());
+    a.b = p.b;
+    a.l = p.l;
+    for (int i = 0; i < p.b; ++i) a.spos[i] = p.spos[i];
+    a.ntiles = 1ull << (kout - p.b);
+    a.L_in = L_in;
+    a.rank_base = rank << m;
+    CK(launch_tile(st->stream, a));
+    st->stats.kernels_launched++;
+    bytes = 16 * (L_in + L_out);
+  } else {
+    const PhysGate& g = p.gates[0];
+    const uint64_t gpc = g.pc & ~lmask;                  // controls on rank bits
+    const bool rank_ok = ((rank << m) & gpc) == gpc;
+    const uint64_t lc = g.pc & lmask;
+    if (!rank_ok) {
+      // identity on this rank; the expanded region still has to read as zero
+      qgpu_status s = zero_fill(st, L_in, L_out);
+      if (s) return s;
+      bytes = 16 * (L_out - L_in);
+    } else if (p.kind == PK_PAIR || p.kind == PK_QUAD) {
+      const bool full = g.expands_target || !st->cfg.prune;
+      const int krun = full ? kout : kin;
+      if (!full) {
+        qgpu_status s = zero_fill(st, L_in, L_out);
+        if (s) return s;
+      }
+      const int nlc = std::popcount(lc);
+      const bool ctl_in_range = (lc >> krun) == 0;
+      if (p.kind == PK_PAIR) {
+        PairArgs a{};
+        a.psi = st->psi;
+        for (int i = 0; i < 4; ++i) a.u[i] = make_double2(g.U[i].re, g.U[i].im);
+        a.t = g.p[0];
+        sorted_positions(lc | (1ull << g.p[0]), a.ins, &a.nins);
+        sorted_positions(lc, a.ins_c, &a.nins_c);
+        a.cset = lc;
+        a.npairs = ctl_in_range ? (1ull << (krun - 1 - nlc)) : 0;
+        a.L_in = L_in;
+        const bool shfl = g.p[0] < 5 && krun >= 5 && (lc & 31) == 0;
+        CK(launch_pair(st->stream, a, shfl));
+        bytes = 32 * a.npairs + (full ? 0 : 16 * (L_out - L_in));
+      } else {
+        QuadArgs a{};
+        a.psi = st->psi;
+        for (int i = 0; i < 16; ++i) a.u[i] = make_double2(g.U[i].re, g.U[i].im);
+        a.t0 = g.p[0];
+        a.t1 = g.p[1];
+        sorted_positions(lc | (1ull << g.p[0]) | (1ull << g.p[1]), a.ins, &a.nins);
+        a.cset = lc;
+        a.nquads = ctl_in_range ? (1ull << (krun - 2 - nlc)) : 0;
+        a.L_in = L_in;
+        CK(launch_quad(st->stream, a));
+        bytes = 64 * a.nquads + (full ? 0 : 16 * (L_out - L_in));
+      }
+      st->stats.kernels_launched++;
+    } else {  // PK_DIAG: the expanded region stays zero under a diagonal gate
+      qgpu_status s = zero_fill(st, L_in, L_out);
+      if (s) return s;
+      PhaseArgs a{};
+      a.psi = st->psi;
+      a.nt = g.nt;
+      a.t0 = g.p[0];
+      a.t1 = g.p[1];
+      const int dim = 1 << g.nt;
+      int n_not1 = 0, which = 0;
+      for (int v = 0; v < dim; ++v) {
+        const cplx d = g.U[v * (dim + 1)];
+        a.d[v] = make_double2(d.re, d.im);
+        if (!(d.re == 1.0 && d.im == 0.0)) { ++n_not1; which = v; }
+      }
+      // TODO(sharded): targets on rank bits select the entry per rank
+      uint64_t fixed = lc, insmask = lc;
+      if (n_not1 == 1) {
+        for (int j = 0; j < g.nt; ++j) {
+          insmask |= 1ull << g.p[j];
+          if (which >> j & 1) fixed |= 1ull << g.p[j];
+        }
+      }
+      a.fixed = fixed;
+      sorted_positions(insmask, a.ins, &a.nins);
+      const bool in_range = (insmask >> kin) == 0;
+      a.count = (n_not1 == 0 || !in_range) ? 0 : (1ull << (kin - a.nins));
+      CK(launch_phase(st->stream, a));
+      st->stats.kernels_launched++;
+      bytes = 32 * a.count + 16 * (L_out - L_in);
+    }
+  }
+  if (timing) {
+    CK(cudaEventRecord(tl.b, st->stream));
+    tl.bytes = bytes;
+    st->pending.push_back(tl);
+  }
+  account(st, L_out, bytes);
+  st->stats.unfused_bytes += p.unfused_bytes;
+  return QGPU_OK;
+}
+
+qgpu_status ensure_ops(qgpu_state* st, size_t n) {
+  if (n <= st->ops_cap) return QGPU_OK;
+  size_t cap = std::max<size_t>(n, 2 * st->ops_cap);
+  cap = std::max<size_t>(cap, 1024);
+  CK(cudaStreamSynchronize(st->stream));
+  if (st->d_ops) CK(cudaFree(st->d_ops));
+  if (st->h_ops) CK(cudaFreeHost(st->h_ops));
+  st->d_ops = nullptr;
+  st->h_ops = nullptr;
+  CK(cudaMalloc(&st->d_ops, cap * sizeof(DevOp)));
+  CK(cudaMallocHost(&st->h_ops, cap * sizeof(DevOp)));
+  st->ops_cap = cap;
+  return QGPU_OK;
+}
+
+qgpu_status run_plan(qgpu_state* st, const std::vector<Pass>& passes) {
+  size_t nops = 0;
+  for (const Pass& p : passes) nops += p.ops.size();
+  std::vector<size_t> off(passes.size(), 0);
+  if (nops) {
+    qgpu_status s = ensure_ops(st, nops);
+    if (s) return s;
+    // the pinned staging buffer may still be read by the previous upload
+    CK(cudaEventSynchronize(st->ops_evt));
+    size_t o = 0;
+    for (size_t i = 0; i < passes.size(); ++i) {
+      off[i] = o;
+      if (!passes[i].ops.empty())
+        std::memcpy(st->h_ops + o, passes[i].ops.data(), passes[i].ops.size() * sizeof(DevOp));
+      o += passes[i].ops.size();
+    }
+    CK(cudaMemcpyAsync(st->d_ops, st->h_ops, nops * sizeof(DevOp), cudaMemcpyHostToDevice,
+                       st->stream));
+    CK(cudaEventRecord(st->ops_evt, st->stream));
+  }
+  for (size_t i = 0; i < passes.size(); ++i) {
+    qgpu_status s = exec_pass(st, passes[i], st->d_ops + off[i]);
+    if (s) return s;
+  }
+  return QGPU_OK;
+}
+
+void record_trace(qgpu_state* st, const std::vector<int>& order, const std::vector<uint64_t>& inv,
+                  uint64_t base) {
+  const uint64_t full = (st->n >= 64) ? ~0ull : ((1ull << st->n) - 1);
+  for (size_t k = 0; k < order.size(); ++k) {
+    if (st->stats.ops_before_full_involvement < 0 && inv[k] == full)
+      st->stats.ops_before_full_involvement = int64_t(st->trace_order.size());
+    st->trace_order.push_back(base + uint64_t(order[k]));
+    st->trace_inv.push_back(inv[k]);
+  }
+  st->stats.gates_applied += order.size();
+}
+
+qgpu_status check_state(qgpu_state* st) {
+  if (!st) return fail(QGPU_ERR_INVALID_ARG, "state is NULL");
+  if (st->poisoned) return fail(QGPU_ERR_STATE, "state poisoned by an earlier CUDA/NCCL failure");
+  return QGPU_OK;
+}
+
+qgpu_status init_amplitudes(qgpu_state* st) {
+  if (!st->cfg.prune) CK(cudaMemsetAsync(st->psi, 0, (1ull << st->m) * sizeof(double2), st->stream));
+  if (st->cfg.rank == 0) CK(launch_set_amp(st->stream, st->psi, 0, 1.0, 0.0));
+  return QGPU_OK;
+}
+
+PlanOptions plan_options(const qgpu_config& cfg, bool fuse) {
+  PlanOptions o;
+  o.fuse_bits = fuse ? cfg.fuse_bits : 0;
+  o.prune = cfg.prune != 0;
+  return o;
+}
+
+}  // namespace
+
+extern "C" {
+
+const char* qgpu_last_error(void) { return g_err.c_str(); }
+
+const char* qgpu_version(void) {
+  return "qgpu abi " "1" " sm_100a (B200) complex128";
+}
+
+qgpu_status qgpu_config_init(qgpu_config* cfg) {
+  if (!cfg) return fail(QGPU_ERR_INVALID_ARG, "cfg is NULL");
+  std::memset(cfg, 0, sizeof(*cfg));
+  cfg->struct_size = sizeof(qgpu_config);
+  cfg->world_size = 1;
+  cfg->chunk_bits = 21;
+  cfg->prune = 1;
+  cfg->reorder = 2;
+  cfg->fuse_bits = 12;
+  cfg->swap_slab_bytes = 256ull << 20;
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out) {
+  try {
+    if (!out) return fail(QGPU_ERR_INVALID_ARG, "out is NULL");
+    *out = nullptr;
+    qgpu_config cfg;
+    qgpu_config_init(&cfg);
+    if (cfg_in) {
+      if (cfg_in->struct_size != sizeof(qgpu_config))
+        return fail(QGPU_ERR_INVALID_ARG, "qgpu_config.struct_size mismatch (%u != %zu)",
+                    cfg_in->struct_size, sizeof(qgpu_config));
+      cfg = *cfg_in;
+    }
+    if (n < 1 || n > kMaxQubits) return fail(QGPU_ERR_INVALID_ARG, "n_qubits %d out of [1, %d]", n, kMaxQubits);
+    if (cfg.world_size < 1 || (cfg.world_size & (cfg.world_size - 1)))
+      return fail(QGPU_ERR_INVALID_ARG, "world_size %d is not a power of two", cfg.world_size);
+    if (cfg.rank < 0 || cfg.rank >= cfg.world_size)
+      return fail(QGPU_ERR_INVALID_ARG, "rank %d out of range", cfg.rank);
+    const int g = std::countr_zero(unsigned(cfg.world_size));
+    if (n - g < 5) return fail(QGPU_ERR_INVALID_ARG, "need n - log2(world_size) >= 5");
+    if (cfg.fuse_bits < 0 || cfg.fuse_bits > kMaxTileBits - 1)
+      return fail(QGPU_ERR_INVALID_ARG, "fuse_bits %d out of [0, %d]", cfg.fuse_bits, kMaxTileBits - 1);
+    if (cfg.fuse_bits > 0 && cfg.fuse_bits < 7)
+      return fail(QGPU_ERR_INVALID_ARG, "fuse_bits must be 0 or >= 7");
+    if (cfg.reorder < 0 || cfg.reorder > 2) return fail(QGPU_ERR_INVALID_ARG, "reorder must be 0, 1 or 2");
+    cfg.chunk_bits = std::min(std::max(cfg.chunk_bits, 0), n - g);
+    auto* st = new qgpu_state();
+    st->cfg = cfg;
+    st->n = n;
+    st->g = g;
+    st->m = n - g;
+    st->map.init(n, st->m);
+    std::memset(&st->stats, 0, sizeof(st->stats));
+    st->stats.ops_before_full_involvement = -1;
+    auto bail = [&](qgpu_status s) {
+      qgpu_state_destroy(st);
+      return s;
+    };
+    cudaError_t e = cudaSetDevice(cfg.device);
+    if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaSetDevice(%d): %s", cfg.device, cudaGetErrorString(e)));
+    if (cfg.stream) {
+      st->stream = static_cast<cudaStream_t>(cfg.stream);
+    } else {
+      e = cudaStreamCreateWithFlags(&st->stream, cudaStreamNonBlocking);
+      if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaStreamCreate: %s", cudaGetErrorString(e)));
+      st->own_stream = true;
+    }
+    const uint64_t need = (1ull << st->m) * sizeof(double2);
+    if (cfg.state_buffer) {
+      if (cfg.state_buffer_bytes < need)
+        return bail(fail(QGPU_ERR_OUT_OF_MEMORY, "state_buffer has %llu bytes, need %llu",
+                         (unsigned long long)cfg.state_buffer_bytes, (unsigned long long)need));
+      if (reinterpret_cast<uintptr_t>(cfg.state_buffer) % 16)
+        return bail(fail(QGPU_ERR_INVALID_ARG, "state_buffer must be 16-byte aligned"));
+      st->psi = static_cast<double2*>(cfg.state_buffer);
+    } else {
+      e = cudaMalloc(&st->psi, need);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        return bail(fail(QGPU_ERR_OUT_OF_MEMORY, "cudaMalloc(%llu): %s", (unsigned long long)need,
+                         cudaGetErrorString(e)));
+      }
+      st->own_buf = true;
+    }
+    st->cap_amps = 1ull << st->m;
+    e = cudaEventCreateWithFlags(&st->ops_evt, cudaEventDisableTiming);
+    if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e)));
+    if (cfg.world_size > 1) {
+      qgpu_status s = comm_create(&st->comm, cfg, st->stream, &g_err);
+      if (s) return bail(s);
+    }
+    qgpu_status s = init_amplitudes(st);
+    if (s) return bail(s);
+    *out = st;
+    return QGPU_OK;
+  } catch (const std::exception& ex) {
+    return fail(QGPU_ERR_OUT_OF_MEMORY, "exception: %s", ex.what());
+  }
+}
+
+qgpu_status qgpu_state_destroy(qgpu_state* st) {
+  if (!st) return QGPU_OK;
+  if (st->stream) cudaStreamSynchronize(st->stream);
+  for (auto& t : st->pending) {
+    cudaEventDestroy(t.a);
+    cudaEventDestroy(t.b);
+  }
+  for (auto e : st->event_pool) cudaEventDestroy(e);
+  if (st->comm) comm_destroy(st->comm);
+  if (st->own_buf && st->psi) cudaFree(st->psi);
+  if (st->d_ops) cudaFree(st->d_ops);
+  if (st->h_ops) cudaFreeHost(st->h_ops);
+  if (st->d_scratch) cudaFree(st->d_scratch);
+  if (st->ops_evt) cudaEventDestroy(st->ops_evt);
+  if (st->own_stream && st->stream) cudaStreamDestroy(st->stream);
+  delete st;
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_state_reset(qgpu_state* st) {
+  if (qgpu_status s = check_state(st)) return s;
+  st->map.init(st->n, st->m);
+  st->trace_order.clear();
+  st->trace_inv.clear();
+  st->gate_counter = 0;
+  if (qgpu_status s = drain_timing(st)) return s;
+  std::memset(&st->stats, 0, sizeof(st->stats));
+  st->stats.ops_before_full_involvement = -1;
+  return init_amplitudes(st);
+}
+
+qgpu_status qgpu_set_amplitudes(qgpu_state* st, const double* amps) {
+  if (qgpu_status s = check_state(st)) return s;
+  if (!amps) return fail(QGPU_ERR_INVALID_ARG, "amps is NULL");
+  if (st->g > 0) return fail(QGPU_ERR_UNSUPPORTED, "set_amplitudes is single-GPU only");
+  CK(cudaMemcpyAsync(st->psi, amps, (1ull << st->n) * sizeof(double2), cudaMemcpyHostToDevice, st->stream));
+  CK(cudaStreamSynchronize(st->stream));
+  st->map.init(st->n, st->m);
+  for (int q = 0; q < st->n; ++q) {
+    st->map.pos[q] = q;
+    st->map.lq[q] = q;
+  }
+  st->map.kl = st->n;
+  st->map.involvement = (st->n >= 64) ? ~0ull : ((1ull << st->n) - 1);
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_synchronize(qgpu_state* st) {
+  if (qgpu_status s = check_state(st)) return s;
+  CK(cudaStreamSynchronize(st->stream));
+  return drain_timing(st);
+}
+
+qgpu_status qgpu_state_info(const qgpu_state* st, int* n, int* nl, void** dev) {
+  if (!st) return fail(QGPU_ERR_INVALID_ARG, "state is NULL");
+  if (n) *n = st->n;
+  if (nl) *nl = st->m;
+  if (dev) *dev = st->psi;
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_apply_gate(qgpu_state* st, const double* U, int nt, const int* targets, int nc,
+                            const int* controls) {
+  try {
+    if (qgpu_status s = check_state(st)) return s;
+    if (!U || !targets) return fail(QGPU_ERR_INVALID_ARG, "U/targets is NULL");
+    if (nt < 1 || nt > 2) return fail(QGPU_ERR_INVALID_ARG, "n_targets must be 1 or 2");
+    if (nc < 0 || (nc > 0 && !controls)) return fail(QGPU_ERR_INVALID_ARG, "bad controls");
+    Gate g;
+    g.nt = nt;
+    uint64_t seen = 0;
+    for (int j = 0; j < nt + nc; ++j) {
+      const int q = j < nt ? targets[j] : controls[j - nt];
+      if (q < 0 || q >= st->n) return fail(QGPU_ERR_INVALID_ARG, "qubit %d out of range [0, %d)", q, st->n);
+      if (seen >> q & 1) return fail(QGPU_ERR_INVALID_ARG, "qubit %d repeated", q);
+      seen |= 1ull << q;
+      if (j < nt) g.t[j] = q;
+      else g.cmask |= 1ull << q;
+    }
+    const int dim = 1 << nt;
+    for (int i = 0; i < dim * dim; ++i) g.U[i] = cplx{U[2 * i], U[2 * i + 1]};
+    g.diag = is_diagonal(g.U, nt);
+    g.relabel = false;  // an explicit gate call always moves data
+    std::vector<Gate> gs{g};
+    std::vector<int> order{0};
+    std::vector<Pass> passes;
+    std::vector<uint64_t> inv;
+    plan_circuit(gs, order, st->map, plan_options(st->cfg, false), &passes, &inv);
+    record_trace(st, order, inv, st->gate_counter);
+    st->gate_counter++;
+    return run_plan(st, passes);
+  } catch (const std::exception& ex) {
+    return fail(QGPU_ERR_OUT_OF_MEMORY, "exception: %s", ex.what());
+  }
+}
+
+qgpu_status qgpu_apply_circuit(qgpu_state* st, const qgpu_circuit* c) {
+  try {
+    if (qgpu_status s = check_state(st)) return s;
+    if (!c) return fail(QGPU_ERR_INVALID_ARG, "circuit is NULL");
+    if (c->c.n > st->n) return fail(QGPU_ERR_INVALID_ARG, "circuit has %d qubits, state %d", c->c.n, st->n);
+    std::vector<int> order = reorder(c->c.gates, st->cfg.reorder);
+    std::vector<Pass> passes;
+    std::vector<uint64_t> inv;
+    plan_circuit(c->c.gates, order, st->map, plan_options(st->cfg, st->cfg.fuse_bits > 0), &passes, &inv);
+    record_trace(st, order, inv, 0);
+    for (const Gate& g : c->c.gates) st->stats.relabels += g.relabel ? 1 : 0;
+    return run_plan(st, passes);
+  } catch (const std::exception& ex) {
+    return fail(QGPU_ERR_OUT_OF_MEMORY, "exception: %s", ex.what());
+  }
+}
+
+qgpu_status qgpu_get_amplitudes_device(qgpu_state* st, uint64_t start, uint64_t count, double* dev_out) {
+  if (qgpu_status s = check_state(st)) return s;
+  if (!dev_out && count) return fail(QGPU_ERR_INVALID_ARG, "dev_out is NULL");
+  if (start + count > (1ull << st->n) || start + count < start)
+    return fail(QGPU_ERR_INVALID_ARG, "range [%llu, +%llu) outside 2^%d", (unsigned long long)start,
+                (unsigned long long)count, st->n);
+  if (st->g > 0) return fail(QGPU_ERR_UNSUPPORTED, "sharded get_amplitudes: use qgpu_get_amplitudes");
+  GatherArgs a{};
+  a.psi = st->psi;
+  a.out = reinterpret_cast<double2*>(dev_out);
+  a.start = start;
+  a.count = count;
+  a.n = st->n;
+  a.m = st->m;
+  a.rank = uint64_t(st->cfg.rank);
+  for (int q = 0; q < st->n; ++q) {
+    a.pos[q] = st->map.pos[q] < 0 ? 0 : st->map.pos[q];
+    if (st->map.pos[q] < 0) a.unassigned |= 1ull << q;
+  }
+  a.L = live(st, st->map.kl);
+  CK(launch_gather(st->stream, a));
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_get_amplitudes(qgpu_state* st, uint64_t start, uint64_t count, double* out) {
+  if (qgpu_status s = check_state(st)) return s;
+  if (!out && count) return fail(QGPU_ERR_INVALID_ARG, "out is NULL");
+  if (st->g > 0) return comm_get_amplitudes(st->comm, st, start, count, out);
+  const uint64_t chunk = std::min<uint64_t>(count, 1ull << 24);
+  if (chunk > st->scratch_cap / 2) {
+    CK(cudaStreamSynchronize(st->stream));
+    if (st->d_scratch) CK(cudaFree(st->d_scratch));
+    st->d_scratch = nullptr;
+    CK(cudaMalloc(&st->d_scratch, chunk * 2 * sizeof(double)));
+    st->scratch_cap = chunk * 2;
+  }
+  for (uint64_t done = 0; done < count; done += chunk) {
+    const uint64_t c = std::min(chunk, count - done);
+    if (qgpu_status s = qgpu_get_amplitudes_device(st, start + done, c, st->d_scratch)) return s;
+    CK(cudaMemcpyAsync(out + 2 * done, st->d_scratch, c * 2 * sizeof(double), cudaMemcpyDeviceToHost, st->stream));
+  }
+  CK(cudaStreamSynchronize(st->stream));
+  return drain_timing(st);
+}
+
+qgpu_status qgpu_probabilities(qgpu_state* st, int mq, const int* qubits, double* out) {
+  if (qgpu_status s = check_state(st)) return s;
+  if (mq < 0 || mq > 30) return fail(QGPU_ERR_INVALID_ARG, "m=%d out of [0, 30]", mq);
+  if (!out || (mq > 0 && !qubits)) return fail(QGPU_ERR_INVALID_ARG, "NULL argument");
+  ProbArgs a{};
+  a.psi = st->psi;
+  a.m = mq;
+  uint64_t seen = 0;
+  uint64_t rank_fixed = 0;  // requested qubits on rank bits (sharded)
+  for (int j = 0; j < mq; ++j) {
+    const int q = qubits[j];
+    if (q < 0 || q >= st->n || (seen >> q & 1)) return fail(QGPU_ERR_INVALID_ARG, "bad qubit %d", q);
+    seen |= 1ull << q;
+    const int p = st->map.pos[q];
+    a.ppos[j] = (p < 0 || p >= st->m) ? 63 : p;
+    if (p >= st->m && (uint64_t(st->cfg.rank) >> (p - st->m) & 1)) rank_fixed |= 1ull << j;
+  }
+  a.L = live(st, st->map.kl);
+  const bool active = st->g == 0 || (uint64_t(st->cfg.rank) >> st->map.kg) == 0;
+  if (!active) a.L = 0;
+  const size_t B = size_t(1) << mq;
+  const size_t need = B + probs_scratch_doubles(mq);
+  if (need > st->scratch_cap) {
+    CK(cudaStreamSynchronize(st->stream));
+    if (st->d_scratch) CK(cudaFree(st->d_scratch));
+    st->d_scratch = nullptr;
+    CK(cudaMalloc(&st->d_scratch, need * sizeof(double)));
+    st->scratch_cap = need;
+  }
+  a.out = st->d_scratch;
+  CK(launch_probs(st->stream, a, st->d_scratch + B));
+  if (st->g > 0) {
+    qgpu_status s = comm_probabilities_finish(st->comm, st->d_scratch, mq, rank_fixed, st->stream);
+    if (s) return s;
+  }
+  CK(cudaMemcpyAsync(out, st->d_scratch, B * sizeof(double), cudaMemcpyDeviceToHost, st->stream));
+  CK(cudaStreamSynchronize(st->stream));
+  return drain_timing(st);
+}
+
+qgpu_status qgpu_circuit_from_qasm(const char* text, size_t len, qgpu_circuit** out) {
+  try {
+    if (!text || !out) return fail(QGPU_ERR_INVALID_ARG, "NULL argument");
+    *out = nullptr;
+    auto* c = new qgpu_circuit();
+    std::string err;
+    qgpu_status s = parse_qasm(text, len, &c->c, &err);
+    if (s) {
+      delete c;
+      return fail(s, "%s", err.c_str());
+    }
+    *out = c;
+    return QGPU_OK;
+  } catch (const std::exception& ex) {
+    return fail(QGPU_ERR_OUT_OF_MEMORY, "exception: %s", ex.what());
+  }
+}
+
+qgpu_status qgpu_circuit_info(const qgpu_circuit* c, int* n, uint64_t* ng) {
+  if (!c) return fail(QGPU_ERR_INVALID_ARG, "circuit is NULL");
+  if (n) *n = c->c.n;
+  if (ng) *ng = c->c.gates.size();
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_circuit_destroy(qgpu_circuit* c) {
+  delete c;
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_circuit_reorder(const qgpu_circuit* c, int mode, uint64_t* order, uint64_t cap, uint64_t* n) {
+  try {
+    if (!c) return fail(QGPU_ERR_INVALID_ARG, "circuit is NULL");
+    if (mode < 0 || mode > 2) return fail(QGPU_ERR_INVALID_ARG, "mode must be 0, 1 or 2");
+    std::vector<int> o = reorder(c->c.gates, mode);
+    if (n) *n = o.size();
+    if (order)
+      for (uint64_t i = 0; i < std::min<uint64_t>(cap, o.size()); ++i) order[i] = uint64_t(o[i]);
+    return QGPU_OK;
+  } catch (const std::exception& ex) {
+    return fail(QGPU_ERR_OUT_OF_MEMORY, "exception: %s", ex.what());
+  }
+}
+
+qgpu_status qgpu_circuit_plan(const qgpu_circuit* c, int n, int world, int reorder_mode, int fuse_bits,
+                              int64_t* info, uint64_t cap, uint64_t* n_passes) {
+  try {
+    if (!c) return fail(QGPU_ERR_INVALID_ARG, "circuit is NULL");
+    if (n < c->c.n || n > kMaxQubits) return fail(QGPU_ERR_INVALID_ARG, "bad n");
+    if (world < 1 || (world & (world - 1))) return fail(QGPU_ERR_INVALID_ARG, "bad world size");
+    const int g = std::countr_zero(unsigned(world));
+    QubitMap map;
+    map.init(n, n - g);
+    PlanOptions o;
+    o.fuse_bits = fuse_bits;
+    std::vector<Pass> passes;
+    plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode), map, o, &passes, nullptr);
+    if (n_passes) *n_passes = passes.size();
+    for (uint64_t i = 0; info && i < std::min<uint64_t>(cap, passes.size()); ++i) {
+      const Pass& p = passes[i];
+      uint64_t S = 0;
+      for (int j = 0; j < p.b; ++j) S |= 1ull << p.spos[j];
+      int64_t* r = info + 8 * i;
+      r[0] = p.first; r[1] = p.count; r[2] = p.kind; r[3] = p.k_in; r[4] = p.k_out; r[5] = p.b;
+      r[6] = int64_t(S & 0xffffffffull);
+      r[7] = int64_t(S >> 32);
+    }
+    return QGPU_OK;
+  } catch (const std::exception& ex) {
+    return fail(QGPU_ERR_OUT_OF_MEMORY, "exception: %s", ex.what());
+  }
+}
+
+qgpu_status qgpu_get_involvement(qgpu_state* st, uint64_t* mask) {
+  if (!st || !mask) return fail(QGPU_ERR_INVALID_ARG, "NULL argument");
+  *mask = st->map.involvement;
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_get_chunk_bitmap(qgpu_state* st, int c, uint64_t* words, uint64_t n_words) {
+  if (!st || !words) return fail(QGPU_ERR_INVALID_ARG, "NULL argument");
+  if (c < 0 || c > st->n) return fail(QGPU_ERR_INVALID_ARG, "chunk_bits out of range");
+  const uint64_t nch = 1ull << (st->n - c);
+  if (n_words < (nch + 63) / 64) return fail(QGPU_ERR_INVALID_ARG, "n_words too small");
+  std::memset(words, 0, n_words * sizeof(uint64_t));
+  const uint64_t full = (st->n >= 64) ? ~0ull : ((1ull << st->n) - 1);
+  const uint64_t uninv = ~st->map.involvement & full;
+  // bit j set iff ((j << c) & ~involvement) == 0 (Alg.1 l.7)
+  for (uint64_t j = 0; j < nch; ++j)
+    if (((j << c) & uninv) == 0) words[j >> 6] |= 1ull << (j & 63);
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_get_schedule(qgpu_state* st, uint64_t* order, uint64_t* inv, uint64_t cap, uint64_t* n) {
+  if (!st) return fail(QGPU_ERR_INVALID_ARG, "state is NULL");
+  const uint64_t len = st->trace_order.size();
+  if (n) *n = len;
+  for (uint64_t i = 0; i < std::min(cap, len); ++i) {
+    if (order) order[i] = st->trace_order[i];
+    if (inv) inv[i] = st->trace_inv[i];
+  }
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_get_qubit_map(qgpu_state* st, int* pos) {
+  if (!st || !pos) return fail(QGPU_ERR_INVALID_ARG, "NULL argument");
+  for (int q = 0; q < st->n; ++q) pos[q] = st->map.pos[q];
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_get_stats(qgpu_state* st, qgpu_stats* out) {
+  if (!st || !out) return fail(QGPU_ERR_INVALID_ARG, "NULL argument");
+  if (!st->pending.empty()) {
+    if (qgpu_status s = drain_timing(st)) return s;
+  }
+  *out = st->stats;
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_reset_stats(qgpu_state* st) {
+  if (!st) return fail(QGPU_ERR_INVALID_ARG, "state is NULL");
+  if (qgpu_status s = drain_timing(st)) return s;
+  const int64_t obf = st->stats.ops_before_full_involvement;
+  std::memset(&st->stats, 0, sizeof(st->stats));
+  st->stats.ops_before_full_involvement = obf;
+  return QGPU_OK;
+}
+
+}  // extern "C"

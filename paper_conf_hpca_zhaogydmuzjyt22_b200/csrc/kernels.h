@@ -1,0 +1,85 @@
+// Kernel argument blocks and launchers (kernels.cu). Passed by value as kernel parameters.
+#pragma once
+
+#include <cuda_runtime.h>
+
+#include "qgpu_internal.h"
+
+namespace qgpu {
+
+struct PairArgs {
+  double2* psi;
+  double2 u[4];            // row-major 2x2
+  int t;                   // target position
+  int nins;                // inserted zero positions for pair enumeration (target + controls)
+  int ins[kMaxQubits];
+  int nins_c;              // controls only (shuffle variant: per-amplitude enumeration)
+  int ins_c[kMaxQubits];
+  uint64_t cset;           // local control bits forced to 1
+  uint64_t npairs;         // live pairs with controls satisfied
+  uint64_t L_in;           // reads at index >= L_in are implicit zeros (first-touch expand)
+};
+
+struct QuadArgs {
+  double2* psi;
+  double2 u[16];
+  int t0, t1;              // bit 0 / bit 1 of U's index
+  int nins;
+  int ins[kMaxQubits];
+  uint64_t cset;
+  uint64_t nquads;
+  uint64_t L_in;
+};
+
+struct PhaseArgs {
+  double2* psi;
+  double2 d[4];            // diagonal entries indexed by target bits
+  int nt, t0, t1;
+  int nins;
+  int ins[kMaxQubits];     // positions fixed by `fixed`
+  uint64_t fixed;          // bits forced to 1 (controls, and targets in the single-term form)
+  uint64_t count;          // amplitudes enumerated
+};
+
+struct TileArgs {
+  double2* psi;
+  const DevOp* ops;
+  int nops;
+  int b, l;
+  int spos[kMaxTileBits];
+  uint64_t ntiles;
+  uint64_t L_in;
+  uint64_t rank_base;      // rank << m (global bits for tile-uniform conditions)
+};
+
+struct GatherArgs {
+  const double2* psi;
+  double2* out;
+  uint64_t start, count;
+  int n, m;
+  uint64_t rank;
+  int pos[kMaxQubits];
+  uint64_t unassigned;     // logical qubits never involved (their |1> half is zero)
+  uint64_t L;              // live local size
+};
+
+struct ProbArgs {
+  const double2* psi;
+  uint64_t L;
+  int m;
+  int ppos[32];            // physical position of each requested qubit (63 = never set)
+  double* out;
+  double* partial;
+};
+
+size_t tile_smem_bytes(int b, int l);
+size_t probs_scratch_doubles(int m);
+cudaError_t launch_pair(cudaStream_t st, const PairArgs& a, bool shfl);
+cudaError_t launch_quad(cudaStream_t st, const QuadArgs& a);
+cudaError_t launch_phase(cudaStream_t st, const PhaseArgs& a);
+cudaError_t launch_tile(cudaStream_t st, const TileArgs& a);
+cudaError_t launch_gather(cudaStream_t st, const GatherArgs& a);
+cudaError_t launch_probs(cudaStream_t st, ProbArgs a, double* scratch);
+cudaError_t launch_set_amp(cudaStream_t st, double2* psi, uint64_t i, double re, double im);
+
+}  // namespace qgpu

@@ -1,0 +1,143 @@
+// Internal declarations of libqgpu (not part of the ABI).
+//
+// Layering:
+//   qasm.cpp    a1  OpenQASM-2 subset -> circuit IR (gate matrices in gates.cpp)
+//   sched.cpp   a2  dependency DAG + Alg.2 / Alg.3 reorder
+//               a3  involvement flags, first-touch qubit placement, chunk bitmap
+//               a4  pass planner: cuts the order into consecutive fused HBM passes
+//   kernels.cu  a5-a9, a11  sm_100a kernels (pair, quad, diag, fused tile, gather, reduce)
+//   comm.cpp    a10 global-local swaps over NCCL (sharded mode)
+//   api.cpp     the C ABI (include/qgpu.h)
+#pragma once
+
+#include <cstdint>
+#include <string>
+#include <vector>
+
+#include "../../include/qgpu.h"
+
+namespace qgpu {
+
+struct cplx {
+  double re, im;
+};
+
+constexpr int kMaxQubits = 40;
+
+// ------------------------------------------------------------------------------------ IR
+// One gate after lowering: target matrix U (2^nt x 2^nt, row-major, bit j of
+// the row/column index <-> t[j]) acting where every control in cmask is |1>.
+struct Gate {
+  int nt = 1;
+  int t[2] = {0, 0};
+  uint64_t cmask = 0;
+  cplx U[16];
+  bool diag = false;     // U is diagonal (z s t p rz cp cz crz rzz ...)
+  bool relabel = false;  // uncontrolled SWAP: executed as a qubit-map relabel
+  int line = 0;
+  uint64_t tmask() const {
+    uint64_t m = 1ull << t[0];
+    if (nt == 2) m |= 1ull << t[1];
+    return m;
+  }
+  uint64_t qmask() const { return tmask() | cmask; }  // qubits it involves (P:229 l.11)
+};
+
+struct Circuit {
+  int n = 0;
+  std::vector<Gate> gates;
+};
+
+qgpu_status parse_qasm(const char* text, size_t len, Circuit* out, std::string* err);
+// Lower a gate name: fills the arity and the target matrix; false if the name is unknown.
+bool gate_matrix(const std::string& name, const std::vector<double>& p, int* n_params,
+                 int* n_qubits, int* n_controls, cplx* U, bool build);
+bool is_diagonal(const cplx* U, int nt);
+bool is_swap_matrix(const cplx* U, int nt);
+
+// ------------------------------------------------------------------------------ schedule
+std::vector<int> reorder(const std::vector<Gate>& gates, int mode);  // 0, 1 (Alg.2), 2 (Alg.3)
+
+// Qubit map + involvement (a3). Physical positions 0..m-1 are local index bits, m..n-1 are
+// global (rank) bits when sharded. Positions are handed out in first-touch order, local ones
+// first, so the live part of every active rank's buffer is the prefix [0, 2^kl).
+struct QubitMap {
+  int n = 0, m = 0;              // total and local qubits
+  int pos[kMaxQubits];           // logical -> physical, -1 = never involved
+  int lq[kMaxQubits];            // physical -> logical, -1 = free
+  int kl = 0;                    // assigned local positions (live local size 2^kl)
+  int kg = 0;                    // assigned global positions (active ranks 2^kg)
+  uint64_t involvement = 0;      // P:223 flags (logical)
+  void init(int n_, int m_);
+  // Set involvement bits (P:229 l.11) and place the not-yet-placed qubits of `mask`
+  // (ascending logical index).
+  void touch(uint64_t mask);
+  uint64_t phys_mask(uint64_t logical_mask) const;
+  void swap_positions(int pa, int pb);  // exchange the logical qubits at two positions
+};
+
+// --------------------------------------------------------------------------- device ops
+enum OpKind : int { OP_U1 = 0, OP_U2 = 1, OP_PHASE = 2 };
+
+// One operation of a fused tile pass. Target bits t0/t1 and the per-amplitude condition
+// (lmask/lmatch) are in TILE-LOCAL bits; omask/omatch are physical local-index bits outside
+// the tile and gmask/gmatch rank bits: both are tile-uniform conditions.
+struct DevOp {
+  int kind;
+  int t0, t1;
+  uint32_t lmask, lmatch;
+  uint64_t omask, omatch;
+  double m[32];  // U1: 4 complex, U2: 16 complex, PHASE: 1 complex (re, im interleaved)
+};
+
+constexpr int kMaxTileBits = 13;
+
+// A gate in physical positions at its execution time.
+struct PhysGate {
+  int gate = -1;          // index into the circuit
+  int nt = 1;
+  int p[2] = {0, 0};      // physical targets
+  uint64_t pc = 0;        // physical control mask (may include global positions)
+  cplx U[16];
+  bool diag = false;
+  bool expands_target = false;  // a target was first touched by this gate
+};
+
+enum PassKind : int {
+  PK_TILE = 0, PK_PAIR = 1, PK_QUAD = 2, PK_DIAG = 3, PK_RELABEL = 4, PK_SWAP = 5
+};
+
+struct Pass {
+  int kind = PK_TILE;
+  int first = 0, count = 0;     // range in the execution order
+  int k_in = 0, k_out = 0;      // log2 local live size before / after the pass
+  // fused tile pass
+  int b = 0, l = 0;
+  int spos[kMaxTileBits];
+  std::vector<PhysGate> gates;  // gates of the pass (tile) or the single gate (pair/quad/diag)
+  std::vector<DevOp> ops;       // built at pass close (tile)
+  // swap pass (sharded)
+  int nswap = 0;
+  int swap_global[8], swap_local[8];
+  uint64_t unfused_bytes = 0;   // bytes the pass's gates would move one gate per pass
+};
+
+struct PlanOptions {
+  int fuse_bits = 12;   // b
+  int l_min = 5;        // minimum contiguous low tile bits (2^5 * 16 B = 512 B runs)
+  int max_u_ops = 24;   // non-diagonal ops per fused pass (FP64 / smem budget)
+  int max_ops = 256;    // all ops per fused pass
+  bool prune = true;
+};
+
+// Cut `order` of `gates` into passes, updating `map` (involvement, placement) exactly as the
+// execution will. inv_after[k] = involvement after the k-th executed gate.
+void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order, QubitMap& map,
+                  const PlanOptions& opt, std::vector<Pass>* passes,
+                  std::vector<uint64_t>* inv_after);
+// Build the device ops of a tile pass from its gates and tile positions.
+void build_tile_ops(Pass& p, int m);
+// Unfused byte model of one gate on live size 2^k.
+uint64_t unfused_gate_bytes(const PhysGate& g, int k_in, int k_out);
+
+}  // namespace qgpu

@@ -1,0 +1,350 @@
+// Host-side scheduler of the product path (independent of oracle/schedule.py).
+//
+// a2  Dependency DAG and reordering: Alg.2 greedy and Alg.3
+//     forward-looking. Readings: Q3 minimum search starts at +inf;
+//     Q4 deterministic tie-break, minimum of (cost, costCurrent, position in exeList), newly
+//     ready gates appended in ascending program index; Q5 one DAG edge per distinct
+//     most-recent predecessor on each operand qubit.
+// a3  involvement flags (Alg.1 l.11) and first-touch placement: a qubit receives the
+//     next free physical position the first time a gate involves it, so the non-zero part of
+//     the state ("2^n - 2^(n-m) amplitudes are zero") is the contiguous prefix
+//     [0, 2^k) of the buffer -- Alg.1's chunk skipping becomes "stop at the live prefix".
+// a4  pass planner: cuts the executed order into CONSECUTIVE runs (the per-gate involvement
+//     trace is unchanged); each run is one fused HBM pass over tiles of 2^b amplitudes.
+#include <algorithm>
+#include <bit>
+#include <cstring>
+#include <limits>
+
+#include "qgpu_internal.h"
+
+namespace qgpu {
+
+// ----------------------------------------------------------------------------------- a2
+namespace {
+
+struct Dag {
+  std::vector<uint64_t> q;                 // qubit mask per gate
+  std::vector<std::vector<int>> desc;      // descendants, ascending
+  std::vector<int> npred;
+};
+
+Dag build_dag(const std::vector<Gate>& gates) {
+  Dag d;
+  const int G = int(gates.size());
+  d.q.resize(G);
+  d.desc.assign(G, {});
+  d.npred.assign(G, 0);
+  int last[64];
+  std::fill(last, last + 64, -1);
+  for (int i = 0; i < G; ++i) {
+    d.q[i] = gates[i].qmask();
+    std::vector<int> preds;
+    for (uint64_t m = d.q[i]; m; m &= m - 1) {
+      const int qb = std::countr_zero(m);
+      if (last[qb] >= 0 && std::find(preds.begin(), preds.end(), last[qb]) == preds.end())
+        preds.push_back(last[qb]);
+    }
+    for (uint64_t m = d.q[i]; m; m &= m - 1) last[std::countr_zero(m)] = i;
+    d.npred[i] = int(preds.size());
+    for (int p : preds) d.desc[p].push_back(i);
+  }
+  for (auto& v : d.desc) std::sort(v.begin(), v.end());
+  return d;
+}
+
+inline int newq(uint64_t q, uint64_t involved) { return std::popcount(q & ~involved); }
+
+}  // namespace
+
+std::vector<int> reorder(const std::vector<Gate>& gates, int mode) {
+  const int G = int(gates.size());
+  std::vector<int> out;
+  out.reserve(G);
+  if (mode == 0) {
+    for (int i = 0; i < G; ++i) out.push_back(i);
+    return out;
+  }
+  Dag d = build_dag(gates);
+  std::vector<int> exe;
+  for (int i = 0; i < G; ++i)
+    if (d.npred[i] == 0) exe.push_back(i);
+  uint64_t involved = 0;
+  std::vector<int> look;
+  while (!exe.empty()) {
+    int best_pos = -1;
+    long best_cost = std::numeric_limits<long>::max(), best_cur = best_cost;
+    for (int pos = 0; pos < int(exe.size()); ++pos) {
+      const int g = exe[pos];
+      const long cur = newq(d.q[g], involved);          // Alg.3 l.3-6 (= Alg.2 cost)
+      long cost = cur;
+      if (mode == 2) {
+        const uint64_t inv2 = involved | d.q[g];
+        long la = std::numeric_limits<long>::max();       // Q3: +inf
+        for (int h : exe)                                   // Alg.3 l.7, l.12-18
+          if (h != g) la = std::min<long>(la, newq(d.q[h], inv2));
+        for (int h : d.desc[g])                             // Alg.3 l.8-10
+          if (d.npred[h] == 1) la = std::min<long>(la, newq(d.q[h], inv2));
+        if (la == std::numeric_limits<long>::max()) la = 0;
+        cost = cur + la;                                    // Alg.3 l.19
+      }
+      // key (cost, costCurrent, position): strict '<' keeps the earliest position
+      if (cost < best_cost || (cost == best_cost && cur < best_cur)) {
+        best_cost = cost;
+        best_cur = cur;
+        best_pos = pos;
+      }
+    }
+    const int next = exe[best_pos];
+    exe.erase(exe.begin() + best_pos);                      // Alg.2 l.16
+    out.push_back(next);                                    // Alg.2 l.17
+    involved |= d.q[next];
+    for (int h : d.desc[next])                              // Alg.2 l.18-21
+      if (--d.npred[h] == 0) exe.push_back(h);
+  }
+  return out;
+}
+
+// ----------------------------------------------------------------------------------- a3
+void QubitMap::init(int n_, int m_) {
+  n = n_;
+  m = m_;
+  kl = kg = 0;
+  involvement = 0;
+  std::fill(pos, pos + kMaxQubits, -1);
+  std::fill(lq, lq + kMaxQubits, -1);
+}
+
+void QubitMap::touch(uint64_t mask) {
+  involvement |= mask;                                      // Alg.1 l.11
+  for (uint64_t r = mask; r; r &= r - 1) {
+    const int q = std::countr_zero(r);
+    if (pos[q] >= 0) continue;
+    const int p = (kl < m) ? kl++ : m + kg++;               // local first, then global
+    pos[q] = p;
+    lq[p] = q;
+  }
+}
+
+uint64_t QubitMap::phys_mask(uint64_t lm) const {
+  uint64_t r = 0;
+  for (; lm; lm &= lm - 1) r |= 1ull << pos[std::countr_zero(lm)];
+  return r;
+}
+
+void QubitMap::swap_positions(int pa, int pb) {
+  const int qa = lq[pa], qb = lq[pb];
+  lq[pa] = qb;
+  lq[pb] = qa;
+  if (qa >= 0) pos[qa] = pb;
+  if (qb >= 0) pos[qb] = pa;
+}
+
+// ----------------------------------------------------------------------------------- a4
+uint64_t unfused_gate_bytes(const PhysGate& g, int k_in, int k_out) {
+  const double L = double(1ull << k_out);
+  if (g.diag) {
+    // amplitudes whose diagonal entry differs from 1, times read+write
+    int ones = 0;
+    for (int v = 0; v < (1 << g.nt); ++v) {
+      const cplx d = g.U[v * ((1 << g.nt) + 1)];
+      ones += (d.re == 1.0 && d.im == 0.0);
+    }
+    const double frac = double((1 << g.nt) - ones) / double(1 << g.nt);
+    const int nc = std::popcount(g.pc);
+    return uint64_t(32.0 * frac * double(1ull << k_in) / double(1ull << nc));
+  }
+  const int nc = std::popcount(g.pc);
+  if (k_out > k_in) return uint64_t(16.0 * double(1ull << k_in) + 16.0 * L);
+  return uint64_t(32.0 * L / double(1ull << nc));
+}
+
+namespace {
+
+// tile-local bits of a physical mask (positions outside the tile dropped)
+uint32_t to_local(uint64_t phys, const Pass& p) {
+  uint32_t r = 0;
+  for (int i = 0; i < p.b; ++i)
+    if (phys >> p.spos[i] & 1) r |= 1u << i;
+  return r;
+}
+uint64_t outside(uint64_t phys, const Pass& p) {
+  for (int i = 0; i < p.b; ++i) phys &= ~(1ull << p.spos[i]);
+  return phys;
+}
+int local_bit(int pos, const Pass& p) {
+  for (int i = 0; i < p.b; ++i)
+    if (p.spos[i] == pos) return i;
+  return -1;
+}
+
+}  // namespace
+
+void build_tile_ops(Pass& p, int /*m*/) {
+  p.ops.clear();
+  for (const PhysGate& g : p.gates) {
+    if (!g.diag) {
+      DevOp o{};
+      o.kind = g.nt == 1 ? OP_U1 : OP_U2;
+      o.t0 = local_bit(g.p[0], p);
+      o.t1 = g.nt == 2 ? local_bit(g.p[1], p) : 0;
+      o.lmask = o.lmatch = to_local(g.pc, p);
+      o.omask = o.omatch = outside(g.pc, p);
+      const int dim = 1 << g.nt;
+      for (int i = 0; i < dim * dim; ++i) {
+        o.m[2 * i] = g.U[i].re;
+        o.m[2 * i + 1] = g.U[i].im;
+      }
+      p.ops.push_back(o);
+    } else {
+      // diagonal: one phase term per diagonal entry that is not exactly 1
+      const int dim = 1 << g.nt;
+      uint64_t tmask = 1ull << g.p[0];
+      if (g.nt == 2) tmask |= 1ull << g.p[1];
+      for (int v = 0; v < dim; ++v) {
+        const cplx d = g.U[v * (dim + 1)];
+        if (d.re == 1.0 && d.im == 0.0) continue;
+        uint64_t match = g.pc;
+        for (int j = 0; j < g.nt; ++j)
+          if (v >> j & 1) match |= 1ull << g.p[j];
+        const uint64_t mask = g.pc | tmask;
+        DevOp o{};
+        o.kind = OP_PHASE;
+        o.lmask = to_local(mask, p);
+        o.lmatch = to_local(match, p);
+        o.omask = outside(mask, p);
+        o.omatch = outside(match, p);
+        o.m[0] = d.re;
+        o.m[1] = d.im;
+        p.ops.push_back(o);
+      }
+    }
+  }
+}
+
+namespace {
+
+struct Builder {
+  const std::vector<Gate>& gates;
+  QubitMap& map;
+  const PlanOptions& opt;
+  std::vector<Pass>* out;
+  bool open = false;
+  Pass cur;
+  uint64_t used = 0;   // physical positions that must be tile bits (non-diagonal targets)
+  int n_u = 0;
+
+  void close() {
+    if (!open) return;
+    Pass& p = cur;
+    const int kt = p.k_out;
+    if (p.kind == PK_TILE) {
+      const int b = std::min(opt.fuse_bits, kt);
+      uint64_t S = used;
+      for (int pos = 0; pos < kt && std::popcount(S) < b; ++pos) S |= 1ull << pos;
+      p.b = std::popcount(S);
+      int i = 0;
+      for (uint64_t r = S; r; r &= r - 1) p.spos[i++] = std::countr_zero(r);
+      p.l = 0;
+      while (p.l < p.b && p.spos[p.l] == p.l) ++p.l;
+      build_tile_ops(p, map.m);
+    }
+    out->push_back(std::move(p));
+    cur = Pass();
+    open = false;
+    used = 0;
+    n_u = 0;
+  }
+
+  void start(int kind, int first, int k_in) {
+    cur = Pass();
+    cur.kind = kind;
+    cur.first = first;
+    cur.k_in = k_in;
+    cur.k_out = k_in;
+    open = true;
+    used = 0;
+    n_u = 0;
+  }
+
+  bool fits(uint64_t need, int n_ops_new) const {
+    if (int(cur.ops.size()) + n_ops_new > opt.max_ops) return false;
+    if (need && n_u + 1 > opt.max_u_ops) return false;
+    const int lm = std::min(opt.l_min, std::max(cur.k_out, 0));
+    uint64_t S = used | need | ((lm > 0) ? ((1ull << lm) - 1) : 0);
+    return std::popcount(S) <= opt.fuse_bits;
+  }
+};
+
+}  // namespace
+
+void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order, QubitMap& map,
+                  const PlanOptions& opt, std::vector<Pass>* passes,
+                  std::vector<uint64_t>* inv_after) {
+  Builder B{gates, map, opt, passes};
+  const bool fuse = opt.fuse_bits > 0;
+  for (int k = 0; k < int(order.size()); ++k) {
+    const Gate& g = gates[order[k]];
+    const int k_before = map.kl;
+    const uint64_t fresh = g.qmask() & ~map.involvement;
+    map.touch(g.qmask());
+    if (inv_after) inv_after->push_back(map.involvement);
+    if (g.relabel) {
+      const int pa = map.pos[g.t[0]], pb = map.pos[g.t[1]];
+      if (fuse && B.open && B.cur.kind == PK_TILE) {
+        // relabels move no data; inside a tile pass they only re-map later gates
+        map.swap_positions(pa, pb);
+        B.cur.k_out = map.kl;
+        B.cur.count++;
+        continue;
+      }
+      B.close();
+      B.start(PK_RELABEL, k, k_before);
+      map.swap_positions(pa, pb);
+      B.cur.k_out = map.kl;
+      B.cur.count = 1;
+      B.close();
+      continue;
+    }
+    PhysGate pg;
+    pg.gate = order[k];
+    pg.nt = g.nt;
+    pg.p[0] = map.pos[g.t[0]];
+    pg.p[1] = g.nt == 2 ? map.pos[g.t[1]] : 0;
+    pg.pc = map.phys_mask(g.cmask);
+    std::memcpy(pg.U, g.U, sizeof(g.U));
+    pg.diag = g.diag;
+    pg.expands_target = (g.tmask() & fresh) != 0;
+    // TODO(sharded): swap planning for non-diagonal targets on global positions
+    if (fuse) {
+      uint64_t need = 0;
+      if (!g.diag) {
+        need |= 1ull << pg.p[0];
+        if (g.nt == 2) need |= 1ull << pg.p[1];
+      }
+      int n_new_ops = g.diag ? (1 << g.nt) : 1;
+      if (!(B.open && B.cur.kind == PK_TILE && B.fits(need, n_new_ops))) {
+        B.close();
+        B.start(PK_TILE, k, k_before);
+      }
+      B.used |= need;
+      if (need) B.n_u++;
+      B.cur.gates.push_back(pg);
+      B.cur.ops.resize(B.cur.ops.size() + n_new_ops);  // placeholder count; rebuilt at close
+      B.cur.count++;
+      B.cur.k_out = map.kl;
+      B.cur.unfused_bytes += unfused_gate_bytes(pg, k_before, map.kl);
+    } else {
+      B.close();
+      B.start(g.diag ? PK_DIAG : (g.nt == 1 ? PK_PAIR : PK_QUAD), k, k_before);
+      B.cur.gates.push_back(pg);
+      B.cur.count = 1;
+      B.cur.k_out = map.kl;
+      B.cur.unfused_bytes = unfused_gate_bytes(pg, k_before, map.kl);
+      B.close();
+    }
+  }
+  B.close();
+}
+
+}  // namespace qgpu

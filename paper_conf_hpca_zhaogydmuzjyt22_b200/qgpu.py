@@ -1,0 +1,272 @@
+"""Thin ctypes binding of libqgpu.so (include/qgpu.h): argument marshalling only.
+
+Every step of the hot path runs in the library's CUDA kernels. If the shared library is
+missing the import fails loudly -- there is no CPU fallback. PyTorch, when used by the caller,
+only supplies device memory (``state_buffer``) and the stream.
+"""
+from __future__ import annotations
+
+import ctypes
+import os
+from typing import Optional, Sequence
+
+import numpy as np
+
+_PKG = os.path.dirname(os.path.abspath(__file__))
+LIB_PATH = os.path.join(_PKG, "libqgpu.so")
+
+QGPU_OK = 0
+STATUS = {0: "OK", 1: "INVALID_ARG", 2: "OUT_OF_MEMORY", 3: "UNSUPPORTED", 4: "PARSE",
+          5: "CUDA", 6: "NCCL", 7: "STATE"}
+
+EXPORTS = [
+    "qgpu_config_init", "qgpu_state_create", "qgpu_state_destroy", "qgpu_state_reset",
+    "qgpu_set_amplitudes", "qgpu_synchronize", "qgpu_state_info", "qgpu_apply_gate",
+    "qgpu_apply_circuit", "qgpu_get_amplitudes", "qgpu_get_amplitudes_device",
+    "qgpu_probabilities", "qgpu_circuit_from_qasm", "qgpu_circuit_info", "qgpu_circuit_destroy",
+    "qgpu_circuit_reorder", "qgpu_circuit_plan", "qgpu_get_involvement", "qgpu_get_chunk_bitmap",
+    "qgpu_get_schedule", "qgpu_get_qubit_map", "qgpu_get_stats", "qgpu_reset_stats",
+    "qgpu_last_error", "qgpu_version",
+]
+
+
+class QgpuError(RuntimeError):
+    def __init__(self, status: int, msg: str):
+        super().__init__(f"qgpu {STATUS.get(status, status)}: {msg}")
+        self.status = status
+        self.kind = STATUS.get(status, str(status))
+
+
+class Config(ctypes.Structure):
+    _fields_ = [
+        ("struct_size", ctypes.c_uint32), ("device", ctypes.c_int), ("stream", ctypes.c_void_p),
+        ("state_buffer", ctypes.c_void_p), ("state_buffer_bytes", ctypes.c_uint64),
+        ("rank", ctypes.c_int), ("world_size", ctypes.c_int), ("nccl_unique_id", ctypes.c_void_p),
+        ("chunk_bits", ctypes.c_int), ("prune", ctypes.c_int), ("reorder", ctypes.c_int),
+        ("fuse_bits", ctypes.c_int), ("timing", ctypes.c_int), ("swap_slab_bytes", ctypes.c_uint64),
+    ]
+
+
+class Stats(ctypes.Structure):
+    _fields_ = [(n, ctypes.c_uint64) for n in (
+        "gates_applied", "passes", "kernels_launched", "relabels", "amps_processed", "amps_full",
+        "chunks_processed", "chunks_skipped", "algo_bytes", "unfused_bytes", "swaps", "swap_bytes")] + [
+        ("ops_before_full_involvement", ctypes.c_int64), ("kernel_ms", ctypes.c_double),
+        ("tile_kernel_ms", ctypes.c_double), ("tile_kernel_launches", ctypes.c_uint64),
+        ("tile_algo_bytes", ctypes.c_uint64), ("swap_ms", ctypes.c_double)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
+_lib = None
+
+
+def load(path: str = LIB_PATH) -> ctypes.CDLL:
+    """Load libqgpu.so (raises if it has not been built: no fallback)."""
+    global _lib
+    if _lib is not None:
+        return _lib
+    if not os.path.exists(path):
+        raise ImportError(f"{path} not built: run `python -m paper_conf_hpca_zhaogydmuzjyt22_b200.build`")
+    lib = ctypes.CDLL(path)
+    P, I, U64 = ctypes.c_void_p, ctypes.c_int, ctypes.c_uint64
+    sig = {
+        "qgpu_config_init": [P], "qgpu_state_create": [I, P, P], "qgpu_state_destroy": [P],
+        "qgpu_state_reset": [P], "qgpu_set_amplitudes": [P, P], "qgpu_synchronize": [P],
+        "qgpu_state_info": [P, P, P, P], "qgpu_apply_gate": [P, P, I, P, I, P],
+        "qgpu_apply_circuit": [P, P], "qgpu_get_amplitudes": [P, U64, U64, P],
+        "qgpu_get_amplitudes_device": [P, U64, U64, P], "qgpu_probabilities": [P, I, P, P],
+        "qgpu_circuit_from_qasm": [ctypes.c_char_p, ctypes.c_size_t, P],
+        "qgpu_circuit_info": [P, P, P], "qgpu_circuit_destroy": [P],
+        "qgpu_circuit_reorder": [P, I, P, U64, P], "qgpu_circuit_plan": [P, I, I, I, I, P, U64, P],
+        "qgpu_get_involvement": [P, P], "qgpu_get_chunk_bitmap": [P, I, P, U64],
+        "qgpu_get_schedule": [P, P, P, U64, P], "qgpu_get_qubit_map": [P, P],
+        "qgpu_get_stats": [P, P], "qgpu_reset_stats": [P],
+    }
+    for name, args in sig.items():
+        f = getattr(lib, name)
+        f.argtypes = args
+        f.restype = ctypes.c_int
+    lib.qgpu_last_error.restype = ctypes.c_char_p
+    lib.qgpu_last_error.argtypes = []
+    lib.qgpu_version.restype = ctypes.c_char_p
+    lib.qgpu_version.argtypes = []
+    _lib = lib
+    return lib
+
+
+def _check(rc: int) -> None:
+    if rc != QGPU_OK:
+        raise QgpuError(rc, load().qgpu_last_error().decode(errors="replace"))
+
+
+def config(**kw) -> Config:
+    cfg = Config()
+    _check(load().qgpu_config_init(ctypes.byref(cfg)))
+    for k, v in kw.items():
+        if k == "nccl_unique_id" and v is not None and not isinstance(v, int):
+            buf = ctypes.create_string_buffer(bytes(v), 128)
+            cfg._nccl_id_buf = buf  # keep alive
+            v = ctypes.addressof(buf)
+        setattr(cfg, k, v)
+    return cfg
+
+
+class Circuit:
+    """A parsed OpenQASM-2 circuit (qgpu_circuit_from_qasm)."""
+
+    def __init__(self, qasm_text: str):
+        lib = load()
+        self._h = ctypes.c_void_p()
+        data = qasm_text.encode()
+        _check(lib.qgpu_circuit_from_qasm(data, len(data), ctypes.byref(self._h)))
+
+    @property
+    def handle(self):
+        return self._h
+
+    def info(self):
+        n, g = ctypes.c_int(), ctypes.c_uint64()
+        _check(load().qgpu_circuit_info(self._h, ctypes.byref(n), ctypes.byref(g)))
+        return n.value, g.value
+
+    def reorder(self, mode: int) -> np.ndarray:
+        _, ng = self.info()
+        out = np.zeros(max(ng, 1), dtype=np.uint64)
+        cnt = ctypes.c_uint64()
+        _check(load().qgpu_circuit_reorder(self._h, mode, out.ctypes.data, ng, ctypes.byref(cnt)))
+        return out[:cnt.value].astype(np.int64)
+
+    def plan(self, n: int, world_size: int = 1, reorder: int = 2, fuse_bits: int = 12) -> np.ndarray:
+        cnt = ctypes.c_uint64()
+        _check(load().qgpu_circuit_plan(self._h, n, world_size, reorder, fuse_bits, None, 0,
+                                        ctypes.byref(cnt)))
+        info = np.zeros((max(cnt.value, 1), 8), dtype=np.int64)
+        _check(load().qgpu_circuit_plan(self._h, n, world_size, reorder, fuse_bits,
+                                        info.ctypes.data, cnt.value, ctypes.byref(cnt)))
+        return info[:cnt.value]
+
+    def close(self):
+        if self._h:
+            load().qgpu_circuit_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+
+class State:
+    """An n-qubit state vector on one GPU (or one shard of it), starting in |0...0>."""
+
+    def __init__(self, n: int, cfg: Optional[Config] = None, **kw):
+        lib = load()
+        self.cfg = cfg if cfg is not None else config(**kw)
+        self._h = ctypes.c_void_p()
+        _check(lib.qgpu_state_create(n, ctypes.byref(self.cfg), ctypes.byref(self._h)))
+        self.n = n
+
+    @property
+    def handle(self):
+        return self._h
+
+    def close(self):
+        if self._h:
+            load().qgpu_state_destroy(self._h)
+            self._h = ctypes.c_void_p()
+
+    def __del__(self):
+        try:
+            self.close()
+        except Exception:
+            pass
+
+    def __enter__(self):
+        return self
+
+    def __exit__(self, *a):
+        self.close()
+
+    def reset(self):
+        _check(load().qgpu_state_reset(self._h))
+
+    def synchronize(self):
+        _check(load().qgpu_synchronize(self._h))
+
+    def info(self):
+        n, nl, p = ctypes.c_int(), ctypes.c_int(), ctypes.c_void_p()
+        _check(load().qgpu_state_info(self._h, ctypes.byref(n), ctypes.byref(nl), ctypes.byref(p)))
+        return n.value, nl.value, p.value
+
+    def set_amplitudes(self, psi: np.ndarray):
+        psi = np.ascontiguousarray(psi, dtype=np.complex128)
+        assert psi.size == 1 << self.n
+        _check(load().qgpu_set_amplitudes(self._h, psi.ctypes.data))
+
+    def apply_gate(self, U, targets: Sequence[int], controls: Sequence[int] = ()):
+        U = np.ascontiguousarray(U, dtype=np.complex128)
+        t = np.ascontiguousarray(targets, dtype=np.int32)
+        c = np.ascontiguousarray(controls if len(controls) else [0], dtype=np.int32)
+        assert U.shape == (1 << len(t), 1 << len(t))
+        _check(load().qgpu_apply_gate(self._h, U.ctypes.data, len(t), t.ctypes.data, len(controls),
+                                      c.ctypes.data if len(controls) else None))
+
+    def apply_circuit(self, circ: Circuit):
+        _check(load().qgpu_apply_circuit(self._h, circ.handle))
+
+    def amplitudes(self, start: int = 0, count: Optional[int] = None) -> np.ndarray:
+        if count is None:
+            count = (1 << self.n) - start
+        out = np.empty(count, dtype=np.complex128)
+        _check(load().qgpu_get_amplitudes(self._h, start, count, out.ctypes.data))
+        return out
+
+    def amplitudes_device(self, start: int, count: int, dev_ptr: int):
+        _check(load().qgpu_get_amplitudes_device(self._h, start, count, dev_ptr))
+
+    def probabilities(self, qubits: Sequence[int]) -> np.ndarray:
+        q = np.ascontiguousarray(qubits if len(qubits) else [0], dtype=np.int32)
+        out = np.empty(1 << len(qubits), dtype=np.float64)
+        _check(load().qgpu_probabilities(self._h, len(qubits), q.ctypes.data, out.ctypes.data))
+        return out
+
+    def involvement(self) -> int:
+        v = ctypes.c_uint64()
+        _check(load().qgpu_get_involvement(self._h, ctypes.byref(v)))
+        return v.value
+
+    def chunk_bitmap(self, chunk_bits: int) -> np.ndarray:
+        nch = 1 << (self.n - chunk_bits)
+        words = np.zeros((nch + 63) // 64, dtype=np.uint64)
+        _check(load().qgpu_get_chunk_bitmap(self._h, chunk_bits, words.ctypes.data, words.size))
+        bits = np.unpackbits(words.view(np.uint8), bitorder="little")[:nch]
+        return bits.astype(np.uint8)
+
+    def schedule(self):
+        cnt = ctypes.c_uint64()
+        _check(load().qgpu_get_schedule(self._h, None, None, 0, ctypes.byref(cnt)))
+        o = np.zeros(max(cnt.value, 1), dtype=np.uint64)
+        iv = np.zeros(max(cnt.value, 1), dtype=np.uint64)
+        _check(load().qgpu_get_schedule(self._h, o.ctypes.data, iv.ctypes.data, cnt.value,
+                                        ctypes.byref(cnt)))
+        return o[:cnt.value].astype(np.int64), iv[:cnt.value]
+
+    def qubit_map(self) -> np.ndarray:
+        pos = np.zeros(self.n, dtype=np.int32)
+        _check(load().qgpu_get_qubit_map(self._h, pos.ctypes.data))
+        return pos
+
+    def stats(self) -> dict:
+        s = Stats()
+        _check(load().qgpu_get_stats(self._h, ctypes.byref(s)))
+        return s.as_dict()
+
+    def reset_stats(self):
+        _check(load().qgpu_reset_stats(self._h))
+
+
+def version() -> str:
+    return load().qgpu_version().decode()

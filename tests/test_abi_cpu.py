@@ -1,0 +1,151 @@
+"""CPU-only checks of the C ABI library: it builds/loads, exports every declared symbol, and its
+host logic (QASM loader, Alg.2/3 reorder, pass planner) agrees with the oracle. No GPU calls."""
+import os
+import re
+
+import numpy as np
+import pytest
+
+from oracle import qasm as oq
+from oracle import schedule as osch
+from workloads import circuits as wc
+
+ROOT = os.path.dirname(os.path.dirname(os.path.abspath(__file__)))
+
+
+@pytest.fixture(scope="module")
+def q():
+    from paper_conf_hpca_zhaogydmuzjyt22_b200 import build, qgpu
+    build.build()
+    qgpu.load()
+    return qgpu
+
+
+def test_exports_every_declared_symbol(q):
+    hdr = open(os.path.join(ROOT, "include", "qgpu.h")).read()
+    declared = set(re.findall(r"\b(qgpu_[a-z_]+)\s*\(", hdr))
+    assert len(declared) >= 20
+    lib = q.load()
+    for name in declared:
+        assert hasattr(lib, name), name
+    assert declared <= set(q.EXPORTS) | {"qgpu_last_error", "qgpu_version"}
+    assert "sm_100a" in q.version()
+
+
+def test_config_struct_size(q):
+    import ctypes
+    cfg = q.config()
+    assert cfg.struct_size == ctypes.sizeof(q.Config)
+    assert (cfg.prune, cfg.reorder, cfg.chunk_bits, cfg.fuse_bits, cfg.world_size) == (1, 2, 21, 12, 1)
+
+
+CIRCS = {
+    "ghz_qft5": lambda: wc.ghz_qft(5),
+    "qft12": lambda: wc.qft(12),
+    "qft9x": lambda: wc.qft(9, x=300),
+    "qaoa14": lambda: wc.qaoa(14, 2, seed=1),
+    "rqc12": lambda: wc.rqc(12, 10, seed=3),
+    "gs3x4": lambda: wc.gs(3, 4),
+    "hlf3x4": lambda: wc.hlf(3, 4, seed=2),
+    "bv9": lambda: wc.bv(9, 0b10110101),
+    "iqp8": lambda: wc.iqp(8),
+    "rand8": lambda: wc.random_circuit(8, 150, seed=11),
+    "rand10": lambda: wc.random_circuit(10, 300, seed=12),
+}
+
+
+@pytest.mark.parametrize("name", sorted(CIRCS))
+def test_loader_matches_oracle_parser(q, name):
+    c = CIRCS[name]()
+    text = c.qasm()
+    n, gates = oq.parse(text)
+    qc = q.Circuit(text)
+    assert qc.info() == (n, len(gates))
+
+
+@pytest.mark.parametrize("name", sorted(CIRCS))
+@pytest.mark.parametrize("mode", [0, 1, 2])
+def test_reorder_bit_exact_vs_oracle(q, name, mode):
+    """oracle and library schedules must be identical (Alg.2/Alg.3 + Q4)."""
+    c = CIRCS[name]()
+    text = c.qasm()
+    _, gates = oq.parse(text)
+    ref = osch.reorder(gates, mode)
+    got = q.Circuit(text).reorder(mode)
+    assert list(got) == list(ref)
+
+
+def test_reorder_gs5_walkthrough(q):
+    """forward-looking reorder of the gs_5 example gives 1,2,2,3,3,4,4,4,5."""
+    text = ('OPENQASM 2.0;\ninclude "qelib1.inc";\nqreg q[5];\nh q[0];\nh q[1];\nh q[2];\nh q[3];\n'
+            'h q[4];\ncx q[0],q[1];\ncx q[0],q[2];\ncx q[1],q[3];\ncx q[2],q[3];\n')
+    order = q.Circuit(text).reorder(2)
+    _, gates = oq.parse(text)
+    cnt = [bin(i).count("1") for i in osch.involvement_trace(gates, list(order))]
+    assert cnt == [1, 2, 2, 3, 3, 4, 4, 4, 5]
+
+
+@pytest.mark.parametrize("name", ["qft12", "qaoa14", "rqc12", "rand10", "hlf3x4"])
+@pytest.mark.parametrize("fuse", [0, 7, 9, 12])
+def test_plan_invariants(q, name, fuse):
+    """a4: passes are consecutive runs of the reordered list; tile passes have <= b tile bits
+    that include the low contiguous run; live sizes never shrink."""
+    c = CIRCS[name]()
+    qc = q.Circuit(c.qasm())
+    n, ng = qc.info()
+    plan = qc.plan(n, 1, 2, fuse)
+    pos = 0
+    k_prev = 0
+    for first, count, kind, kin, kout, b, slo, shi in plan:
+        assert first == pos and count >= 1
+        pos += count
+        assert kin == k_prev and kout >= kin
+        k_prev = kout
+        if fuse == 0:
+            assert kind in (1, 2, 3, 4)
+            assert count == 1
+        else:
+            assert kind in (0, 4)
+            if kind == 0:
+                S = int(slo) | (int(shi) << 32)
+                assert bin(S).count("1") == b <= fuse
+                assert b == min(fuse, kout)
+                lm = min(5, kout)
+                assert S & ((1 << lm) - 1) == (1 << lm) - 1
+                assert S >> kout == 0
+    assert pos == ng
+    assert k_prev == n or ng == 0 or k_prev == bin(osch.involvement_trace(oq.parse(c.qasm())[1])[-1]).count("1")
+
+
+def test_fused_qft28_is_few_passes(q):
+    """QFT_28 (config C2) with Alg.3 and b=12 collapses into a handful of HBM passes."""
+    qc = q.Circuit(wc.qft(28).qasm())
+    plan = qc.plan(28, 1, 2, 12)
+    assert len(plan) <= 40
+
+
+def test_parse_errors(q):
+    with pytest.raises(q.QgpuError) as e:
+        q.Circuit("OPENQASM 2.0;\nqreg q[2];\nh q[0]\ncx q[0],q[1];\n")
+    assert e.value.kind == "PARSE" and "line 4" in str(e.value)
+    with pytest.raises(q.QgpuError) as e:
+        q.Circuit("OPENQASM 2.0;\nqreg q[2];\nreset q[0];\n")
+    assert e.value.kind == "UNSUPPORTED"
+    with pytest.raises(q.QgpuError) as e:
+        q.Circuit("OPENQASM 2.0;\nqreg q[2];\nfoo q[0];\n")
+    assert e.value.kind == "UNSUPPORTED"
+    with pytest.raises(q.QgpuError) as e:
+        q.Circuit("OPENQASM 2.0;\nqreg q[2];\ncx q[0],q[0];\n")
+    assert e.value.kind == "INVALID_ARG"
+    c = q.Circuit("OPENQASM 2.0;\nqreg a[2];\nqreg b[3];\ncreg c[5];\nh b;\ncx a[1],b[2];\n"
+                  "rx(-pi/2^2 + 2*sin(pi/6)) a[0];\nbarrier a;\nmeasure a[0] -> c[0];\n")
+    assert c.info() == (5, 5)
+
+
+def test_state_create_without_gpu_fails_cleanly(q):
+    import torch
+    if torch.cuda.is_available():
+        pytest.skip("GPU present")
+    with pytest.raises(q.QgpuError) as e:
+        q.State(10)
+    assert e.value.kind in ("CUDA", "OUT_OF_MEMORY")
