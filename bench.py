@@ -1,0 +1,406 @@
+#!/usr/bin/env python
+"""Benchmark of the B200 Q-GPU hot path (one JSON line on rank 0).
+
+Default workload (BASELINE.json configs[1]): QFT_28 on 1x B200 with delayed qubit involvement
+and pruning (reorder=2, prune=1, fused passes b=12). A step = qgpu_state_reset +
+qgpu_apply_circuit of the whole circuit (every gate, the state resident in HBM); the metric
+is circuit seconds (lower is better). See DESIGN.md §7 for the byte model and peaks.
+
+    python bench.py [--gpus N --steps K --warmup W] [--workload qft28|qaoa32|rqc|gs|hlf]
+    python bench.py --impl reference ...     # the oracle (plain CPU simulator) as the baseline arm
+
+N > 1 (torchrun): each rank runs its own replica of the workload (weak scaling, no data-path
+collective; the sharded path is DESIGN.md §8), timed on the device, max over ranks.
+"""
+from __future__ import annotations
+
+import argparse
+import json
+import math
+import os
+import statistics
+import subprocess
+import sys
+import tempfile
+import threading
+import time
+
+ROOT = os.path.dirname(os.path.abspath(__file__))
+sys.path.insert(0, ROOT)
+
+METRIC = "circuit sec & gate-apply HBM GB/s vs peak, 28–36 qubits, 1/2/4/8 B200"
+
+
+def workload(name: str, n: int | None):
+    from workloads import circuits as wc
+    if name == "qft28":
+        nn = n or 28
+        return wc.qft(nn), f"qft_{nn} (configs[1]: {nn}-qubit QFT on 1xB200, |0...0>, delayed involvement)"
+    if name == "qaoa32":
+        nn = n or 32
+        return wc.qaoa(nn, 2, seed=1), f"qaoa_{nn} MaxCut p=2, 3-regular seed 1 (configs[2])"
+    if name == "rqc":
+        nn = n or 30
+        return wc.rqc(nn, 20, seed=3), f"rqc_{nn} depth 20 seed 3 (configs[3] shape)"
+    if name == "gs":
+        return wc.gs(6, 6), "gs_36 6x6 grid (configs[4])"
+    if name == "hlf":
+        return wc.hlf(6, 6, seed=2), "hlf_36 6x6 grid seed 2 (configs[4])"
+    raise SystemExit(f"unknown workload {name}")
+
+
+def peaks():
+    p = os.path.join(ROOT, "MEASURED_PEAKS.json")
+    if os.path.exists(p):
+        d = json.load(open(p))
+        return float(d["hbm_gbs"]), "measured (MEASURED_PEAKS.json hbm_gbs, torch copy)"
+    return 6650.0, "fallback (B200_PROFILING.md: 6.65 TB/s)"
+
+
+class ClockSampler:
+    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
+              "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
+              "clocks_event_reasons.sw_power_cap")
+
+    def __init__(self, device: int):
+        self.device = device
+        self.proc = None
+        self.f = None
+
+    def __enter__(self):
+        try:
+            self.f = tempfile.NamedTemporaryFile("w+", delete=False, suffix=".csv")
+            self.proc = subprocess.Popen(
+                ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}",
+                 "--format=csv,noheader,nounits", "-lms", "200"], stdout=self.f,
+                stderr=subprocess.DEVNULL)
+        except Exception:
+            self.proc = None
+        return self
+
+    def __exit__(self, *a):
+        if self.proc is not None:
+            self.proc.terminate()
+            try:
+                self.proc.wait(timeout=5)
+            except Exception:
+                self.proc.kill()
+
+    def summary(self):
+        if self.proc is None:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
+        self.f.flush()
+        rows = []
+        for line in open(self.f.name):
+            parts = [x.strip() for x in line.split(",")]
+            if len(parts) == 6 and parts[0].isdigit():
+                rows.append(parts)
+        os.unlink(self.f.name)
+        if not rows:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
+        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
+        reasons = sorted({names[i] for r in rows for i in range(4) if r[2 + i] == "Active"})
+        return {"sm_mhz": statistics.median(int(r[0]) for r in rows),
+                "sm_max_mhz": max(int(r[1]) for r in rows), "reasons": reasons,
+                "samples": len(rows)}
+
+
+def dist_setup(args):
+    import torch
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    local = int(os.environ.get("LOCAL_RANK", "0"))
+    if world > 1:
+        import torch.distributed as dist
+        torch.cuda.set_device(local)
+        dist.init_process_group("nccl", device_id=torch.device("cuda", local))
+    return world, rank, local
+
+
+def barrier(world):
+    if world > 1:
+        import torch.distributed as dist
+        dist.barrier()
+
+
+def allreduce_max(x: float, world: int, device) -> float:
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.MAX)
+    return float(t.item())
+
+
+def allreduce_sum(x: float, world: int, device) -> float:
+    if world == 1:
+        return x
+    import torch
+    import torch.distributed as dist
+    t = torch.tensor([x], dtype=torch.float64, device=device)
+    dist.all_reduce(t, op=dist.ReduceOp.SUM)
+    return float(t.item())
+
+
+# ----------------------------------------------------------------------------- oracle arm
+
+def oracle_sample(text: str, budget_s: float, start_gate: int = 0, max_gates: int | None = None):
+    """Time the oracle (as it stands: program order, no pruning) on the first gates of the
+    workload at full size until `budget_s` elapses; returns (sec_per_circuit, sample)."""
+    from oracle import qasm as oq
+    from oracle import statevector as osv
+    n, gates = oq.parse(text)
+    threads = osv.default_threads()
+    psi = osv.zero_state(n)
+    for i in range(min(start_gate, len(gates))):
+        pass  # the sample always starts from |0...0>: every oracle gate visits all 2^n indices
+    t0 = time.perf_counter()
+    done = 0
+    while done < len(gates) and (time.perf_counter() - t0) < budget_s:
+        g = gates[(start_gate + done) % len(gates)]
+        osv.apply_gate(psi, n, g.U, g.targets, g.controls, threads)
+        done += 1
+        if max_gates and done >= max_gates:
+            break
+    dt = time.perf_counter() - t0
+    per_gate = dt / max(done, 1)
+    return per_gate * len(gates), {"gates_timed": done, "gates_total": len(gates),
+                                   "seconds": dt, "threads": threads, "n": n}
+
+
+def run_reference(args):
+    world = int(os.environ.get("WORLD_SIZE", "1"))
+    rank = int(os.environ.get("RANK", "0"))
+    if rank != 0:
+        return
+    circ, desc = workload(args.workload, args.n)
+    text = circ.qasm()
+    from oracle import statevector as osv
+    osv.build()
+    for _ in range(args.warmup):
+        oracle_sample(text, 0.0, max_gates=1)
+    vals, samples = [], []
+    for k in range(args.steps):
+        v, smp = oracle_sample(text, args.ref_step_seconds, start_gate=0, max_gates=args.ref_gates)
+        vals.append(v)
+        samples.append(smp)
+    value = statistics.mean(vals)
+    cores = samples[0]["threads"]
+    sample = (f"per step: first {samples[0]['gates_timed']} of {samples[0]['gates_total']} gates "
+              f"of the workload in program order on the full 2^{samples[0]['n']} state, "
+              f"extrapolated linearly to the whole circuit")
+    line = {
+        "impl": "reference", "metric": METRIC, "value": value, "unit": "s", "n_gpus": world,
+        "steps": args.steps, "warmup": args.warmup, "ms_per_step": value * 1e3,
+        "higher_is_better": False, "scaling": "weak", "vs_baseline": None, "dtype": "c128",
+        "data": "synthetic", "config": {"workload": desc, "parallelism": "cpu oracle"},
+        "cpu_baseline": {"value": value, "unit": "s", "cores": cores, "kind": "oracle", "sample": sample},
+        "e2e": {"value": value, "unit": "s", "h2d_bytes_per_step": 0, "d2h_bytes_per_step": 0},
+    }
+    print(json.dumps(line), flush=True)
+
+
+# ----------------------------------------------------------------------------- GPU arm
+
+def single_qubit_sweep(q, torch, n: int, reps: int = 3):
+    """a6 microbenchmark: one generic 1-qubit gate at every target position on a fully involved
+    2^n state (SURVEY §8d 'formal >= 70%' number). Bytes = 32 * 2^n per gate."""
+    import numpy as np
+    stream = torch.cuda.Stream()
+    s = q.State(n, stream=stream.cuda_stream, fuse_bits=0)
+    H = np.array([[1, 1], [1, -1]], dtype=complex) / math.sqrt(2)
+    for t in range(n):
+        s.apply_gate(H, [t])
+    s.synchronize()
+    rng = np.random.default_rng(1)
+    U = np.linalg.qr(rng.normal(size=(2, 2)) + 1j * rng.normal(size=(2, 2)))[0]
+    res = []
+    for t in range(n):
+        s.apply_gate(U, [t])
+        e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+        e0.record(stream)
+        for _ in range(reps):
+            s.apply_gate(U, [t])
+        e1.record(stream)
+        e1.synchronize()
+        ms = e0.elapsed_time(e1) / reps
+        res.append(32.0 * (1 << n) / (ms * 1e-3) / 1e9)
+    s.close()
+    return res
+
+
+def run_ours(args):
+    import numpy as np
+    import torch
+
+    world, rank, local = dist_setup(args)
+    device = torch.device("cuda", local)
+    torch.cuda.set_device(device)
+    from paper_conf_hpca_zhaogydmuzjyt22_b200 import build as qbuild
+    if rank == 0 or world == 1:
+        qbuild.build()
+    barrier(world)
+    from paper_conf_hpca_zhaogydmuzjyt22_b200 import qgpu as q
+    q.load()
+
+    circ, desc = workload(args.workload, args.n)
+    text = circ.qasm()
+    n = circ.n
+    stream = torch.cuda.Stream(device=device)
+    cfg = dict(device=local, stream=stream.cuda_stream, fuse_bits=args.fuse_bits, reorder=args.reorder,
+               prune=int(not args.no_prune), timing=1)
+    st = q.State(n, **cfg)
+    c = q.Circuit(text)
+    ngates = c.info()[1]
+    flush = torch.empty(64 << 20, dtype=torch.float32, device=device)  # 256 MiB > 126 MB L2
+
+    def step():
+        st.reset()
+        st.apply_circuit(c)
+
+    for _ in range(args.warmup):
+        step()
+    st.synchronize()
+
+    times, stats = [], []
+    barrier(world)
+    torch.cuda.synchronize(device)
+    with ClockSampler(local) as clk:
+        for _ in range(args.steps):
+            with torch.cuda.stream(stream):
+                flush.zero_()          # L2 flush between timed steps (untimed)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            step()
+            e1.record(stream)
+            e1.synchronize()
+            times.append(e0.elapsed_time(e1))
+            stats.append(st.stats())
+        torch.cuda.synchronize(device)
+    barrier(world)
+    ms_local = statistics.mean(times)
+    ms = allreduce_max(ms_local, world, device)
+    clocks = clk.summary()
+
+    # roofline of the dominant kernel (fused tile pass): algorithmic bytes / event-timed duration
+    tile_ms = statistics.mean(s["tile_kernel_ms"] for s in stats)
+    tile_bytes = statistics.mean(s["tile_algo_bytes"] for s in stats)
+    tile_launches = statistics.mean(s["tile_kernel_launches"] for s in stats)
+    kernel_ms = statistics.mean(s["kernel_ms"] for s in stats)
+    algo_bytes = statistics.mean(s["algo_bytes"] for s in stats)
+    unfused = statistics.mean(s["unfused_bytes"] for s in stats)
+    peak, peak_src = peaks()
+    achieved = tile_bytes / (tile_ms * 1e-3) / 1e9 if tile_ms > 0 else 0.0
+    traffic = None
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    if os.path.exists(tp):
+        try:
+            t = json.load(open(tp))
+            if t.get("workload") == args.workload and t.get("n") == n:
+                traffic = t.get("dram_bytes_per_launch")
+        except Exception:
+            traffic = None
+    s0 = stats[-1]
+
+    # e2e through the public API with host buffers: QASM text -> parse -> reset -> apply ->
+    # probabilities of 10 qubits back to the host (pinned copies inside the library)
+    e2e_qubits = list(range(min(10, n)))
+    e2e_times = []
+    h2d = d2h = 0
+    barrier(world)
+    for k in range(max(1, args.steps)):
+        torch.cuda.synchronize(device)
+        t0 = time.perf_counter()
+        cc = q.Circuit(text)
+        st.reset()
+        st.apply_circuit(cc)
+        p = st.probabilities(e2e_qubits)
+        e2e_times.append(time.perf_counter() - t0)
+        ss = st.stats()
+        h2d, d2h = ss["h2d_bytes"], ss["d2h_bytes"]
+        cc.close()
+    e2e_val = allreduce_max(statistics.mean(e2e_times), world, device)
+    assert abs(p.sum() - 1) < 1e-9, "e2e readout not normalised"
+
+    launches = s0["kernels_launched"]
+    line = {
+        "metric": METRIC, "value": ms / 1e3, "unit": "s", "n_gpus": world, "steps": args.steps,
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False, "scaling": "weak",
+        "vs_baseline": None, "dtype": "c128", "data": "synthetic (seeded generator, QASM text)",
+        "config": {"workload": desc, "n_qubits": n, "gates": ngates, "reorder": args.reorder,
+                   "prune": int(not args.no_prune), "fuse_bits": args.fuse_bits,
+                   "replicas_per_gpu": 1, "parallelism": f"replicas x{world}" if world > 1 else "1 GPU",
+                   "l2": "flushed between timed steps (256 MiB write) and state 16*2^n B > L2"},
+        "roofline": {"kernel": "tile_kernel (fused pass)", "bound": "hbm", "achieved": achieved,
+                     "peak": peak, "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
+                     "peak_source": peak_src, "algo_bytes_per_launch": tile_bytes / max(tile_launches, 1),
+                     "launches_per_step": tile_launches, "tile_ms_per_step": tile_ms,
+                     "share_of_step": tile_ms / ms if ms else None,
+                     "frac_of_8TBs_spec": achieved / 8000.0},
+        "gates_per_s": ngates / (ms / 1e3),
+        "gate_apply_GBps": {"algorithmic": algo_bytes / (ms / 1e3) / 1e9,
+                            "unfused_equivalent": unfused / (ms / 1e3) / 1e9,
+                            "kernel_ms_per_step": kernel_ms},
+        "pruning": {"chunks_processed": s0["chunks_processed"], "chunks_skipped": s0["chunks_skipped"],
+                    "amps_processed": s0["amps_processed"], "amps_full": s0["amps_full"],
+                    "ops_before_full_involvement": s0["ops_before_full_involvement"],
+                    "passes": s0["passes"], "relabels": s0["relabels"]},
+        "e2e": {"value": e2e_val, "unit": "s", "h2d_bytes_per_step": h2d, "d2h_bytes_per_step": d2h,
+                "path": "qgpu_circuit_from_qasm + qgpu_state_reset + qgpu_apply_circuit + qgpu_probabilities(10 qubits)"},
+        "gpu_launches": launches * args.steps,
+        "gpu_launches_per_step": launches,
+        "clocks": clocks,
+    }
+    st.close()
+
+    if args.micro and rank == 0:
+        nm = args.micro_n
+        gbs = single_qubit_sweep(q, torch, nm)
+        line["single_qubit_gate"] = {"n": nm, "GBps_min": min(gbs), "GBps_median": statistics.median(gbs),
+                                     "GBps_per_target": [round(x, 1) for x in gbs],
+                                     "frac_min": min(gbs) / peak, "frac_median": statistics.median(gbs) / peak,
+                                     "frac_min_of_8TBs": min(gbs) / 8000.0}
+
+    if rank == 0 and world == 1 and not args.no_cpu_baseline:
+        v, smp = oracle_sample(text, args.cpu_seconds)
+        line["cpu_baseline"] = {"value": v, "unit": "s", "cores": smp["threads"], "kind": "oracle",
+                                "sample": f"first {smp['gates_timed']} of {smp['gates_total']} gates of "
+                                          f"{args.workload} (program order, unpruned, full 2^{n} state, "
+                                          f"{smp['seconds']:.1f} s), extrapolated linearly to the circuit"}
+    if rank == 0:
+        print(json.dumps(line), flush=True)
+    if world > 1:
+        import torch.distributed as dist
+        dist.destroy_process_group()
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--gpus", type=int, default=1)
+    ap.add_argument("--steps", type=int, default=5)
+    ap.add_argument("--warmup", type=int, default=3)
+    ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
+    ap.add_argument("--workload", default="qft28")
+    ap.add_argument("--n", type=int, default=None)
+    ap.add_argument("--fuse-bits", type=int, default=12)
+    ap.add_argument("--reorder", type=int, default=2)
+    ap.add_argument("--no-prune", action="store_true")
+    ap.add_argument("--micro", type=int, default=1)
+    ap.add_argument("--micro-n", type=int, default=30)
+    ap.add_argument("--no-cpu-baseline", action="store_true")
+    ap.add_argument("--cpu-seconds", type=float, default=20.0)
+    ap.add_argument("--ref-step-seconds", type=float, default=8.0)
+    ap.add_argument("--ref-gates", type=int, default=None)
+    args = ap.parse_args()
+    if args.warmup < 3:
+        args.warmup = 3
+    if args.impl == "reference":
+        run_reference(args)
+    else:
+        run_ours(args)
+
+
+if __name__ == "__main__":
+    main()

@@ -90,6 +90,8 @@ typedef struct {
   uint64_t tile_kernel_launches;
   uint64_t tile_algo_bytes;    /* algorithmic bytes of fused tile kernels only               */
   double swap_ms;              /* timing=1: time in swaps                                    */
+  uint64_t h2d_bytes;          /* host->device bytes copied by the library (ops, amplitudes) */
+  uint64_t d2h_bytes;          /* device->host bytes copied by readout calls                 */
 } qgpu_stats;
 
 /* ---- configuration and state ---------------------------------------------------------- */

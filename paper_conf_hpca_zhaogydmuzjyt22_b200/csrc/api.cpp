@@ -57,8 +57,8 @@ struct qgpu_state {
   qgpu_stats stats;
   bool poisoned = false;
   // device op arena (fused tile passes read their ops from here)
-  DevOp* d_ops = nullptr;
-  DevOp* h_ops = nullptr;
+  unsigned char* d_ops = nullptr;
+  unsigned char* h_ops = nullptr;
   size_t ops_cap = 0;
   cudaEvent_t ops_evt = nullptr;
   // readout scratch
@@ -150,7 +150,7 @@ qgpu_status zero_fill(qgpu_state* st, uint64_t from, uint64_t to) {
 }
 
 // Execute one planned pass on this rank's local buffer.
-qgpu_status exec_pass(qgpu_state* st, const Pass& p, const DevOp* d_ops) {
+qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops) {
   const int m = st->m;
   const uint64_t lmask = (m >= 64) ? ~0ull : ((1ull << m) - 1);
   const int kin = st->cfg.prune ? p.k_in : m, kout = st->cfg.prune ? p.k_out : m;
@@ -177,8 +177,11 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const DevOp* d_ops) {
   if (p.kind == PK_TILE) {
     TileArgs a{};
     a.psi = st->psi;
-    a.ops = d_ops;
+    a.blob = d_ops;
     a.nops = int(p.ops.size());
+    a.nscalar = p.nscalar;
+    a.ops_bytes = int(p.ops_bytes());
+    a.npool = int(p.pool.size());
     a.b = p.b;
     a.l = p.l;
     for (int i = 0; i < p.b; ++i) a.spos[i] = p.spos[i];
@@ -279,36 +282,39 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const DevOp* d_ops) {
 qgpu_status ensure_ops(qgpu_state* st, size_t n) {
   if (n <= st->ops_cap) return QGPU_OK;
   size_t cap = std::max<size_t>(n, 2 * st->ops_cap);
-  cap = std::max<size_t>(cap, 1024);
+  cap = std::max<size_t>(cap, 1 << 16);
   CK(cudaStreamSynchronize(st->stream));
   if (st->d_ops) CK(cudaFree(st->d_ops));
   if (st->h_ops) CK(cudaFreeHost(st->h_ops));
   st->d_ops = nullptr;
   st->h_ops = nullptr;
-  CK(cudaMalloc(&st->d_ops, cap * sizeof(DevOp)));
-  CK(cudaMallocHost(&st->h_ops, cap * sizeof(DevOp)));
+  CK(cudaMalloc(&st->d_ops, cap));
+  CK(cudaMallocHost(&st->h_ops, cap));
   st->ops_cap = cap;
   return QGPU_OK;
 }
 
 qgpu_status run_plan(qgpu_state* st, const std::vector<Pass>& passes) {
-  size_t nops = 0;
-  for (const Pass& p : passes) nops += p.ops.size();
+  size_t nbytes = 0;
   std::vector<size_t> off(passes.size(), 0);
-  if (nops) {
-    qgpu_status s = ensure_ops(st, nops);
+  for (size_t i = 0; i < passes.size(); ++i) {
+    off[i] = nbytes;
+    nbytes += passes[i].blob_bytes();
+  }
+  if (nbytes) {
+    qgpu_status s = ensure_ops(st, nbytes);
     if (s) return s;
     // the pinned staging buffer may still be read by the previous upload
     CK(cudaEventSynchronize(st->ops_evt));
-    size_t o = 0;
     for (size_t i = 0; i < passes.size(); ++i) {
-      off[i] = o;
-      if (!passes[i].ops.empty())
-        std::memcpy(st->h_ops + o, passes[i].ops.data(), passes[i].ops.size() * sizeof(DevOp));
-      o += passes[i].ops.size();
+      const Pass& p = passes[i];
+      if (p.ops.empty()) continue;
+      std::memset(st->h_ops + off[i], 0, p.ops_bytes());
+      std::memcpy(st->h_ops + off[i], p.ops.data(), p.ops.size() * sizeof(TileOp));
+      std::memcpy(st->h_ops + off[i] + p.ops_bytes(), p.pool.data(), p.pool.size() * sizeof(cplx));
     }
-    CK(cudaMemcpyAsync(st->d_ops, st->h_ops, nops * sizeof(DevOp), cudaMemcpyHostToDevice,
-                       st->stream));
+    CK(cudaMemcpyAsync(st->d_ops, st->h_ops, nbytes, cudaMemcpyHostToDevice, st->stream));
+    st->stats.h2d_bytes += nbytes;
     CK(cudaEventRecord(st->ops_evt, st->stream));
   }
   for (size_t i = 0; i < passes.size(); ++i) {
@@ -338,7 +344,10 @@ qgpu_status check_state(qgpu_state* st) {
 
 qgpu_status init_amplitudes(qgpu_state* st) {
   if (!st->cfg.prune) CK(cudaMemsetAsync(st->psi, 0, (1ull << st->m) * sizeof(double2), st->stream));
-  if (st->cfg.rank == 0) CK(launch_set_amp(st->stream, st->psi, 0, 1.0, 0.0));
+  if (st->cfg.rank == 0) {
+    CK(launch_set_amp(st->stream, st->psi, 0, 1.0, 0.0));
+    st->stats.kernels_launched++;
+  }
   return QGPU_OK;
 }
 
@@ -585,6 +594,7 @@ qgpu_status qgpu_get_amplitudes_device(qgpu_state* st, uint64_t start, uint64_t 
   }
   a.L = live(st, st->map.kl);
   CK(launch_gather(st->stream, a));
+  st->stats.kernels_launched++;
   return QGPU_OK;
 }
 
@@ -604,6 +614,7 @@ qgpu_status qgpu_get_amplitudes(qgpu_state* st, uint64_t start, uint64_t count, 
     const uint64_t c = std::min(chunk, count - done);
     if (qgpu_status s = qgpu_get_amplitudes_device(st, start + done, c, st->d_scratch)) return s;
     CK(cudaMemcpyAsync(out + 2 * done, st->d_scratch, c * 2 * sizeof(double), cudaMemcpyDeviceToHost, st->stream));
+    st->stats.d2h_bytes += c * 2 * sizeof(double);
   }
   CK(cudaStreamSynchronize(st->stream));
   return drain_timing(st);
@@ -640,11 +651,13 @@ qgpu_status qgpu_probabilities(qgpu_state* st, int mq, const int* qubits, double
   }
   a.out = st->d_scratch;
   CK(launch_probs(st->stream, a, st->d_scratch + B));
+  st->stats.kernels_launched += (mq <= 12) ? 2 : 1;
   if (st->g > 0) {
     qgpu_status s = comm_probabilities_finish(st->comm, st->d_scratch, mq, rank_fixed, st->stream);
     if (s) return s;
   }
   CK(cudaMemcpyAsync(out, st->d_scratch, B * sizeof(double), cudaMemcpyDeviceToHost, st->stream));
+  st->stats.d2h_bytes += B * sizeof(double);
   CK(cudaStreamSynchronize(st->stream));
   return drain_timing(st);
 }

@@ -177,20 +177,48 @@ __global__ void __launch_bounds__(kThreads) phase_kernel(PhaseArgs a) {
 
 // ------------------------------------------------------------------------------ a9 tile
 // One CTA processes tiles of T = 2^b amplitudes: tile-local bit i <-> physical position
-// spos[i]; spos[0..l) = 0..l-1, so a warp moves 32 consecutive amplitudes (512 B).
-// Non-tile bits of the live range index the tiles. Op conditions on bits outside the tile
-// (omask/omatch over rank_base | base) are uniform over a tile; PHASE ops whose condition is
-// entirely outside the tile are a per-tile scalar (they commute with every op of the pass,
-// which acts on tile bits only) applied once at load.
+// spos[i]; spos[0..l) = 0..l-1, so a warp moves 32 consecutive amplitudes (512 B). The
+// non-tile bits of the live range index the tiles (grid-stride, persistent CTAs).
+//  * load: cp.async (LDGSTS) global -> shared, 16 B per request, every request of the tile in
+//    flight at once with no register staging; requests at index >= L_in use src-size 0, i.e.
+//    the hardware zero-fills them (first-touch expansion, a5).
+//  * op conditions on bits outside the tile are tile-uniform: evaluated once per tile into
+//    `active`. PHASE ops whose condition lies entirely outside the tile multiply the whole
+//    tile by one scalar; they commute with every op of the pass (which act on tile bits only),
+//    so their product is applied once, at the store.
+//  * U1/U2 ops: pairs/quads read-modify-write in shared memory, one barrier per op.
+//  * runs of PHASE ops: each thread keeps its 16 amplitudes in registers across the run; the
+//    condition on the thread's fixed tile bits is tested once per op and thread.
 constexpr int kTileMaxPer = 16;  // amplitudes per thread (T <= 16 * kThreads = 4096)
 
-__global__ void __launch_bounds__(kThreads) tile_kernel(TileArgs a) {
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
+  const unsigned sa = static_cast<unsigned>(__cvta_generic_to_shared(smem));
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(sa), "l"(gmem), "r"(src_bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() {
+  asm volatile("cp.async.wait_all;\n" ::: "memory");
+}
+
+__global__ void __launch_bounds__(kThreads, 2) tile_kernel(TileArgs a) {
   extern __shared__ __align__(16) unsigned char smem_raw[];
-  double2* s = reinterpret_cast<double2*>(smem_raw);
   const int b = a.b, l = a.l;
   const uint32_t T = 1u << b;
-  uint64_t* hiOff = reinterpret_cast<uint64_t*>(s + T);
   const int nh = 1 << (b - l);
+  double2* s = reinterpret_cast<double2*>(smem_raw);
+  uint64_t* hiOff = reinterpret_cast<uint64_t*>(s + T);
+  unsigned char* blob = reinterpret_cast<unsigned char*>(hiOff + ((nh + 1) & ~1));
+  const TileOp* ops = reinterpret_cast<const TileOp*>(blob);
+  const double2* pool = reinterpret_cast<const double2*>(blob + a.ops_bytes);
+  unsigned char* active = blob + a.ops_bytes + size_t(a.npool) * 16;
+  double2* scal_s = reinterpret_cast<double2*>(active + ((a.nops + 15) & ~15));
+
+  {  // stage the pass's ops and matrices in shared memory (once per CTA)
+    const int4* src = reinterpret_cast<const int4*>(a.blob);
+    int4* dst = reinterpret_cast<int4*>(blob);
+    const int n16 = (a.ops_bytes + a.npool * 16) / 16;
+    for (int i = threadIdx.x; i < n16; i += kThreads) dst[i] = src[i];
+  }
   for (int h = threadIdx.x; h < nh; h += kThreads) {
     uint64_t off = 0;
     for (int i = l; i < b; ++i)
@@ -198,80 +226,91 @@ __global__ void __launch_bounds__(kThreads) tile_kernel(TileArgs a) {
     hiOff[h] = off;
   }
   __syncthreads();
-  const uint64_t lowmask = (1ull << l) - 1;
-  const DevOp* __restrict__ ops = a.ops;
+  const uint32_t lowmask = (1u << l) - 1;
   const int per = (T + kThreads - 1) / kThreads;
+  const uint32_t tid = threadIdx.x;
+  const int warp = tid >> 5, lane = tid & 31;
 
   for (uint64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x) {
     const uint64_t base = deposit(tile, a.spos, b);
     const uint64_t gbase = a.rank_base | base;
-    // tile-uniform scalar of the PHASE ops that live entirely outside the tile
-    double2 scal = make_double2(1.0, 0.0);
-    bool has_scal = false;
-    for (int k = 0; k < a.nops; ++k) {
-      if (ops[k].kind == OP_PHASE && ops[k].lmask == 0 && (gbase & ops[k].omask) == ops[k].omatch) {
-        scal = cmul(scal, make_double2(ops[k].m[0], ops[k].m[1]));
-        has_scal = true;
-      }
-    }
-    // ---- load (all loads in flight before the first shared-memory store)
-    double2 v[kTileMaxPer];
+    // ---- issue every load of the tile
 #pragma unroll
     for (int r = 0; r < kTileMaxPer; ++r) {
-      if (r < per) {
-        const uint32_t j = threadIdx.x + r * kThreads;
+      const uint32_t j = tid + r * kThreads;
+      if (r < per && j < T) {
         const uint64_t idx = base | (j & lowmask) | hiOff[j >> l];
-        v[r] = (j < T && idx < a.L_in) ? ld_stream(a.psi + idx) : make_double2(0, 0);
+        const bool live = idx < a.L_in;
+        cp_async16(s + j, a.psi + (live ? idx : 0), live ? 16 : 0);
       }
     }
+    asm volatile("cp.async.commit_group;\n" ::: "memory");
+    // ---- tile-uniform op conditions (overlaps the loads)
+    for (int k = tid; k < a.nops; k += kThreads)
+      active[k] = (gbase & ops[k].omask) == ops[k].omatch;
+    __syncthreads();
+    if (warp == 0) {  // product of outside-only phases: lane-strided, then butterfly
+      double2 sc = make_double2(1.0, 0.0);
+      for (int k = lane; k < a.nscalar; k += 32)
+        if (active[k]) sc = cmul(sc, pool[ops[k].moff]);
 #pragma unroll
-    for (int r = 0; r < kTileMaxPer; ++r) {
-      if (r < per) {
-        const uint32_t j = threadIdx.x + r * kThreads;
-        if (j < T) s[j] = has_scal ? cmul(v[r], scal) : v[r];
+      for (int o = 16; o > 0; o >>= 1) {
+        double2 t;
+        t.x = __shfl_xor_sync(0xffffffffu, sc.x, o);
+        t.y = __shfl_xor_sync(0xffffffffu, sc.y, o);
+        sc = cmul(sc, t);
       }
+      if (lane == 0) *scal_s = sc;
     }
+    cp_async_wait_all();
     __syncthreads();
     // ---- apply the pass's ops in order
-    int i = 0;
+    int i = a.nscalar;
     while (i < a.nops) {
       const int kind = ops[i].kind;
       if (kind == OP_PHASE) {
-        int j = i;
-        while (j < a.nops && ops[j].kind == OP_PHASE) ++j;
-        // owned amplitudes in registers across the whole run of phase ops
+        // a run of commuting phase terms, grouped by their condition on the owned index r:
+        // accumulate each group's product per thread, then multiply the matching amplitudes
+        double2 v[kTileMaxPer];
 #pragma unroll
         for (int r = 0; r < kTileMaxPer; ++r) {
-          const uint32_t jj = threadIdx.x + r * kThreads;
+          const uint32_t jj = tid + r * kThreads;
           if (r < per && jj < T) v[r] = s[jj];
         }
-        for (int k = i; k < j; ++k) {
-          const uint32_t lm = ops[k].lmask;
-          if (lm == 0) continue;  // folded into the tile scalar
-          if ((gbase & ops[k].omask) != ops[k].omatch) continue;
-          const uint32_t lt = ops[k].lmatch;
-          const double2 ph = make_double2(ops[k].m[0], ops[k].m[1]);
-#pragma unroll
-          for (int r = 0; r < kTileMaxPer; ++r) {
-            const uint32_t jj = threadIdx.x + r * kThreads;
-            if (r < per && (jj & lm) == lt) v[r] = cmul(v[r], ph);
+        double2 acc = make_double2(1.0, 0.0);
+        bool any = false;
+        for (;; ++i) {
+          const TileOp& o = ops[i];
+          if (active[i] && (tid & o.lmask & (kThreads - 1)) == (o.lmatch & (kThreads - 1))) {
+            acc = cmul(acc, pool[o.moff]);
+            any = true;
           }
+          if (o.t0) {  // end of group: apply to the owned amplitudes whose r matches
+            if (any) {
+              const uint32_t mh = o.lmask >> 8, th = o.lmatch >> 8;
+#pragma unroll
+              for (int r = 0; r < kTileMaxPer; ++r)
+                if (r < per && (uint32_t(r) & mh) == th) v[r] = cmul(v[r], acc);
+            }
+            acc = make_double2(1.0, 0.0);
+            any = false;
+          }
+          if (o.t1) break;
         }
+        ++i;
 #pragma unroll
         for (int r = 0; r < kTileMaxPer; ++r) {
-          const uint32_t jj = threadIdx.x + r * kThreads;
+          const uint32_t jj = tid + r * kThreads;
           if (r < per && jj < T) s[jj] = v[r];
         }
         __syncthreads();
-        i = j;
       } else if (kind == OP_U1) {
-        if ((gbase & ops[i].omask) == ops[i].omatch) {
+        if (active[i]) {
           const int t = ops[i].t0;
           const uint32_t lm = ops[i].lmask;
-          const double* m = ops[i].m;
-          const double2 u00 = make_double2(m[0], m[1]), u01 = make_double2(m[2], m[3]);
-          const double2 u10 = make_double2(m[4], m[5]), u11 = make_double2(m[6], m[7]);
-          for (uint32_t p = threadIdx.x; p < T / 2; p += kThreads) {
+          const double2* u = pool + ops[i].moff;
+          const double2 u00 = u[0], u01 = u[1], u10 = u[2], u11 = u[3];
+          for (uint32_t p = tid; p < T / 2; p += kThreads) {
             const uint32_t i0 = uint32_t(insert0(p, t));
             if ((i0 & lm) != lm) continue;
             const uint32_t i1 = i0 | (1u << t);
@@ -283,28 +322,24 @@ __global__ void __launch_bounds__(kThreads) tile_kernel(TileArgs a) {
         }
         ++i;
       } else {  // OP_U2
-        if ((gbase & ops[i].omask) == ops[i].omatch) {
+        if (active[i]) {
           const int t0 = ops[i].t0, t1 = ops[i].t1;
           const int lo = min(t0, t1), hi = max(t0, t1);
           const uint32_t lm = ops[i].lmask;
-          const double* m = ops[i].m;
-          double2 u[16];
-#pragma unroll
-          for (int e = 0; e < 16; ++e) u[e] = make_double2(m[2 * e], m[2 * e + 1]);
-          const uint32_t o[4] = {0u, 1u << t0, 1u << t1, (1u << t0) | (1u << t1)};
-          for (uint32_t p = threadIdx.x; p < T / 4; p += kThreads) {
+          const double2* u = pool + ops[i].moff;
+          const uint32_t o1 = 1u << t0, o2 = 1u << t1;
+          for (uint32_t p = tid; p < T / 4; p += kThreads) {
             const uint32_t i0 = uint32_t(insert0(insert0(p, lo), hi));
             if ((i0 & lm) != lm) continue;
-            double2 x[4];
-#pragma unroll
-            for (int e = 0; e < 4; ++e) x[e] = s[i0 | o[e]];
+            const double2 x0 = s[i0], x1 = s[i0 | o1], x2 = s[i0 | o2], x3 = s[i0 | o1 | o2];
 #pragma unroll
             for (int row = 0; row < 4; ++row) {
-              double2 y = cmul(u[row * 4], x[0]);
-              y = cfma(u[row * 4 + 1], x[1], y);
-              y = cfma(u[row * 4 + 2], x[2], y);
-              y = cfma(u[row * 4 + 3], x[3], y);
-              s[i0 | o[row]] = y;
+              double2 y = cmul(u[row * 4], x0);
+              y = cfma(u[row * 4 + 1], x1, y);
+              y = cfma(u[row * 4 + 2], x2, y);
+              y = cfma(u[row * 4 + 3], x3, y);
+              const uint32_t o = (row & 1 ? o1 : 0u) | (row & 2 ? o2 : 0u);
+              s[i0 | o] = y;
             }
           }
           __syncthreads();
@@ -312,12 +347,15 @@ __global__ void __launch_bounds__(kThreads) tile_kernel(TileArgs a) {
         ++i;
       }
     }
-    // ---- store (every amplitude of the tile, including the expanded zero region)
+    // ---- store every amplitude of the tile (including the expanded zero region)
+    const double2 sc = *scal_s;
+    const bool has_sc = !(sc.x == 1.0 && sc.y == 0.0);
 #pragma unroll
     for (int r = 0; r < kTileMaxPer; ++r) {
-      if (r < per) {
-        const uint32_t j = threadIdx.x + r * kThreads;
-        if (j < T) st_stream(a.psi + (base | (j & lowmask) | hiOff[j >> l]), s[j]);
+      const uint32_t j = tid + r * kThreads;
+      if (r < per && j < T) {
+        const double2 x = has_sc ? cmul(s[j], sc) : s[j];
+        st_stream(a.psi + (base | (j & lowmask) | hiOff[j >> l]), x);
       }
     }
     __syncthreads();
@@ -382,7 +420,6 @@ __global__ void set_amp_kernel(double2* psi, uint64_t i, double2 v) { psi[i] = v
 // --------------------------------------------------------------------------- launchers
 namespace {
 int g_num_sms = 0;
-int g_tile_bps = 0;
 int num_sms() {
   if (!g_num_sms) {
     int dev = 0;
@@ -399,8 +436,10 @@ unsigned grid_for(uint64_t work_items, int per_block, int blocks_per_sm) {
 }
 }  // namespace
 
-size_t tile_smem_bytes(int b, int l) {
-  return (size_t(1) << b) * 16 + (size_t(1) << (b - l)) * 8;
+size_t tile_smem_bytes(int b, int l, int nops, int ops_bytes, int npool) {
+  const size_t nh = size_t(1) << (b - l);
+  return (size_t(1) << b) * 16 + ((nh + 1) & ~size_t(1)) * 8 + size_t(ops_bytes) +
+         size_t(npool) * 16 + size_t((nops + 15) & ~15) + 16;
 }
 
 cudaError_t launch_pair(cudaStream_t st, const PairArgs& a, bool shfl) {
@@ -435,14 +474,15 @@ cudaError_t launch_phase(cudaStream_t st, const PhaseArgs& a) {
 
 cudaError_t launch_tile(cudaStream_t st, const TileArgs& a) {
   if (a.ntiles == 0) return cudaSuccess;
-  const size_t smem = tile_smem_bytes(a.b, a.l);
-  static size_t configured = 0;
-  if (smem > configured) {
+  const size_t smem = tile_smem_bytes(a.b, a.l, a.nops, a.ops_bytes, a.npool);
+  static bool configured = false;
+  if (!configured) {
     cudaError_t e = cudaFuncSetAttribute(tile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
-                                         int(std::max<size_t>(smem, tile_smem_bytes(kMaxTileBits, 5))));
+                                         227 * 1024);
     if (e != cudaSuccess) return e;
-    configured = std::max<size_t>(smem, tile_smem_bytes(kMaxTileBits, 5));
+    configured = true;
   }
+  if (smem > 227 * 1024) return cudaErrorInvalidValue;
   int bps = 0;
   cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, tile_kernel, kThreads, smem);
   if (bps <= 0) bps = 1;

@@ -43,8 +43,11 @@ struct PhaseArgs {
 
 struct TileArgs {
   double2* psi;
-  const DevOp* ops;
+  const void* blob;        // [TileOp x nops, padded to 16 B | double2 x npool]
   int nops;
+  int nscalar;             // leading OP_PHASE_SCALAR ops (tile-uniform phases)
+  int ops_bytes;
+  int npool;
   int b, l;
   int spos[kMaxTileBits];
   uint64_t ntiles;
@@ -72,7 +75,7 @@ struct ProbArgs {
   double* partial;
 };
 
-size_t tile_smem_bytes(int b, int l);
+size_t tile_smem_bytes(int b, int l, int nops, int ops_bytes, int npool);
 size_t probs_scratch_doubles(int m);
 cudaError_t launch_pair(cudaStream_t st, const PairArgs& a, bool shfl);
 cudaError_t launch_quad(cudaStream_t st, const QuadArgs& a);

@@ -181,21 +181,20 @@ int local_bit(int pos, const Pass& p) {
 }  // namespace
 
 void build_tile_ops(Pass& p, int /*m*/) {
-  p.ops.clear();
+  std::vector<TileOp> raw;
+  std::vector<cplx> pool;
   for (const PhysGate& g : p.gates) {
     if (!g.diag) {
-      DevOp o{};
+      TileOp o{};
       o.kind = g.nt == 1 ? OP_U1 : OP_U2;
       o.t0 = local_bit(g.p[0], p);
       o.t1 = g.nt == 2 ? local_bit(g.p[1], p) : 0;
       o.lmask = o.lmatch = to_local(g.pc, p);
       o.omask = o.omatch = outside(g.pc, p);
+      o.moff = uint32_t(pool.size());
       const int dim = 1 << g.nt;
-      for (int i = 0; i < dim * dim; ++i) {
-        o.m[2 * i] = g.U[i].re;
-        o.m[2 * i + 1] = g.U[i].im;
-      }
-      p.ops.push_back(o);
+      for (int i = 0; i < dim * dim; ++i) pool.push_back(g.U[i]);
+      raw.push_back(o);
     } else {
       // diagonal: one phase term per diagonal entry that is not exactly 1
       const int dim = 1 << g.nt;
@@ -208,17 +207,38 @@ void build_tile_ops(Pass& p, int /*m*/) {
         for (int j = 0; j < g.nt; ++j)
           if (v >> j & 1) match |= 1ull << g.p[j];
         const uint64_t mask = g.pc | tmask;
-        DevOp o{};
-        o.kind = OP_PHASE;
+        TileOp o{};
         o.lmask = to_local(mask, p);
         o.lmatch = to_local(match, p);
         o.omask = outside(mask, p);
         o.omatch = outside(match, p);
-        o.m[0] = d.re;
-        o.m[1] = d.im;
-        p.ops.push_back(o);
+        o.kind = o.lmask == 0 ? OP_PHASE_SCALAR : OP_PHASE;
+        o.moff = uint32_t(pool.size());
+        pool.push_back(d);
+        raw.push_back(o);
       }
     }
+  }
+  p.ops.clear();
+  p.pool = std::move(pool);
+  for (const TileOp& o : raw)
+    if (o.kind == OP_PHASE_SCALAR) p.ops.push_back(o);
+  p.nscalar = int(p.ops.size());
+  for (size_t i = 0; i < raw.size();) {
+    if (raw[i].kind == OP_PHASE_SCALAR) { ++i; continue; }
+    if (raw[i].kind != OP_PHASE) { p.ops.push_back(raw[i]); ++i; continue; }
+    std::vector<TileOp> run;
+    size_t j = i;
+    for (; j < raw.size() && (raw[j].kind == OP_PHASE || raw[j].kind == OP_PHASE_SCALAR); ++j)
+      if (raw[j].kind == OP_PHASE) run.push_back(raw[j]);
+    auto key = [](const TileOp& o) { return (uint64_t(o.lmask >> 8) << 32) | (o.lmatch >> 8); };
+    std::stable_sort(run.begin(), run.end(), [&](const TileOp& x, const TileOp& y) { return key(x) < key(y); });
+    for (size_t k = 0; k < run.size(); ++k) {
+      run[k].t0 = (k + 1 == run.size() || key(run[k + 1]) != key(run[k])) ? 1 : 0;
+      run[k].t1 = (k + 1 == run.size()) ? 1 : 0;
+      p.ops.push_back(run[k]);
+    }
+    i = j;
   }
 }
 
@@ -268,7 +288,7 @@ struct Builder {
   }
 
   bool fits(uint64_t need, int n_ops_new) const {
-    if (int(cur.ops.size()) + n_ops_new > opt.max_ops) return false;
+    if (cur.n_est + n_ops_new > opt.max_ops) return false;
     if (need && n_u + 1 > opt.max_u_ops) return false;
     const int lm = std::min(opt.l_min, std::max(cur.k_out, 0));
     uint64_t S = used | need | ((lm > 0) ? ((1ull << lm) - 1) : 0);
@@ -330,7 +350,7 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
       B.used |= need;
       if (need) B.n_u++;
       B.cur.gates.push_back(pg);
-      B.cur.ops.resize(B.cur.ops.size() + n_new_ops);  // placeholder count; rebuilt at close
+      B.cur.n_est += n_new_ops;
       B.cur.count++;
       B.cur.k_out = map.kl;
       B.cur.unfused_bytes += unfused_gate_bytes(pg, k_before, map.kl);

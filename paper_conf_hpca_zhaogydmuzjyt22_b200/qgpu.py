@@ -53,7 +53,8 @@ class Stats(ctypes.Structure):
         "chunks_processed", "chunks_skipped", "algo_bytes", "unfused_bytes", "swaps", "swap_bytes")] + [
         ("ops_before_full_involvement", ctypes.c_int64), ("kernel_ms", ctypes.c_double),
         ("tile_kernel_ms", ctypes.c_double), ("tile_kernel_launches", ctypes.c_uint64),
-        ("tile_algo_bytes", ctypes.c_uint64), ("swap_ms", ctypes.c_double)]
+        ("tile_algo_bytes", ctypes.c_uint64), ("swap_ms", ctypes.c_double),
+        ("h2d_bytes", ctypes.c_uint64), ("d2h_bytes", ctypes.c_uint64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
