@@ -69,6 +69,9 @@ typedef struct {
                                  0 = one kernel per gate (pair/quad/diag kernels)          */
   int timing;                 /* 1: time every launch with CUDA events into qgpu_stats     */
   uint64_t swap_slab_bytes;   /* staging bytes per all-to-all slab (sharded mode)          */
+  int jit;                    /* fused passes: 0 = generic tile kernel only; 1 (default) = NVRTC-
+                                 specialised kernel for passes of >= 2^16 amplitudes; 2 = always.
+                                 Falls back to the generic kernel if NVRTC is unavailable   */
 } qgpu_config;
 
 typedef struct {
@@ -92,6 +95,9 @@ typedef struct {
   double swap_ms;              /* timing=1: time in swaps                                    */
   uint64_t h2d_bytes;          /* host->device bytes copied by the library (ops, amplitudes) */
   uint64_t d2h_bytes;          /* device->host bytes copied by readout calls                 */
+  uint64_t jit_launches;       /* fused passes run by an NVRTC-specialised kernel            */
+  uint64_t jit_compiles;       /* kernels compiled (cache misses)                            */
+  double jit_ms;               /* host time spent compiling                                  */
 } qgpu_stats;
 
 /* ---- configuration and state ---------------------------------------------------------- */
@@ -178,6 +184,13 @@ qgpu_status qgpu_circuit_reorder(const qgpu_circuit* c, int mode, uint64_t* orde
  * 3 diag, 4 relabel, 5 swap. */
 qgpu_status qgpu_circuit_plan(const qgpu_circuit* c, int n_qubits, int world_size, int reorder,
                               int fuse_bits, int64_t* info, uint64_t cap, uint64_t* n_passes);
+
+/* Host-only (no GPU needed): generate the NVRTC-specialised kernel source of every fused pass of
+ * the plan (as qgpu_circuit_plan) and compile it for sm_100a. *n_compiled = passes compiled.
+ * Returns UNSUPPORTED if NVRTC cannot be loaded, CUDA (with the NVRTC log in
+ * qgpu_last_error) if a pass fails to compile. */
+qgpu_status qgpu_circuit_jit_check(const qgpu_circuit* c, int n_qubits, int reorder, int fuse_bits,
+                                   int* n_compiled);
 
 /* ---- scheduler state (tests / diagnostics) ---------------------------------------------- */
 

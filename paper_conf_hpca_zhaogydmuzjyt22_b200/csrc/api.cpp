@@ -6,12 +6,14 @@
 #include <bit>
 #include <cstdarg>
 #include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <exception>
 #include <string>
 #include <vector>
 
 #include "comm.h"
+#include "jit.h"
 #include "kernels.h"
 #include "qgpu_internal.h"
 
@@ -26,7 +28,7 @@ namespace {
 thread_local std::string g_err;
 
 qgpu_status fail(qgpu_status s, const char* fmt, ...) {
-  char buf[1024];
+  static thread_local char buf[1 << 16];
   va_list ap;
   va_start(ap, fmt);
   vsnprintf(buf, sizeof(buf), fmt, ap);
@@ -177,18 +179,40 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops)
   if (p.kind == PK_TILE) {
     TileArgs a{};
     a.psi = st->psi;
+    const TileProgram& P = p.prog;
     a.blob = d_ops;
-    a.nops = int(p.ops.size());
-    a.nscalar = p.nscalar;
-    a.ops_bytes = int(p.ops_bytes());
-    a.npool = int(p.pool.size());
+    a.blob_bytes = int(P.bytes);
+    a.nops = int(P.ops.size());
+    a.npat = int(P.patterns.size());
+    a.nscalar = int(P.scalar.size());
+    a.off_entries = int(P.off_entries);
+    a.off_patterns = int(P.off_patterns);
+    a.off_terms = int(P.off_terms);
+    a.off_scalar = int(P.off_scalar);
+    a.off_pool = int(P.off_pool);
+    a.nr = P.nr;
+    a.nw = P.nw;
     a.b = p.b;
     a.l = p.l;
     for (int i = 0; i < p.b; ++i) a.spos[i] = p.spos[i];
     a.ntiles = 1ull << (kout - p.b);
     a.L_in = L_in;
     a.rank_base = rank << m;
-    CK(launch_tile(st->stream, a));
+    const int jit = st->cfg.jit;
+    cudaError_t e = cudaErrorNotSupported;
+    if (jit == 2 || (jit == 1 && kout >= 16)) {
+      double ms = 0;
+      e = launch_tile_jit(st->stream, p, a, tile_smem_bytes(a), device_num_sms(), &ms);
+      if (e == cudaSuccess) {
+        st->stats.jit_launches++;
+        if (ms > 0) {
+          st->stats.jit_compiles++;
+          st->stats.jit_ms += ms;
+        }
+      }
+    }
+    if (e == cudaErrorNotSupported) e = launch_tile(st->stream, a);
+    CK(e);
     st->stats.kernels_launched++;
     bytes = 16 * (L_in + L_out);
   } else {
@@ -299,20 +323,15 @@ qgpu_status run_plan(qgpu_state* st, const std::vector<Pass>& passes) {
   std::vector<size_t> off(passes.size(), 0);
   for (size_t i = 0; i < passes.size(); ++i) {
     off[i] = nbytes;
-    nbytes += passes[i].blob_bytes();
+    if (passes[i].kind == PK_TILE) nbytes += (passes[i].prog.bytes + 15) / 16 * 16;
   }
   if (nbytes) {
     qgpu_status s = ensure_ops(st, nbytes);
     if (s) return s;
     // the pinned staging buffer may still be read by the previous upload
     CK(cudaEventSynchronize(st->ops_evt));
-    for (size_t i = 0; i < passes.size(); ++i) {
-      const Pass& p = passes[i];
-      if (p.ops.empty()) continue;
-      std::memset(st->h_ops + off[i], 0, p.ops_bytes());
-      std::memcpy(st->h_ops + off[i], p.ops.data(), p.ops.size() * sizeof(TileOp));
-      std::memcpy(st->h_ops + off[i] + p.ops_bytes(), p.pool.data(), p.pool.size() * sizeof(cplx));
-    }
+    for (size_t i = 0; i < passes.size(); ++i)
+      if (passes[i].kind == PK_TILE) passes[i].prog.pack(st->h_ops + off[i]);
     CK(cudaMemcpyAsync(st->d_ops, st->h_ops, nbytes, cudaMemcpyHostToDevice, st->stream));
     st->stats.h2d_bytes += nbytes;
     CK(cudaEventRecord(st->ops_evt, st->stream));
@@ -378,6 +397,7 @@ qgpu_status qgpu_config_init(qgpu_config* cfg) {
   cfg->reorder = 2;
   cfg->fuse_bits = 12;
   cfg->swap_slab_bytes = 256ull << 20;
+  cfg->jit = 1;
   return QGPU_OK;
 }
 
@@ -406,6 +426,8 @@ qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out
       return fail(QGPU_ERR_INVALID_ARG, "fuse_bits must be 0 or >= 7");
     if (cfg.reorder < 0 || cfg.reorder > 2) return fail(QGPU_ERR_INVALID_ARG, "reorder must be 0, 1 or 2");
     cfg.chunk_bits = std::min(std::max(cfg.chunk_bits, 0), n - g);
+    if (const char* ev = std::getenv("QGPU_JIT")) cfg.jit = std::atoi(ev);
+    if (cfg.jit < 0 || cfg.jit > 2) return fail(QGPU_ERR_INVALID_ARG, "jit must be 0, 1 or 2");
     auto* st = new qgpu_state();
     st->cfg = cfg;
     st->n = n;
@@ -728,6 +750,32 @@ qgpu_status qgpu_circuit_plan(const qgpu_circuit* c, int n, int world, int reord
       r[0] = p.first; r[1] = p.count; r[2] = p.kind; r[3] = p.k_in; r[4] = p.k_out; r[5] = p.b;
       r[6] = int64_t(S & 0xffffffffull);
       r[7] = int64_t(S >> 32);
+    }
+    return QGPU_OK;
+  } catch (const std::exception& ex) {
+    return fail(QGPU_ERR_OUT_OF_MEMORY, "exception: %s", ex.what());
+  }
+}
+
+qgpu_status qgpu_circuit_jit_check(const qgpu_circuit* c, int n, int reorder_mode, int fuse_bits,
+                                   int* n_compiled) {
+  try {
+    if (!c || n < c->c.n || n > kMaxQubits) return fail(QGPU_ERR_INVALID_ARG, "bad arguments");
+    if (n_compiled) *n_compiled = 0;
+    QubitMap map;
+    map.init(n, n);
+    PlanOptions o;
+    o.fuse_bits = fuse_bits;
+    std::vector<Pass> passes;
+    plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode), map, o, &passes, nullptr);
+    std::string cubin, log;
+    for (const Pass& p : passes) {
+      if (p.kind != PK_TILE) continue;
+      if (!jit_compile_cubin(tile_jit_source(p), &cubin, &log)) {
+        if (log == "libnvrtc not found") return fail(QGPU_ERR_UNSUPPORTED, "%s", log.c_str());
+        return fail(QGPU_ERR_CUDA, "NVRTC: %s\n--- source ---\n%s", log.c_str(), tile_jit_source(p).c_str());
+      }
+      if (n_compiled) (*n_compiled)++;
     }
     return QGPU_OK;
   } catch (const std::exception& ex) {

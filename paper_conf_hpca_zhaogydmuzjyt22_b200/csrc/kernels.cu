@@ -21,24 +21,7 @@ namespace qgpu {
 
 namespace {
 
-__device__ __forceinline__ double2 cmul(double2 a, double2 b) {
-  return make_double2(fma(a.x, b.x, -a.y * b.y), fma(a.x, b.y, a.y * b.x));
-}
-// a*b + c
-__device__ __forceinline__ double2 cfma(double2 a, double2 b, double2 c) {
-  return make_double2(fma(a.x, b.x, fma(-a.y, b.y, c.x)), fma(a.x, b.y, fma(a.y, b.x, c.y)));
-}
-__device__ __forceinline__ uint64_t insert0(uint64_t v, int b) {
-  const uint64_t lo = v & ((1ull << b) - 1);
-  return ((v >> b) << (b + 1)) | lo;
-}
-// insert zero bits at the (ascending) positions ins[0..nins)
-__device__ __forceinline__ uint64_t deposit(uint64_t v, const int* ins, int nins) {
-  for (int i = 0; i < nins; ++i) v = insert0(v, ins[i]);
-  return v;
-}
 __device__ __forceinline__ double2 ld_stream(const double2* p) { return __ldcs(p); }
-__device__ __forceinline__ void st_stream(double2* p, double2 v) { __stcs(p, v); }
 
 constexpr int kThreads = 256;
 
@@ -176,190 +159,78 @@ __global__ void __launch_bounds__(kThreads) phase_kernel(PhaseArgs a) {
 }
 
 // ------------------------------------------------------------------------------ a9 tile
-// One CTA processes tiles of T = 2^b amplitudes: tile-local bit i <-> physical position
-// spos[i]; spos[0..l) = 0..l-1, so a warp moves 32 consecutive amplitudes (512 B). The
-// non-tile bits of the live range index the tiles (grid-stride, persistent CTAs).
-//  * load: cp.async (LDGSTS) global -> shared, 16 B per request, every request of the tile in
-//    flight at once with no register staging; requests at index >= L_in use src-size 0, i.e.
-//    the hardware zero-fills them (first-touch expansion, a5).
-//  * op conditions on bits outside the tile are tile-uniform: evaluated once per tile into
-//    `active`. PHASE ops whose condition lies entirely outside the tile multiply the whole
-//    tile by one scalar; they commute with every op of the pass (which act on tile bits only),
-//    so their product is applied once, at the store.
-//  * U1/U2 ops: pairs/quads read-modify-write in shared memory, one barrier per op.
-//  * runs of PHASE ops: each thread keeps its 16 amplitudes in registers across the run; the
-//    condition on the thread's fixed tile bits is tested once per op and thread.
-constexpr int kTileMaxPer = 16;  // amplitudes per thread (T <= 16 * kThreads = 4096)
-
-__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
-  const unsigned sa = static_cast<unsigned>(__cvta_generic_to_shared(smem));
-  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(sa), "l"(gmem), "r"(src_bytes)
-               : "memory");
-}
-__device__ __forceinline__ void cp_async_wait_all() {
-  asm volatile("cp.async.wait_all;\n" ::: "memory");
-}
-
-__global__ void __launch_bounds__(kThreads, 2) tile_kernel(TileArgs a) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  const int b = a.b, l = a.l;
-  const uint32_t T = 1u << b;
-  const int nh = 1 << (b - l);
-  double2* s = reinterpret_cast<double2*>(smem_raw);
-  uint64_t* hiOff = reinterpret_cast<uint64_t*>(s + T);
-  unsigned char* blob = reinterpret_cast<unsigned char*>(hiOff + ((nh + 1) & ~1));
-  const TileOp* ops = reinterpret_cast<const TileOp*>(blob);
-  const double2* pool = reinterpret_cast<const double2*>(blob + a.ops_bytes);
-  unsigned char* active = blob + a.ops_bytes + size_t(a.npool) * 16;
-  double2* scal_s = reinterpret_cast<double2*>(active + ((a.nops + 15) & ~15));
-
-  {  // stage the pass's ops and matrices in shared memory (once per CTA)
-    const int4* src = reinterpret_cast<const int4*>(a.blob);
-    int4* dst = reinterpret_cast<int4*>(blob);
-    const int n16 = (a.ops_bytes + a.npool * 16) / 16;
-    for (int i = threadIdx.x; i < n16; i += kThreads) dst[i] = src[i];
+// The generic (interpreted) fused-pass kernel: the pass program is walked op by op. The
+// persistent tile loop, loads, constants and store are tile_driver (tile_common.cuh); the JIT
+// path (jit.cpp) replaces this body by straight-line code specialised to one pass.
+template <int NR>
+struct InterpBody {
+  int nops;
+  __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c) const {
+    for (int i = 1; i < nops; ++i) {
+      const TileOp& op = c.ops[i];
+      switch (op.kind) {
+        case OP_RUN:
+          op_run<NR>(v, op, c, mp, op.a0, op.a1, op.cls, int(op.tmask), int(op.tmatch));
+          break;
+        case OP_U1R: {
+          if (!op_active(op, c.gbase) || (mp.base & op.tmask) != op.tmatch) break;
+          const double2* u = c.pool + op.moff;
+          switch (op.a0 * 4 + op.cls) {
+#define QGPU_U1R(K, CL) \
+  case K * 4 + CL: op_u1r<NR, K, CL>(v, u, op.rmask, op.rmatch); break;
+            QGPU_U1R(0, 0) QGPU_U1R(0, 1) QGPU_U1R(0, 2) QGPU_U1R(1, 0) QGPU_U1R(1, 1) QGPU_U1R(1, 2)
+            QGPU_U1R(2, 0) QGPU_U1R(2, 1) QGPU_U1R(2, 2) QGPU_U1R(3, 0) QGPU_U1R(3, 1) QGPU_U1R(3, 2)
+#undef QGPU_U1R
+            default: break;
+          }
+          break;
+        }
+        case OP_U1L: {
+          if (!op_active(op, c.gbase)) break;
+          const bool tc = (mp.base & op.tmask) == op.tmatch;
+          const double2* u = c.pool + op.moff;
+          if (op.cls == MAT_X) op_u1l<NR, MAT_X>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch);
+          else if (op.cls == MAT_REAL) op_u1l<NR, MAT_REAL>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch);
+          else op_u1l<NR, MAT_GENERIC>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch);
+          break;
+        }
+        case OP_U2R: {
+          if (!op_active(op, c.gbase) || (mp.base & op.tmask) != op.tmatch) break;
+          const double2* u = c.pool + op.moff;
+          switch (op.a0 * 4 + op.a1) {
+#define QGPU_U2R(A, B) \
+  case A * 4 + B: op_u2r<NR, A, B>(v, u, op.rmask, op.rmatch); break;
+            QGPU_U2R(0, 1) QGPU_U2R(0, 2) QGPU_U2R(0, 3) QGPU_U2R(1, 0) QGPU_U2R(1, 2) QGPU_U2R(1, 3)
+            QGPU_U2R(2, 0) QGPU_U2R(2, 1) QGPU_U2R(2, 3) QGPU_U2R(3, 0) QGPU_U2R(3, 1) QGPU_U2R(3, 2)
+#undef QGPU_U2R
+            default: break;
+          }
+          break;
+        }
+        case OP_REMAP:
+          tile_spill<NR>(v, c, mp);
+          mp = make_mapping<NR>(op, c.nw, c.lane, c.warp);
+          tile_reload<NR>(v, c, mp);
+          break;
+        default: {  // OP_SMEM1 / OP_SMEM2 (tile-uniform condition is uniform: barriers are safe)
+          if (!op_active(op, c.gbase)) break;
+          tile_spill<NR>(v, c, mp);
+          if (op.kind == OP_SMEM2) op_smem2(c, op);
+          else if (op.cls == MAT_X) op_smem1<MAT_X>(c, op);
+          else if (op.cls == MAT_REAL) op_smem1<MAT_REAL>(c, op);
+          else op_smem1<MAT_GENERIC>(c, op);
+          tile_reload<NR>(v, c, mp);
+          break;
+        }
+      }
+    }
   }
-  for (int h = threadIdx.x; h < nh; h += kThreads) {
-    uint64_t off = 0;
-    for (int i = l; i < b; ++i)
-      if (h >> (i - l) & 1) off |= 1ull << a.spos[i];
-    hiOff[h] = off;
-  }
-  __syncthreads();
-  const uint32_t lowmask = (1u << l) - 1;
-  const int per = (T + kThreads - 1) / kThreads;
-  const uint32_t tid = threadIdx.x;
-  const int warp = tid >> 5, lane = tid & 31;
+};
 
-  for (uint64_t tile = blockIdx.x; tile < a.ntiles; tile += gridDim.x) {
-    const uint64_t base = deposit(tile, a.spos, b);
-    const uint64_t gbase = a.rank_base | base;
-    // ---- issue every load of the tile
-#pragma unroll
-    for (int r = 0; r < kTileMaxPer; ++r) {
-      const uint32_t j = tid + r * kThreads;
-      if (r < per && j < T) {
-        const uint64_t idx = base | (j & lowmask) | hiOff[j >> l];
-        const bool live = idx < a.L_in;
-        cp_async16(s + j, a.psi + (live ? idx : 0), live ? 16 : 0);
-      }
-    }
-    asm volatile("cp.async.commit_group;\n" ::: "memory");
-    // ---- tile-uniform op conditions (overlaps the loads)
-    for (int k = tid; k < a.nops; k += kThreads)
-      active[k] = (gbase & ops[k].omask) == ops[k].omatch;
-    __syncthreads();
-    if (warp == 0) {  // product of outside-only phases: lane-strided, then butterfly
-      double2 sc = make_double2(1.0, 0.0);
-      for (int k = lane; k < a.nscalar; k += 32)
-        if (active[k]) sc = cmul(sc, pool[ops[k].moff]);
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) {
-        double2 t;
-        t.x = __shfl_xor_sync(0xffffffffu, sc.x, o);
-        t.y = __shfl_xor_sync(0xffffffffu, sc.y, o);
-        sc = cmul(sc, t);
-      }
-      if (lane == 0) *scal_s = sc;
-    }
-    cp_async_wait_all();
-    __syncthreads();
-    // ---- apply the pass's ops in order
-    int i = a.nscalar;
-    while (i < a.nops) {
-      const int kind = ops[i].kind;
-      if (kind == OP_PHASE) {
-        // a run of commuting phase terms, grouped by their condition on the owned index r:
-        // accumulate each group's product per thread, then multiply the matching amplitudes
-        double2 v[kTileMaxPer];
-#pragma unroll
-        for (int r = 0; r < kTileMaxPer; ++r) {
-          const uint32_t jj = tid + r * kThreads;
-          if (r < per && jj < T) v[r] = s[jj];
-        }
-        double2 acc = make_double2(1.0, 0.0);
-        bool any = false;
-        for (;; ++i) {
-          const TileOp& o = ops[i];
-          if (active[i] && (tid & o.lmask & (kThreads - 1)) == (o.lmatch & (kThreads - 1))) {
-            acc = cmul(acc, pool[o.moff]);
-            any = true;
-          }
-          if (o.t0) {  // end of group: apply to the owned amplitudes whose r matches
-            if (any) {
-              const uint32_t mh = o.lmask >> 8, th = o.lmatch >> 8;
-#pragma unroll
-              for (int r = 0; r < kTileMaxPer; ++r)
-                if (r < per && (uint32_t(r) & mh) == th) v[r] = cmul(v[r], acc);
-            }
-            acc = make_double2(1.0, 0.0);
-            any = false;
-          }
-          if (o.t1) break;
-        }
-        ++i;
-#pragma unroll
-        for (int r = 0; r < kTileMaxPer; ++r) {
-          const uint32_t jj = tid + r * kThreads;
-          if (r < per && jj < T) s[jj] = v[r];
-        }
-        __syncthreads();
-      } else if (kind == OP_U1) {
-        if (active[i]) {
-          const int t = ops[i].t0;
-          const uint32_t lm = ops[i].lmask;
-          const double2* u = pool + ops[i].moff;
-          const double2 u00 = u[0], u01 = u[1], u10 = u[2], u11 = u[3];
-          for (uint32_t p = tid; p < T / 2; p += kThreads) {
-            const uint32_t i0 = uint32_t(insert0(p, t));
-            if ((i0 & lm) != lm) continue;
-            const uint32_t i1 = i0 | (1u << t);
-            const double2 x0 = s[i0], x1 = s[i1];
-            s[i0] = cfma(u00, x0, cmul(u01, x1));
-            s[i1] = cfma(u10, x0, cmul(u11, x1));
-          }
-          __syncthreads();
-        }
-        ++i;
-      } else {  // OP_U2
-        if (active[i]) {
-          const int t0 = ops[i].t0, t1 = ops[i].t1;
-          const int lo = min(t0, t1), hi = max(t0, t1);
-          const uint32_t lm = ops[i].lmask;
-          const double2* u = pool + ops[i].moff;
-          const uint32_t o1 = 1u << t0, o2 = 1u << t1;
-          for (uint32_t p = tid; p < T / 4; p += kThreads) {
-            const uint32_t i0 = uint32_t(insert0(insert0(p, lo), hi));
-            if ((i0 & lm) != lm) continue;
-            const double2 x0 = s[i0], x1 = s[i0 | o1], x2 = s[i0 | o2], x3 = s[i0 | o1 | o2];
-#pragma unroll
-            for (int row = 0; row < 4; ++row) {
-              double2 y = cmul(u[row * 4], x0);
-              y = cfma(u[row * 4 + 1], x1, y);
-              y = cfma(u[row * 4 + 2], x2, y);
-              y = cfma(u[row * 4 + 3], x3, y);
-              const uint32_t o = (row & 1 ? o1 : 0u) | (row & 2 ? o2 : 0u);
-              s[i0 | o] = y;
-            }
-          }
-          __syncthreads();
-        }
-        ++i;
-      }
-    }
-    // ---- store every amplitude of the tile (including the expanded zero region)
-    const double2 sc = *scal_s;
-    const bool has_sc = !(sc.x == 1.0 && sc.y == 0.0);
-#pragma unroll
-    for (int r = 0; r < kTileMaxPer; ++r) {
-      const uint32_t j = tid + r * kThreads;
-      if (r < per && j < T) {
-        const double2 x = has_sc ? cmul(s[j], sc) : s[j];
-        st_stream(a.psi + (base | (j & lowmask) | hiOff[j >> l]), x);
-      }
-    }
-    __syncthreads();
-  }
+template <int NR>
+__global__ void __launch_bounds__(256, 1) tile_kernel(TileArgs a) {
+  InterpBody<NR> body{a.nops};
+  tile_driver<NR>(a, body);
 }
 
 // ------------------------------------------------------------------------------ a11
@@ -436,10 +307,12 @@ unsigned grid_for(uint64_t work_items, int per_block, int blocks_per_sm) {
 }
 }  // namespace
 
-size_t tile_smem_bytes(int b, int l, int nops, int ops_bytes, int npool) {
-  const size_t nh = size_t(1) << (b - l);
-  return (size_t(1) << b) * 16 + ((nh + 1) & ~size_t(1)) * 8 + size_t(ops_bytes) +
-         size_t(npool) * 16 + size_t((nops + 15) & ~15) + 16;
+int device_num_sms() { return num_sms(); }
+
+size_t tile_smem_bytes(const TileArgs& a) {
+  const size_t nh = size_t(1) << (a.b - a.l);
+  return 2 * (size_t(1) << a.b) * 16 + ((nh + 1) & ~size_t(1)) * 8 + size_t(a.blob_bytes) +
+         size_t(a.npat + 1) * 16;
 }
 
 cudaError_t launch_pair(cudaStream_t st, const PairArgs& a, bool shfl) {
@@ -472,23 +345,35 @@ cudaError_t launch_phase(cudaStream_t st, const PhaseArgs& a) {
   return cudaGetLastError();
 }
 
-cudaError_t launch_tile(cudaStream_t st, const TileArgs& a) {
-  if (a.ntiles == 0) return cudaSuccess;
-  const size_t smem = tile_smem_bytes(a.b, a.l, a.nops, a.ops_bytes, a.npool);
+template <int NR>
+cudaError_t launch_tile_nr(cudaStream_t st, const TileArgs& a, size_t smem) {
   static bool configured = false;
   if (!configured) {
-    cudaError_t e = cudaFuncSetAttribute(tile_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(tile_kernel<NR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          227 * 1024);
     if (e != cudaSuccess) return e;
     configured = true;
   }
-  if (smem > 227 * 1024) return cudaErrorInvalidValue;
+  const int threads = 32 << a.nw;
   int bps = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, tile_kernel, kThreads, smem);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, tile_kernel<NR>, threads, smem);
   if (bps <= 0) bps = 1;
   const unsigned g = unsigned(std::min<uint64_t>(a.ntiles, uint64_t(num_sms()) * bps));
-  tile_kernel<<<g, kThreads, smem, st>>>(a);
+  tile_kernel<NR><<<g, threads, smem, st>>>(a);
   return cudaGetLastError();
+}
+
+cudaError_t launch_tile(cudaStream_t st, const TileArgs& a) {
+  if (a.ntiles == 0) return cudaSuccess;
+  const size_t smem = tile_smem_bytes(a);
+  if (smem > 227 * 1024) return cudaErrorInvalidValue;
+  switch (a.nr) {
+    case 0: return launch_tile_nr<0>(st, a, smem);
+    case 1: return launch_tile_nr<1>(st, a, smem);
+    case 2: return launch_tile_nr<2>(st, a, smem);
+    case 3: return launch_tile_nr<3>(st, a, smem);
+    default: return launch_tile_nr<4>(st, a, smem);
+  }
 }
 
 cudaError_t launch_gather(cudaStream_t st, const GatherArgs& a) {

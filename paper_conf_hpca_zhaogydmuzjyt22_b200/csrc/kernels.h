@@ -41,20 +41,6 @@ struct PhaseArgs {
   uint64_t count;          // amplitudes enumerated
 };
 
-struct TileArgs {
-  double2* psi;
-  const void* blob;        // [TileOp x nops, padded to 16 B | double2 x npool]
-  int nops;
-  int nscalar;             // leading OP_PHASE_SCALAR ops (tile-uniform phases)
-  int ops_bytes;
-  int npool;
-  int b, l;
-  int spos[kMaxTileBits];
-  uint64_t ntiles;
-  uint64_t L_in;
-  uint64_t rank_base;      // rank << m (global bits for tile-uniform conditions)
-};
-
 struct GatherArgs {
   const double2* psi;
   double2* out;
@@ -75,7 +61,8 @@ struct ProbArgs {
   double* partial;
 };
 
-size_t tile_smem_bytes(int b, int l, int nops, int ops_bytes, int npool);
+size_t tile_smem_bytes(const TileArgs& a);
+int device_num_sms();
 size_t probs_scratch_doubles(int m);
 cudaError_t launch_pair(cudaStream_t st, const PairArgs& a, bool shfl);
 cudaError_t launch_quad(cudaStream_t st, const QuadArgs& a);

@@ -15,6 +15,7 @@
 #include <vector>
 
 #include "../../include/qgpu.h"
+#include "tile_common.cuh"
 
 namespace qgpu {
 
@@ -77,27 +78,22 @@ struct QubitMap {
 };
 
 // --------------------------------------------------------------------------- device ops
-enum OpKind : int { OP_U1 = 0, OP_U2 = 1, OP_PHASE = 2, OP_PHASE_SCALAR = 3 };
-
-// One operation of a fused tile pass (copied to shared memory by every CTA). Target bits
-// t0/t1 and the per-amplitude condition (lmask/lmatch) are TILE-LOCAL bits; omask/omatch are
-// bits of (rank << m | local index) outside the tile: a tile-uniform condition. The matrix
-// (U1: 4, U2: 16, PHASE: 1 complex) is pool[moff...].
-// Diagonal terms commute with each other, so a maximal run of consecutive PHASE terms is
-// re-sorted on the host by their condition on the "register" tile bits (bits >= 8, i.e. the
-// amplitude index r a thread owns); t0 = 1 marks the last term of such a group and t1 = 1
-// the last term of the run. Terms whose condition lies entirely outside the tile
-// (OP_PHASE_SCALAR) commute with every op of the pass and are listed first.
-struct TileOp {
-  int kind;
-  int t0, t1;
-  uint32_t moff;
-  uint32_t lmask, lmatch;
-  uint64_t omask, omatch;
+// Device-side program structures (TileOp, RunEntry, PhaseTerm, Pattern) live in
+// tile_common.cuh, shared with the kernels and the NVRTC-compiled pass kernels.
+struct TileProgram {
+  std::vector<TileOp> ops;
+  std::vector<RunEntry> entries;
+  std::vector<Pattern> patterns;
+  std::vector<PhaseTerm> terms;
+  std::vector<PhaseTerm> scalar;   // tile-uniform diagonal terms (commute with the whole pass)
+  std::vector<cplx> pool;          // U matrices
+  int nr = 0, nw = 0;
+  // byte offsets of each region inside the blob (all multiples of 16)
+  size_t off_entries = 0, off_patterns = 0, off_terms = 0, off_scalar = 0, off_pool = 0, bytes = 0;
+  void layout();
+  void pack(unsigned char* dst) const;
 };
-static_assert(sizeof(TileOp) == 40, "TileOp layout is shared with the kernel");
 
-constexpr int kMaxTileBits = 13;
 
 // A gate in physical positions at its execution time.
 struct PhysGate {
@@ -122,13 +118,8 @@ struct Pass {
   int b = 0, l = 0;
   int spos[kMaxTileBits];
   std::vector<PhysGate> gates;  // gates of the pass (tile) or the single gate (pair/quad/diag)
-  std::vector<TileOp> ops;      // built at pass close (tile)
-  std::vector<cplx> pool;       // matrices of the ops
+  TileProgram prog;             // built at pass close (tile)
   int n_est = 0;                // op-count estimate while the pass is open
-  int nscalar = 0;              // leading OP_PHASE_SCALAR ops
-  // bytes of the device blob [ops (padded to 16 B) | pool]
-  size_t ops_bytes() const { return (ops.size() * sizeof(TileOp) + 15) / 16 * 16; }
-  size_t blob_bytes() const { return ops_bytes() + pool.size() * sizeof(cplx); }
   // swap pass (sharded)
   int nswap = 0;
   int swap_global[8], swap_local[8];

@@ -13,6 +13,8 @@
 //     trace is unchanged); each run is one fused HBM pass over tiles of 2^b amplitudes.
 #include <algorithm>
 #include <bit>
+#include <cstdio>
+#include <cstdlib>
 #include <cstring>
 #include <limits>
 
@@ -180,23 +182,77 @@ int local_bit(int pos, const Pass& p) {
 
 }  // namespace
 
+void TileProgram::layout() {
+  size_t o = ops.size() * sizeof(TileOp);
+  off_entries = o;
+  o += entries.size() * sizeof(RunEntry);
+  off_patterns = o;
+  o += patterns.size() * sizeof(Pattern);
+  off_terms = o;
+  o += terms.size() * sizeof(PhaseTerm);
+  off_scalar = o;
+  o += scalar.size() * sizeof(PhaseTerm);
+  off_pool = o;
+  o += pool.size() * sizeof(cplx);
+  bytes = o;
+}
+
+void TileProgram::pack(unsigned char* dst) const {
+  std::memcpy(dst, ops.data(), ops.size() * sizeof(TileOp));
+  std::memcpy(dst + off_entries, entries.data(), entries.size() * sizeof(RunEntry));
+  std::memcpy(dst + off_patterns, patterns.data(), patterns.size() * sizeof(Pattern));
+  std::memcpy(dst + off_terms, terms.data(), terms.size() * sizeof(PhaseTerm));
+  std::memcpy(dst + off_scalar, scalar.data(), scalar.size() * sizeof(PhaseTerm));
+  std::memcpy(dst + off_pool, pool.data(), pool.size() * sizeof(cplx));
+}
+
+namespace {
+
+struct RawOp {
+  int kind;                 // 0: U1, 1: U2, 2: phase term
+  int t[2];                 // tile-local targets
+  uint32_t lmask, lmatch;   // tile-local condition (controls / diagonal pattern)
+  uint64_t omask, omatch;   // condition outside the tile (tile-uniform)
+  cplx U[16];
+  cplx ph;
+};
+
+int mat_class(const cplx* U, int nt) {
+  const int d = 1 << nt;
+  bool real = true;
+  for (int i = 0; i < d * d; ++i)
+    if (U[i].im != 0.0) real = false;
+  if (nt == 1 && real && U[0].re == 0.0 && U[3].re == 0.0 && U[1].re == 1.0 && U[2].re == 1.0)
+    return MAT_X;
+  return real ? MAT_REAL : MAT_GENERIC;
+}
+
+}  // namespace
+
+// Build the device program of a tile pass (a9). Steps:
+//  1. lower the pass's gates to tile-local ops (U1/U2 with conditions, one phase term per
+//     diagonal entry != 1);
+//  2. sink every phase term past the following U ops whose targets it does not touch
+//     (a diagonal operator that does not depend on the target bits commutes with a
+//     controlled U), so diagonal terms gather into few, long runs; terms whose condition lies
+//     entirely outside the tile commute with the whole pass and become the tile scalar;
+//  3. assign register bits per segment (earliest next use), encode conditions relative to
+//     the mapping, and group each run's terms into distinct patterns.
 void build_tile_ops(Pass& p, int /*m*/) {
-  std::vector<TileOp> raw;
-  std::vector<cplx> pool;
+  TileProgram& P = p.prog;
+  P = TileProgram();
+  std::vector<RawOp> raw;
   for (const PhysGate& g : p.gates) {
     if (!g.diag) {
-      TileOp o{};
-      o.kind = g.nt == 1 ? OP_U1 : OP_U2;
-      o.t0 = local_bit(g.p[0], p);
-      o.t1 = g.nt == 2 ? local_bit(g.p[1], p) : 0;
+      RawOp o{};
+      o.kind = g.nt == 1 ? 0 : 1;
+      o.t[0] = local_bit(g.p[0], p);
+      o.t[1] = g.nt == 2 ? local_bit(g.p[1], p) : 0;
       o.lmask = o.lmatch = to_local(g.pc, p);
       o.omask = o.omatch = outside(g.pc, p);
-      o.moff = uint32_t(pool.size());
-      const int dim = 1 << g.nt;
-      for (int i = 0; i < dim * dim; ++i) pool.push_back(g.U[i]);
+      std::memcpy(o.U, g.U, sizeof(g.U));
       raw.push_back(o);
     } else {
-      // diagonal: one phase term per diagonal entry that is not exactly 1
       const int dim = 1 << g.nt;
       uint64_t tmask = 1ull << g.p[0];
       if (g.nt == 2) tmask |= 1ull << g.p[1];
@@ -207,38 +263,202 @@ void build_tile_ops(Pass& p, int /*m*/) {
         for (int j = 0; j < g.nt; ++j)
           if (v >> j & 1) match |= 1ull << g.p[j];
         const uint64_t mask = g.pc | tmask;
-        TileOp o{};
+        RawOp o{};
+        o.kind = 2;
         o.lmask = to_local(mask, p);
         o.lmatch = to_local(match, p);
         o.omask = outside(mask, p);
         o.omatch = outside(match, p);
-        o.kind = o.lmask == 0 ? OP_PHASE_SCALAR : OP_PHASE;
-        o.moff = uint32_t(pool.size());
-        pool.push_back(d);
-        raw.push_back(o);
+        o.ph = d;
+        if (o.lmask == 0) P.scalar.push_back(PhaseTerm{o.omask, o.omatch, d.re, d.im});
+        else raw.push_back(o);
       }
     }
   }
-  p.ops.clear();
-  p.pool = std::move(pool);
-  for (const TileOp& o : raw)
-    if (o.kind == OP_PHASE_SCALAR) p.ops.push_back(o);
-  p.nscalar = int(p.ops.size());
-  for (size_t i = 0; i < raw.size();) {
-    if (raw[i].kind == OP_PHASE_SCALAR) { ++i; continue; }
-    if (raw[i].kind != OP_PHASE) { p.ops.push_back(raw[i]); ++i; continue; }
-    std::vector<TileOp> run;
-    size_t j = i;
-    for (; j < raw.size() && (raw[j].kind == OP_PHASE || raw[j].kind == OP_PHASE_SCALAR); ++j)
-      if (raw[j].kind == OP_PHASE) run.push_back(raw[j]);
-    auto key = [](const TileOp& o) { return (uint64_t(o.lmask >> 8) << 32) | (o.lmatch >> 8); };
-    std::stable_sort(run.begin(), run.end(), [&](const TileOp& x, const TileOp& y) { return key(x) < key(y); });
-    for (size_t k = 0; k < run.size(); ++k) {
-      run[k].t0 = (k + 1 == run.size() || key(run[k + 1]) != key(run[k])) ? 1 : 0;
-      run[k].t1 = (k + 1 == run.size()) ? 1 : 0;
-      p.ops.push_back(run[k]);
+  // 2. sink phase terms
+  std::vector<RawOp> seq, pending;
+  for (const RawOp& o : raw) {
+    if (o.kind == 2) {
+      pending.push_back(o);
+      continue;
     }
-    i = j;
+    uint32_t tb = 1u << o.t[0];
+    if (o.kind == 1) tb |= 1u << o.t[1];
+    std::vector<RawOp> keep;
+    for (const RawOp& ph : pending) (ph.lmask & tb ? seq : keep).push_back(ph);
+    pending.swap(keep);
+    seq.push_back(o);
+  }
+  for (const RawOp& ph : pending) seq.push_back(ph);
+
+  // 3. mapping
+  const int b = p.b;
+  const int lanes = std::min(5, b);
+  const int nonlane = b - lanes;
+  const int nr = std::min(4, nonlane), nw = nonlane - nr;
+  P.nr = nr;
+  P.nw = nw;
+  const size_t INF = ~size_t(0);
+  auto next_use = [&](int bit, size_t from) {
+    for (size_t i = from; i < seq.size(); ++i) {
+      const RawOp& o = seq[i];
+      if (o.kind == 2) continue;
+      if (o.t[0] == bit || (o.kind == 1 && o.t[1] == bit)) return i;
+    }
+    return INF;
+  };
+  int R[4] = {0, 0, 0, 0}, W[3] = {0, 0, 0};
+  auto choose = [&](uint32_t need, size_t from) {
+    std::vector<int> cand;
+    for (int t = lanes; t < b; ++t) cand.push_back(t);
+    std::stable_sort(cand.begin(), cand.end(), [&](int x, int y) {
+      const bool nx = need >> x & 1, ny = need >> y & 1;
+      if (nx != ny) return nx;
+      const size_t ux = next_use(x, from), uy = next_use(y, from);
+      if (ux != uy) return ux < uy;
+      return x > y;
+    });
+    for (int k = 0; k < nr; ++k) R[k] = cand[k];
+    std::vector<int> w(cand.begin() + nr, cand.end());
+    std::sort(w.begin(), w.end());
+    for (int k = 0; k < nw; ++k) W[k] = w[k];
+    TileOp op{};
+    op.kind = OP_REMAP;
+    for (int k = 0; k < nr; ++k) op.a0 |= R[k] << (4 * k);
+    for (int k = 0; k < nw; ++k) op.a1 |= W[k] << (4 * k);
+    P.ops.push_back(op);
+  };
+  auto ridx = [&](int bit) {
+    for (int k = 0; k < nr; ++k)
+      if (R[k] == bit) return k;
+    return -1;
+  };
+  auto split = [&](uint32_t lmask, uint32_t lmatch, uint32_t* tm, uint32_t* tt, uint32_t* rm, uint32_t* rt) {
+    *rm = *rt = 0;
+    uint32_t rbits = 0;
+    for (int k = 0; k < nr; ++k) {
+      rbits |= 1u << R[k];
+      if (lmask >> R[k] & 1) {
+        *rm |= 1u << k;
+        if (lmatch >> R[k] & 1) *rt |= 1u << k;
+      }
+    }
+    *tm = lmask & ~rbits;
+    *tt = lmatch & *tm;
+  };
+  choose(0, 0);
+  for (size_t i = 0; i < seq.size();) {
+    const RawOp& o = seq[i];
+    if (o.kind == 2) {  // a run of phase terms -> distinct patterns
+      size_t j = i;
+      std::vector<std::pair<uint64_t, std::vector<const RawOp*>>> pats;
+      for (; j < seq.size() && seq[j].kind == 2; ++j) {
+        const uint64_t key = (uint64_t(seq[j].lmask) << 32) | seq[j].lmatch;
+        auto it = std::find_if(pats.begin(), pats.end(), [&](auto& e) { return e.first == key; });
+        if (it == pats.end()) pats.push_back({key, {&seq[j]}});
+        else it->second.push_back(&seq[j]);
+      }
+      std::vector<RunEntry> ents;
+      for (auto& pe : pats) {
+        Pattern pt{uint32_t(P.terms.size()), uint32_t(pe.second.size()), 0, 0};
+        for (const RawOp* t : pe.second) P.terms.push_back(PhaseTerm{t->omask, t->omatch, t->ph.re, t->ph.im});
+        RunEntry e{};
+        uint32_t tm, tt, rm, rt;
+        split(uint32_t(pe.first >> 32), uint32_t(pe.first), &tm, &tt, &rm, &rt);
+        e.tmask = tm;
+        e.tmatch = tt;
+        e.rmask = uint16_t(rm);
+        e.rmatch = uint16_t(rt);
+        e.pat = uint16_t(P.patterns.size());
+        P.patterns.push_back(pt);
+        ents.push_back(e);
+      }
+      // slots: 0 = thread constant (no condition on r), 1+k = exactly "r bit k set",
+      // 5 = general condition on r (grouped by (rmask, rmatch), applied with predication)
+      auto slot = [](const RunEntry& e) {
+        if (e.rmask == 0) return 0;
+        for (int k = 0; k < 4; ++k)
+          if (e.rmask == (1u << k) && e.rmatch == (1u << k)) return 1 + k;
+        return 5;
+      };
+      std::stable_sort(ents.begin(), ents.end(), [&](const RunEntry& x, const RunEntry& y) {
+        const int sx = slot(x), sy = slot(y);
+        if (sx != sy) return sx < sy;
+        return (uint32_t(x.rmask) << 16 | x.rmatch) < (uint32_t(y.rmask) << 16 | y.rmatch);
+      });
+      int nslot[6] = {0, 0, 0, 0, 0, 0};
+      for (auto& e : ents) nslot[slot(e)]++;
+      for (size_t k = 0; k < ents.size(); ++k)
+        ents[k].gend = (k + 1 == ents.size() || ents[k + 1].rmask != ents[k].rmask ||
+                        ents[k + 1].rmatch != ents[k].rmatch) ? 1 : 0;
+      TileOp op{};
+      op.kind = OP_RUN;
+      op.moff = uint32_t(P.entries.size());
+      op.cnt = uint32_t(ents.size());
+      op.a0 = nslot[0];
+      op.a1 = nslot[1];
+      op.cls = nslot[2];
+      op.tmask = uint32_t(nslot[3]);
+      op.tmatch = uint32_t(nslot[4]);
+      for (auto& e : ents) P.entries.push_back(e);
+      P.ops.push_back(op);
+      i = j;
+      continue;
+    }
+    TileOp op{};
+    op.cls = mat_class(o.U, o.kind + 1);
+    op.omask = o.omask;
+    op.omatch = o.omatch;
+    op.moff = uint32_t(P.pool.size());
+    const int dim = o.kind == 0 ? 2 : 4;
+    for (int e = 0; e < dim * dim; ++e) P.pool.push_back(o.U[e]);
+    if (o.kind == 0) {
+      const int t = o.t[0];
+      if (t < lanes) {
+        op.kind = OP_U1L;
+        op.a0 = t;
+      } else if (nr > 0) {
+        if (ridx(t) < 0) choose(1u << t, i);
+        op.kind = OP_U1R;
+        op.a0 = ridx(t);
+      } else {
+        op.kind = OP_SMEM1;
+        op.a0 = t;
+      }
+    } else {
+      const int t0 = o.t[0], t1 = o.t[1];
+      if (t0 >= lanes && t1 >= lanes && nr >= 2) {
+        if (ridx(t0) < 0 || ridx(t1) < 0) choose((1u << t0) | (1u << t1), i);
+        op.kind = OP_U2R;
+        op.a0 = ridx(t0);
+        op.a1 = ridx(t1);
+      } else {
+        op.kind = OP_SMEM2;
+        op.a0 = t0;
+        op.a1 = t1;
+      }
+    }
+    if (op.kind == OP_SMEM1 || op.kind == OP_SMEM2) {
+      op.tmask = o.lmask;
+      op.tmatch = o.lmatch;
+    } else {
+      split(o.lmask, o.lmatch, &op.tmask, &op.tmatch, &op.rmask, &op.rmatch);
+    }
+    P.ops.push_back(op);
+    ++i;
+  }
+  P.layout();
+  if (std::getenv("QGPU_DEBUG_PLAN")) {
+    int cnt[7] = {0, 0, 0, 0, 0, 0, 0}, groups = 0;
+    for (const TileOp& o : P.ops) cnt[o.kind]++;
+    for (const RunEntry& e : P.entries) groups += e.gend;
+    std::fprintf(stderr,
+                 "tile pass k %d->%d b=%d nr=%d nw=%d gates=%zu ops=%zu remap=%d u1r=%d u1l=%d u2r=%d smem=%d "
+                 "runs=%d entries=%zu groups=%d patterns=%zu terms=%zu scalar=%zu S=",
+                 p.k_in, p.k_out, p.b, nr, nw, p.gates.size(), P.ops.size(), cnt[0], cnt[1], cnt[2], cnt[3],
+                 cnt[4] + cnt[5], cnt[6], P.entries.size(), groups, P.patterns.size(), P.terms.size(),
+                 P.scalar.size());
+    for (int i = 0; i < p.b; ++i) std::fprintf(stderr, "%d%s", p.spos[i], i + 1 < p.b ? "," : "\n");
   }
 }
 

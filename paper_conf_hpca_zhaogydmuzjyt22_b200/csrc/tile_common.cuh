@@ -1,0 +1,437 @@
+// Device code of the fused tile pass (a9), self-contained so that it is compiled both into
+// libqgpu.so (the generic, interpreted tile kernel in kernels.cu) and, as source text, by NVRTC
+// into per-pass specialised kernels (jit.cpp). No host headers.
+//
+// Thread/amplitude mapping: a tile holds T = 2^b amplitudes (tile-local index j); tile bits
+// 0..4 are the lane bits (physical positions 0..4, so a warp moves 512 contiguous bytes), the
+// other b-5 tile bits are split into NR <= 4 REGISTER bits (each thread owns the 2^NR
+// amplitudes that differ in them) and nw = b-5-NR WARP bits. OP_REMAP re-distributes the tile
+// through shared memory so that other tile bits become register bits; gates on register bits
+// run in registers, gates on lane bits use warp shuffles, everything else is a shared-memory op.
+#pragma once
+
+#ifdef __CUDACC_RTC__
+typedef unsigned int uint32_t;
+typedef unsigned short uint16_t;
+typedef unsigned long long uint64_t;
+#else
+#include <cstdint>
+#endif
+
+namespace qgpu {
+
+constexpr int kMaxTileBits = 13;
+constexpr int kRegAmps = 16;
+
+enum OpKind : int {
+  OP_REMAP = 0,  // a0: packed register bits (4 bits each), a1: packed warp bits
+  OP_U1R = 1,    // 1-qubit U on register bit index a0
+  OP_U1L = 2,    // 1-qubit U on lane bit a0
+  OP_U2R = 3,    // 2-qubit U on register bit indices a0 (U bit 0), a1 (U bit 1)
+  OP_SMEM1 = 4,  // 1-qubit U on tile bit a0 via shared memory (tmask/tmatch: full condition)
+  OP_SMEM2 = 5,  // 2-qubit U on tile bits a0, a1 via shared memory
+  OP_RUN = 6     // run of diagonal phase patterns: entries [moff, moff + cnt)
+};
+enum MatClass : int { MAT_GENERIC = 0, MAT_REAL = 1, MAT_X = 2 };
+
+struct TileOp {
+  int kind;
+  int a0, a1;
+  int cls;                 // matrix class (U ops); RUN: entries of slot 2
+  uint32_t tmask, tmatch;  // condition on the thread's fixed tile bits (lane + warp bits)
+  uint32_t rmask, rmatch;  // condition on the owned register index r
+  uint32_t moff, cnt;      // matrix offset in the pool (complex units) / run entries
+  uint64_t omask, omatch;  // tile-uniform condition on (rank << m | index) bits outside the tile
+  uint64_t pad;
+};
+static_assert(sizeof(TileOp) == 64, "TileOp layout");
+
+// One distinct diagonal pattern of a run: the product of its active terms is computed once per
+// tile, then applied to the amplitudes matching (tmask,tmatch) x (rmask,rmatch).
+struct RunEntry {
+  uint32_t tmask, tmatch;
+  uint16_t rmask, rmatch, pat, gend;  // gend: last entry of a group with equal (rmask, rmatch)
+};
+static_assert(sizeof(RunEntry) == 16, "RunEntry layout");
+struct PhaseTerm {
+  uint64_t omask, omatch;  // tile-uniform condition
+  double re, im;           // phase factor
+};
+struct Pattern {
+  uint32_t first, count, pad0, pad1;  // range of PhaseTerms
+};
+
+#if defined(__CUDACC__)
+
+struct TileArgs {
+  double2* psi;
+  const void* blob;        // TileProgram blob (ops | entries | patterns | terms | scalar | pool)
+  int blob_bytes;
+  int nops, npat, nscalar;
+  int off_entries, off_patterns, off_terms, off_scalar, off_pool;
+  int nr, nw;              // register / warp bits of the thread mapping
+  int b, l;
+  int spos[kMaxTileBits];
+  uint64_t ntiles;
+  uint64_t L_in;
+  uint64_t rank_base;      // rank << m (global bits for tile-uniform conditions)
+};
+
+__device__ __forceinline__ double2 cmul(double2 a, double2 b) {
+  return make_double2(fma(a.x, b.x, -a.y * b.y), fma(a.x, b.y, a.y * b.x));
+}
+// a*b + c
+__device__ __forceinline__ double2 cfma(double2 a, double2 b, double2 c) {
+  return make_double2(fma(a.x, b.x, fma(-a.y, b.y, c.x)), fma(a.x, b.y, fma(a.y, b.x, c.y)));
+}
+__device__ __forceinline__ uint64_t insert0(uint64_t v, int b) {
+  const uint64_t lo = v & ((1ull << b) - 1);
+  return ((v >> b) << (b + 1)) | lo;
+}
+// insert zero bits at the (ascending) positions ins[0..nins)
+__device__ __forceinline__ uint64_t deposit(uint64_t v, const int* ins, int nins) {
+  for (int i = 0; i < nins; ++i) v = insert0(v, ins[i]);
+  return v;
+}
+__device__ __forceinline__ void st_stream(double2* p, double2 v) { __stcs(p, v); }
+
+__device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
+  const unsigned sa = static_cast<unsigned>(__cvta_generic_to_shared(smem));
+  asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(sa), "l"(gmem), "r"(src_bytes)
+               : "memory");
+}
+__device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
+
+// (x0, x1) <- U (x0, x1), U = [[u0 u1] [u2 u3]], with the matrix-class shortcut
+template <int CLS>
+__device__ __forceinline__ void apply2(double2& x0, double2& x1, const double2 (&u)[4]) {
+  if (CLS == MAT_X) {
+    const double2 t = x0;
+    x0 = x1;
+    x1 = t;
+  } else if (CLS == MAT_REAL) {
+    const double a = u[0].x, bq = u[1].x, c = u[2].x, d = u[3].x;
+    const double2 y0 = make_double2(fma(a, x0.x, bq * x1.x), fma(a, x0.y, bq * x1.y));
+    const double2 y1 = make_double2(fma(c, x0.x, d * x1.x), fma(c, x0.y, d * x1.y));
+    x0 = y0;
+    x1 = y1;
+  } else {
+    const double2 y0 = cfma(u[0], x0, cmul(u[1], x1));
+    const double2 y1 = cfma(u[2], x0, cmul(u[3], x1));
+    x0 = y0;
+    x1 = y1;
+  }
+}
+
+struct Mapping {
+  uint32_t base;   // tile index of the thread's r = 0 amplitude (lane + warp bits)
+  uint32_t rb[4];  // tile-index bit of each register bit
+  __device__ __forceinline__ uint32_t j(int r) const {
+    return base | ((r & 1) ? rb[0] : 0u) | ((r & 2) ? rb[1] : 0u) | ((r & 4) ? rb[2] : 0u) |
+           ((r & 8) ? rb[3] : 0u);
+  }
+};
+
+template <int NR>
+__device__ __forceinline__ Mapping make_mapping(const TileOp& op, int nw, int lane, int warp) {
+  Mapping mp;
+  mp.base = uint32_t(lane);
+  for (int k = 0; k < nw; ++k)
+    if (warp >> k & 1) mp.base |= 1u << ((op.a1 >> (4 * k)) & 15);
+#pragma unroll
+  for (int k = 0; k < 4; ++k) mp.rb[k] = (k < NR) ? (1u << ((op.a0 >> (4 * k)) & 15)) : 0u;
+  return mp;
+}
+
+// Per-tile context handed to the program body.
+struct TileCtx {
+  double2* s;            // current tile buffer (natural order)
+  const TileOp* ops;
+  const RunEntry* ents;
+  const double2* pool;
+  const double2* C;      // per-tile pattern constants
+  uint64_t gbase;        // rank << m | tile base index
+  uint32_t T;
+  int nthr, tid, lane, warp, nw;
+  bool own;              // this lane owns amplitudes (b >= 5 always)
+};
+
+template <int NR>
+__device__ __forceinline__ void tile_spill(const double2 (&v)[kRegAmps], const TileCtx& c, const Mapping& mp) {
+  __syncthreads();
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r)
+    if (c.own) c.s[mp.j(r)] = v[r];
+  __syncthreads();
+}
+template <int NR>
+__device__ __forceinline__ void tile_reload(double2 (&v)[kRegAmps], const TileCtx& c, const Mapping& mp) {
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r) v[r] = c.own ? c.s[mp.j(r)] : make_double2(0, 0);
+}
+
+__device__ __forceinline__ bool op_active(const TileOp& op, uint64_t gbase) {
+  return (gbase & op.omask) == op.omatch;
+}
+
+// 1-qubit U on register bit K for every owned pair whose r satisfies (r & rm) == rt
+template <int NR, int K, int CLS>
+__device__ __forceinline__ void op_u1r(double2 (&v)[kRegAmps], const double2* up, uint32_t rm, uint32_t rt) {
+  const double2 u[4] = {up[0], up[1], up[2], up[3]};
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r) {
+    if (r >> K & 1) continue;
+    if ((uint32_t(r) & rm) == rt) apply2<CLS>(v[r], v[r | (1 << K)], u);
+  }
+}
+
+// 1-qubit U on lane bit t: partner amplitude by warp shuffle
+template <int NR, int CLS>
+__device__ __forceinline__ void op_u1l(double2 (&v)[kRegAmps], const double2* up, int t, int lane, bool tc,
+                                       uint32_t rm, uint32_t rt) {
+  const bool hi = (lane >> t) & 1;
+  const double2 c0 = hi ? up[2] : up[0], c1 = hi ? up[3] : up[1];
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r) {
+    if ((uint32_t(r) & rm) != rt) continue;
+    double2 pv;
+    pv.x = __shfl_xor_sync(0xffffffffu, v[r].x, 1 << t);
+    pv.y = __shfl_xor_sync(0xffffffffu, v[r].y, 1 << t);
+    const double2 a0 = hi ? pv : v[r], a1 = hi ? v[r] : pv;
+    double2 y;
+    if (CLS == MAT_X) y = pv;
+    else if (CLS == MAT_REAL) y = make_double2(fma(c0.x, a0.x, c1.x * a1.x), fma(c0.x, a0.y, c1.x * a1.y));
+    else y = cfma(c0, a0, cmul(c1, a1));
+    if (tc) v[r] = y;
+  }
+}
+
+// 2-qubit U on register bits K0 (U index bit 0) and K1 (bit 1)
+template <int NR, int K0, int K1>
+__device__ __forceinline__ void op_u2r(double2 (&v)[kRegAmps], const double2* u, uint32_t rm, uint32_t rt) {
+  constexpr int m0 = 1 << K0, m1 = 1 << K1;
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r) {
+    if (r & (m0 | m1)) continue;
+    if ((uint32_t(r) & rm) != rt) continue;
+    const double2 x0 = v[r], x1 = v[r | m0], x2 = v[r | m1], x3 = v[r | m0 | m1];
+#pragma unroll
+    for (int row = 0; row < 4; ++row) {
+      double2 y = cmul(u[row * 4], x0);
+      y = cfma(u[row * 4 + 1], x1, y);
+      y = cfma(u[row * 4 + 2], x2, y);
+      y = cfma(u[row * 4 + 3], x3, y);
+      v[r | (row & 1 ? m0 : 0) | (row & 2 ? m1 : 0)] = y;
+    }
+  }
+}
+
+// Run of diagonal patterns. Slot 0 (no condition on r): one factor for all owned amplitudes;
+// slots 1..4 ("r bit k set"): one factor per bit, the 2^NR table is built by doubling; the
+// remaining entries have a general condition on r and are applied group by group.
+template <int NR>
+__device__ __forceinline__ void op_run(double2 (&v)[kRegAmps], const TileOp& op, const TileCtx& c,
+                                       const Mapping& mp, int n0, int n1, int n2, int n3, int n4) {
+  uint32_t e = op.moff;
+  double2 t0 = make_double2(1.0, 0.0);
+  for (const uint32_t end = e + uint32_t(n0); e < end; ++e) {
+    const RunEntry en = c.ents[e];
+    if ((mp.base & en.tmask) == en.tmatch) t0 = cmul(t0, c.C[en.pat]);
+  }
+  double2 ek[4];
+  const int ne[4] = {n1, n2, n3, n4};
+#pragma unroll
+  for (int k = 0; k < 4; ++k) {
+    ek[k] = make_double2(1.0, 0.0);
+    for (const uint32_t end = e + uint32_t(ne[k]); e < end; ++e) {
+      const RunEntry en = c.ents[e];
+      if ((mp.base & en.tmask) == en.tmatch) ek[k] = cmul(ek[k], c.C[en.pat]);
+    }
+  }
+  if (n0 + n1 + n2 + n3 + n4 > 0) {
+    double2 P[kRegAmps];
+    P[0] = t0;
+#pragma unroll
+    for (int k = 0; k < NR; ++k)
+#pragma unroll
+      for (int r = 0; r < (1 << k); ++r) P[r | (1 << k)] = cmul(P[r], ek[k]);
+#pragma unroll
+    for (int r = 0; r < (1 << NR); ++r) v[r] = cmul(v[r], P[r]);
+  }
+  double2 acc = make_double2(1.0, 0.0);
+  for (const uint32_t end = op.moff + op.cnt; e < end; ++e) {
+    const RunEntry en = c.ents[e];
+    if ((mp.base & en.tmask) == en.tmatch) acc = cmul(acc, c.C[en.pat]);
+    if (en.gend) {
+#pragma unroll
+      for (int r = 0; r < (1 << NR); ++r) {
+        const bool mt = (uint32_t(r) & en.rmask) == en.rmatch;
+        v[r] = cmul(v[r], mt ? acc : make_double2(1.0, 0.0));
+      }
+      acc = make_double2(1.0, 0.0);
+    }
+  }
+}
+
+// Shared-memory fallback ops (tile in natural order in c.s; caller spills/reloads)
+template <int CLS>
+__device__ __forceinline__ void op_smem1(const TileCtx& c, const TileOp& op) {
+  const int t = op.a0;
+  const double2* up = c.pool + op.moff;
+  const double2 u[4] = {up[0], up[1], up[2], up[3]};
+  for (uint32_t pp = c.tid; pp < c.T / 2; pp += c.nthr) {
+    const uint32_t i0 = uint32_t(insert0(pp, t));
+    if ((i0 & op.tmask) != op.tmatch) continue;
+    const uint32_t i1 = i0 | (1u << t);
+    double2 x0 = c.s[i0], x1 = c.s[i1];
+    apply2<CLS>(x0, x1, u);
+    c.s[i0] = x0;
+    c.s[i1] = x1;
+  }
+  __syncthreads();
+}
+
+__device__ __forceinline__ void op_smem2(const TileCtx& c, const TileOp& op) {
+  const int t0 = op.a0, t1 = op.a1;
+  const int lo = min(t0, t1), hi = max(t0, t1);
+  const double2* u = c.pool + op.moff;
+  const uint32_t o1 = 1u << t0, o2 = 1u << t1;
+  for (uint32_t pp = c.tid; pp < c.T / 4; pp += c.nthr) {
+    const uint32_t i0 = uint32_t(insert0(insert0(pp, lo), hi));
+    if ((i0 & op.tmask) != op.tmatch) continue;
+    const double2 x0 = c.s[i0], x1 = c.s[i0 | o1], x2 = c.s[i0 | o2], x3 = c.s[i0 | o1 | o2];
+#pragma unroll
+    for (int row = 0; row < 4; ++row) {
+      double2 y = cmul(u[row * 4], x0);
+      y = cfma(u[row * 4 + 1], x1, y);
+      y = cfma(u[row * 4 + 2], x2, y);
+      y = cfma(u[row * 4 + 3], x3, y);
+      c.s[i0 | (row & 1 ? o1 : 0u) | (row & 2 ? o2 : 0u)] = y;
+    }
+  }
+  __syncthreads();
+}
+
+__device__ __forceinline__ void issue_tile_loads(double2* buf, const TileArgs& a, const uint64_t* hiOff,
+                                                 uint64_t tile, uint32_t T, int nthr, int tid, int nld,
+                                                 uint32_t lowmask, int l) {
+  const uint64_t base = deposit(tile, a.spos, a.b);
+#pragma unroll
+  for (int r = 0; r < kRegAmps; ++r) {
+    const uint32_t j = uint32_t(tid) + uint32_t(r) * nthr;
+    if (r < nld && j < T) {
+      const uint64_t idx = base | (j & lowmask) | hiOff[j >> l];
+      const bool live = idx < a.L_in;
+      cp_async16(buf + j, a.psi + (live ? idx : 0), live ? 16 : 0);
+    }
+  }
+  asm volatile("cp.async.commit_group;\n" ::: "memory");
+}
+
+// The persistent tile loop shared by the interpreted and the JIT kernels: one CTA per SM, two
+// tile buffers (the loads of tile i+1 fly while tile i is computed in registers), per-tile
+// pattern constants and tile-uniform phase computed right after the tile lands.
+// Body: void operator()(double2 (&v)[16], Mapping& mp, const TileCtx& c).
+template <int NR, class Body>
+__device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
+  extern __shared__ __align__(16) unsigned char smem_raw[];
+  const int b = a.b, l = a.l, nw = a.nw;
+  const uint32_t T = 1u << b;
+  const int nh = 1 << (b - l);
+  const int nthr = blockDim.x;
+  double2* bufs = reinterpret_cast<double2*>(smem_raw);  // 2 x T
+  uint64_t* hiOff = reinterpret_cast<uint64_t*>(bufs + 2 * T);
+  unsigned char* blob = reinterpret_cast<unsigned char*>(hiOff + ((nh + 1) & ~1));
+  const TileOp* ops = reinterpret_cast<const TileOp*>(blob);
+  const RunEntry* ents = reinterpret_cast<const RunEntry*>(blob + a.off_entries);
+  const Pattern* pats = reinterpret_cast<const Pattern*>(blob + a.off_patterns);
+  const PhaseTerm* terms = reinterpret_cast<const PhaseTerm*>(blob + a.off_terms);
+  const PhaseTerm* scal = reinterpret_cast<const PhaseTerm*>(blob + a.off_scalar);
+  const double2* pool = reinterpret_cast<const double2*>(blob + a.off_pool);
+  double2* C = reinterpret_cast<double2*>(blob + a.blob_bytes);  // pattern constants
+  double2* scal_s = C + a.npat;
+
+  {
+    const int4* src = reinterpret_cast<const int4*>(a.blob);
+    int4* dst = reinterpret_cast<int4*>(blob);
+    for (int i = threadIdx.x; i < a.blob_bytes / 16; i += nthr) dst[i] = src[i];
+  }
+  for (int h = threadIdx.x; h < nh; h += nthr) {
+    uint64_t off = 0;
+    for (int i = l; i < b; ++i)
+      if (h >> (i - l) & 1) off |= 1ull << a.spos[i];
+    hiOff[h] = off;
+  }
+  __syncthreads();
+  const uint32_t lowmask = (1u << l) - 1;
+  const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
+  const int nld = (T + nthr - 1) / nthr;  // natural-order amplitudes per thread
+  TileCtx c;
+  c.ops = ops;
+  c.ents = ents;
+  c.pool = pool;
+  c.C = C;
+  c.T = T;
+  c.nthr = nthr;
+  c.tid = tid;
+  c.lane = lane;
+  c.warp = warp;
+  c.nw = nw;
+  c.own = lane < int(T);
+
+  uint64_t tile = blockIdx.x;
+  if (tile < a.ntiles) issue_tile_loads(bufs, a, hiOff, tile, T, nthr, tid, nld, lowmask, l);
+  for (int it = 0; tile < a.ntiles; tile += gridDim.x, ++it) {
+    double2* s = bufs + (it & 1) * T;
+    const uint64_t base = deposit(tile, a.spos, b);
+    const uint64_t gbase = a.rank_base | base;
+    cp_async_wait_all();
+    __syncthreads();  // tile `it` landed; the other buffer is free (previous store done)
+    if (tile + gridDim.x < a.ntiles)
+      issue_tile_loads(bufs + ((it + 1) & 1) * T, a, hiOff, tile + gridDim.x, T, nthr, tid, nld, lowmask, l);
+    for (int pi = tid; pi < a.npat; pi += nthr) {
+      double2 cc = make_double2(1.0, 0.0);
+      const Pattern pt = pats[pi];
+      for (uint32_t k = pt.first; k < pt.first + pt.count; ++k)
+        if ((gbase & terms[k].omask) == terms[k].omatch) cc = cmul(cc, make_double2(terms[k].re, terms[k].im));
+      C[pi] = cc;
+    }
+    if (warp == 0) {
+      double2 sc = make_double2(1.0, 0.0);
+      for (int k = lane; k < a.nscalar; k += 32)
+        if ((gbase & scal[k].omask) == scal[k].omatch) sc = cmul(sc, make_double2(scal[k].re, scal[k].im));
+#pragma unroll
+      for (int o = 16; o > 0; o >>= 1) {
+        double2 t;
+        t.x = __shfl_xor_sync(0xffffffffu, sc.x, o);
+        t.y = __shfl_xor_sync(0xffffffffu, sc.y, o);
+        sc = cmul(sc, t);
+      }
+      if (lane == 0) *scal_s = sc;
+    }
+    c.s = s;
+    c.gbase = gbase;
+    double2 v[kRegAmps];
+    Mapping mp = make_mapping<NR>(ops[0], nw, lane, warp);  // ops[0] is always OP_REMAP
+    tile_reload<NR>(v, c, mp);
+    __syncthreads();  // constants visible
+    body(v, mp, c);
+    // back to natural order, then store (times the tile-uniform phase)
+    tile_spill<NR>(v, c, mp);
+    const double2 sc = *scal_s;
+    const bool has_sc = !(sc.x == 1.0 && sc.y == 0.0);
+#pragma unroll
+    for (int r = 0; r < kRegAmps; ++r) {
+      const uint32_t j = uint32_t(tid) + uint32_t(r) * nthr;
+      if (r < nld && j < T) {
+        const double2 x = has_sc ? cmul(s[j], sc) : s[j];
+        st_stream(a.psi + (base | (j & lowmask) | hiOff[j >> l]), x);
+      }
+    }
+  }
+  cp_async_wait_all();
+}
+
+#endif  // __CUDACC__
+
+}  // namespace qgpu

@@ -24,7 +24,7 @@ EXPORTS = [
     "qgpu_set_amplitudes", "qgpu_synchronize", "qgpu_state_info", "qgpu_apply_gate",
     "qgpu_apply_circuit", "qgpu_get_amplitudes", "qgpu_get_amplitudes_device",
     "qgpu_probabilities", "qgpu_circuit_from_qasm", "qgpu_circuit_info", "qgpu_circuit_destroy",
-    "qgpu_circuit_reorder", "qgpu_circuit_plan", "qgpu_get_involvement", "qgpu_get_chunk_bitmap",
+    "qgpu_circuit_reorder", "qgpu_circuit_plan", "qgpu_circuit_jit_check", "qgpu_get_involvement", "qgpu_get_chunk_bitmap",
     "qgpu_get_schedule", "qgpu_get_qubit_map", "qgpu_get_stats", "qgpu_reset_stats",
     "qgpu_last_error", "qgpu_version",
 ]
@@ -44,6 +44,7 @@ class Config(ctypes.Structure):
         ("rank", ctypes.c_int), ("world_size", ctypes.c_int), ("nccl_unique_id", ctypes.c_void_p),
         ("chunk_bits", ctypes.c_int), ("prune", ctypes.c_int), ("reorder", ctypes.c_int),
         ("fuse_bits", ctypes.c_int), ("timing", ctypes.c_int), ("swap_slab_bytes", ctypes.c_uint64),
+        ("jit", ctypes.c_int),
     ]
 
 
@@ -54,7 +55,8 @@ class Stats(ctypes.Structure):
         ("ops_before_full_involvement", ctypes.c_int64), ("kernel_ms", ctypes.c_double),
         ("tile_kernel_ms", ctypes.c_double), ("tile_kernel_launches", ctypes.c_uint64),
         ("tile_algo_bytes", ctypes.c_uint64), ("swap_ms", ctypes.c_double),
-        ("h2d_bytes", ctypes.c_uint64), ("d2h_bytes", ctypes.c_uint64)]
+        ("h2d_bytes", ctypes.c_uint64), ("d2h_bytes", ctypes.c_uint64),
+        ("jit_launches", ctypes.c_uint64), ("jit_compiles", ctypes.c_uint64), ("jit_ms", ctypes.c_double)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
@@ -81,6 +83,7 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
         "qgpu_circuit_from_qasm": [ctypes.c_char_p, ctypes.c_size_t, P],
         "qgpu_circuit_info": [P, P, P], "qgpu_circuit_destroy": [P],
         "qgpu_circuit_reorder": [P, I, P, U64, P], "qgpu_circuit_plan": [P, I, I, I, I, P, U64, P],
+        "qgpu_circuit_jit_check": [P, I, I, I, P],
         "qgpu_get_involvement": [P, P], "qgpu_get_chunk_bitmap": [P, I, P, U64],
         "qgpu_get_schedule": [P, P, P, U64, P], "qgpu_get_qubit_map": [P, P],
         "qgpu_get_stats": [P, P], "qgpu_reset_stats": [P],
@@ -147,6 +150,12 @@ class Circuit:
         _check(load().qgpu_circuit_plan(self._h, n, world_size, reorder, fuse_bits,
                                         info.ctypes.data, cnt.value, ctypes.byref(cnt)))
         return info[:cnt.value]
+
+    def jit_check(self, n: int, reorder: int = 2, fuse_bits: int = 12) -> int:
+        """Compile the NVRTC-specialised kernel of every fused pass (no GPU needed)."""
+        k = ctypes.c_int()
+        _check(load().qgpu_circuit_jit_check(self._h, n, reorder, fuse_bits, ctypes.byref(k)))
+        return k.value
 
     def close(self):
         if self._h:
