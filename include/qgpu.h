@@ -70,7 +70,7 @@ typedef struct {
   int timing;                 /* 1: time every launch with CUDA events into qgpu_stats     */
   uint64_t swap_slab_bytes;   /* staging bytes per all-to-all slab (sharded mode)          */
   int jit;                    /* fused passes: 0 = generic tile kernel only; 1 (default) = NVRTC-
-                                 specialised kernel for passes of >= 2^16 amplitudes; 2 = always.
+                                 specialised kernel for passes of >= 2^20 amplitudes; 2 = always.
                                  Falls back to the generic kernel if NVRTC is unavailable   */
 } qgpu_config;
 
@@ -186,7 +186,8 @@ qgpu_status qgpu_circuit_plan(const qgpu_circuit* c, int n_qubits, int world_siz
                               int fuse_bits, int64_t* info, uint64_t cap, uint64_t* n_passes);
 
 /* Host-only (no GPU needed): generate the NVRTC-specialised kernel source of every fused pass of
- * the plan (as qgpu_circuit_plan) and compile it for sm_100a. *n_compiled = passes compiled.
+ * the plan (as qgpu_circuit_plan) and compile it for sm_100a into the on-disk cubin cache
+ * ($QGPU_JIT_CACHE, else <dir of libqgpu.so>/build/jitcache). *n_compiled = passes compiled.
  * Returns UNSUPPORTED if NVRTC cannot be loaded, CUDA (with the NVRTC log in
  * qgpu_last_error) if a pass fails to compile. */
 qgpu_status qgpu_circuit_jit_check(const qgpu_circuit* c, int n_qubits, int reorder, int fuse_bits,

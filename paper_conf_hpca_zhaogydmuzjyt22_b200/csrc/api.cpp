@@ -25,6 +25,8 @@ struct qgpu_circuit {
 
 namespace {
 
+constexpr int kJitMinBits = 20;  // jit=1: specialise passes whose live range is >= 2^20
+
 thread_local std::string g_err;
 
 qgpu_status fail(qgpu_status s, const char* fmt, ...) {
@@ -195,21 +197,25 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops)
     a.b = p.b;
     a.l = p.l;
     for (int i = 0; i < p.b; ++i) a.spos[i] = p.spos[i];
+    a.nsrun = 0;
+    for (int i = 0; i < p.b;) {
+      int j = i;
+      while (j + 1 < p.b && p.spos[j + 1] == p.spos[j] + 1) ++j;
+      a.srun_pos[a.nsrun] = p.spos[i];
+      a.srun_len[a.nsrun] = j - i + 1;
+      a.nsrun++;
+      i = j + 1;
+    }
     a.ntiles = 1ull << (kout - p.b);
     a.L_in = L_in;
     a.rank_base = rank << m;
     const int jit = st->cfg.jit;
     cudaError_t e = cudaErrorNotSupported;
-    if (jit == 2 || (jit == 1 && kout >= 16)) {
+    if (jit == 2 || (jit == 1 && p.k_out >= kJitMinBits)) {
       double ms = 0;
       e = launch_tile_jit(st->stream, p, a, tile_smem_bytes(a), device_num_sms(), &ms);
-      if (e == cudaSuccess) {
-        st->stats.jit_launches++;
-        if (ms > 0) {
-          st->stats.jit_compiles++;
-          st->stats.jit_ms += ms;
-        }
-      }
+      if (e == cudaSuccess) st->stats.jit_launches++;
+      st->stats.jit_ms += ms;
     }
     if (e == cudaErrorNotSupported) e = launch_tile(st->stream, a);
     CK(e);
@@ -335,6 +341,15 @@ qgpu_status run_plan(qgpu_state* st, const std::vector<Pass>& passes) {
     CK(cudaMemcpyAsync(st->d_ops, st->h_ops, nbytes, cudaMemcpyHostToDevice, st->stream));
     st->stats.h2d_bytes += nbytes;
     CK(cudaEventRecord(st->ops_evt, st->stream));
+  }
+  if (st->cfg.jit) {
+    std::vector<const Pass*> want;
+    for (const Pass& p : passes)
+      if (p.kind == PK_TILE && (st->cfg.jit == 2 || p.k_out >= kJitMinBits)) want.push_back(&p);
+    double ms = 0;
+    const int k = jit_prepare(want, &ms);
+    st->stats.jit_compiles += uint64_t(k);
+    st->stats.jit_ms += ms;
   }
   for (size_t i = 0; i < passes.size(); ++i) {
     qgpu_status s = exec_pass(st, passes[i], st->d_ops + off[i]);
@@ -771,7 +786,7 @@ qgpu_status qgpu_circuit_jit_check(const qgpu_circuit* c, int n, int reorder_mod
     std::string cubin, log;
     for (const Pass& p : passes) {
       if (p.kind != PK_TILE) continue;
-      if (!jit_compile_cubin(tile_jit_source(p), &cubin, &log)) {
+      if (!jit_cubin_cached(tile_jit_source(p), &cubin, &log, nullptr)) {
         if (log == "libnvrtc not found") return fail(QGPU_ERR_UNSUPPORTED, "%s", log.c_str());
         return fail(QGPU_ERR_CUDA, "NVRTC: %s\n--- source ---\n%s", log.c_str(), tile_jit_source(p).c_str());
       }

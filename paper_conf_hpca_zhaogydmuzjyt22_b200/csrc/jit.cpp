@@ -13,13 +13,20 @@
 #include <dlfcn.h>
 #include <nvrtc.h>
 
+#include <algorithm>
+#include <atomic>
 #include <chrono>
+#include <fstream>
+#include <sys/stat.h>
+#include <unistd.h>
 #include <cstdio>
 #include <cstdlib>
 #include <mutex>
+#include <thread>
 #include <sstream>
 #include <string>
 #include <unordered_map>
+#include <vector>
 
 #include "jit.h"
 #include "kernels.h"
@@ -98,7 +105,71 @@ bool load_driver(JitLib& L) {
   return true;
 }
 
+// ---- on-disk cubin cache: <dir>/<fnv1a64(source|options)>.cubin
+// dir = $QGPU_JIT_CACHE, else <directory of libqgpu.so>/build/jitcache
+std::string cache_dir() {
+  if (const char* ev = std::getenv("QGPU_JIT_CACHE")) return ev;
+  Dl_info info;
+  if (dladdr(reinterpret_cast<void*>(&cache_dir), &info) && info.dli_fname) {
+    std::string so = info.dli_fname;
+    const size_t k = so.find_last_of('/');
+    return (k == std::string::npos ? std::string(".") : so.substr(0, k)) + "/build/jitcache";
+  }
+  return "";
+}
+
+std::string cache_key(const std::string& src) {
+  uint64_t h = 1469598103934665603ull;
+  auto mix = [&](const std::string& x) {
+    for (unsigned char ch : x) {
+      h ^= ch;
+      h *= 1099511628211ull;
+    }
+  };
+  mix(src);
+  mix("|sm_100a|-std=c++17|-lineinfo|");
+  if (const char* ev = std::getenv("QGPU_JIT_OPTS")) mix(ev);
+  char buf[32];
+  std::snprintf(buf, sizeof(buf), "%016llx", static_cast<unsigned long long>(h));
+  return buf;
+}
+
+bool cache_read(const std::string& key, std::string* cubin) {
+  const std::string d = cache_dir();
+  if (d.empty()) return false;
+  std::ifstream f(d + "/" + key + ".cubin", std::ios::binary);
+  if (!f) return false;
+  cubin->assign(std::istreambuf_iterator<char>(f), std::istreambuf_iterator<char>());
+  return !cubin->empty();
+}
+
+void cache_write(const std::string& key, const std::string& cubin) {
+  const std::string d = cache_dir();
+  if (d.empty()) return;
+  ::mkdir((d.substr(0, d.find_last_of('/'))).c_str(), 0755);
+  ::mkdir(d.c_str(), 0755);
+  const std::string tmp = d + "/" + key + ".tmp." + std::to_string(::getpid());
+  {
+    std::ofstream f(tmp, std::ios::binary);
+    if (!f) return;
+    f.write(cubin.data(), std::streamsize(cubin.size()));
+  }
+  std::rename(tmp.c_str(), (d + "/" + key + ".cubin").c_str());
+}
+
 }  // namespace
+
+bool jit_cubin_cached(const std::string& src, std::string* cubin, std::string* log, bool* hit) {
+  const std::string key = cache_key(src);
+  if (cache_read(key, cubin)) {
+    if (hit) *hit = true;
+    return true;
+  }
+  if (hit) *hit = false;
+  if (!jit_compile_cubin(src, cubin, log)) return false;
+  cache_write(key, *cubin);
+  return true;
+}
 
 std::string tile_jit_source(const Pass& p) {
   const TileProgram& P = p.prog;
@@ -116,10 +187,46 @@ std::string tile_jit_source(const Pass& p) {
     const bool thr = op.tmask != 0;       // condition on the thread's fixed bits present
     o << "    { const TileOp& op = ops[" << i << "];\n";
     switch (op.kind) {
-      case OP_RUN:
-        o << "      op_run<" << NR << ">(v, op, c, mp, " << op.a0 << ", " << op.a1 << ", " << op.cls << ", "
-          << op.tmask << ", " << op.tmatch << ");\n";
+      case OP_RUN: {
+        // entries are compile-time: slot 0 (all owned amplitudes), slots 1..4 (r bit k set),
+        // then general groups (compile-time r condition)
+        const int ns[5] = {op.a0, op.a1, op.cls, int(op.tmask), int(op.tmatch)};
+        const char* acc[5] = {"t0", "e0", "e1", "e2", "e3"};
+        uint32_t e = op.moff;
+        o << "      const uint32_t tb = mp.base; (void)tb;\n";
+        o << "      double2 t0 = make_double2(1.0, 0.0), e0 = t0, e1 = t0, e2 = t0, e3 = t0;\n";
+        int used = 0;
+        for (int sl = 0; sl < 5; ++sl) {
+          for (int k = 0; k < ns[sl]; ++k, ++e) {
+            const RunEntry& en = P.entries[e];
+            used |= 1 << sl;
+            o << "      ";
+            if (en.tmask) o << "if ((tb & " << en.tmask << "u) == " << en.tmatch << "u) ";
+            o << acc[sl] << " = cmul(" << acc[sl] << ", c.C[" << en.pat << "]);\n";
+          }
+        }
+        if (used)
+          o << "      run_apply_table<" << NR << ", " << ((used >> 1) & 1 ? "true" : "false") << ", "
+            << ((used >> 2) & 1 ? "true" : "false") << ", " << ((used >> 3) & 1 ? "true" : "false") << ", "
+            << ((used >> 4) & 1 ? "true" : "false") << ">(v, t0, e0, e1, e2, e3);\n";
+        const uint32_t end = op.moff + op.cnt;
+        bool open_group = false;
+        for (; e < end; ++e) {
+          const RunEntry& en = P.entries[e];
+          if (!open_group) {
+            o << "      { double2 acc = make_double2(1.0, 0.0);\n";
+            open_group = true;
+          }
+          o << "        ";
+          if (en.tmask) o << "if ((tb & " << en.tmask << "u) == " << en.tmatch << "u) ";
+          o << "acc = cmul(acc, c.C[" << en.pat << "]);\n";
+          if (en.gend) {
+            o << "        run_apply_group<" << NR << ", " << en.rmask << "u, " << en.rmatch << "u>(v, acc); }\n";
+            open_group = false;
+          }
+        }
         break;
+      }
       case OP_U1R:
         o << "      if (" << (uni ? "op_active(op, c.gbase)" : "true") << (thr ? " && (mp.base & op.tmask) == op.tmatch" : "")
           << ") op_u1r<" << NR << ", " << op.a0 << ", " << op.cls << ">(v, c.pool + op.moff, " << op.rmask << "u, "
@@ -157,7 +264,7 @@ std::string tile_jit_source(const Pass& p) {
   return o.str();
 }
 
-bool jit_compile_cubin(const std::string& src, std::string* cubin, std::string* log) {
+bool jit_compile_cubin(const std::string& src, std::string* cubin, std::string* log) {  // NOLINT
   JitLib& L = lib();
   if (!L.createProgram && !load_nvrtc(L)) {
     *log = L.err;
@@ -170,8 +277,14 @@ bool jit_compile_cubin(const std::string& src, std::string* cubin, std::string* 
     *log = "nvrtcCreateProgram failed";
     return false;
   }
-  const char* opts[] = {"-arch=sm_100a", "-std=c++17", "-lineinfo", "-DQGPU_JIT=1"};
-  const nvrtcResult rc = L.compileProgram(prog, 4, opts);
+  std::vector<const char*> opts = {"-arch=sm_100a", "-std=c++17", "-lineinfo", "-DQGPU_JIT=1"};
+  std::vector<std::string> extra;
+  if (const char* ev = std::getenv("QGPU_JIT_OPTS")) {  // e.g. "-Xptxas -O2" (experiments)
+    std::istringstream is(ev);
+    for (std::string w; is >> w;) extra.push_back(w);
+  }
+  for (auto& w : extra) opts.push_back(w.c_str());
+  const nvrtcResult rc = L.compileProgram(prog, int(opts.size()), opts.data());
   size_t n = 0;
   L.getLogSize(prog, &n);
   log->assign(n, '\0');
@@ -200,6 +313,54 @@ bool jit_available(std::string* why) {
   return L.ok;
 }
 
+// Make sure the kernels of `passes` are loaded: cubins come from the disk cache or are compiled
+// in parallel (one NVRTC program per pass, up to hardware_concurrency threads).
+int jit_prepare(const std::vector<const Pass*>& passes, double* compile_ms) {
+  if (passes.empty() || !jit_available(nullptr)) return 0;
+  JitLib& L = lib();
+  const auto t0 = std::chrono::steady_clock::now();
+  std::vector<std::string> srcs;
+  {
+    std::lock_guard<std::mutex> g(L.mu);
+    for (const Pass* p : passes) {
+      std::string src = tile_jit_source(*p);
+      if (!L.cache.count(src) && std::find(srcs.begin(), srcs.end(), src) == srcs.end()) srcs.push_back(std::move(src));
+    }
+  }
+  if (srcs.empty()) return 0;
+  std::vector<std::string> cubins(srcs.size());
+  std::vector<char> ok(srcs.size(), 0);
+  std::atomic<size_t> next{0};
+  auto work = [&]() {
+    for (size_t i; (i = next.fetch_add(1)) < srcs.size();) {
+      std::string log;
+      ok[i] = jit_cubin_cached(srcs[i], &cubins[i], &log, nullptr) ? 1 : 0;
+      if (!ok[i]) std::fprintf(stderr, "qgpu: JIT compile failed:\n%s\n", log.c_str());
+    }
+  };
+  const unsigned nt = std::max(1u, std::min<unsigned>(std::thread::hardware_concurrency(), unsigned(srcs.size())));
+  std::vector<std::thread> th;
+  for (unsigned t = 1; t < nt; ++t) th.emplace_back(work);
+  work();
+  for (auto& t : th) t.join();
+  cudaFree(nullptr);
+  int loaded = 0;
+  for (size_t i = 0; i < srcs.size(); ++i) {
+    if (!ok[i]) continue;
+    CUmodule mod = nullptr;
+    CUfunction fn = nullptr;
+    if (L.moduleLoadData(&mod, cubins[i].data()) != CUDA_SUCCESS) continue;
+    if (L.moduleGetFunction(&fn, mod, "qgpu_tile_pass") != CUDA_SUCCESS) continue;
+    if (L.funcSetAttribute(fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, 227 * 1024) != CUDA_SUCCESS) continue;
+    std::lock_guard<std::mutex> g(L.mu);
+    L.cache.emplace(srcs[i], fn);
+    ++loaded;
+  }
+  if (compile_ms)
+    *compile_ms += std::chrono::duration<double, std::milli>(std::chrono::steady_clock::now() - t0).count();
+  return loaded;
+}
+
 // Compile (or fetch from the cache) and launch the specialised kernel of pass p.
 // Returns cudaErrorNotSupported when the JIT is unavailable (caller falls back).
 cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, size_t smem, int num_sms,
@@ -216,7 +377,8 @@ cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, s
   if (!fn) {
     const auto t0 = std::chrono::steady_clock::now();
     std::string cubin, log;
-    if (!jit_compile_cubin(src, &cubin, &log)) {
+    bool hit = false;
+    if (!jit_cubin_cached(src, &cubin, &log, &hit)) {
       std::fprintf(stderr, "qgpu: JIT compile failed, using the interpreted tile kernel:\n%s\n", log.c_str());
       return cudaErrorNotSupported;
     }
@@ -227,7 +389,7 @@ cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, s
     if (L.funcSetAttribute(fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, 227 * 1024) != CUDA_SUCCESS)
       return cudaErrorNotSupported;
     const auto t1 = std::chrono::steady_clock::now();
-    if (compile_ms) *compile_ms += std::chrono::duration<double, std::milli>(t1 - t0).count();
+    if (compile_ms) *compile_ms += std::max(1e-3, std::chrono::duration<double, std::milli>(t1 - t0).count());
     std::lock_guard<std::mutex> g(L.mu);
     L.cache.emplace(src, fn);
   }

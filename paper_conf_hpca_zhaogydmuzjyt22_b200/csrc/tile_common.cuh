@@ -72,6 +72,8 @@ struct TileArgs {
   int nr, nw;              // register / warp bits of the thread mapping
   int b, l;
   int spos[kMaxTileBits];
+  int nsrun;                      // maximal runs of consecutive tile positions (for deposit)
+  int srun_pos[kMaxTileBits], srun_len[kMaxTileBits];
   uint64_t ntiles;
   uint64_t L_in;
   uint64_t rank_base;      // rank << m (global bits for tile-uniform conditions)
@@ -94,6 +96,15 @@ __device__ __forceinline__ uint64_t deposit(uint64_t v, const int* ins, int nins
   return v;
 }
 __device__ __forceinline__ void st_stream(double2* p, double2 v) { __stcs(p, v); }
+
+// tile index -> base amplitude index: insert the tile positions (as runs of consecutive bits)
+__device__ __forceinline__ uint64_t tile_base(uint64_t t, const TileArgs& a) {
+  for (int i = 0; i < a.nsrun; ++i) {
+    const int p = a.srun_pos[i];
+    t = ((t >> p) << (p + a.srun_len[i])) | (t & ((1ull << p) - 1));
+  }
+  return t;
+}
 
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
   const unsigned sa = static_cast<unsigned>(__cvta_generic_to_shared(smem));
@@ -273,6 +284,29 @@ __device__ __forceinline__ void op_run(double2 (&v)[kRegAmps], const TileOp& op,
   }
 }
 
+// JIT helpers for a run whose entries are compile-time: multiply the owned amplitudes by the
+// table P[r] = t0 * prod_{k: r_k = 1} e_k (built by doubling; bits without entries skipped).
+template <int NR, bool E0, bool E1, bool E2, bool E3>
+__device__ __forceinline__ void run_apply_table(double2 (&v)[kRegAmps], double2 t0, double2 e0, double2 e1,
+                                                double2 e2, double2 e3) {
+  double2 P[kRegAmps];
+  P[0] = t0;
+  const double2 ek[4] = {e0, e1, e2, e3};
+  const bool has[4] = {E0, E1, E2, E3};
+#pragma unroll
+  for (int k = 0; k < NR; ++k)
+#pragma unroll
+    for (int r = 0; r < (1 << k); ++r) P[r | (1 << k)] = has[k] ? cmul(P[r], ek[k]) : P[r];
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r) v[r] = cmul(v[r], P[r]);
+}
+template <int NR, unsigned RM, unsigned RT>
+__device__ __forceinline__ void run_apply_group(double2 (&v)[kRegAmps], double2 acc) {
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r)
+    if ((unsigned(r) & RM) == RT) v[r] = cmul(v[r], acc);
+}
+
 // Shared-memory fallback ops (tile in natural order in c.s; caller spills/reloads)
 template <int CLS>
 __device__ __forceinline__ void op_smem1(const TileCtx& c, const TileOp& op) {
@@ -315,7 +349,7 @@ __device__ __forceinline__ void op_smem2(const TileCtx& c, const TileOp& op) {
 __device__ __forceinline__ void issue_tile_loads(double2* buf, const TileArgs& a, const uint64_t* hiOff,
                                                  uint64_t tile, uint32_t T, int nthr, int tid, int nld,
                                                  uint32_t lowmask, int l) {
-  const uint64_t base = deposit(tile, a.spos, a.b);
+  const uint64_t base = tile_base(tile, a);
 #pragma unroll
   for (int r = 0; r < kRegAmps; ++r) {
     const uint32_t j = uint32_t(tid) + uint32_t(r) * nthr;
@@ -383,7 +417,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   if (tile < a.ntiles) issue_tile_loads(bufs, a, hiOff, tile, T, nthr, tid, nld, lowmask, l);
   for (int it = 0; tile < a.ntiles; tile += gridDim.x, ++it) {
     double2* s = bufs + (it & 1) * T;
-    const uint64_t base = deposit(tile, a.spos, b);
+    const uint64_t base = tile_base(tile, a);
     const uint64_t gbase = a.rank_base | base;
     cp_async_wait_all();
     __syncthreads();  // tile `it` landed; the other buffer is free (previous store done)

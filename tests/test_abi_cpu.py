@@ -149,3 +149,17 @@ def test_state_create_without_gpu_fails_cleanly(q):
     with pytest.raises(q.QgpuError) as e:
         q.State(10)
     assert e.value.kind in ("CUDA", "OUT_OF_MEMORY")
+
+
+def test_jit_sources_compile_without_gpu(q):
+    """The per-pass NVRTC sources compile for sm_100a on the CPU box (no GPU)."""
+    for c in (wc.ghz_qft(5), wc.random_circuit(9, 80, seed=3)):
+        qc = q.Circuit(c.qasm())
+        try:
+            k = qc.jit_check(c.n, 2, 7)
+        except q.QgpuError as e:
+            if e.kind == "UNSUPPORTED":
+                pytest.skip("NVRTC not available")
+            raise
+        n_tile = sum(1 for r in qc.plan(c.n, 1, 2, 7) if r[2] == 0)
+        assert k == n_tile

@@ -295,3 +295,40 @@ def test_torch_buffer_and_stream(q):
     for lq, p in enumerate(pos):
         idx |= ((xs >> lq) & 1) << p
     assert np.abs(got[idx] - ref).max() <= TOL
+
+
+# ----------------------------------------------------------------------------- JIT path
+JIT_CIRCS = {
+    "fuzz12": lambda: wc.random_circuit(12, 300, seed=41),
+    "fuzz14": lambda: wc.random_circuit(14, 300, seed=42),
+    "qft16x": lambda: wc.qft(16, x=4321),
+    "qaoa14": lambda: wc.qaoa(14, 2, seed=1),
+    "rqc14": lambda: wc.rqc(14, 10, seed=3),
+    "hlf4x4": lambda: wc.hlf(4, 4, seed=2),
+}
+
+
+@pytest.mark.parametrize("name", sorted(JIT_CIRCS))
+@pytest.mark.parametrize("fuse", [9, 12])
+def test_jit_specialised_kernels_vs_oracle(q, name, fuse):
+    """jit=2: every fused pass runs an NVRTC-specialised kernel; parity vs the oracle and
+    agreement with the interpreted tile kernel (jit=0)."""
+    c = JIT_CIRCS[name]()
+    text = c.qasm()
+    qc = q.Circuit(text)
+    with q.State(c.n, fuse_bits=fuse, jit=2) as s:
+        s.apply_circuit(qc)
+        got = s.amplitudes()
+        st = s.stats()
+    assert st["jit_launches"] > 0
+    ref = oracle_run(text)
+    assert np.abs(got - ref).max() <= TOL
+    interp = gpu_run(q, text, fuse_bits=fuse, jit=0)
+    assert np.abs(got - interp).max() <= 1e-13
+
+
+def test_jit_pruning_neutrality_exact(q):
+    text = wc.random_circuit(15, 250, seed=21).qasm()
+    a = gpu_run(q, text, fuse_bits=12, prune=1, jit=2)
+    b = gpu_run(q, text, fuse_bits=12, prune=0, jit=2)
+    assert np.array_equal(a, b)
