@@ -68,6 +68,7 @@ struct qgpu_state {
   // readout scratch
   double* d_scratch = nullptr;
   size_t scratch_cap = 0;  // doubles
+  double2* d_zero = nullptr;  // zero amplitudes: source of the expanded region in tile loads
   // timing
   std::vector<TimedLaunch> pending;
   std::vector<cudaEvent_t> event_pool;
@@ -209,6 +210,13 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops)
     a.ntiles = 1ull << (kout - p.b);
     a.L_in = L_in;
     a.rank_base = rank << m;
+    a.zero = st->d_zero;
+    a.bulk = p.l >= 7 ? 1 : 0;
+    a.remaps = 0;
+    for (size_t i = 1; i < P.ops.size(); ++i)
+      if (P.ops[i].kind == OP_REMAP || P.ops[i].kind == OP_SMEM1 || P.ops[i].kind == OP_SMEM2) a.remaps = 1;
+    a.nbuf = 3;
+    if (tile_smem_bytes(a) > 227 * 1024) a.nbuf = 2;
     const int jit = st->cfg.jit;
     cudaError_t e = cudaErrorNotSupported;
     if (jit == 2 || (jit == 1 && p.k_out >= kJitMinBits)) {
@@ -388,6 +396,8 @@ qgpu_status init_amplitudes(qgpu_state* st) {
 PlanOptions plan_options(const qgpu_config& cfg, bool fuse) {
   PlanOptions o;
   o.fuse_bits = fuse ? cfg.fuse_bits : 0;
+  if (const char* ev = std::getenv("QGPU_REGBITS")) o.reg_bits = std::atoi(ev);
+  if (const char* ev = std::getenv("QGPU_MAX_UOPS")) o.max_u_ops = std::atoi(ev);
   o.prune = cfg.prune != 0;
   return o;
 }
@@ -482,6 +492,9 @@ qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out
       st->own_buf = true;
     }
     st->cap_amps = 1ull << st->m;
+    e = cudaMalloc(&st->d_zero, sizeof(double2) << kMaxTileBits);
+    if (e == cudaSuccess) e = cudaMemset(st->d_zero, 0, sizeof(double2) << kMaxTileBits);
+    if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "zero buffer: %s", cudaGetErrorString(e)));
     e = cudaEventCreateWithFlags(&st->ops_evt, cudaEventDisableTiming);
     if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e)));
     if (cfg.world_size > 1) {
@@ -510,6 +523,7 @@ qgpu_status qgpu_state_destroy(qgpu_state* st) {
   if (st->d_ops) cudaFree(st->d_ops);
   if (st->h_ops) cudaFreeHost(st->h_ops);
   if (st->d_scratch) cudaFree(st->d_scratch);
+  if (st->d_zero) cudaFree(st->d_zero);
   if (st->ops_evt) cudaEventDestroy(st->ops_evt);
   if (st->own_stream && st->stream) cudaStreamDestroy(st->stream);
   delete st;

@@ -259,7 +259,8 @@ std::string tile_jit_source(const Pass& p) {
     o << "    }\n";
   }
   o << "  }\n};\n";
-  o << "extern \"C\" __global__ void __launch_bounds__(256, 1) qgpu_tile_pass(const TileArgs a) {\n";
+  o << "extern \"C\" __global__ void __launch_bounds__(" << (NR >= 4 ? 256 : 512)
+    << ", 1) qgpu_tile_pass(const TileArgs a) {\n";
   o << "  JitBody body;\n  tile_driver<" << NR << ">(a, body);\n}\n";
   return o.str();
 }

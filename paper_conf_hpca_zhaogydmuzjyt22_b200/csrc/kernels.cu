@@ -228,7 +228,7 @@ struct InterpBody {
 };
 
 template <int NR>
-__global__ void __launch_bounds__(256, 1) tile_kernel(TileArgs a) {
+__global__ void __launch_bounds__(NR >= 4 ? 256 : 512, 1) tile_kernel(TileArgs a) {
   InterpBody<NR> body{a.nops};
   tile_driver<NR>(a, body);
 }
@@ -311,8 +311,8 @@ int device_num_sms() { return num_sms(); }
 
 size_t tile_smem_bytes(const TileArgs& a) {
   const size_t nh = size_t(1) << (a.b - a.l);
-  return 2 * (size_t(1) << a.b) * 16 + ((nh + 1) & ~size_t(1)) * 8 + size_t(a.blob_bytes) +
-         size_t(a.npat + 1) * 16;
+  return size_t(a.nbuf) * (size_t(1) << a.b) * 16 + 32 + ((nh + 1) & ~size_t(1)) * 8 +
+         size_t(a.blob_bytes) + size_t(a.npat + 1) * 16;
 }
 
 cudaError_t launch_pair(cudaStream_t st, const PairArgs& a, bool shfl) {

@@ -131,6 +131,7 @@ struct PlanOptions {
   int l_min = 5;        // minimum contiguous low tile bits (2^5 * 16 B = 512 B runs)
   int max_u_ops = 24;   // non-diagonal ops per fused pass (FP64 / smem budget)
   int max_ops = 256;    // all ops per fused pass
+  int reg_bits = 4;     // register bits per thread (2^reg_bits amplitudes in registers)
   bool prune = true;
 };
 
@@ -140,7 +141,7 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
                   const PlanOptions& opt, std::vector<Pass>* passes,
                   std::vector<uint64_t>* inv_after);
 // Build the device ops of a tile pass from its gates and tile positions.
-void build_tile_ops(Pass& p, int m);
+void build_tile_ops(Pass& p, int m, int reg_bits = 4);
 // Unfused byte model of one gate on live size 2^k.
 uint64_t unfused_gate_bytes(const PhysGate& g, int k_in, int k_out);
 

@@ -238,7 +238,7 @@ int mat_class(const cplx* U, int nt) {
 //     entirely outside the tile commute with the whole pass and become the tile scalar;
 //  3. assign register bits per segment (earliest next use), encode conditions relative to
 //     the mapping, and group each run's terms into distinct patterns.
-void build_tile_ops(Pass& p, int /*m*/) {
+void build_tile_ops(Pass& p, int /*m*/, int reg_bits) {
   TileProgram& P = p.prog;
   P = TileProgram();
   std::vector<RawOp> raw;
@@ -295,7 +295,7 @@ void build_tile_ops(Pass& p, int /*m*/) {
   const int b = p.b;
   const int lanes = std::min(5, b);
   const int nonlane = b - lanes;
-  const int nr = std::min(4, nonlane), nw = nonlane - nr;
+  const int nr = std::min(std::min(4, std::max(reg_bits, 3)), nonlane), nw = nonlane - nr;
   P.nr = nr;
   P.nw = nw;
   const size_t INF = ~size_t(0);
@@ -487,7 +487,7 @@ struct Builder {
       for (uint64_t r = S; r; r &= r - 1) p.spos[i++] = std::countr_zero(r);
       p.l = 0;
       while (p.l < p.b && p.spos[p.l] == p.l) ++p.l;
-      build_tile_ops(p, map.m);
+      build_tile_ops(p, map.m, opt.reg_bits);
     }
     out->push_back(std::move(p));
     cur = Pass();

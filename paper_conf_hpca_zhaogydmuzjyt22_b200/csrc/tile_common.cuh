@@ -77,6 +77,10 @@ struct TileArgs {
   uint64_t ntiles;
   uint64_t L_in;
   uint64_t rank_base;      // rank << m (global bits for tile-uniform conditions)
+  const double2* zero;     // >= 2^kMaxTileBits zero amplitudes (source of the expanded region)
+  int nbuf;                // tile buffers in shared memory (2 or 3)
+  int bulk;                // 1: bulk async copies (runs of >= 2^7 amplitudes), 0: per-thread
+  int remaps;              // the program contains REMAP / shared-memory ops
 };
 
 __device__ __forceinline__ double2 cmul(double2 a, double2 b) {
@@ -112,6 +116,37 @@ __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src
                : "memory");
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
+
+// ---- bulk asynchronous copies (TMA bulk path, SASS UBLKCP) with an mbarrier per buffer
+__device__ __forceinline__ uint32_t smem_u32(const void* p) {
+  return static_cast<uint32_t>(__cvta_generic_to_shared(p));
+}
+__device__ __forceinline__ void mbar_init(uint64_t* bar, uint32_t count) {
+  asm volatile("mbarrier.init.shared::cta.b64 [%0], %1;\n" ::"r"(smem_u32(bar)), "r"(count) : "memory");
+}
+__device__ __forceinline__ void mbar_arrive_expect_tx(uint64_t* bar, uint32_t bytes) {
+  asm volatile("{\n.reg .b64 st;\nmbarrier.arrive.expect_tx.shared::cta.b64 st, [%0], %1;\n}\n"
+               ::"r"(smem_u32(bar)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
+  uint32_t done = 0;
+  do {
+    asm volatile("{\n.reg .pred p;\nmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\nselp.u32 %0, 1, 0, p;\n}\n"
+                 : "=r"(done) : "r"(smem_u32(bar)), "r"(parity) : "memory");
+  } while (!done);
+}
+__device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
+  asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n"
+               ::"r"(smem_u32(dst)), "l"(src), "r"(bytes), "r"(smem_u32(bar)) : "memory");
+}
+__device__ __forceinline__ void bulk_s2g(void* dst, const void* src, uint32_t bytes) {
+  asm volatile("cp.async.bulk.global.shared::cta.bulk_group [%0], [%1], %2;\n"
+               ::"l"(dst), "r"(smem_u32(src)), "r"(bytes) : "memory");
+}
+__device__ __forceinline__ void bulk_commit() { asm volatile("cp.async.bulk.commit_group;\n" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_read() { asm volatile("cp.async.bulk.wait_group.read 0;\n" ::: "memory"); }
+__device__ __forceinline__ void bulk_wait_all() { asm volatile("cp.async.bulk.wait_group 0;\n" ::: "memory"); }
+__device__ __forceinline__ void fence_proxy_async() { asm volatile("fence.proxy.async.shared::cta;\n" ::: "memory"); }
 
 // (x0, x1) <- U (x0, x1), U = [[u0 u1] [u2 u3]], with the matrix-class shortcut
 template <int CLS>
@@ -346,15 +381,42 @@ __device__ __forceinline__ void op_smem2(const TileCtx& c, const TileOp& op) {
   __syncthreads();
 }
 
-__device__ __forceinline__ void issue_tile_loads(double2* buf, const TileArgs& a, const uint64_t* hiOff,
-                                                 uint64_t tile, uint32_t T, int nthr, int tid, int nld,
-                                                 uint32_t lowmask, int l) {
+// Tile loads of one tile: warp 0 issues one bulk copy per contiguous run of 2^l amplitudes
+// (runs at index >= L_in are copied from the zero buffer: first-touch expansion, a5); the
+// buffer's mbarrier completes when all T*16 bytes have landed.
+__device__ __forceinline__ void issue_tile_loads_bulk(double2* buf, uint64_t* bar, const TileArgs& a,
+                                                      const uint64_t* hiOff, uint64_t tile, int lane) {
   const uint64_t base = tile_base(tile, a);
+  const int nrun = 1 << (a.b - a.l);
+  const uint64_t rl = 1ull << a.l;
+  if (lane == 0) mbar_arrive_expect_tx(bar, uint32_t(16u << a.b));
+  __syncwarp();
+  for (int h = lane; h < nrun; h += 32) {
+    const uint64_t idx = base | hiOff[h];
+    double2* dst = buf + (uint64_t(h) << a.l);
+    if (idx + rl <= a.L_in) {
+      bulk_g2s(dst, a.psi + idx, uint32_t(rl * 16), bar);
+    } else if (idx >= a.L_in) {
+      bulk_g2s(dst, a.zero, uint32_t(rl * 16), bar);
+    } else {  // L_in < 2^l: the live part, then zeros
+      const uint64_t live = a.L_in - idx;
+      bulk_g2s(dst, a.psi + idx, uint32_t(live * 16), bar);
+      bulk_g2s(dst + live, a.zero, uint32_t((rl - live) * 16), bar);
+    }
+  }
+}
+
+// Per-thread variant for short runs (l < 7): one 16-B cp.async (LDGSTS) per amplitude,
+// src-size 0 (hardware zero-fill) beyond L_in.
+__device__ __forceinline__ void issue_tile_loads_thr(double2* buf, const TileArgs& a, const uint64_t* hiOff,
+                                                     uint64_t tile, uint32_t T, int nthr, int tid) {
+  const uint64_t base = tile_base(tile, a);
+  const uint32_t lowmask = (1u << a.l) - 1;
 #pragma unroll
   for (int r = 0; r < kRegAmps; ++r) {
     const uint32_t j = uint32_t(tid) + uint32_t(r) * nthr;
-    if (r < nld && j < T) {
-      const uint64_t idx = base | (j & lowmask) | hiOff[j >> l];
+    if (j < T) {
+      const uint64_t idx = base | (j & lowmask) | hiOff[j >> a.l];
       const bool live = idx < a.L_in;
       cp_async16(buf + j, a.psi + (live ? idx : 0), live ? 16 : 0);
     }
@@ -362,19 +424,32 @@ __device__ __forceinline__ void issue_tile_loads(double2* buf, const TileArgs& a
   asm volatile("cp.async.commit_group;\n" ::: "memory");
 }
 
-// The persistent tile loop shared by the interpreted and the JIT kernels: one CTA per SM, two
-// tile buffers (the loads of tile i+1 fly while tile i is computed in registers), per-tile
-// pattern constants and tile-uniform phase computed right after the tile lands.
+__device__ __forceinline__ void issue_tile_stores(double2* buf, const TileArgs& a, const uint64_t* hiOff,
+                                                  uint64_t base, int lane) {
+  const int nrun = 1 << (a.b - a.l);
+  const uint32_t bytes = 16u << a.l;
+  for (int h = lane; h < nrun; h += 32) bulk_s2g(a.psi + (base | hiOff[h]), buf + (uint64_t(h) << a.l), bytes);
+  bulk_commit();
+}
+
+// The persistent tile loop shared by the interpreted and the JIT kernels: one CTA (or two) per
+// SM, nbuf (3, else 2) tile buffers: the loads of tile i+1 fly while tile i is computed in
+// registers; tile i is written back while tile i+1 computes. Long contiguous runs (l >= 7)
+// move with bulk async copies issued by warp 0 (mbarrier-tracked loads, bulk-group stores);
+// short runs with per-thread cp.async / streaming stores. Per tile the pattern constants and
+// the tile-uniform phase are computed while the tile lands.
 // Body: void operator()(double2 (&v)[16], Mapping& mp, const TileCtx& c).
 template <int NR, class Body>
 __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
-  extern __shared__ __align__(16) unsigned char smem_raw[];
-  const int b = a.b, l = a.l, nw = a.nw;
+  extern __shared__ __align__(128) unsigned char smem_raw[];
+  const int b = a.b, l = a.l, nw = a.nw, nbuf = a.nbuf;
+  const bool bulk = a.bulk != 0;
   const uint32_t T = 1u << b;
   const int nh = 1 << (b - l);
   const int nthr = blockDim.x;
-  double2* bufs = reinterpret_cast<double2*>(smem_raw);  // 2 x T
-  uint64_t* hiOff = reinterpret_cast<uint64_t*>(bufs + 2 * T);
+  double2* bufs = reinterpret_cast<double2*>(smem_raw);             // nbuf x T
+  uint64_t* bars = reinterpret_cast<uint64_t*>(bufs + nbuf * T);    // 4 mbarriers
+  uint64_t* hiOff = bars + 4;
   unsigned char* blob = reinterpret_cast<unsigned char*>(hiOff + ((nh + 1) & ~1));
   const TileOp* ops = reinterpret_cast<const TileOp*>(blob);
   const RunEntry* ents = reinterpret_cast<const RunEntry*>(blob + a.off_entries);
@@ -396,10 +471,13 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       if (h >> (i - l) & 1) off |= 1ull << a.spos[i];
     hiOff[h] = off;
   }
+  if (threadIdx.x == 0) {
+    for (int q = 0; q < 4; ++q) mbar_init(&bars[q], 1);
+    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
+  }
   __syncthreads();
-  const uint32_t lowmask = (1u << l) - 1;
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
-  const int nld = (T + nthr - 1) / nthr;  // natural-order amplitudes per thread
+  const uint32_t lowmask = (1u << l) - 1;
   TileCtx c;
   c.ops = ops;
   c.ents = ents;
@@ -414,26 +492,42 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   c.own = lane < int(T);
 
   uint64_t tile = blockIdx.x;
-  if (tile < a.ntiles) issue_tile_loads(bufs, a, hiOff, tile, T, nthr, tid, nld, lowmask, l);
+  if (tile < a.ntiles) {
+    if (!bulk) issue_tile_loads_thr(bufs, a, hiOff, tile, T, nthr, tid);
+    else if (warp == 0) issue_tile_loads_bulk(bufs, &bars[0], a, hiOff, tile, lane);
+  }
+  int k = 0;
+  uint32_t phase = 0;  // mbarrier parity per buffer
   for (int it = 0; tile < a.ntiles; tile += gridDim.x, ++it) {
-    double2* s = bufs + (it & 1) * T;
+    double2* s = bufs + k * T;
+    const int kn = (k + 1 == nbuf) ? 0 : k + 1;
     const uint64_t base = tile_base(tile, a);
     const uint64_t gbase = a.rank_base | base;
-    cp_async_wait_all();
-    __syncthreads();  // tile `it` landed; the other buffer is free (previous store done)
-    if (tile + gridDim.x < a.ntiles)
-      issue_tile_loads(bufs + ((it + 1) & 1) * T, a, hiOff, tile + gridDim.x, T, nthr, tid, nld, lowmask, l);
-    for (int pi = tid; pi < a.npat; pi += nthr) {
+    // prefetch the next tile into buffer kn (its stores were issued nbuf-1 tiles ago)
+    const bool more = tile + gridDim.x < a.ntiles;
+    if (more) {
+      if (!bulk) {
+        issue_tile_loads_thr(bufs + kn * T, a, hiOff, tile + gridDim.x, T, nthr, tid);
+      } else if (warp == 0) {
+        if (nbuf >= 3) asm volatile("cp.async.bulk.wait_group.read 1;\n" ::: "memory");
+        else bulk_wait_read();
+        __syncwarp();
+        issue_tile_loads_bulk(bufs + kn * T, &bars[kn], a, hiOff, tile + gridDim.x, lane);
+      }
+    }
+    // pattern constants, spread over the warps (pattern pi -> warp pi % nwarps)
+    const int nwarps = nthr >> 5;
+    for (int pi = warp + nwarps * lane; pi < a.npat; pi += nthr) {
       double2 cc = make_double2(1.0, 0.0);
       const Pattern pt = pats[pi];
-      for (uint32_t k = pt.first; k < pt.first + pt.count; ++k)
-        if ((gbase & terms[k].omask) == terms[k].omatch) cc = cmul(cc, make_double2(terms[k].re, terms[k].im));
+      for (uint32_t q = pt.first; q < pt.first + pt.count; ++q)
+        if ((gbase & terms[q].omask) == terms[q].omatch) cc = cmul(cc, make_double2(terms[q].re, terms[q].im));
       C[pi] = cc;
     }
-    if (warp == 0) {
+    if (warp == nthr / 32 - 1) {  // the last warp: product of the tile-uniform phases
       double2 sc = make_double2(1.0, 0.0);
-      for (int k = lane; k < a.nscalar; k += 32)
-        if ((gbase & scal[k].omask) == scal[k].omatch) sc = cmul(sc, make_double2(scal[k].re, scal[k].im));
+      for (int q = lane; q < a.nscalar; q += 32)
+        if ((gbase & scal[q].omask) == scal[q].omatch) sc = cmul(sc, make_double2(scal[q].re, scal[q].im));
 #pragma unroll
       for (int o = 16; o > 0; o >>= 1) {
         double2 t;
@@ -443,27 +537,46 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       }
       if (lane == 0) *scal_s = sc;
     }
+    if (bulk) {
+      mbar_wait(&bars[k], (phase >> k) & 1u);  // tile `it` landed
+      phase ^= 1u << k;
+    } else {
+      if (more) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
+      else cp_async_wait_all();
+    }
+    __syncthreads();  // tile and constants visible to every thread
     c.s = s;
     c.gbase = gbase;
     double2 v[kRegAmps];
     Mapping mp = make_mapping<NR>(ops[0], nw, lane, warp);  // ops[0] is always OP_REMAP
     tile_reload<NR>(v, c, mp);
-    __syncthreads();  // constants visible
     body(v, mp, c);
-    // back to natural order, then store (times the tile-uniform phase)
-    tile_spill<NR>(v, c, mp);
+    // back to natural order (times the tile-uniform phase), then store
     const double2 sc = *scal_s;
-    const bool has_sc = !(sc.x == 1.0 && sc.y == 0.0);
+    if (!(sc.x == 1.0 && sc.y == 0.0)) {
 #pragma unroll
-    for (int r = 0; r < kRegAmps; ++r) {
-      const uint32_t j = uint32_t(tid) + uint32_t(r) * nthr;
-      if (r < nld && j < T) {
-        const double2 x = has_sc ? cmul(s[j], sc) : s[j];
-        st_stream(a.psi + (base | (j & lowmask) | hiOff[j >> l]), x);
+      for (int r = 0; r < (1 << NR); ++r) v[r] = cmul(v[r], sc);
+    }
+    // without remaps each thread writes back exactly the slots it read: no barrier needed
+    if (a.remaps) __syncthreads();
+#pragma unroll
+    for (int r = 0; r < (1 << NR); ++r)
+      if (c.own) s[mp.j(r)] = v[r];
+    if (bulk) {
+      fence_proxy_async();
+      __syncthreads();
+      if (warp == 0) issue_tile_stores(s, a, hiOff, base, lane);
+    } else {
+      __syncthreads();
+#pragma unroll
+      for (int r = 0; r < kRegAmps; ++r) {
+        const uint32_t j = uint32_t(tid) + uint32_t(r) * nthr;
+        if (j < T) st_stream(a.psi + (base | (j & lowmask) | hiOff[j >> l]), s[j]);
       }
     }
+    k = kn;
   }
-  cp_async_wait_all();
+  if (bulk && warp == 0) bulk_wait_all();
 }
 
 #endif  // __CUDACC__
