@@ -58,7 +58,10 @@ typedef struct {
   void* state_buffer;         /* optional caller-owned device memory (e.g. a torch tensor) */
   uint64_t state_buffer_bytes;/* its size; must be >= 16 * 2^(n - log2 world_size)          */
   int rank, world_size;       /* world_size = 2^g GPUs; 1 = single GPU                     */
-  const void* nccl_unique_id; /* 128-byte ncclUniqueId (world_size > 1), same on all ranks */
+  const void* nccl_unique_id; /* 128-byte ncclUniqueId (world_size > 1), same on all ranks.
+                                 NULL with world_size > 1: "virtual ranks" -- all 2^g shards
+                                 live in this process on `device` (tests the sharded path,
+                                 rank-bit conditions and swaps, on one GPU)               */
   int chunk_bits;             /* c: bitmap/pruning unit 2^c amplitudes;
                                  default 21, clamped to [0, n]                             */
   int prune;                  /* 1 (default): pruning + delayed involvement;
@@ -185,6 +188,17 @@ qgpu_status qgpu_circuit_reorder(const qgpu_circuit* c, int mode, uint64_t* orde
 qgpu_status qgpu_circuit_plan(const qgpu_circuit* c, int n_qubits, int world_size, int reorder,
                               int fuse_bits, int64_t* info, uint64_t cap, uint64_t* n_passes);
 
+/* Host-only (no GPU needed): the physical plan as text, for diagnostics and for executing the
+ * sharded protocol independently in tests. One line per pass
+ *   "P kind k_in k_out kg kg_from nswap g0 l0 g1 l1 ..." (kind as in qgpu_circuit_plan; 6 =
+ *   activation of ranks [2^kg_from, 2^kg); 5 = swap of rank bit positions g with local l),
+ * followed by one line per gate of the pass in physical positions at execution time
+ *   "G nt p0 p1 control_mask diag re im re im ..." (the (2^nt)^2 matrix, row-major),
+ * and a final "M pos_0 ... pos_{n-1}" with the final qubit map (-1 = never involved).
+ * Writes at most cap bytes (NUL-terminated); *len = bytes needed (without the NUL). */
+qgpu_status qgpu_circuit_plan_text(const qgpu_circuit* c, int n_qubits, int world_size, int reorder,
+                                   int fuse_bits, char* buf, size_t cap, size_t* len);
+
 /* Host-only (no GPU needed): generate the NVRTC-specialised kernel source of every fused pass of
  * the plan (as qgpu_circuit_plan) and compile it for sm_100a into the on-disk cubin cache
  * ($QGPU_JIT_CACHE, else <dir of libqgpu.so>/build/jitcache). *n_compiled = passes compiled.
@@ -215,6 +229,10 @@ qgpu_status qgpu_get_qubit_map(qgpu_state* st, int* pos);
 
 qgpu_status qgpu_get_stats(qgpu_state* st, qgpu_stats* out);
 qgpu_status qgpu_reset_stats(qgpu_state* st);
+
+/* Host: a fresh 128-byte ncclUniqueId (rank 0 creates it, the caller broadcasts it, e.g. with
+ * torch.distributed). UNSUPPORTED if libnccl.so.2 cannot be loaded ($QGPU_NCCL_LIB). */
+qgpu_status qgpu_nccl_unique_id(void* out, size_t len);
 
 /* Thread-local detail of the last error on this thread (valid until the next call). */
 const char* qgpu_last_error(void);

@@ -47,9 +47,17 @@ struct TimedLaunch {
 
 }  // namespace
 
+struct Shard {
+  int rank = 0;
+  double2* psi = nullptr;
+  bool own = false;
+};
+
 struct qgpu_state {
   qgpu_config cfg;
   int n = 0, g = 0, m = 0;
+  std::vector<Shard> shards;  // 1 per process (NCCL) or world_size (virtual ranks, one GPU)
+  bool virt = false;
   cudaStream_t stream = nullptr;
   bool own_stream = false;
   double2* psi = nullptr;
@@ -149,39 +157,57 @@ void sorted_positions(uint64_t mask, int* out, int* n) {
   for (; mask; mask &= mask - 1) out[(*n)++] = std::countr_zero(mask);
 }
 
-qgpu_status zero_fill(qgpu_state* st, uint64_t from, uint64_t to) {
-  if (to > from) CK(cudaMemsetAsync(st->psi + from, 0, (to - from) * sizeof(double2), st->stream));
+qgpu_status zero_fill(qgpu_state* st, double2* psi, uint64_t from, uint64_t to) {
+  if (to > from) CK(cudaMemsetAsync(psi + from, 0, (to - from) * sizeof(double2), st->stream));
   return QGPU_OK;
 }
 
-// Execute one planned pass on this rank's local buffer.
-qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops) {
+// Global-local swap (a10): exchange rank bit (swap_global - m) with local position swap_local,
+// one pair at a time. Virtual ranks: in-device swap of the two halves; NCCL: pack, send/recv with
+// the partner rank in slabs through bounded staging, unpack (in place: the received half lands
+// in the slots of the half that was sent).
+qgpu_status exec_swap(qgpu_state* st, const Pass& p, uint64_t* bytes) {
+  const int m = st->m;
+  const uint64_t half = 1ull << (m - 1);
+  const uint64_t active = 1ull << p.kg;
+  for (int i = 0; i < p.nswap; ++i) {
+    const int j = p.swap_global[i] - m, lp = p.swap_local[i];
+    if (st->virt) {
+      for (Shard& sh : st->shards) {
+        const uint64_t r = uint64_t(sh.rank);
+        if (r >= active || (r >> j & 1)) continue;
+        const uint64_t partner = r | (1ull << j);
+        CK(launch_swap_halves(st->stream, sh.psi, st->shards[partner].psi, lp, half));
+        st->stats.kernels_launched++;
+      }
+    } else {
+      for (Shard& sh : st->shards) {
+        if (uint64_t(sh.rank) >= active) continue;
+        qgpu_status s = comm_swap_bit(st->comm, sh.psi, m, sh.rank, j, lp, st->stream, &g_err);
+        if (s) {
+          st->poisoned = true;
+          return s;
+        }
+      }
+    }
+    *bytes += 16 * half;
+    st->stats.swaps++;
+    st->stats.swap_bytes += 16 * half;
+  }
+  return QGPU_OK;
+}
+
+// Execute one compute pass (tile / pair / quad / diag) on one rank's local buffer.
+qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_ops, double2* psi,
+                         uint64_t rank, uint64_t* bytes_out) {
   const int m = st->m;
   const uint64_t lmask = (m >= 64) ? ~0ull : ((1ull << m) - 1);
   const int kin = st->cfg.prune ? p.k_in : m, kout = st->cfg.prune ? p.k_out : m;
   const uint64_t L_in = 1ull << kin, L_out = 1ull << kout;
-  const bool timing = st->cfg.timing != 0;
-  TimedLaunch tl{};
   uint64_t bytes = 0;
-  if (p.kind == PK_RELABEL) {
-    if (kout > kin) {
-      qgpu_status s = zero_fill(st, L_in, L_out);
-      if (s) return s;
-      st->stats.kernels_launched++;
-      account(st, L_out, 16 * (L_out - L_in));
-    }
-    return QGPU_OK;
-  }
-  if (timing) {
-    tl.a = get_event(st);
-    tl.b = get_event(st);
-    tl.kind = p.kind;
-    CK(cudaEventRecord(tl.a, st->stream));
-  }
-  const uint64_t rank = uint64_t(st->cfg.rank);
   if (p.kind == PK_TILE) {
     TileArgs a{};
-    a.psi = st->psi;
+    a.psi = psi;
     const TileProgram& P = p.prog;
     a.blob = d_ops;
     a.blob_bytes = int(P.bytes);
@@ -236,21 +262,21 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops)
     const uint64_t lc = g.pc & lmask;
     if (!rank_ok) {
       // identity on this rank; the expanded region still has to read as zero
-      qgpu_status s = zero_fill(st, L_in, L_out);
+      qgpu_status s = zero_fill(st, psi, L_in, L_out);
       if (s) return s;
       bytes = 16 * (L_out - L_in);
     } else if (p.kind == PK_PAIR || p.kind == PK_QUAD) {
       const bool full = g.expands_target || !st->cfg.prune;
       const int krun = full ? kout : kin;
       if (!full) {
-        qgpu_status s = zero_fill(st, L_in, L_out);
+        qgpu_status s = zero_fill(st, psi, L_in, L_out);
         if (s) return s;
       }
       const int nlc = std::popcount(lc);
       const bool ctl_in_range = (lc >> krun) == 0;
       if (p.kind == PK_PAIR) {
         PairArgs a{};
-        a.psi = st->psi;
+        a.psi = psi;
         for (int i = 0; i < 4; ++i) a.u[i] = make_double2(g.U[i].re, g.U[i].im);
         a.t = g.p[0];
         sorted_positions(lc | (1ull << g.p[0]), a.ins, &a.nins);
@@ -263,7 +289,7 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops)
         bytes = 32 * a.npairs + (full ? 0 : 16 * (L_out - L_in));
       } else {
         QuadArgs a{};
-        a.psi = st->psi;
+        a.psi = psi;
         for (int i = 0; i < 16; ++i) a.u[i] = make_double2(g.U[i].re, g.U[i].im);
         a.t0 = g.p[0];
         a.t1 = g.p[1];
@@ -276,26 +302,39 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops)
       }
       st->stats.kernels_launched++;
     } else {  // PK_DIAG: the expanded region stays zero under a diagonal gate
-      qgpu_status s = zero_fill(st, L_in, L_out);
+      qgpu_status s = zero_fill(st, psi, L_in, L_out);
       if (s) return s;
       PhaseArgs a{};
-      a.psi = st->psi;
-      a.nt = g.nt;
-      a.t0 = g.p[0];
-      a.t1 = g.p[1];
+      a.psi = psi;
+      // targets on rank bits are fixed by this rank: keep the entries that match them
+      int lt[2], nlt = 0, gfix = 0, gsel = 0;
+      for (int j = 0; j < g.nt; ++j) {
+        if (g.p[j] >= m) {
+          gsel |= 1 << j;
+          if ((rank >> (g.p[j] - m)) & 1) gfix |= 1 << j;
+        } else {
+          lt[nlt++] = j;
+        }
+      }
+      a.nt = nlt;
+      a.t0 = nlt > 0 ? g.p[lt[0]] : 0;
+      a.t1 = nlt > 1 ? g.p[lt[1]] : 0;
       const int dim = 1 << g.nt;
       int n_not1 = 0, which = 0;
-      for (int v = 0; v < dim; ++v) {
+      for (int w = 0; w < (1 << nlt); ++w) {
+        int v = gfix;
+        for (int q = 0; q < nlt; ++q)
+          if (w >> q & 1) v |= 1 << lt[q];
         const cplx d = g.U[v * (dim + 1)];
-        a.d[v] = make_double2(d.re, d.im);
-        if (!(d.re == 1.0 && d.im == 0.0)) { ++n_not1; which = v; }
+        a.d[w] = make_double2(d.re, d.im);
+        if (!(d.re == 1.0 && d.im == 0.0)) { ++n_not1; which = w; }
       }
-      // TODO(sharded): targets on rank bits select the entry per rank
+      (void)gsel;
       uint64_t fixed = lc, insmask = lc;
       if (n_not1 == 1) {
-        for (int j = 0; j < g.nt; ++j) {
-          insmask |= 1ull << g.p[j];
-          if (which >> j & 1) fixed |= 1ull << g.p[j];
+        for (int q = 0; q < nlt; ++q) {
+          insmask |= 1ull << g.p[lt[q]];
+          if (which >> q & 1) fixed |= 1ull << g.p[lt[q]];
         }
       }
       a.fixed = fixed;
@@ -307,13 +346,69 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops)
       bytes = 32 * a.count + 16 * (L_out - L_in);
     }
   }
+  *bytes_out = bytes;
+  return QGPU_OK;
+}
+
+// Execute one planned pass: compute passes on every active local shard (ranks >= 2^kg hold
+// only zeros and skip the work), swaps through the communicator, activations as memsets.
+qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops) {
+  const int m = st->m;
+  const int kin = st->cfg.prune ? p.k_in : m, kout = st->cfg.prune ? p.k_out : m;
+  const uint64_t L_in = 1ull << kin, L_out = 1ull << kout;
+  const uint64_t active = 1ull << p.kg;
+  if (p.kind == PK_RELABEL) {
+    if (kout > kin) {
+      for (Shard& sh : st->shards)
+        if (uint64_t(sh.rank) < active) {
+          qgpu_status s = zero_fill(st, sh.psi, L_in, L_out);
+          if (s) return s;
+        }
+      st->stats.kernels_launched++;
+      account(st, L_out, 16 * (L_out - L_in));
+    }
+    return QGPU_OK;
+  }
+  if (p.kind == PK_ACTIVATE) {
+    for (Shard& sh : st->shards)
+      if (uint64_t(sh.rank) >= (1ull << p.kg_from) && uint64_t(sh.rank) < active) {
+        qgpu_status s = zero_fill(st, sh.psi, 0, 1ull << m);
+        if (s) return s;
+      }
+    return QGPU_OK;
+  }
+  const bool timing = st->cfg.timing != 0;
+  TimedLaunch tl{};
+  if (timing) {
+    tl.a = get_event(st);
+    tl.b = get_event(st);
+    tl.kind = p.kind;
+    CK(cudaEventRecord(tl.a, st->stream));
+  }
+  uint64_t bytes = 0;
+  if (p.kind == PK_SWAP) {
+    qgpu_status s = exec_swap(st, p, &bytes);
+    if (s) return s;
+  } else {
+    bool first = true;
+    for (Shard& sh : st->shards) {
+      if (uint64_t(sh.rank) >= active) continue;
+      uint64_t b = 0;
+      qgpu_status s = exec_compute(st, p, d_ops, sh.psi, uint64_t(sh.rank), &b);
+      if (s) return s;
+      if (first) bytes = b;
+      first = false;
+    }
+  }
   if (timing) {
     CK(cudaEventRecord(tl.b, st->stream));
     tl.bytes = bytes;
     st->pending.push_back(tl);
   }
-  account(st, L_out, bytes);
-  st->stats.unfused_bytes += p.unfused_bytes;
+  if (p.kind != PK_SWAP) {
+    account(st, L_out, bytes);
+    st->stats.unfused_bytes += p.unfused_bytes;
+  }
   return QGPU_OK;
 }
 
@@ -385,10 +480,12 @@ qgpu_status check_state(qgpu_state* st) {
 }
 
 qgpu_status init_amplitudes(qgpu_state* st) {
-  if (!st->cfg.prune) CK(cudaMemsetAsync(st->psi, 0, (1ull << st->m) * sizeof(double2), st->stream));
-  if (st->cfg.rank == 0) {
-    CK(launch_set_amp(st->stream, st->psi, 0, 1.0, 0.0));
-    st->stats.kernels_launched++;
+  for (Shard& sh : st->shards) {
+    if (!st->cfg.prune) CK(cudaMemsetAsync(sh.psi, 0, (1ull << st->m) * sizeof(double2), st->stream));
+    if (sh.rank == 0) {
+      CK(launch_set_amp(st->stream, sh.psi, 0, 1.0, 0.0));
+      st->stats.kernels_launched++;
+    }
   }
   return QGPU_OK;
 }
@@ -475,30 +572,41 @@ qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out
       st->own_stream = true;
     }
     const uint64_t need = (1ull << st->m) * sizeof(double2);
-    if (cfg.state_buffer) {
-      if (cfg.state_buffer_bytes < need)
-        return bail(fail(QGPU_ERR_OUT_OF_MEMORY, "state_buffer has %llu bytes, need %llu",
-                         (unsigned long long)cfg.state_buffer_bytes, (unsigned long long)need));
-      if (reinterpret_cast<uintptr_t>(cfg.state_buffer) % 16)
-        return bail(fail(QGPU_ERR_INVALID_ARG, "state_buffer must be 16-byte aligned"));
-      st->psi = static_cast<double2*>(cfg.state_buffer);
-    } else {
-      e = cudaMalloc(&st->psi, need);
-      if (e != cudaSuccess) {
-        cudaGetLastError();
-        return bail(fail(QGPU_ERR_OUT_OF_MEMORY, "cudaMalloc(%llu): %s", (unsigned long long)need,
-                         cudaGetErrorString(e)));
+    // world_size > 1 without an NCCL id: "virtual ranks", every shard in this process on this
+    // GPU (exercises the sharded path -- rank-bit conditions, activation, swaps -- on one GPU)
+    st->virt = cfg.world_size > 1 && cfg.nccl_unique_id == nullptr;
+    const int nshard = st->virt ? cfg.world_size : 1;
+    if (st->virt && cfg.state_buffer) return bail(fail(QGPU_ERR_UNSUPPORTED, "virtual ranks allocate their own shards"));
+    for (int r = 0; r < nshard; ++r) {
+      Shard sh;
+      sh.rank = st->virt ? r : cfg.rank;
+      if (cfg.state_buffer) {
+        if (cfg.state_buffer_bytes < need)
+          return bail(fail(QGPU_ERR_OUT_OF_MEMORY, "state_buffer has %llu bytes, need %llu",
+                           (unsigned long long)cfg.state_buffer_bytes, (unsigned long long)need));
+        if (reinterpret_cast<uintptr_t>(cfg.state_buffer) % 16)
+          return bail(fail(QGPU_ERR_INVALID_ARG, "state_buffer must be 16-byte aligned"));
+        sh.psi = static_cast<double2*>(cfg.state_buffer);
+      } else {
+        e = cudaMalloc(&sh.psi, need);
+        if (e != cudaSuccess) {
+          cudaGetLastError();
+          return bail(fail(QGPU_ERR_OUT_OF_MEMORY, "cudaMalloc(%llu): %s", (unsigned long long)need,
+                           cudaGetErrorString(e)));
+        }
+        sh.own = true;
       }
-      st->own_buf = true;
+      st->shards.push_back(sh);
     }
+    st->psi = st->shards[0].psi;
     st->cap_amps = 1ull << st->m;
     e = cudaMalloc(&st->d_zero, sizeof(double2) << kMaxTileBits);
     if (e == cudaSuccess) e = cudaMemset(st->d_zero, 0, sizeof(double2) << kMaxTileBits);
     if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "zero buffer: %s", cudaGetErrorString(e)));
     e = cudaEventCreateWithFlags(&st->ops_evt, cudaEventDisableTiming);
     if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e)));
-    if (cfg.world_size > 1) {
-      qgpu_status s = comm_create(&st->comm, cfg, st->stream, &g_err);
+    if (cfg.world_size > 1 && !st->virt) {
+      qgpu_status s = comm_create(&st->comm, cfg, st->stream, (1ull << st->m), &g_err);
       if (s) return bail(s);
     }
     qgpu_status s = init_amplitudes(st);
@@ -519,7 +627,8 @@ qgpu_status qgpu_state_destroy(qgpu_state* st) {
   }
   for (auto e : st->event_pool) cudaEventDestroy(e);
   if (st->comm) comm_destroy(st->comm);
-  if (st->own_buf && st->psi) cudaFree(st->psi);
+  for (Shard& sh : st->shards)
+    if (sh.own && sh.psi) cudaFree(sh.psi);
   if (st->d_ops) cudaFree(st->d_ops);
   if (st->h_ops) cudaFreeHost(st->h_ops);
   if (st->d_scratch) cudaFree(st->d_scratch);
@@ -546,6 +655,7 @@ qgpu_status qgpu_set_amplitudes(qgpu_state* st, const double* amps) {
   if (qgpu_status s = check_state(st)) return s;
   if (!amps) return fail(QGPU_ERR_INVALID_ARG, "amps is NULL");
   if (st->g > 0) return fail(QGPU_ERR_UNSUPPORTED, "set_amplitudes is single-GPU only");
+  st->psi = st->shards[0].psi;
   CK(cudaMemcpyAsync(st->psi, amps, (1ull << st->n) * sizeof(double2), cudaMemcpyHostToDevice, st->stream));
   CK(cudaStreamSynchronize(st->stream));
   st->map.init(st->n, st->m);
@@ -630,29 +740,37 @@ qgpu_status qgpu_get_amplitudes_device(qgpu_state* st, uint64_t start, uint64_t 
   if (start + count > (1ull << st->n) || start + count < start)
     return fail(QGPU_ERR_INVALID_ARG, "range [%llu, +%llu) outside 2^%d", (unsigned long long)start,
                 (unsigned long long)count, st->n);
-  if (st->g > 0) return fail(QGPU_ERR_UNSUPPORTED, "sharded get_amplitudes: use qgpu_get_amplitudes");
-  GatherArgs a{};
-  a.psi = st->psi;
-  a.out = reinterpret_cast<double2*>(dev_out);
-  a.start = start;
-  a.count = count;
-  a.n = st->n;
-  a.m = st->m;
-  a.rank = uint64_t(st->cfg.rank);
-  for (int q = 0; q < st->n; ++q) {
-    a.pos[q] = st->map.pos[q] < 0 ? 0 : st->map.pos[q];
-    if (st->map.pos[q] < 0) a.unassigned |= 1ull << q;
+  if (!count) return QGPU_OK;
+  const bool sharded = st->g > 0;
+  if (sharded) CK(cudaMemsetAsync(dev_out, 0, count * 2 * sizeof(double), st->stream));
+  for (Shard& sh : st->shards) {
+    if (sharded && (uint64_t(sh.rank) >> st->map.kg) != 0) continue;  // inactive: all zero
+    GatherArgs a{};
+    a.psi = sh.psi;
+    a.out = reinterpret_cast<double2*>(dev_out);
+    a.start = start;
+    a.count = count;
+    a.n = st->n;
+    a.m = st->m;
+    a.rank = uint64_t(sh.rank);
+    a.only_owned = sharded ? 1 : 0;
+    for (int q = 0; q < st->n; ++q) {
+      a.pos[q] = st->map.pos[q] < 0 ? 0 : st->map.pos[q];
+      if (st->map.pos[q] < 0) a.unassigned |= 1ull << q;
+    }
+    a.L = live(st, st->map.kl);
+    CK(launch_gather(st->stream, a));
+    st->stats.kernels_launched++;
   }
-  a.L = live(st, st->map.kl);
-  CK(launch_gather(st->stream, a));
-  st->stats.kernels_launched++;
+  if (sharded && st->comm) {  // every rank gets the full range (collective)
+    if (qgpu_status s = comm_allreduce_sum(st->comm, dev_out, count * 2, st->stream, &g_err)) return s;
+  }
   return QGPU_OK;
 }
 
 qgpu_status qgpu_get_amplitudes(qgpu_state* st, uint64_t start, uint64_t count, double* out) {
   if (qgpu_status s = check_state(st)) return s;
   if (!out && count) return fail(QGPU_ERR_INVALID_ARG, "out is NULL");
-  if (st->g > 0) return comm_get_amplitudes(st->comm, st, start, count, out);
   const uint64_t chunk = std::min<uint64_t>(count, 1ull << 24);
   if (chunk > st->scratch_cap / 2) {
     CK(cudaStreamSynchronize(st->stream));
@@ -676,23 +794,18 @@ qgpu_status qgpu_probabilities(qgpu_state* st, int mq, const int* qubits, double
   if (mq < 0 || mq > 30) return fail(QGPU_ERR_INVALID_ARG, "m=%d out of [0, 30]", mq);
   if (!out || (mq > 0 && !qubits)) return fail(QGPU_ERR_INVALID_ARG, "NULL argument");
   ProbArgs a{};
-  a.psi = st->psi;
   a.m = mq;
   uint64_t seen = 0;
-  uint64_t rank_fixed = 0;  // requested qubits on rank bits (sharded)
   for (int j = 0; j < mq; ++j) {
     const int q = qubits[j];
     if (q < 0 || q >= st->n || (seen >> q & 1)) return fail(QGPU_ERR_INVALID_ARG, "bad qubit %d", q);
     seen |= 1ull << q;
     const int p = st->map.pos[q];
     a.ppos[j] = (p < 0 || p >= st->m) ? 63 : p;
-    if (p >= st->m && (uint64_t(st->cfg.rank) >> (p - st->m) & 1)) rank_fixed |= 1ull << j;
   }
-  a.L = live(st, st->map.kl);
-  const bool active = st->g == 0 || (uint64_t(st->cfg.rank) >> st->map.kg) == 0;
-  if (!active) a.L = 0;
   const size_t B = size_t(1) << mq;
-  const size_t need = B + probs_scratch_doubles(mq);
+  const size_t nsh = st->shards.size();
+  const size_t need = B * (nsh > 1 ? 2 : 1) + probs_scratch_doubles(mq);
   if (need > st->scratch_cap) {
     CK(cudaStreamSynchronize(st->stream));
     if (st->d_scratch) CK(cudaFree(st->d_scratch));
@@ -700,17 +813,40 @@ qgpu_status qgpu_probabilities(qgpu_state* st, int mq, const int* qubits, double
     CK(cudaMalloc(&st->d_scratch, need * sizeof(double)));
     st->scratch_cap = need;
   }
-  a.out = st->d_scratch;
-  CK(launch_probs(st->stream, a, st->d_scratch + B));
-  st->stats.kernels_launched += (mq <= 12) ? 2 : 1;
-  if (st->g > 0) {
-    qgpu_status s = comm_probabilities_finish(st->comm, st->d_scratch, mq, rank_fixed, st->stream);
-    if (s) return s;
+  double* acc = st->d_scratch;
+  double* tmp = st->d_scratch + B;
+  double* part = st->d_scratch + B * (nsh > 1 ? 2 : 1);
+  for (size_t i = 0; i < nsh; ++i) {
+    const Shard& sh = st->shards[i];
+    ProbArgs pa = a;
+    pa.psi = sh.psi;
+    pa.yfixed = 0;
+    for (int j = 0; j < mq; ++j) {  // requested qubits on rank bits: fixed by this rank
+      const int p = st->map.pos[qubits[j]];
+      if (p >= st->m && ((uint64_t(sh.rank) >> (p - st->m)) & 1)) pa.yfixed |= 1ull << j;
+    }
+    const bool active = st->g == 0 || (uint64_t(sh.rank) >> st->map.kg) == 0;
+    pa.L = active ? live(st, st->map.kl) : 0;
+    pa.out = i == 0 ? acc : tmp;
+    CK(launch_probs(st->stream, pa, part));
+    st->stats.kernels_launched += (mq <= 12) ? 2 : 1;
+    if (i > 0) CK(launch_add(st->stream, acc, tmp, B));
   }
-  CK(cudaMemcpyAsync(out, st->d_scratch, B * sizeof(double), cudaMemcpyDeviceToHost, st->stream));
+  if (st->comm) {
+    if (qgpu_status s = comm_allreduce_sum(st->comm, acc, B, st->stream, &g_err)) return s;
+  }
+  CK(cudaMemcpyAsync(out, acc, B * sizeof(double), cudaMemcpyDeviceToHost, st->stream));
   st->stats.d2h_bytes += B * sizeof(double);
   CK(cudaStreamSynchronize(st->stream));
   return drain_timing(st);
+}
+
+qgpu_status qgpu_nccl_unique_id(void* out, size_t len) {
+  if (!out || len < 128) return fail(QGPU_ERR_INVALID_ARG, "need a 128-byte buffer");
+  std::string err;
+  qgpu_status s = comm_unique_id(out, &err);
+  if (s) return fail(s, "%s", err.c_str());
+  return QGPU_OK;
 }
 
 qgpu_status qgpu_circuit_from_qasm(const char* text, size_t len, qgpu_circuit** out) {
@@ -779,6 +915,57 @@ qgpu_status qgpu_circuit_plan(const qgpu_circuit* c, int n, int world, int reord
       r[0] = p.first; r[1] = p.count; r[2] = p.kind; r[3] = p.k_in; r[4] = p.k_out; r[5] = p.b;
       r[6] = int64_t(S & 0xffffffffull);
       r[7] = int64_t(S >> 32);
+    }
+    return QGPU_OK;
+  } catch (const std::exception& ex) {
+    return fail(QGPU_ERR_OUT_OF_MEMORY, "exception: %s", ex.what());
+  }
+}
+
+qgpu_status qgpu_circuit_plan_text(const qgpu_circuit* c, int n, int world, int reorder_mode, int fuse_bits,
+                                   char* buf, size_t cap, size_t* len) {
+  try {
+    if (!c) return fail(QGPU_ERR_INVALID_ARG, "circuit is NULL");
+    if (n < c->c.n || n > kMaxQubits) return fail(QGPU_ERR_INVALID_ARG, "bad n");
+    if (world < 1 || (world & (world - 1))) return fail(QGPU_ERR_INVALID_ARG, "bad world size");
+    const int g = std::countr_zero(unsigned(world));
+    if (n - g < 3) return fail(QGPU_ERR_INVALID_ARG, "too few local qubits");
+    QubitMap map;
+    map.init(n, n - g);
+    PlanOptions o;
+    o.fuse_bits = fuse_bits;
+    std::vector<Pass> passes;
+    plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode), map, o, &passes, nullptr);
+    std::string t;
+    char line[512];
+    for (const Pass& p : passes) {
+      std::snprintf(line, sizeof(line), "P %d %d %d %d %d %d", p.kind, p.k_in, p.k_out, p.kg, p.kg_from, p.nswap);
+      t += line;
+      for (int i = 0; i < p.nswap; ++i) {
+        std::snprintf(line, sizeof(line), " %d %d", p.swap_global[i], p.swap_local[i]);
+        t += line;
+      }
+      t += "\n";
+      for (const PhysGate& pg : p.gates) {
+        std::snprintf(line, sizeof(line), "G %d %d %d %llu %d", pg.nt, pg.p[0], pg.p[1],
+                      static_cast<unsigned long long>(pg.pc), pg.diag ? 1 : 0);
+        t += line;
+        const int dim = 1 << pg.nt;
+        for (int e = 0; e < dim * dim; ++e) {
+          std::snprintf(line, sizeof(line), " %.17g %.17g", pg.U[e].re, pg.U[e].im);
+          t += line;
+        }
+        t += "\n";
+      }
+    }
+    t += "M";
+    for (int q = 0; q < n; ++q) t += " " + std::to_string(map.pos[q]);
+    t += "\n";
+    if (len) *len = t.size();
+    if (buf && cap) {
+      const size_t k = std::min(cap - 1, t.size());
+      std::memcpy(buf, t.data(), k);
+      buf[k] = 0;
     }
     return QGPU_OK;
   } catch (const std::exception& ex) {

@@ -243,8 +243,13 @@ __global__ void gather_kernel(GatherArgs a) {
       uint64_t phys = 0;
       for (int q = 0; q < a.n; ++q)
         if (X >> q & 1) phys |= 1ull << a.pos[q];
-      if ((phys >> a.m) == a.rank && (phys & ((1ull << a.m) - 1)) < a.L)
-        v = a.psi[phys & ((1ull << a.m) - 1)];
+      if ((phys >> a.m) == a.rank) {
+        if ((phys & ((1ull << a.m) - 1)) < a.L) v = a.psi[phys & ((1ull << a.m) - 1)];
+      } else if (a.only_owned) {
+        continue;
+      }
+    } else if (a.only_owned) {
+      continue;
     }
     a.out[x] = v;
   }
@@ -260,7 +265,7 @@ __global__ void __launch_bounds__(kThreads) probs_block_kernel(ProbArgs a) {
   const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
   for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < a.L; i += stride) {
     const double2 v = a.psi[i];
-    uint32_t y = 0;
+    uint32_t y = uint32_t(a.yfixed);
     for (int j = 0; j < a.m; ++j) y |= uint32_t((i >> a.ppos[j]) & 1) << j;
     atomicAdd(&hist[y], v.x * v.x + v.y * v.y);
   }
@@ -280,13 +285,40 @@ __global__ void probs_global_kernel(ProbArgs a) {
   const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
   for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < a.L; i += stride) {
     const double2 v = a.psi[i];
-    uint64_t y = 0;
+    uint64_t y = a.yfixed;
     for (int j = 0; j < a.m; ++j) y |= ((i >> a.ppos[j]) & 1) << j;
     atomicAdd(&a.out[y], v.x * v.x + v.y * v.y);
   }
 }
 
 __global__ void set_amp_kernel(double2* psi, uint64_t i, double2 v) { psi[i] = v; }
+
+// a10 (virtual ranks): exchange the lp=1 half of shard a with the lp=0 half of shard b
+__global__ void swap_halves_kernel(double2* a, double2* b, int lp, uint64_t half) {
+  const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+  for (uint64_t t = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < half; t += stride) {
+    const uint64_t i0 = insert0(t, lp);
+    const uint64_t ia = i0 | (1ull << lp);
+    const double2 x = __ldcs(a + ia), y = __ldcs(b + i0);
+    __stcs(a + ia, y);
+    __stcs(b + i0, x);
+  }
+}
+// a10 (NCCL): gather / scatter slab [t0, t0+count) of the half with local bit lp == bit
+__global__ void pack_half_kernel(const double2* psi, double2* buf, int lp, int bit, uint64_t t0, uint64_t count) {
+  const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+  for (uint64_t t = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < count; t += stride)
+    buf[t] = __ldcs(psi + (insert0(t0 + t, lp) | (uint64_t(bit) << lp)));
+}
+__global__ void unpack_half_kernel(double2* psi, const double2* buf, int lp, int bit, uint64_t t0, uint64_t count) {
+  const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+  for (uint64_t t = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < count; t += stride)
+    __stcs(psi + (insert0(t0 + t, lp) | (uint64_t(bit) << lp)), buf[t]);
+}
+__global__ void add_kernel(double* out, const double* in, uint64_t count) {
+  const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+  for (uint64_t t = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < count; t += stride) out[t] += in[t];
+}
 
 // --------------------------------------------------------------------------- launchers
 namespace {
@@ -405,6 +437,26 @@ cudaError_t launch_probs(cudaStream_t st, ProbArgs a, double* scratch) {
   if (a.L == 0) return cudaSuccess;
   const unsigned g = grid_for(a.L, 256, 8);
   probs_global_kernel<<<g, 256, 0, st>>>(a);
+  return cudaGetLastError();
+}
+
+cudaError_t launch_swap_halves(cudaStream_t st, double2* a, double2* b, int lp, uint64_t half) {
+  swap_halves_kernel<<<grid_for(half, 256 * 4, 8), 256, 0, st>>>(a, b, lp, half);
+  return cudaGetLastError();
+}
+cudaError_t launch_pack_half(cudaStream_t st, const double2* psi, double2* buf, int lp, int bit, uint64_t t0,
+                             uint64_t count) {
+  pack_half_kernel<<<grid_for(count, 256 * 4, 8), 256, 0, st>>>(psi, buf, lp, bit, t0, count);
+  return cudaGetLastError();
+}
+cudaError_t launch_unpack_half(cudaStream_t st, double2* psi, const double2* buf, int lp, int bit, uint64_t t0,
+                               uint64_t count) {
+  unpack_half_kernel<<<grid_for(count, 256 * 4, 8), 256, 0, st>>>(psi, buf, lp, bit, t0, count);
+  return cudaGetLastError();
+}
+cudaError_t launch_add(cudaStream_t st, double* out, const double* in, uint64_t count) {
+  if (!count) return cudaSuccess;
+  add_kernel<<<grid_for(count, 256 * 4, 8), 256, 0, st>>>(out, in, count);
   return cudaGetLastError();
 }
 

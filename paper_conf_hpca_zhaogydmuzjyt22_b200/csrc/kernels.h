@@ -50,6 +50,7 @@ struct GatherArgs {
   int pos[kMaxQubits];
   uint64_t unassigned;     // logical qubits never involved (their |1> half is zero)
   uint64_t L;              // live local size
+  int only_owned;          // sharded: write only the amplitudes this rank owns
 };
 
 struct ProbArgs {
@@ -57,6 +58,7 @@ struct ProbArgs {
   uint64_t L;
   int m;
   int ppos[32];            // physical position of each requested qubit (63 = never set)
+  uint64_t yfixed;         // bucket bits given by this rank's bits (requested qubits on rank bits)
   double* out;
   double* partial;
 };
@@ -71,5 +73,12 @@ cudaError_t launch_tile(cudaStream_t st, const TileArgs& a);
 cudaError_t launch_gather(cudaStream_t st, const GatherArgs& a);
 cudaError_t launch_probs(cudaStream_t st, ProbArgs a, double* scratch);
 cudaError_t launch_set_amp(cudaStream_t st, double2* psi, uint64_t i, double re, double im);
+// sharded swaps (a10)
+cudaError_t launch_swap_halves(cudaStream_t st, double2* a, double2* b, int lp, uint64_t half);
+cudaError_t launch_pack_half(cudaStream_t st, const double2* psi, double2* buf, int lp, int bit, uint64_t t0,
+                             uint64_t count);
+cudaError_t launch_unpack_half(cudaStream_t st, double2* psi, const double2* buf, int lp, int bit, uint64_t t0,
+                               uint64_t count);
+cudaError_t launch_add(cudaStream_t st, double* out, const double* in, uint64_t count);
 
 }  // namespace qgpu

@@ -107,7 +107,8 @@ struct PhysGate {
 };
 
 enum PassKind : int {
-  PK_TILE = 0, PK_PAIR = 1, PK_QUAD = 2, PK_DIAG = 3, PK_RELABEL = 4, PK_SWAP = 5
+  PK_TILE = 0, PK_PAIR = 1, PK_QUAD = 2, PK_DIAG = 3, PK_RELABEL = 4, PK_SWAP = 5,
+  PK_ACTIVATE = 6  // ranks [2^kg_from, 2^kg) become active (their buffers are zeroed)
 };
 
 struct Pass {
@@ -120,9 +121,11 @@ struct Pass {
   std::vector<PhysGate> gates;  // gates of the pass (tile) or the single gate (pair/quad/diag)
   TileProgram prog;             // built at pass close (tile)
   int n_est = 0;                // op-count estimate while the pass is open
-  // swap pass (sharded)
+  int kg = 0;                   // active ranks 2^kg while the pass runs (sharded)
+  // swap pass (sharded): exchange global positions swap_global[i] with local swap_local[i]
   int nswap = 0;
   int swap_global[8], swap_local[8];
+  int kg_from = 0;              // activation pass
   uint64_t unfused_bytes = 0;   // bytes the pass's gates would move one gate per pass
 };
 

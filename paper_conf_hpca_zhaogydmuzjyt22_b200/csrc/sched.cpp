@@ -502,6 +502,7 @@ struct Builder {
     cur.first = first;
     cur.k_in = k_in;
     cur.k_out = k_in;
+    cur.kg = map.kg;
     open = true;
     used = 0;
     n_u = 0;
@@ -523,12 +524,23 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
                   std::vector<uint64_t>* inv_after) {
   Builder B{gates, map, opt, passes};
   const bool fuse = opt.fuse_bits > 0;
+  const int m = map.m;
   for (int k = 0; k < int(order.size()); ++k) {
     const Gate& g = gates[order[k]];
     const int k_before = map.kl;
+    const int kg_before = map.kg;
     const uint64_t fresh = g.qmask() & ~map.involvement;
     map.touch(g.qmask());
     if (inv_after) inv_after->push_back(map.involvement);
+    if (map.kg > kg_before) {
+      // sharded: a qubit was placed on a rank bit; the ranks that become active hold zeros
+      B.close();
+      B.start(PK_ACTIVATE, k, k_before);
+      B.cur.kg_from = kg_before;
+      B.cur.kg = map.kg;
+      B.cur.k_out = map.kl;
+      B.close();
+    }
     if (g.relabel) {
       const int pa = map.pos[g.t[0]], pb = map.pos[g.t[1]];
       if (fuse && B.open && B.cur.kind == PK_TILE) {
@@ -546,6 +558,33 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
       B.close();
       continue;
     }
+    if (!g.diag) {
+      // a non-diagonal target on a rank bit: swap it with a local position first (a10).
+      // Victims: the highest local positions that are not targets of this gate.
+      int gl[2], ng = 0;
+      uint64_t tloc = 0;
+      for (int j = 0; j < g.nt; ++j) {
+        const int p = map.pos[g.t[j]];
+        if (p >= m) gl[ng++] = p;
+        else tloc |= 1ull << p;
+      }
+      if (ng) {
+        B.close();
+        B.start(PK_SWAP, k, map.kl);
+        B.cur.count = 0;
+        int victim = m - 1;
+        for (int j = 0; j < ng; ++j) {
+          while (tloc >> victim & 1) --victim;
+          B.cur.swap_global[j] = gl[j];
+          B.cur.swap_local[j] = victim;
+          --victim;
+        }
+        B.cur.nswap = ng;
+        for (int j = 0; j < ng; ++j) map.swap_positions(B.cur.swap_global[j], B.cur.swap_local[j]);
+        B.cur.k_out = map.kl;
+        B.close();
+      }
+    }
     PhysGate pg;
     pg.gate = order[k];
     pg.nt = g.nt;
@@ -555,7 +594,6 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
     std::memcpy(pg.U, g.U, sizeof(g.U));
     pg.diag = g.diag;
     pg.expands_target = (g.tmask() & fresh) != 0;
-    // TODO(sharded): swap planning for non-diagonal targets on global positions
     if (fuse) {
       uint64_t need = 0;
       if (!g.diag) {

@@ -24,9 +24,9 @@ EXPORTS = [
     "qgpu_set_amplitudes", "qgpu_synchronize", "qgpu_state_info", "qgpu_apply_gate",
     "qgpu_apply_circuit", "qgpu_get_amplitudes", "qgpu_get_amplitudes_device",
     "qgpu_probabilities", "qgpu_circuit_from_qasm", "qgpu_circuit_info", "qgpu_circuit_destroy",
-    "qgpu_circuit_reorder", "qgpu_circuit_plan", "qgpu_circuit_jit_check", "qgpu_get_involvement", "qgpu_get_chunk_bitmap",
+    "qgpu_circuit_reorder", "qgpu_circuit_plan", "qgpu_circuit_plan_text", "qgpu_circuit_jit_check", "qgpu_get_involvement", "qgpu_get_chunk_bitmap",
     "qgpu_get_schedule", "qgpu_get_qubit_map", "qgpu_get_stats", "qgpu_reset_stats",
-    "qgpu_last_error", "qgpu_version",
+    "qgpu_nccl_unique_id", "qgpu_last_error", "qgpu_version",
 ]
 
 
@@ -84,9 +84,11 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
         "qgpu_circuit_info": [P, P, P], "qgpu_circuit_destroy": [P],
         "qgpu_circuit_reorder": [P, I, P, U64, P], "qgpu_circuit_plan": [P, I, I, I, I, P, U64, P],
         "qgpu_circuit_jit_check": [P, I, I, I, P],
+        "qgpu_circuit_plan_text": [P, I, I, I, I, P, ctypes.c_size_t, P],
         "qgpu_get_involvement": [P, P], "qgpu_get_chunk_bitmap": [P, I, P, U64],
         "qgpu_get_schedule": [P, P, P, U64, P], "qgpu_get_qubit_map": [P, P],
         "qgpu_get_stats": [P, P], "qgpu_reset_stats": [P],
+        "qgpu_nccl_unique_id": [P, ctypes.c_size_t],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -151,6 +153,15 @@ class Circuit:
                                         info.ctypes.data, cnt.value, ctypes.byref(cnt)))
         return info[:cnt.value]
 
+    def plan_text(self, n: int, world_size: int = 1, reorder: int = 2, fuse_bits: int = 12) -> str:
+        ln = ctypes.c_size_t()
+        _check(load().qgpu_circuit_plan_text(self._h, n, world_size, reorder, fuse_bits, None, 0,
+                                             ctypes.byref(ln)))
+        buf = ctypes.create_string_buffer(ln.value + 1)
+        _check(load().qgpu_circuit_plan_text(self._h, n, world_size, reorder, fuse_bits, buf,
+                                             ln.value + 1, ctypes.byref(ln)))
+        return buf.value.decode()
+
     def jit_check(self, n: int, reorder: int = 2, fuse_bits: int = 12) -> int:
         """Compile the NVRTC-specialised kernel of every fused pass (no GPU needed)."""
         k = ctypes.c_int()
@@ -174,6 +185,8 @@ class State:
 
     def __init__(self, n: int, cfg: Optional[Config] = None, **kw):
         lib = load()
+        if kw.get("nccl_unique_id") is not None and "QGPU_NCCL_LIB" not in os.environ and _nccl_lib_path():
+            os.environ["QGPU_NCCL_LIB"] = _nccl_lib_path()
         self.cfg = cfg if cfg is not None else config(**kw)
         self._h = ctypes.c_void_p()
         _check(lib.qgpu_state_create(n, ctypes.byref(self.cfg), ctypes.byref(self._h)))
@@ -276,6 +289,27 @@ class State:
 
     def reset_stats(self):
         _check(load().qgpu_reset_stats(self._h))
+
+
+def _nccl_lib_path():
+    try:
+        import nvidia.nccl
+        for d in nvidia.nccl.__path__:
+            p = os.path.join(d, "lib", "libnccl.so.2")
+            if os.path.exists(p):
+                return p
+    except Exception:
+        pass
+    return None
+
+
+def nccl_unique_id() -> bytes:
+    """A fresh ncclUniqueId (128 bytes) to broadcast from rank 0 (torch.distributed)."""
+    if "QGPU_NCCL_LIB" not in os.environ and _nccl_lib_path():
+        os.environ["QGPU_NCCL_LIB"] = _nccl_lib_path()
+    buf = ctypes.create_string_buffer(128)
+    _check(load().qgpu_nccl_unique_id(buf, 128))
+    return buf.raw
 
 
 def version() -> str:
