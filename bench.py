@@ -10,7 +10,9 @@ is circuit seconds (lower is better). See DESIGN.md §7 for the byte model and p
     python bench.py --impl reference ...     # the oracle (plain CPU simulator) as the baseline arm
 
 N > 1 (torchrun): each rank runs its own replica of the workload (weak scaling, no data-path
-collective; the sharded path is DESIGN.md §8), timed on the device, max over ranks.
+collective), timed on the device, max over ranks. With --sharded one state is sharded over the N
+ranks (top log2 N qubits on rank bits, global-local swaps over NCCL; configs[3]: --workload rqc
+--n 34 --sharded), strong scaling.
 """
 from __future__ import annotations
 
@@ -154,8 +156,6 @@ def oracle_sample(text: str, budget_s: float, start_gate: int = 0, max_gates: in
     n, gates = oq.parse(text)
     threads = osv.default_threads()
     psi = osv.zero_state(n)
-    for i in range(min(start_gate, len(gates))):
-        pass  # the sample always starts from |0...0>: every oracle gate visits all 2^n indices
     t0 = time.perf_counter()
     done = 0
     while done < len(gates) and (time.perf_counter() - t0) < budget_s:
@@ -251,6 +251,14 @@ def run_ours(args):
     stream = torch.cuda.Stream(device=device)
     cfg = dict(device=local, stream=stream.cuda_stream, fuse_bits=args.fuse_bits, reorder=args.reorder,
                prune=int(not args.no_prune), timing=1)
+    sharded = args.sharded and world > 1
+    if sharded:
+        # one state sharded over the ranks: top log2(N) qubits on rank bits, global-local swaps
+        # over NCCL (a10); the ncclUniqueId goes from rank 0 to all ranks through torch
+        import torch.distributed as dist
+        obj = [q.nccl_unique_id() if rank == 0 else None]
+        dist.broadcast_object_list(obj, src=0)
+        cfg.update(world_size=world, rank=rank, nccl_unique_id=obj[0])
     st = q.State(n, **cfg)
     c = q.Circuit(text)
     ngates = c.info()[1]
@@ -327,11 +335,14 @@ def run_ours(args):
     launches = s0["kernels_launched"]
     line = {
         "metric": METRIC, "value": ms / 1e3, "unit": "s", "n_gpus": world, "steps": args.steps,
-        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False, "scaling": "weak",
+        "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False,
+        "scaling": "strong" if sharded else "weak",
         "vs_baseline": None, "dtype": "c128", "data": "synthetic (seeded generator, QASM text)",
         "config": {"workload": desc, "n_qubits": n, "gates": ngates, "reorder": args.reorder,
                    "prune": int(not args.no_prune), "fuse_bits": args.fuse_bits,
-                   "replicas_per_gpu": 1, "parallelism": f"replicas x{world}" if world > 1 else "1 GPU",
+                   "replicas_per_gpu": 0 if sharded else 1,
+                   "parallelism": (f"sharded x{world} (NCCL global-local swaps)" if sharded else
+                                   f"replicas x{world}" if world > 1 else "1 GPU"),
                    "l2": "flushed between timed steps (256 MiB write) and state 16*2^n B > L2"},
         "roofline": {"kernel": "tile_kernel (fused pass)", "bound": "hbm", "achieved": achieved,
                      "peak": peak, "unit": "GB/s", "frac": achieved / peak, "traffic": traffic,
@@ -393,6 +404,8 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=20.0)
     ap.add_argument("--ref-step-seconds", type=float, default=8.0)
     ap.add_argument("--ref-gates", type=int, default=None)
+    ap.add_argument("--sharded", action="store_true",
+                    help="N>1: shard one state over the ranks (NCCL swaps) instead of N replicas")
     args = ap.parse_args()
     if args.warmup < 3:
         args.warmup = 3

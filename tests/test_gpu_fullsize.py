@@ -1,0 +1,106 @@
+"""Parity at BASELINE.json's full sizes, in the configuration bench.py times (reorder=2,
+prune=1, fused b=12, NVRTC-specialised kernels): closed forms checked on the whole state or on
+sampled ranges, full oracle comparison where the oracle finishes in seconds (28 qubits), and
+properties that hold at any size (norm, mirror U U^dagger = I)."""
+import math
+
+import numpy as np
+import pytest
+
+from oracle import statevector as osv
+from workloads import circuits as wc
+
+pytestmark = [pytest.mark.gpu, pytest.mark.slow]
+
+TOL = 1e-10
+
+
+@pytest.fixture(scope="module")
+def q():
+    import torch
+    if not torch.cuda.is_available():
+        pytest.skip("no CUDA device")
+    from paper_conf_hpca_zhaogydmuzjyt22_b200 import build, qgpu
+    build.build()
+    qgpu.load()
+    return qgpu
+
+
+def test_c2_qft28_basis_state_full_state(q):
+    """configs[1]: QFT_28 on |x> (x from rng seed 2); every amplitude vs e^{2 pi i x y / 2^n} / 2^{n/2}."""
+    c = wc.config_circuit("C2x")
+    n, x = c.n, c.meta["x"]
+    with q.State(n) as s:
+        s.apply_circuit(q.Circuit(c.qasm()))
+        worst = 0.0
+        step = 1 << 24
+        for start in range(0, 1 << n, step):
+            got = s.amplitudes(start, step)
+            y = np.arange(start, start + step, dtype=np.int64)
+            ph = ((x * y) % (1 << n)).astype(np.float64) / (1 << n)
+            exp = np.exp(2j * np.pi * ph) / math.sqrt(1 << n)
+            worst = max(worst, float(np.abs(got - exp).max()))
+        p = s.probabilities([])
+    assert worst <= TOL
+    assert abs(p[0] - 1) <= 1e-12
+
+
+def test_c2_qft28_zero_state_and_stats(q):
+    c = wc.qft(28)
+    with q.State(28, chunk_bits=21) as s:
+        s.apply_circuit(q.Circuit(c.qasm()))
+        a = s.amplitudes(0, 1 << 20)
+        b = s.amplitudes((1 << 28) - (1 << 20), 1 << 20)
+        st = s.stats()
+    u = 1 / math.sqrt(1 << 28)
+    assert np.abs(a - u).max() <= TOL and np.abs(b - u).max() <= TOL
+    assert st["chunks_skipped"] > 0 and st["ops_before_full_involvement"] > 300
+
+
+def test_qaoa28_vs_oracle_full(q):
+    c = wc.qaoa(28, 2, seed=1)
+    text = c.qasm()
+    with q.State(c.n) as s:
+        s.apply_circuit(q.Circuit(text))
+        got = s.amplitudes()
+    ref = osv.simulate(text)
+    assert np.abs(got - ref).max() <= TOL
+
+
+def test_c3_qaoa32_norm_mirror_and_marginals(q):
+    """configs[2]: QAOA MaxCut p=2 at 32 qubits (64 GiB): norm, marginal symmetry of MaxCut
+    (global bit flip: p(y) = p(~y) on any qubit subset), and the mirror returns |0>."""
+    c = wc.config_circuit("C3")
+    with q.State(c.n) as s:
+        s.apply_circuit(q.Circuit(c.qasm()))
+        p = s.probabilities(list(range(8)))
+        assert abs(p.sum() - 1) <= 1e-12
+        assert np.abs(p - p[::-1]).max() <= 1e-12
+        s.reset()
+        s.apply_circuit(q.Circuit(wc.mirror(c).qasm()))
+        a = s.amplitudes(0, 4096)
+    assert abs(a[0] - 1) <= TOL and np.abs(a[1:]).max() <= TOL
+
+
+def test_rqc30_mirror(q):
+    c = wc.rqc(30, 20, seed=3)
+    with q.State(c.n) as s:
+        s.apply_circuit(q.Circuit(wc.mirror(c).qasm()))
+        a = s.amplitudes(0, 4096)
+        p = s.probabilities([])
+    assert abs(a[0] - 1) <= TOL and np.abs(a[1:]).max() <= TOL
+    assert abs(p[0] - 1) <= 1e-12
+
+
+def test_graph_state_30_sampled_ranges(q):
+    c = wc.gs(5, 6)
+    n, edges = c.n, c.meta["edges"]
+    with q.State(n) as s:
+        s.apply_circuit(q.Circuit(c.qasm()))
+        for start in (0, 123456789, (1 << n) - (1 << 16)):
+            got = s.amplitudes(start, 1 << 16)
+            xs = np.arange(start, start + (1 << 16), dtype=np.int64)
+            par = np.zeros_like(xs)
+            for u, v in edges:
+                par ^= ((xs >> u) & 1) & ((xs >> v) & 1)
+            assert np.abs(got - (1 - 2 * par) / math.sqrt(1 << n)).max() <= TOL
