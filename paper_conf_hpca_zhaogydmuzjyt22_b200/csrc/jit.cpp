@@ -174,22 +174,50 @@ bool jit_cubin_cached(const std::string& src, std::string* cubin, std::string* l
 std::string tile_jit_source(const Pass& p) {
   const TileProgram& P = p.prog;
   const int NR = P.nr;
+  // compile-time zero tracking (first-touch expansion, a5): tile bits whose physical position
+  // is >= k_in hold zeros until a non-diagonal op targets them
+  uint32_t zpos = 0;
+  for (int i = 0; i < p.b; ++i)
+    if (p.spos[i] >= p.k_in) zpos |= 1u << i;
+  int R[4] = {0, 0, 0, 0};
+  auto decode = [&](const TileOp& op) {
+    for (int k = 0; k < 4; ++k) R[k] = (op.a0 >> (4 * k)) & 15;
+  };
+  auto zmask = [&]() {
+    unsigned zm = 0;
+    for (int r = 0; r < (1 << NR); ++r)
+      for (int k = 0; k < NR; ++k)
+        if ((r >> k & 1) && (zpos >> R[k] & 1)) zm |= 1u << r;
+    return zm;
+  };
+  decode(P.ops[0]);
   std::ostringstream o;
-  o << "// qgpu tile pass: b=" << p.b << " nr=" << NR << " nw=" << P.nw << " ops=" << P.ops.size() << "\n";
+  o << "// qgpu tile pass: b=" << p.b << " nr=" << NR << " nw=" << P.nw << " ops=" << P.ops.size()
+    << " k_in=" << p.k_in << "\n";
   o << "#include \"tile_common.cuh\"\n";
   o << "using namespace qgpu;\n";
   o << "struct JitBody {\n";
   o << "  __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c) const {\n";
   o << "    const TileOp* ops = c.ops;\n";
+  {
+    const unsigned zm = zmask();
+    if (zm) {  // the initial reload read these slots from the zero region: make them exact zeros
+      o << "    {";
+      for (int r = 0; r < (1 << NR); ++r)
+        if (zm >> r & 1) o << " v[" << r << "] = make_double2(0.0, 0.0);";
+      o << " }\n";
+    }
+  }
   for (size_t i = 1; i < P.ops.size(); ++i) {
     const TileOp& op = P.ops[i];
     const bool uni = op.omask != 0;       // tile-uniform condition present
     const bool thr = op.tmask != 0;       // condition on the thread's fixed bits present
+    const unsigned zm = zmask();
     o << "    { const TileOp& op = ops[" << i << "];\n";
     switch (op.kind) {
       case OP_RUN: {
         // entries are compile-time: slot 0 (all owned amplitudes), slots 1..4 (r bit k set),
-        // then general groups (compile-time r condition)
+        // then general groups (compile-time r condition); zero slots are skipped
         const int ns[5] = {op.a0, op.a1, op.cls, int(op.tmask), int(op.tmatch)};
         const char* acc[5] = {"t0", "e0", "e1", "e2", "e3"};
         uint32_t e = op.moff;
@@ -206,9 +234,9 @@ std::string tile_jit_source(const Pass& p) {
           }
         }
         if (used)
-          o << "      run_apply_table<" << NR << ", " << ((used >> 1) & 1 ? "true" : "false") << ", "
+          o << "      run_apply_table_z<" << NR << ", " << ((used >> 1) & 1 ? "true" : "false") << ", "
             << ((used >> 2) & 1 ? "true" : "false") << ", " << ((used >> 3) & 1 ? "true" : "false") << ", "
-            << ((used >> 4) & 1 ? "true" : "false") << ">(v, t0, e0, e1, e2, e3);\n";
+            << ((used >> 4) & 1 ? "true" : "false") << ", " << zm << "u>(v, t0, e0, e1, e2, e3);\n";
         const uint32_t end = op.moff + op.cnt;
         bool open_group = false;
         for (; e < end; ++e) {
@@ -221,7 +249,8 @@ std::string tile_jit_source(const Pass& p) {
           if (en.tmask) o << "if ((tb & " << en.tmask << "u) == " << en.tmatch << "u) ";
           o << "acc = cmul(acc, c.C[" << en.pat << "]);\n";
           if (en.gend) {
-            o << "        run_apply_group<" << NR << ", " << en.rmask << "u, " << en.rmatch << "u>(v, acc); }\n";
+            o << "        run_apply_group_z<" << NR << ", " << en.rmask << "u, " << en.rmatch << "u, " << zm
+              << "u>(v, acc); }\n";
             open_group = false;
           }
         }
@@ -229,22 +258,26 @@ std::string tile_jit_source(const Pass& p) {
       }
       case OP_U1R:
         o << "      if (" << (uni ? "op_active(op, c.gbase)" : "true") << (thr ? " && (mp.base & op.tmask) == op.tmatch" : "")
-          << ") op_u1r<" << NR << ", " << op.a0 << ", " << op.cls << ">(v, c.pool + op.moff, " << op.rmask << "u, "
-          << op.rmatch << "u);\n";
+          << ") op_u1r_z<" << NR << ", " << op.a0 << ", " << op.cls << ", " << zm << "u>(v, c.pool + op.moff, "
+          << op.rmask << "u, " << op.rmatch << "u);\n";
+        zpos &= ~(1u << R[op.a0]);
         break;
       case OP_U1L:
-        o << "      if (" << (uni ? "op_active(op, c.gbase)" : "true") << ") op_u1l<" << NR << ", " << op.cls
-          << ">(v, c.pool + op.moff, " << op.a0 << ", c.lane, " << (thr ? "(mp.base & op.tmask) == op.tmatch" : "true")
-          << ", " << op.rmask << "u, " << op.rmatch << "u);\n";
+        o << "      if (" << (uni ? "op_active(op, c.gbase)" : "true") << ") op_u1l_z<" << NR << ", " << op.cls
+          << ", " << zm << "u>(v, c.pool + op.moff, " << op.a0 << ", c.lane, "
+          << (thr ? "(mp.base & op.tmask) == op.tmatch" : "true") << ", " << op.rmask << "u, " << op.rmatch << "u);\n";
+        zpos &= ~(1u << op.a0);
         break;
       case OP_U2R:
         o << "      if (" << (uni ? "op_active(op, c.gbase)" : "true") << (thr ? " && (mp.base & op.tmask) == op.tmatch" : "")
-          << ") op_u2r<" << NR << ", " << op.a0 << ", " << op.a1 << ">(v, c.pool + op.moff, " << op.rmask << "u, "
-          << op.rmatch << "u);\n";
+          << ") op_u2r_z<" << NR << ", " << op.a0 << ", " << op.a1 << ", " << zm << "u>(v, c.pool + op.moff, "
+          << op.rmask << "u, " << op.rmatch << "u);\n";
+        zpos &= ~((1u << R[op.a0]) | (1u << R[op.a1]));
         break;
       case OP_REMAP:
         o << "      tile_spill<" << NR << ">(v, c, mp); mp = make_mapping<" << NR
           << ">(op, c.nw, c.lane, c.warp); tile_reload<" << NR << ">(v, c, mp);\n";
+        decode(op);
         break;
       case OP_SMEM1:
       case OP_SMEM2:
@@ -252,6 +285,8 @@ std::string tile_jit_source(const Pass& p) {
         if (op.kind == OP_SMEM2) o << "op_smem2(c, op); ";
         else o << "op_smem1<" << op.cls << ">(c, op); ";
         o << "tile_reload<" << NR << ">(v, c, mp); }\n";
+        zpos &= ~(1u << op.a0);
+        if (op.kind == OP_SMEM2) zpos &= ~(1u << op.a1);
         break;
       default:
         break;

@@ -178,8 +178,9 @@ struct InterpBody {
           switch (op.a0 * 4 + op.cls) {
 #define QGPU_U1R(K, CL) \
   case K * 4 + CL: op_u1r<NR, K, CL>(v, u, op.rmask, op.rmatch); break;
-            QGPU_U1R(0, 0) QGPU_U1R(0, 1) QGPU_U1R(0, 2) QGPU_U1R(1, 0) QGPU_U1R(1, 1) QGPU_U1R(1, 2)
-            QGPU_U1R(2, 0) QGPU_U1R(2, 1) QGPU_U1R(2, 2) QGPU_U1R(3, 0) QGPU_U1R(3, 1) QGPU_U1R(3, 2)
+            QGPU_U1R(0, 0) QGPU_U1R(0, 1) QGPU_U1R(0, 2) QGPU_U1R(0, 3) QGPU_U1R(1, 0) QGPU_U1R(1, 1)
+            QGPU_U1R(1, 2) QGPU_U1R(1, 3) QGPU_U1R(2, 0) QGPU_U1R(2, 1) QGPU_U1R(2, 2) QGPU_U1R(2, 3)
+            QGPU_U1R(3, 0) QGPU_U1R(3, 1) QGPU_U1R(3, 2) QGPU_U1R(3, 3)
 #undef QGPU_U1R
             default: break;
           }
@@ -190,6 +191,7 @@ struct InterpBody {
           const bool tc = (mp.base & op.tmask) == op.tmatch;
           const double2* u = c.pool + op.moff;
           if (op.cls == MAT_X) op_u1l<NR, MAT_X>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch);
+          else if (op.cls == MAT_RI) op_u1l<NR, MAT_RI>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch);
           else if (op.cls == MAT_REAL) op_u1l<NR, MAT_REAL>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch);
           else op_u1l<NR, MAT_GENERIC>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch);
           break;
@@ -217,6 +219,7 @@ struct InterpBody {
           tile_spill<NR>(v, c, mp);
           if (op.kind == OP_SMEM2) op_smem2(c, op);
           else if (op.cls == MAT_X) op_smem1<MAT_X>(c, op);
+          else if (op.cls == MAT_RI) op_smem1<MAT_RI>(c, op);
           else if (op.cls == MAT_REAL) op_smem1<MAT_REAL>(c, op);
           else op_smem1<MAT_GENERIC>(c, op);
           tile_reload<NR>(v, c, mp);

@@ -224,7 +224,9 @@ int mat_class(const cplx* U, int nt) {
     if (U[i].im != 0.0) real = false;
   if (nt == 1 && real && U[0].re == 0.0 && U[3].re == 0.0 && U[1].re == 1.0 && U[2].re == 1.0)
     return MAT_X;
-  return real ? MAT_REAL : MAT_GENERIC;
+  if (real) return MAT_REAL;
+  if (nt == 1 && U[0].im == 0.0 && U[3].im == 0.0 && U[1].re == 0.0 && U[2].re == 0.0) return MAT_RI;
+  return MAT_GENERIC;
 }
 
 }  // namespace

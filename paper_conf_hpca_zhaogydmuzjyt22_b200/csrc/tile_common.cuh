@@ -32,7 +32,12 @@ enum OpKind : int {
   OP_SMEM2 = 5,  // 2-qubit U on tile bits a0, a1 via shared memory
   OP_RUN = 6     // run of diagonal phase patterns: entries [moff, moff + cnt)
 };
-enum MatClass : int { MAT_GENERIC = 0, MAT_REAL = 1, MAT_X = 2 };
+enum MatClass : int {
+  MAT_GENERIC = 0,  // complex 2x2: 16 FP64 per pair
+  MAT_REAL = 1,     // real entries (H, RY): 8 per pair
+  MAT_X = 2,        // exactly X: a swap, no arithmetic
+  MAT_RI = 3        // real diagonal, imaginary off-diagonal (RX, SX up to phase...): 8 per pair
+};
 
 struct TileOp {
   int kind;
@@ -161,6 +166,12 @@ __device__ __forceinline__ void apply2(double2& x0, double2& x1, const double2 (
     const double2 y1 = make_double2(fma(c, x0.x, d * x1.x), fma(c, x0.y, d * x1.y));
     x0 = y0;
     x1 = y1;
+  } else if (CLS == MAT_RI) {  // u = [[a, i b], [i c, d]] with a, b, c, d real
+    const double a = u[0].x, bq = u[1].y, c = u[2].y, d = u[3].x;
+    const double2 y0 = make_double2(fma(a, x0.x, -bq * x1.y), fma(a, x0.y, bq * x1.x));
+    const double2 y1 = make_double2(fma(d, x1.x, -c * x0.y), fma(d, x1.y, c * x0.x));
+    x0 = y0;
+    x1 = y1;
   } else {
     const double2 y0 = cfma(u[0], x0, cmul(u[1], x1));
     const double2 y1 = cfma(u[2], x0, cmul(u[3], x1));
@@ -245,9 +256,17 @@ __device__ __forceinline__ void op_u1l(double2 (&v)[kRegAmps], const double2* up
     pv.y = __shfl_xor_sync(0xffffffffu, v[r].y, 1 << t);
     const double2 a0 = hi ? pv : v[r], a1 = hi ? v[r] : pv;
     double2 y;
-    if (CLS == MAT_X) y = pv;
-    else if (CLS == MAT_REAL) y = make_double2(fma(c0.x, a0.x, c1.x * a1.x), fma(c0.x, a0.y, c1.x * a1.y));
-    else y = cfma(c0, a0, cmul(c1, a1));
+    if (CLS == MAT_X) {
+      y = pv;
+    } else if (CLS == MAT_REAL) {
+      y = make_double2(fma(c0.x, a0.x, c1.x * a1.x), fma(c0.x, a0.y, c1.x * a1.y));
+    } else if (CLS == MAT_RI) {  // lo lane: a x0 + i b x1; hi lane: i c x0 + d x1
+      const double2 own = hi ? a1 : a0, oth = hi ? a0 : a1;
+      const double dg = hi ? up[3].x : up[0].x, od = hi ? up[2].y : up[1].y;
+      y = make_double2(fma(dg, own.x, -od * oth.y), fma(dg, own.y, od * oth.x));
+    } else {
+      y = cfma(c0, a0, cmul(c1, a1));
+    }
     if (tc) v[r] = y;
   }
 }
@@ -317,6 +336,122 @@ __device__ __forceinline__ void op_run(double2 (&v)[kRegAmps], const TileOp& op,
       acc = make_double2(1.0, 0.0);
     }
   }
+}
+
+// ---- JIT variants aware of compile-time zero slots (first-touch expansion, a5): slot r is
+// known to be exactly zero when one of its register bits is a tile position >= L_in that no
+// non-diagonal op has targeted yet. ZM is the 16-bit mask of such slots.
+template <int CLS>
+__device__ __forceinline__ void apply2_x1zero(double2& x0, double2& x1, const double2 (&u)[4]) {
+  // (x0, 0) -> (u00 x0, u10 x0)
+  if (CLS == MAT_X) {
+    x1 = x0;
+    x0 = make_double2(0.0, 0.0);
+  } else if (CLS == MAT_REAL) {
+    x1 = make_double2(u[2].x * x0.x, u[2].x * x0.y);
+    x0 = make_double2(u[0].x * x0.x, u[0].x * x0.y);
+  } else {
+    x1 = cmul(u[2], x0);
+    x0 = cmul(u[0], x0);
+  }
+}
+template <int CLS>
+__device__ __forceinline__ void apply2_x0zero(double2& x0, double2& x1, const double2 (&u)[4]) {
+  // (0, x1) -> (u01 x1, u11 x1)
+  if (CLS == MAT_X) {
+    x0 = x1;
+    x1 = make_double2(0.0, 0.0);
+  } else if (CLS == MAT_REAL) {
+    x0 = make_double2(u[1].x * x1.x, u[1].x * x1.y);
+    x1 = make_double2(u[3].x * x1.x, u[3].x * x1.y);
+  } else {
+    x0 = cmul(u[1], x1);
+    x1 = cmul(u[3], x1);
+  }
+}
+template <int NR, int K, int CLS, unsigned ZM>
+__device__ __forceinline__ void op_u1r_z(double2 (&v)[kRegAmps], const double2* up, uint32_t rm, uint32_t rt) {
+  const double2 u[4] = {up[0], up[1], up[2], up[3]};
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r) {
+    if (r >> K & 1) continue;
+    if ((uint32_t(r) & rm) != rt) continue;
+    const int r1 = r | (1 << K);
+    const bool z0 = (ZM >> r) & 1, z1 = (ZM >> r1) & 1;
+    if (z0 && z1) continue;
+    if (z1) apply2_x1zero<CLS>(v[r], v[r1], u);
+    else if (z0) apply2_x0zero<CLS>(v[r], v[r1], u);
+    else apply2<CLS>(v[r], v[r1], u);
+  }
+}
+template <int NR, int CLS, unsigned ZM>
+__device__ __forceinline__ void op_u1l_z(double2 (&v)[kRegAmps], const double2* up, int t, int lane, bool tc,
+                                         uint32_t rm, uint32_t rt) {
+  const bool hi = (lane >> t) & 1;
+  const double2 c0 = hi ? up[2] : up[0], c1 = hi ? up[3] : up[1];
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r) {
+    if ((uint32_t(r) & rm) != rt) continue;
+    if ((ZM >> r) & 1) continue;  // the partner slot (same r, other lane) is zero as well
+    double2 pv;
+    pv.x = __shfl_xor_sync(0xffffffffu, v[r].x, 1 << t);
+    pv.y = __shfl_xor_sync(0xffffffffu, v[r].y, 1 << t);
+    const double2 a0 = hi ? pv : v[r], a1 = hi ? v[r] : pv;
+    double2 y;
+    if (CLS == MAT_X) {
+      y = pv;
+    } else if (CLS == MAT_REAL) {
+      y = make_double2(fma(c0.x, a0.x, c1.x * a1.x), fma(c0.x, a0.y, c1.x * a1.y));
+    } else if (CLS == MAT_RI) {
+      const double2 own = hi ? a1 : a0, oth = hi ? a0 : a1;
+      const double dg = hi ? up[3].x : up[0].x, od = hi ? up[2].y : up[1].y;
+      y = make_double2(fma(dg, own.x, -od * oth.y), fma(dg, own.y, od * oth.x));
+    } else {
+      y = cfma(c0, a0, cmul(c1, a1));
+    }
+    if (tc) v[r] = y;
+  }
+}
+template <int NR, int K0, int K1, unsigned ZM>
+__device__ __forceinline__ void op_u2r_z(double2 (&v)[kRegAmps], const double2* u, uint32_t rm, uint32_t rt) {
+  constexpr int m0 = 1 << K0, m1 = 1 << K1;
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r) {
+    if (r & (m0 | m1)) continue;
+    if ((uint32_t(r) & rm) != rt) continue;
+    if (((ZM >> r) & 1) && ((ZM >> (r | m0)) & 1) && ((ZM >> (r | m1)) & 1) && ((ZM >> (r | m0 | m1)) & 1))
+      continue;
+    const double2 x0 = v[r], x1 = v[r | m0], x2 = v[r | m1], x3 = v[r | m0 | m1];
+#pragma unroll
+    for (int row = 0; row < 4; ++row) {
+      double2 y = cmul(u[row * 4], x0);
+      y = cfma(u[row * 4 + 1], x1, y);
+      y = cfma(u[row * 4 + 2], x2, y);
+      y = cfma(u[row * 4 + 3], x3, y);
+      v[r | (row & 1 ? m0 : 0) | (row & 2 ? m1 : 0)] = y;
+    }
+  }
+}
+template <int NR, bool E0, bool E1, bool E2, bool E3, unsigned ZM>
+__device__ __forceinline__ void run_apply_table_z(double2 (&v)[kRegAmps], double2 t0, double2 e0, double2 e1,
+                                                  double2 e2, double2 e3) {
+  double2 P[kRegAmps];
+  P[0] = t0;
+  const double2 ek[4] = {e0, e1, e2, e3};
+  const bool has[4] = {E0, E1, E2, E3};
+#pragma unroll
+  for (int k = 0; k < NR; ++k)
+#pragma unroll
+    for (int r = 0; r < (1 << k); ++r) P[r | (1 << k)] = has[k] ? cmul(P[r], ek[k]) : P[r];
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r)
+    if (!((ZM >> r) & 1)) v[r] = cmul(v[r], P[r]);
+}
+template <int NR, unsigned RM, unsigned RT, unsigned ZM>
+__device__ __forceinline__ void run_apply_group_z(double2 (&v)[kRegAmps], double2 acc) {
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r)
+    if ((unsigned(r) & RM) == RT && !((ZM >> r) & 1)) v[r] = cmul(v[r], acc);
 }
 
 // JIT helpers for a run whose entries are compile-time: multiply the owned amplitudes by the
@@ -509,9 +644,6 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       if (!bulk) {
         issue_tile_loads_thr(bufs + kn * T, a, hiOff, tile + gridDim.x, T, nthr, tid);
       } else if (warp == 0) {
-        if (nbuf >= 3) asm volatile("cp.async.bulk.wait_group.read 1;\n" ::: "memory");
-        else bulk_wait_read();
-        __syncwarp();
         issue_tile_loads_bulk(bufs + kn * T, &bars[kn], a, hiOff, tile + gridDim.x, lane);
       }
     }
@@ -545,38 +677,49 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       else cp_async_wait_all();
     }
     __syncthreads();  // tile and constants visible to every thread
+    if (base >= a.L_in) {
+      // the whole tile lies in the zero region of a first-touch expansion and no op of the pass
+      // targets its non-tile bits: it stays zero -> store zeros, skip the program
+      if (c.own) {
+#pragma unroll
+        for (int r = 0; r < kRegAmps; ++r) {
+          const uint32_t j = uint32_t(tid) + uint32_t(r) * nthr;
+          if (j < T) st_stream(a.psi + (base | (j & lowmask) | hiOff[j >> l]), make_double2(0.0, 0.0));
+        }
+      }
+      k = kn;
+      __syncthreads();
+      continue;
+    }
     c.s = s;
     c.gbase = gbase;
     double2 v[kRegAmps];
     Mapping mp = make_mapping<NR>(ops[0], nw, lane, warp);  // ops[0] is always OP_REMAP
     tile_reload<NR>(v, c, mp);
     body(v, mp, c);
-    // back to natural order (times the tile-uniform phase), then store
+    // store straight from registers: the lane bits are physical positions 0..4, so each warp
+    // store writes 32 consecutive amplitudes (512 B); the physical offset of an owned amplitude
+    // is linear in its tile bits, phys(j(r)) = phys(base_j) | OR_k r_k phys(rb_k)
     const double2 sc = *scal_s;
-    if (!(sc.x == 1.0 && sc.y == 0.0)) {
+    const bool has_sc = !(sc.x == 1.0 && sc.y == 0.0);
+    const uint64_t pb = base | (mp.base & lowmask) | hiOff[mp.base >> l];
+    uint64_t prb[4];
 #pragma unroll
-      for (int r = 0; r < (1 << NR); ++r) v[r] = cmul(v[r], sc);
+    for (int q = 0; q < 4; ++q) {
+      const uint32_t bit = mp.rb[q];
+      prb[q] = (q < NR) ? ((bit & lowmask) | hiOff[bit >> l]) : 0ull;
     }
-    // without remaps each thread writes back exactly the slots it read: no barrier needed
-    if (a.remaps) __syncthreads();
+    if (c.own) {
 #pragma unroll
-    for (int r = 0; r < (1 << NR); ++r)
-      if (c.own) s[mp.j(r)] = v[r];
-    if (bulk) {
-      fence_proxy_async();
-      __syncthreads();
-      if (warp == 0) issue_tile_stores(s, a, hiOff, base, lane);
-    } else {
-      __syncthreads();
-#pragma unroll
-      for (int r = 0; r < kRegAmps; ++r) {
-        const uint32_t j = uint32_t(tid) + uint32_t(r) * nthr;
-        if (j < T) st_stream(a.psi + (base | (j & lowmask) | hiOff[j >> l]), s[j]);
+      for (int r = 0; r < (1 << NR); ++r) {
+        const uint64_t off = pb | ((r & 1) ? prb[0] : 0ull) | ((r & 2) ? prb[1] : 0ull) |
+                             ((r & 4) ? prb[2] : 0ull) | ((r & 8) ? prb[3] : 0ull);
+        st_stream(a.psi + off, has_sc ? cmul(v[r], sc) : v[r]);
       }
     }
     k = kn;
+    __syncthreads();  // every thread is done with buffer k before it is refilled
   }
-  if (bulk && warp == 0) bulk_wait_all();
 }
 
 #endif  // __CUDACC__
