@@ -237,11 +237,11 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     a.L_in = L_in;
     a.rank_base = rank << m;
     a.zero = st->d_zero;
-    a.bulk = p.l >= 7 ? 1 : 0;
     a.remaps = 0;
     for (size_t i = 1; i < P.ops.size(); ++i)
       if (P.ops[i].kind == OP_REMAP || P.ops[i].kind == OP_SMEM1 || P.ops[i].kind == OP_SMEM2) a.remaps = 1;
-    a.nbuf = 2;
+    a.nbuf = 3;
+    if (tile_smem_bytes(a) > 227 * 1024) a.nbuf = 2;
     const int jit = st->cfg.jit;
     cudaError_t e = cudaErrorNotSupported;
     if (jit == 2 || (jit == 1 && p.k_out >= kJitMinBits)) {

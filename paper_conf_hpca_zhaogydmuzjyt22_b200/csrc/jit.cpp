@@ -190,13 +190,24 @@ std::string tile_jit_source(const Pass& p) {
         if ((r >> k & 1) && (zpos >> R[k] & 1)) zm |= 1u << r;
     return zm;
   };
+  uint32_t Wmask = 0;  // tile bits that are warp bits in the current mapping
+  auto decode_w = [&](const TileOp& op) {
+    Wmask = 0;
+    for (int k = 0; k < P.nw; ++k) Wmask |= 1u << ((op.a1 >> (4 * k)) & 15);
+  };
   decode(P.ops[0]);
+  decode_w(P.ops[0]);
   std::ostringstream o;
   o << "// qgpu tile pass: b=" << p.b << " nr=" << NR << " nw=" << P.nw << " ops=" << P.ops.size()
     << " k_in=" << p.k_in << "\n";
   o << "#include \"tile_common.cuh\"\n";
   o << "using namespace qgpu;\n";
+  // zero slots / zero warps at the start of the pass (used by the driver to skip loads)
+  const unsigned zm_start = zmask();
+  const uint32_t zw_start = zpos & Wmask;
   o << "struct JitBody {\n";
+  o << "  static constexpr unsigned kZM0 = " << zm_start << "u;\n";
+  o << "  static constexpr uint32_t kZW0 = " << zw_start << "u;\n";
   o << "  __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c) const {\n";
   o << "    const TileOp* ops = c.ops;\n";
   {
@@ -213,7 +224,10 @@ std::string tile_jit_source(const Pass& p) {
     const bool uni = op.omask != 0;       // tile-uniform condition present
     const bool thr = op.tmask != 0;       // condition on the thread's fixed bits present
     const unsigned zm = zmask();
+    const uint32_t zw = zpos & Wmask;  // warps whose fixed bits hit these hold only zeros
     o << "    { const TileOp& op = ops[" << i << "];\n";
+    const bool wguard = zw && (op.kind == OP_RUN || op.kind == OP_U1R || op.kind == OP_U2R || op.kind == OP_U1L);
+    if (wguard) o << "      if ((mp.base & " << zw << "u) == 0u) {\n";
     switch (op.kind) {
       case OP_RUN: {
         // entries are compile-time: slot 0 (all owned amplitudes), slots 1..4 (r bit k set),
@@ -278,6 +292,7 @@ std::string tile_jit_source(const Pass& p) {
         o << "      tile_spill<" << NR << ">(v, c, mp); mp = make_mapping<" << NR
           << ">(op, c.nw, c.lane, c.warp); tile_reload<" << NR << ">(v, c, mp);\n";
         decode(op);
+        decode_w(op);
         break;
       case OP_SMEM1:
       case OP_SMEM2:
@@ -291,6 +306,7 @@ std::string tile_jit_source(const Pass& p) {
       default:
         break;
     }
+    if (wguard) o << "      }\n";
     o << "    }\n";
   }
   o << "  }\n};\n";

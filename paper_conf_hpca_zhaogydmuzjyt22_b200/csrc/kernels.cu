@@ -164,6 +164,8 @@ __global__ void __launch_bounds__(kThreads) phase_kernel(PhaseArgs a) {
 // path (jit.cpp) replaces this body by straight-line code specialised to one pass.
 template <int NR>
 struct InterpBody {
+  static constexpr unsigned kZM0 = 0u;
+  static constexpr uint32_t kZW0 = 0u;
   int nops;
   __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c) const {
     for (int i = 1; i < nops; ++i) {
@@ -346,8 +348,9 @@ int device_num_sms() { return num_sms(); }
 
 size_t tile_smem_bytes(const TileArgs& a) {
   const size_t nh = size_t(1) << (a.b - a.l);
-  return size_t(a.nbuf) * (size_t(1) << a.b) * 16 + 32 + ((nh + 1) & ~size_t(1)) * 8 +
-         size_t(a.blob_bytes) + size_t(a.npat + 1) * 16;
+  const size_t nwarps = size_t(1) << a.nw;
+  return size_t(a.nbuf) * (size_t(1) << a.b) * 16 + ((nh + 1) & ~size_t(1)) * 8 + size_t(a.blob_bytes) +
+         nwarps * size_t(a.npat) * 16 + 16;
 }
 
 cudaError_t launch_pair(cudaStream_t st, const PairArgs& a, bool shfl) {

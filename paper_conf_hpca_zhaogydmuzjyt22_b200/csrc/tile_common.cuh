@@ -516,75 +516,63 @@ __device__ __forceinline__ void op_smem2(const TileCtx& c, const TileOp& op) {
   __syncthreads();
 }
 
-// Tile loads of one tile: warp 0 issues one bulk copy per contiguous run of 2^l amplitudes
-// (runs at index >= L_in are copied from the zero buffer: first-touch expansion, a5); the
-// buffer's mbarrier completes when all T*16 bytes have landed.
-__device__ __forceinline__ void issue_tile_loads_bulk(double2* buf, uint64_t* bar, const TileArgs& a,
-                                                      const uint64_t* hiOff, uint64_t tile, int lane) {
-  const uint64_t base = tile_base(tile, a);
-  const int nrun = 1 << (a.b - a.l);
-  const uint64_t rl = 1ull << a.l;
-  if (lane == 0) mbar_arrive_expect_tx(bar, uint32_t(16u << a.b));
-  __syncwarp();
-  for (int h = lane; h < nrun; h += 32) {
-    const uint64_t idx = base | hiOff[h];
-    double2* dst = buf + (uint64_t(h) << a.l);
-    if (idx + rl <= a.L_in) {
-      bulk_g2s(dst, a.psi + idx, uint32_t(rl * 16), bar);
-    } else if (idx >= a.L_in) {
-      bulk_g2s(dst, a.zero, uint32_t(rl * 16), bar);
-    } else {  // L_in < 2^l: the live part, then zeros
-      const uint64_t live = a.L_in - idx;
-      bulk_g2s(dst, a.psi + idx, uint32_t(live * 16), bar);
-      bulk_g2s(dst + live, a.zero, uint32_t((rl - live) * 16), bar);
-    }
+// Physical offset (within the tile) of an owned slot r under mapping mp: phys is linear in the
+// tile bits, phys(j(r)) = phys(base_j) | OR_k r_k phys(rb_k).
+struct SlotAddr {
+  uint64_t pb;
+  uint64_t prb[4];
+  __device__ __forceinline__ uint64_t at(int r) const {
+    return pb | ((r & 1) ? prb[0] : 0ull) | ((r & 2) ? prb[1] : 0ull) | ((r & 4) ? prb[2] : 0ull) |
+           ((r & 8) ? prb[3] : 0ull);
   }
+};
+template <int NR>
+__device__ __forceinline__ SlotAddr slot_addr(const Mapping& mp, const uint64_t* hiOff, uint32_t lowmask, int l) {
+  SlotAddr sa;
+  sa.pb = (mp.base & lowmask) | hiOff[mp.base >> l];
+#pragma unroll
+  for (int q = 0; q < 4; ++q) {
+    const uint32_t bit = mp.rb[q];
+    sa.prb[q] = (q < NR) ? ((bit & lowmask) | hiOff[bit >> l]) : 0ull;
+  }
+  return sa;
 }
 
-// Per-thread variant for short runs (l < 7): one 16-B cp.async (LDGSTS) per amplitude,
-// src-size 0 (hardware zero-fill) beyond L_in.
-__device__ __forceinline__ void issue_tile_loads_thr(double2* buf, const TileArgs& a, const uint64_t* hiOff,
-                                                     uint64_t tile, uint32_t T, int nthr, int tid) {
-  const uint64_t base = tile_base(tile, a);
-  const uint32_t lowmask = (1u << a.l) - 1;
+// Each thread prefetches exactly the slots it owns under the initial mapping (cp.async, 16 B,
+// src-size 0 = hardware zero-fill beyond L_in): no thread reads another thread's load, so a
+// tile needs no CTA barrier unless its program remaps. ZM: slots known to be zero (skipped).
+template <int NR>
+__device__ __forceinline__ void issue_own_loads(double2* buf, const TileArgs& a, const Mapping& mp0,
+                                                const SlotAddr& sa0, uint64_t base, unsigned zm, bool own) {
+  if (own && base < a.L_in) {
 #pragma unroll
-  for (int r = 0; r < kRegAmps; ++r) {
-    const uint32_t j = uint32_t(tid) + uint32_t(r) * nthr;
-    if (j < T) {
-      const uint64_t idx = base | (j & lowmask) | hiOff[j >> a.l];
+    for (int r = 0; r < (1 << NR); ++r) {
+      if ((zm >> r) & 1) continue;
+      const uint64_t idx = base | sa0.at(r);
       const bool live = idx < a.L_in;
-      cp_async16(buf + j, a.psi + (live ? idx : 0), live ? 16 : 0);
+      cp_async16(buf + mp0.j(r), a.psi + (live ? idx : 0), live ? 16 : 0);
     }
   }
   asm volatile("cp.async.commit_group;\n" ::: "memory");
 }
 
-__device__ __forceinline__ void issue_tile_stores(double2* buf, const TileArgs& a, const uint64_t* hiOff,
-                                                  uint64_t base, int lane) {
-  const int nrun = 1 << (a.b - a.l);
-  const uint32_t bytes = 16u << a.l;
-  for (int h = lane; h < nrun; h += 32) bulk_s2g(a.psi + (base | hiOff[h]), buf + (uint64_t(h) << a.l), bytes);
-  bulk_commit();
-}
-
-// The persistent tile loop shared by the interpreted and the JIT kernels: one CTA (or two) per
-// SM, nbuf (3, else 2) tile buffers: the loads of tile i+1 fly while tile i is computed in
-// registers; tile i is written back while tile i+1 computes. Long contiguous runs (l >= 7)
-// move with bulk async copies issued by warp 0 (mbarrier-tracked loads, bulk-group stores);
-// short runs with per-thread cp.async / streaming stores. Per tile the pattern constants and
-// the tile-uniform phase are computed while the tile lands.
-// Body: void operator()(double2 (&v)[16], Mapping& mp, const TileCtx& c).
+// The persistent tile loop shared by the interpreted and the JIT kernels: one CTA per SM, nbuf
+// tile buffers (3; 2 when the program blob is large). Tile i+1 is prefetched into the slots its
+// threads will own while tile i is computed in registers; stores go straight from registers
+// (lane bits = physical positions 0..4: each warp store writes 512 contiguous bytes). Pattern
+// constants are computed per warp and the tile-uniform phase per lane, so a tile without
+// remaps runs with no CTA-wide barrier.
+// Body: void operator()(double2 (&v)[16], Mapping& mp, const TileCtx& c); Body::kZM0 = slots
+// known zero at the start of the pass, Body::kZW0 = warp bits whose warps hold only zeros.
 template <int NR, class Body>
 __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   extern __shared__ __align__(128) unsigned char smem_raw[];
   const int b = a.b, l = a.l, nw = a.nw, nbuf = a.nbuf;
-  const bool bulk = a.bulk != 0;
   const uint32_t T = 1u << b;
   const int nh = 1 << (b - l);
-  const int nthr = blockDim.x;
-  double2* bufs = reinterpret_cast<double2*>(smem_raw);             // nbuf x T
-  uint64_t* bars = reinterpret_cast<uint64_t*>(bufs + nbuf * T);    // 4 mbarriers
-  uint64_t* hiOff = bars + 4;
+  const int nthr = blockDim.x, nwarps = nthr >> 5;
+  double2* bufs = reinterpret_cast<double2*>(smem_raw);  // nbuf x T
+  uint64_t* hiOff = reinterpret_cast<uint64_t*>(bufs + nbuf * T);
   unsigned char* blob = reinterpret_cast<unsigned char*>(hiOff + ((nh + 1) & ~1));
   const TileOp* ops = reinterpret_cast<const TileOp*>(blob);
   const RunEntry* ents = reinterpret_cast<const RunEntry*>(blob + a.off_entries);
@@ -592,8 +580,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   const PhaseTerm* terms = reinterpret_cast<const PhaseTerm*>(blob + a.off_terms);
   const PhaseTerm* scal = reinterpret_cast<const PhaseTerm*>(blob + a.off_scalar);
   const double2* pool = reinterpret_cast<const double2*>(blob + a.off_pool);
-  double2* C = reinterpret_cast<double2*>(blob + a.blob_bytes);  // pattern constants
-  double2* scal_s = C + a.npat;
+  double2* Cw = reinterpret_cast<double2*>(blob + a.blob_bytes);  // per-warp pattern constants
 
   {
     const int4* src = reinterpret_cast<const int4*>(a.blob);
@@ -606,10 +593,6 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       if (h >> (i - l) & 1) off |= 1ull << a.spos[i];
     hiOff[h] = off;
   }
-  if (threadIdx.x == 0) {
-    for (int q = 0; q < 4; ++q) mbar_init(&bars[q], 1);
-    asm volatile("fence.mbarrier_init.release.cluster;\n" ::: "memory");
-  }
   __syncthreads();
   const int tid = threadIdx.x, lane = tid & 31, warp = tid >> 5;
   const uint32_t lowmask = (1u << l) - 1;
@@ -617,7 +600,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   c.ops = ops;
   c.ents = ents;
   c.pool = pool;
-  c.C = C;
+  c.C = Cw + size_t(warp) * a.npat;
   c.T = T;
   c.nthr = nthr;
   c.tid = tid;
@@ -625,39 +608,44 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   c.warp = warp;
   c.nw = nw;
   c.own = lane < int(T);
+  const Mapping mp0 = make_mapping<NR>(ops[0], nw, lane, warp);  // ops[0] is always OP_REMAP
+  const SlotAddr sa0 = slot_addr<NR>(mp0, hiOff, lowmask, l);
+  const bool wzero = (mp0.base & Body::kZW0) != 0u;  // this warp's slots start in the zero region
+  const unsigned zm0 = wzero ? 0xffffu : Body::kZM0;
+  (void)nwarps;
 
   uint64_t tile = blockIdx.x;
-  if (tile < a.ntiles) {
-    if (!bulk) issue_tile_loads_thr(bufs, a, hiOff, tile, T, nthr, tid);
-    else if (warp == 0) issue_tile_loads_bulk(bufs, &bars[0], a, hiOff, tile, lane);
-  }
+  if (tile < a.ntiles) issue_own_loads<NR>(bufs, a, mp0, sa0, tile_base(tile, a), zm0, c.own);
   int k = 0;
-  uint32_t phase = 0;  // mbarrier parity per buffer
   for (int it = 0; tile < a.ntiles; tile += gridDim.x, ++it) {
     double2* s = bufs + k * T;
     const int kn = (k + 1 == nbuf) ? 0 : k + 1;
     const uint64_t base = tile_base(tile, a);
     const uint64_t gbase = a.rank_base | base;
-    // prefetch the next tile into buffer kn (its stores were issued nbuf-1 tiles ago)
     const bool more = tile + gridDim.x < a.ntiles;
-    if (more) {
-      if (!bulk) {
-        issue_tile_loads_thr(bufs + kn * T, a, hiOff, tile + gridDim.x, T, nthr, tid);
-      } else if (warp == 0) {
-        issue_tile_loads_bulk(bufs + kn * T, &bars[kn], a, hiOff, tile + gridDim.x, lane);
+    if (more) issue_own_loads<NR>(bufs + kn * T, a, mp0, sa0, tile_base(tile + gridDim.x, a), zm0, c.own);
+    if (base >= a.L_in) {
+      // the whole tile lies in the zero region of a first-touch expansion and no op of the pass
+      // targets its non-tile bits: it stays zero -> store zeros, skip the program
+      if (c.own) {
+#pragma unroll
+        for (int r = 0; r < (1 << NR); ++r) st_stream(a.psi + (base | sa0.at(r)), make_double2(0.0, 0.0));
       }
+      k = kn;
+      if (nbuf < 3 && a.remaps) __syncthreads();
+      continue;
     }
-    // pattern constants, spread over the warps (pattern pi -> warp pi % nwarps)
-    const int nwarps = nthr >> 5;
-    for (int pi = warp + nwarps * lane; pi < a.npat; pi += nthr) {
+    // pattern constants of this tile, per warp (lane-strided)
+    for (int pi = lane; pi < a.npat; pi += 32) {
       double2 cc = make_double2(1.0, 0.0);
       const Pattern pt = pats[pi];
       for (uint32_t q = pt.first; q < pt.first + pt.count; ++q)
         if ((gbase & terms[q].omask) == terms[q].omatch) cc = cmul(cc, make_double2(terms[q].re, terms[q].im));
-      C[pi] = cc;
+      Cw[size_t(warp) * a.npat + pi] = cc;
     }
-    if (warp == nthr / 32 - 1) {  // the last warp: product of the tile-uniform phases
-      double2 sc = make_double2(1.0, 0.0);
+    // tile-uniform phase, per lane (lane-strided product, then butterfly)
+    double2 sc = make_double2(1.0, 0.0);
+    if (a.nscalar) {
       for (int q = lane; q < a.nscalar; q += 32)
         if ((gbase & scal[q].omask) == scal[q].omatch) sc = cmul(sc, make_double2(scal[q].re, scal[q].im));
 #pragma unroll
@@ -667,58 +655,27 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
         t.y = __shfl_xor_sync(0xffffffffu, sc.y, o);
         sc = cmul(sc, t);
       }
-      if (lane == 0) *scal_s = sc;
     }
-    if (bulk) {
-      mbar_wait(&bars[k], (phase >> k) & 1u);  // tile `it` landed
-      phase ^= 1u << k;
-    } else {
-      if (more) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
-      else cp_async_wait_all();
-    }
-    __syncthreads();  // tile and constants visible to every thread
-    if (base >= a.L_in) {
-      // the whole tile lies in the zero region of a first-touch expansion and no op of the pass
-      // targets its non-tile bits: it stays zero -> store zeros, skip the program
-      if (c.own) {
-#pragma unroll
-        for (int r = 0; r < kRegAmps; ++r) {
-          const uint32_t j = uint32_t(tid) + uint32_t(r) * nthr;
-          if (j < T) st_stream(a.psi + (base | (j & lowmask) | hiOff[j >> l]), make_double2(0.0, 0.0));
-        }
-      }
-      k = kn;
-      __syncthreads();
-      continue;
-    }
+    if (more) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
+    else cp_async_wait_all();
+    __syncwarp();
     c.s = s;
     c.gbase = gbase;
     double2 v[kRegAmps];
-    Mapping mp = make_mapping<NR>(ops[0], nw, lane, warp);  // ops[0] is always OP_REMAP
-    tile_reload<NR>(v, c, mp);
-    body(v, mp, c);
-    // store straight from registers: the lane bits are physical positions 0..4, so each warp
-    // store writes 32 consecutive amplitudes (512 B); the physical offset of an owned amplitude
-    // is linear in its tile bits, phys(j(r)) = phys(base_j) | OR_k r_k phys(rb_k)
-    const double2 sc = *scal_s;
-    const bool has_sc = !(sc.x == 1.0 && sc.y == 0.0);
-    const uint64_t pb = base | (mp.base & lowmask) | hiOff[mp.base >> l];
-    uint64_t prb[4];
+    Mapping mp = mp0;
 #pragma unroll
-    for (int q = 0; q < 4; ++q) {
-      const uint32_t bit = mp.rb[q];
-      prb[q] = (q < NR) ? ((bit & lowmask) | hiOff[bit >> l]) : 0ull;
-    }
+    for (int r = 0; r < (1 << NR); ++r)
+      v[r] = (c.own && !((zm0 >> r) & 1)) ? s[mp0.j(r)] : make_double2(0.0, 0.0);
+    body(v, mp, c);
+    const bool has_sc = !(sc.x == 1.0 && sc.y == 0.0);
+    const SlotAddr sa = slot_addr<NR>(mp, hiOff, lowmask, l);
     if (c.own) {
 #pragma unroll
-      for (int r = 0; r < (1 << NR); ++r) {
-        const uint64_t off = pb | ((r & 1) ? prb[0] : 0ull) | ((r & 2) ? prb[1] : 0ull) |
-                             ((r & 4) ? prb[2] : 0ull) | ((r & 8) ? prb[3] : 0ull);
-        st_stream(a.psi + off, has_sc ? cmul(v[r], sc) : v[r]);
-      }
+      for (int r = 0; r < (1 << NR); ++r) st_stream(a.psi + (base | sa.at(r)), has_sc ? cmul(v[r], sc) : v[r]);
     }
     k = kn;
-    __syncthreads();  // every thread is done with buffer k before it is refilled
+    // with two buffers the next prefetch refills the buffer other warps read during remaps
+    if (nbuf < 3 && a.remaps) __syncthreads();
   }
 }
 
