@@ -174,6 +174,38 @@ bool jit_cubin_cached(const std::string& src, std::string* cubin, std::string* l
 std::string tile_jit_source(const Pass& p) {
   const TileProgram& P = p.prog;
   const int NR = P.nr;
+  // compile-time slot tables of a mapping: tile-local offset J[r] and physical offset Pq[r]
+  auto jtab = [&](const int* Rb) {
+    std::ostringstream t;
+    t << "{";
+    for (int r = 0; r < 16; ++r) {
+      uint32_t j = 0;
+      for (int k = 0; k < NR; ++k)
+        if (r >> k & 1) j |= 1u << Rb[k];
+      t << (r ? ", " : "") << j << "u";
+    }
+    t << "}";
+    return t.str();
+  };
+  auto ptab = [&](const int* Rb) {
+    std::ostringstream t;
+    t << "{";
+    for (int r = 0; r < 16; ++r) {
+      unsigned long long q = 0;
+      for (int k = 0; k < NR; ++k)
+        if (r >> k & 1) q |= 1ull << p.spos[Rb[k]];
+      t << (r ? ", " : "") << q << "ull";
+    }
+    t << "}";
+    return t.str();
+  };
+  auto base_expr = [&](const TileOp& op) {
+    std::ostringstream t;
+    t << "uint32_t(c.lane)";
+    for (int k = 0; k < P.nw; ++k)
+      t << " | ((c.warp >> " << k << ") & 1 ? " << (1u << ((op.a1 >> (4 * k)) & 15)) << "u : 0u)";
+    return t.str();
+  };
   // compile-time zero tracking (first-touch expansion, a5): tile bits whose physical position
   // is >= k_in hold zeros until a non-diagonal op targets them
   uint32_t zpos = 0;
@@ -205,9 +237,19 @@ std::string tile_jit_source(const Pass& p) {
   // zero slots / zero warps at the start of the pass (used by the driver to skip loads)
   const unsigned zm_start = zmask();
   const uint32_t zw_start = zpos & Wmask;
+  // final mapping (for the store)
+  int RF[4] = {R[0], R[1], R[2], R[3]};
+  for (const TileOp& op : P.ops)
+    if (op.kind == OP_REMAP)
+      for (int k = 0; k < 4; ++k) RF[k] = (op.a0 >> (4 * k)) & 15;
   o << "struct JitBody {\n";
   o << "  static constexpr unsigned kZM0 = " << zm_start << "u;\n";
   o << "  static constexpr uint32_t kZW0 = " << zw_start << "u;\n";
+  o << "  static constexpr bool kStatic = true;\n";
+  o << "  static constexpr bool kHasScalar = " << (P.scalar.empty() ? "false" : "true") << ";\n";
+  o << "  static constexpr uint32_t kJ0[kRegAmps] = " << jtab(R) << ";\n";
+  o << "  static constexpr uint64_t kP0[kRegAmps] = " << ptab(R) << ";\n";
+  o << "  static constexpr uint64_t kPF[kRegAmps] = " << ptab(RF) << ";\n";
   o << "  __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c) const {\n";
   o << "    const TileOp* ops = c.ops;\n";
   {
@@ -288,18 +330,23 @@ std::string tile_jit_source(const Pass& p) {
           << op.rmask << "u, " << op.rmatch << "u);\n";
         zpos &= ~((1u << R[op.a0]) | (1u << R[op.a1]));
         break;
-      case OP_REMAP:
-        o << "      tile_spill<" << NR << ">(v, c, mp); mp = make_mapping<" << NR
-          << ">(op, c.nw, c.lane, c.warp); tile_reload<" << NR << ">(v, c, mp);\n";
+      case OP_REMAP: {
+        o << "      { constexpr uint32_t Jo[kRegAmps] = " << jtab(R) << ";\n";
+        o << "        tile_spill_j<" << NR << ">(v, c, mp.base, Jo); }\n";
         decode(op);
         decode_w(op);
+        o << "      mp.base = " << base_expr(op) << ";\n";
+        o << "      { constexpr uint32_t Jn[kRegAmps] = " << jtab(R) << ";\n";
+        o << "        tile_reload_j<" << NR << ">(v, c, mp.base, Jn); }\n";
         break;
+      }
       case OP_SMEM1:
       case OP_SMEM2:
-        o << "      if (" << (uni ? "op_active(op, c.gbase)" : "true") << ") { tile_spill<" << NR << ">(v, c, mp); ";
+        o << "      if (" << (uni ? "op_active(op, c.gbase)" : "true") << ") { constexpr uint32_t Jc[kRegAmps] = "
+          << jtab(R) << ";\n        tile_spill_j<" << NR << ">(v, c, mp.base, Jc); ";
         if (op.kind == OP_SMEM2) o << "op_smem2(c, op); ";
         else o << "op_smem1<" << op.cls << ">(c, op); ";
-        o << "tile_reload<" << NR << ">(v, c, mp); }\n";
+        o << "tile_reload_j<" << NR << ">(v, c, mp.base, Jc); }\n";
         zpos &= ~(1u << op.a0);
         if (op.kind == OP_SMEM2) zpos &= ~(1u << op.a1);
         break;

@@ -166,6 +166,11 @@ template <int NR>
 struct InterpBody {
   static constexpr unsigned kZM0 = 0u;
   static constexpr uint32_t kZW0 = 0u;
+  static constexpr bool kStatic = false;  // mappings read from the program at run time
+  static constexpr bool kHasScalar = true;
+  static constexpr uint32_t kJ0[kRegAmps] = {};
+  static constexpr uint64_t kP0[kRegAmps] = {};
+  static constexpr uint64_t kPF[kRegAmps] = {};
   int nops;
   __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c) const {
     for (int i = 1; i < nops; ++i) {

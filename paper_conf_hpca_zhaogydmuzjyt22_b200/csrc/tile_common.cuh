@@ -227,6 +227,24 @@ __device__ __forceinline__ void tile_reload(double2 (&v)[kRegAmps], const TileCt
   for (int r = 0; r < (1 << NR); ++r) v[r] = c.own ? c.s[mp.j(r)] : make_double2(0, 0);
 }
 
+// Static-mapping variants (JIT): slot r of the thread sits at tile index base + J[r], J a
+// compile-time table, so every shared-memory access uses an immediate offset.
+template <int NR>
+__device__ __forceinline__ void tile_spill_j(const double2 (&v)[kRegAmps], const TileCtx& c, uint32_t base,
+                                             const uint32_t (&J)[kRegAmps]) {
+  __syncthreads();
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r)
+    if (c.own) c.s[base + J[r]] = v[r];
+  __syncthreads();
+}
+template <int NR>
+__device__ __forceinline__ void tile_reload_j(double2 (&v)[kRegAmps], const TileCtx& c, uint32_t base,
+                                              const uint32_t (&J)[kRegAmps]) {
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r) v[r] = c.own ? c.s[base + J[r]] : make_double2(0, 0);
+}
+
 __device__ __forceinline__ bool op_active(const TileOp& op, uint64_t gbase) {
   return (gbase & op.omask) == op.omatch;
 }
@@ -541,16 +559,24 @@ __device__ __forceinline__ SlotAddr slot_addr(const Mapping& mp, const uint64_t*
 // Each thread prefetches exactly the slots it owns under the initial mapping (cp.async, 16 B,
 // src-size 0 = hardware zero-fill beyond L_in): no thread reads another thread's load, so a
 // tile needs no CTA barrier unless its program remaps. ZM: slots known to be zero (skipped).
-template <int NR>
+template <int NR, class Body>
 __device__ __forceinline__ void issue_own_loads(double2* buf, const TileArgs& a, const Mapping& mp0,
                                                 const SlotAddr& sa0, uint64_t base, unsigned zm, bool own) {
   if (own && base < a.L_in) {
 #pragma unroll
     for (int r = 0; r < (1 << NR); ++r) {
       if ((zm >> r) & 1) continue;
-      const uint64_t idx = base | sa0.at(r);
+      uint64_t idx;
+      uint32_t j;
+      if constexpr (Body::kStatic) {
+        idx = (base | sa0.pb) + Body::kP0[r];  // the register bits are disjoint from base_j's
+        j = mp0.base + Body::kJ0[r];
+      } else {
+        idx = base | sa0.at(r);
+        j = mp0.j(r);
+      }
       const bool live = idx < a.L_in;
-      cp_async16(buf + mp0.j(r), a.psi + (live ? idx : 0), live ? 16 : 0);
+      cp_async16(buf + j, a.psi + (live ? idx : 0), live ? 16 : 0);
     }
   }
   asm volatile("cp.async.commit_group;\n" ::: "memory");
@@ -615,7 +641,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   (void)nwarps;
 
   uint64_t tile = blockIdx.x;
-  if (tile < a.ntiles) issue_own_loads<NR>(bufs, a, mp0, sa0, tile_base(tile, a), zm0, c.own);
+  if (tile < a.ntiles) issue_own_loads<NR, Body>(bufs, a, mp0, sa0, tile_base(tile, a), zm0, c.own);
   int k = 0;
   for (int it = 0; tile < a.ntiles; tile += gridDim.x, ++it) {
     double2* s = bufs + k * T;
@@ -623,7 +649,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     const uint64_t base = tile_base(tile, a);
     const uint64_t gbase = a.rank_base | base;
     const bool more = tile + gridDim.x < a.ntiles;
-    if (more) issue_own_loads<NR>(bufs + kn * T, a, mp0, sa0, tile_base(tile + gridDim.x, a), zm0, c.own);
+    if (more) issue_own_loads<NR, Body>(bufs + kn * T, a, mp0, sa0, tile_base(tile + gridDim.x, a), zm0, c.own);
     if (base >= a.L_in) {
       // the whole tile lies in the zero region of a first-touch expansion and no op of the pass
       // targets its non-tile bits: it stays zero -> store zeros, skip the program
@@ -645,7 +671,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     }
     // tile-uniform phase, per lane (lane-strided product, then butterfly)
     double2 sc = make_double2(1.0, 0.0);
-    if (a.nscalar) {
+    if (Body::kHasScalar && a.nscalar) {
       for (int q = lane; q < a.nscalar; q += 32)
         if ((gbase & scal[q].omask) == scal[q].omatch) sc = cmul(sc, make_double2(scal[q].re, scal[q].im));
 #pragma unroll
@@ -664,14 +690,27 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     double2 v[kRegAmps];
     Mapping mp = mp0;
 #pragma unroll
-    for (int r = 0; r < (1 << NR); ++r)
-      v[r] = (c.own && !((zm0 >> r) & 1)) ? s[mp0.j(r)] : make_double2(0.0, 0.0);
+    for (int r = 0; r < (1 << NR); ++r) {
+      uint32_t j;
+      if constexpr (Body::kStatic) j = mp0.base + Body::kJ0[r];
+      else j = mp0.j(r);
+      v[r] = (c.own && !((zm0 >> r) & 1)) ? s[j] : make_double2(0.0, 0.0);
+    }
     body(v, mp, c);
-    const bool has_sc = !(sc.x == 1.0 && sc.y == 0.0);
-    const SlotAddr sa = slot_addr<NR>(mp, hiOff, lowmask, l);
-    if (c.own) {
+    if (Body::kHasScalar && !(sc.x == 1.0 && sc.y == 0.0)) {
 #pragma unroll
-      for (int r = 0; r < (1 << NR); ++r) st_stream(a.psi + (base | sa.at(r)), has_sc ? cmul(v[r], sc) : v[r]);
+      for (int r = 0; r < (1 << NR); ++r) v[r] = cmul(v[r], sc);
+    }
+    if (c.own) {
+      if constexpr (Body::kStatic) {
+        const uint64_t pb = base | (mp.base & lowmask) | hiOff[mp.base >> l];
+#pragma unroll
+        for (int r = 0; r < (1 << NR); ++r) st_stream(a.psi + (pb + Body::kPF[r]), v[r]);
+      } else {
+        const SlotAddr sa = slot_addr<NR>(mp, hiOff, lowmask, l);
+#pragma unroll
+        for (int r = 0; r < (1 << NR); ++r) st_stream(a.psi + (base | sa.at(r)), v[r]);
+      }
     }
     k = kn;
     // with two buffers the next prefetch refills the buffer other warps read during remaps
