@@ -713,6 +713,9 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       }
     }
     k = kn;
+    // the lanes of this warp are done reading this tile's pattern constants before the next
+    // tile's constants are written
+    __syncwarp();
     // with two buffers the next prefetch refills the buffer other warps read during remaps
     if (nbuf < 3 && a.remaps) __syncthreads();
   }

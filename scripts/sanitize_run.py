@@ -1,0 +1,34 @@
+"""Small circuits through every kernel family, for compute-sanitizer (memcheck / racecheck /
+synccheck). Exits non-zero on a parity failure.
+
+    compute-sanitizer --tool racecheck python scripts/sanitize_run.py [--jit 0|2]
+"""
+import argparse
+import os
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+import numpy as np  # noqa: E402
+
+from oracle import statevector as osv  # noqa: E402
+from paper_conf_hpca_zhaogydmuzjyt22_b200 import qgpu as q  # noqa: E402
+from workloads import circuits as wc  # noqa: E402
+
+ap = argparse.ArgumentParser()
+ap.add_argument("--jit", type=int, default=0)
+ap.add_argument("--big", action="store_true", help="multi-tile-per-CTA cases (buffer reuse)")
+args = ap.parse_args()
+cases = [(wc.random_circuit(13, 120, seed=1), 12, 1), (wc.qft(14, x=99), 12, 1), (wc.qaoa(12, 1, seed=2), 9, 1),
+         (wc.rqc(13, 4, seed=3), 12, 2), (wc.random_circuit(12, 80, seed=4), 0, 1)]
+if args.big:  # > 3 tiles per CTA: exercises the prefetch / triple-buffer reuse and remaps
+    cases = [(wc.random_circuit(21, 60, seed=7), 12, 1), (wc.qaoa(20, 1, seed=3), 12, 1),
+             (wc.qft(21, x=12345), 12, 1)]
+worst = 0.0
+for c, fuse, world in cases:
+    with q.State(c.n, fuse_bits=fuse, jit=args.jit, world_size=world) as s:
+        s.apply_circuit(q.Circuit(c.qasm()))
+        got = s.amplitudes()
+        s.probabilities([0, 3, 5])
+    worst = max(worst, float(np.abs(got - osv.simulate(c.qasm())).max()))
+print("max |delta| =", worst)
+sys.exit(0 if worst <= 1e-10 else 1)
