@@ -24,8 +24,33 @@ struct qgpu_circuit {
 };
 
 namespace {
+// A planned circuit for a given starting qubit map: passes (with their resolved JIT kernels)
+// and the device copy of their programs. Reused when the same circuit is applied again from
+// the same map (e.g. after qgpu_state_reset): no host planning, no upload.
+struct CachedPlan {
+  uint64_t key = 0;
+  std::vector<int> order;
+  std::vector<uint64_t> inv;
+  std::vector<Pass> passes;
+  std::vector<size_t> off;
+  unsigned char* d_blob = nullptr;
+  size_t blob_bytes = 0;
+  qgpu::QubitMap map_after;
+  uint64_t relabels = 0;
+  uint64_t last_use = 0;
+};
+}  // namespace
 
-constexpr int kJitMinBits = 20;  // jit=1: specialise passes whose live range is >= 2^20
+namespace {
+
+// jit=1: specialise fused passes whose live range is >= 2^jit_min_bits amplitudes
+int jit_min_bits() {
+  static const int v = [] {
+    const char* ev = std::getenv("QGPU_JIT_MIN_BITS");
+    return ev ? std::atoi(ev) : 12;
+  }();
+  return v;
+}
 
 thread_local std::string g_err;
 
@@ -81,6 +106,8 @@ struct qgpu_state {
   std::vector<TimedLaunch> pending;
   std::vector<cudaEvent_t> event_pool;
   Comm* comm = nullptr;
+  std::vector<CachedPlan> plans;  // small LRU (kMaxPlans)
+  uint64_t plan_clock = 0;
 };
 
 namespace {
@@ -244,7 +271,7 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     if (tile_smem_bytes(a) > 227 * 1024) a.nbuf = 2;
     const int jit = st->cfg.jit;
     cudaError_t e = cudaErrorNotSupported;
-    if (jit == 2 || (jit == 1 && p.k_out >= kJitMinBits)) {
+    if (jit == 2 || (jit == 1 && p.k_out >= jit_min_bits())) {
       double ms = 0;
       e = launch_tile_jit(st->stream, p, a, tile_smem_bytes(a), device_num_sms(), &ms);
       if (e == cudaSuccess) st->stats.jit_launches++;
@@ -426,6 +453,8 @@ qgpu_status ensure_ops(qgpu_state* st, size_t n) {
   return QGPU_OK;
 }
 
+void prepare_jit(qgpu_state* st, const std::vector<Pass>& passes);
+
 qgpu_status run_plan(qgpu_state* st, const std::vector<Pass>& passes) {
   size_t nbytes = 0;
   std::vector<size_t> off(passes.size(), 0);
@@ -444,15 +473,7 @@ qgpu_status run_plan(qgpu_state* st, const std::vector<Pass>& passes) {
     st->stats.h2d_bytes += nbytes;
     CK(cudaEventRecord(st->ops_evt, st->stream));
   }
-  if (st->cfg.jit) {
-    std::vector<const Pass*> want;
-    for (const Pass& p : passes)
-      if (p.kind == PK_TILE && (st->cfg.jit == 2 || p.k_out >= kJitMinBits)) want.push_back(&p);
-    double ms = 0;
-    const int k = jit_prepare(want, &ms);
-    st->stats.jit_compiles += uint64_t(k);
-    st->stats.jit_ms += ms;
-  }
+  prepare_jit(st, passes);
   for (size_t i = 0; i < passes.size(); ++i) {
     qgpu_status s = exec_pass(st, passes[i], st->d_ops + off[i]);
     if (s) return s;
@@ -487,6 +508,59 @@ qgpu_status init_amplitudes(qgpu_state* st) {
     }
   }
   return QGPU_OK;
+}
+
+constexpr size_t kMaxPlans = 8;
+
+uint64_t plan_key(const qgpu_state* st, const qgpu_circuit* c) {
+  uint64_t h = c->c.hash ? c->c.hash : circuit_hash(c->c);
+  auto mix = [&](uint64_t v) {
+    h ^= v + 0x9e3779b97f4a7c15ull + (h << 6) + (h >> 2);
+  };
+  mix(uint64_t(st->cfg.reorder));
+  mix(uint64_t(st->cfg.fuse_bits));
+  mix(uint64_t(st->m));
+  mix(st->map.involvement);
+  mix(uint64_t(st->map.kl) | uint64_t(st->map.kg) << 8);
+  for (int q = 0; q < st->n; ++q) mix(uint64_t(uint32_t(st->map.pos[q])));
+  if (const char* ev = std::getenv("QGPU_REGBITS")) mix(uint64_t(std::atoi(ev)) << 32);
+  if (const char* ev = std::getenv("QGPU_MAX_UOPS")) mix(uint64_t(std::atoi(ev)) << 40);
+  return h;
+}
+
+PlanOptions plan_options(const qgpu_config& cfg, bool fuse);
+
+// Copy the programs of a plan's fused passes to a device buffer owned by the plan.
+qgpu_status upload_plan(qgpu_state* st, CachedPlan* cp) {
+  size_t nbytes = 0;
+  cp->off.assign(cp->passes.size(), 0);
+  for (size_t i = 0; i < cp->passes.size(); ++i) {
+    cp->off[i] = nbytes;
+    if (cp->passes[i].kind == PK_TILE) nbytes += (cp->passes[i].prog.bytes + 15) / 16 * 16;
+  }
+  cp->blob_bytes = nbytes;
+  if (!nbytes) return QGPU_OK;
+  qgpu_status s = ensure_ops(st, nbytes);
+  if (s) return s;
+  CK(cudaEventSynchronize(st->ops_evt));
+  for (size_t i = 0; i < cp->passes.size(); ++i)
+    if (cp->passes[i].kind == PK_TILE) cp->passes[i].prog.pack(st->h_ops + cp->off[i]);
+  CK(cudaMalloc(&cp->d_blob, nbytes));
+  CK(cudaMemcpyAsync(cp->d_blob, st->h_ops, nbytes, cudaMemcpyHostToDevice, st->stream));
+  st->stats.h2d_bytes += nbytes;
+  CK(cudaEventRecord(st->ops_evt, st->stream));
+  return QGPU_OK;
+}
+
+void prepare_jit(qgpu_state* st, const std::vector<Pass>& passes) {
+  if (!st->cfg.jit) return;
+  std::vector<const Pass*> want;
+  for (const Pass& p : passes)
+    if (p.kind == PK_TILE && (st->cfg.jit == 2 || p.k_out >= jit_min_bits())) want.push_back(&p);
+  double ms = 0;
+  const int k = jit_prepare(want, &ms);
+  st->stats.jit_compiles += uint64_t(k);
+  st->stats.jit_ms += ms;
 }
 
 PlanOptions plan_options(const qgpu_config& cfg, bool fuse) {
@@ -632,6 +706,8 @@ qgpu_status qgpu_state_destroy(qgpu_state* st) {
   if (st->h_ops) cudaFreeHost(st->h_ops);
   if (st->d_scratch) cudaFree(st->d_scratch);
   if (st->d_zero) cudaFree(st->d_zero);
+  for (CachedPlan& cp : st->plans)
+    if (cp.d_blob) cudaFree(cp.d_blob);
   if (st->ops_evt) cudaEventDestroy(st->ops_evt);
   if (st->own_stream && st->stream) cudaStreamDestroy(st->stream);
   delete st;
@@ -721,13 +797,40 @@ qgpu_status qgpu_apply_circuit(qgpu_state* st, const qgpu_circuit* c) {
     if (qgpu_status s = check_state(st)) return s;
     if (!c) return fail(QGPU_ERR_INVALID_ARG, "circuit is NULL");
     if (c->c.n > st->n) return fail(QGPU_ERR_INVALID_ARG, "circuit has %d qubits, state %d", c->c.n, st->n);
-    std::vector<int> order = reorder(c->c.gates, st->cfg.reorder);
-    std::vector<Pass> passes;
-    std::vector<uint64_t> inv;
-    plan_circuit(c->c.gates, order, st->map, plan_options(st->cfg, st->cfg.fuse_bits > 0), &passes, &inv);
-    record_trace(st, order, inv, 0);
-    for (const Gate& g : c->c.gates) st->stats.relabels += g.relabel ? 1 : 0;
-    return run_plan(st, passes);
+    const uint64_t key = plan_key(st, c);
+    CachedPlan* hit = nullptr;
+    for (CachedPlan& cp : st->plans)
+      if (cp.key == key) hit = &cp;
+    if (!hit) {
+      CachedPlan cp;
+      cp.key = key;
+      cp.order = reorder(c->c.gates, st->cfg.reorder);
+      QubitMap map = st->map;
+      plan_circuit(c->c.gates, cp.order, map, plan_options(st->cfg, st->cfg.fuse_bits > 0), &cp.passes, &cp.inv);
+      cp.map_after = map;
+      for (const Gate& g : c->c.gates) cp.relabels += g.relabel ? 1 : 0;
+      if (qgpu_status s = upload_plan(st, &cp)) return s;
+      if (st->plans.size() >= kMaxPlans) {  // evict the least recently used
+        size_t lru = 0;
+        for (size_t i = 1; i < st->plans.size(); ++i)
+          if (st->plans[i].last_use < st->plans[lru].last_use) lru = i;
+        CK(cudaStreamSynchronize(st->stream));
+        if (st->plans[lru].d_blob) cudaFree(st->plans[lru].d_blob);
+        st->plans.erase(st->plans.begin() + lru);
+      }
+      st->plans.push_back(std::move(cp));
+      hit = &st->plans.back();
+      prepare_jit(st, hit->passes);
+    }
+    hit->last_use = ++st->plan_clock;
+    record_trace(st, hit->order, hit->inv, 0);
+    st->stats.relabels += hit->relabels;
+    st->map = hit->map_after;
+    for (size_t i = 0; i < hit->passes.size(); ++i) {
+      qgpu_status s = exec_pass(st, hit->passes[i], hit->d_blob ? hit->d_blob + hit->off[i] : nullptr);
+      if (s) return s;
+    }
+    return QGPU_OK;
   } catch (const std::exception& ex) {
     return fail(QGPU_ERR_OUT_OF_MEMORY, "exception: %s", ex.what());
   }
@@ -859,6 +962,7 @@ qgpu_status qgpu_circuit_from_qasm(const char* text, size_t len, qgpu_circuit** 
       delete c;
       return fail(s, "%s", err.c_str());
     }
+    c->c.hash = circuit_hash(c->c);
     *out = c;
     return QGPU_OK;
   } catch (const std::exception& ex) {

@@ -466,9 +466,10 @@ cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, s
                             double* compile_ms) {
   if (!jit_available(nullptr)) return cudaErrorNotSupported;
   JitLib& L = lib();
-  const std::string src = tile_jit_source(p);
-  CUfunction fn = nullptr;
-  {
+  CUfunction fn = static_cast<CUfunction>(p.jit_fn);
+  std::string src;
+  if (!fn) {
+    src = tile_jit_source(p);
     std::lock_guard<std::mutex> g(L.mu);
     auto it = L.cache.find(src);
     if (it != L.cache.end()) fn = it->second;
@@ -492,6 +493,7 @@ cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, s
     std::lock_guard<std::mutex> g(L.mu);
     L.cache.emplace(src, fn);
   }
+  p.jit_fn = fn;
   const unsigned threads = 32u << a.nw;
   const unsigned grid = unsigned(std::min<uint64_t>(a.ntiles, uint64_t(num_sms)));
   TileArgs args = a;

@@ -47,7 +47,9 @@ struct Gate {
 struct Circuit {
   int n = 0;
   std::vector<Gate> gates;
+  uint64_t hash = 0;  // content hash (gates, matrices), set by the parser / on demand
 };
+uint64_t circuit_hash(const Circuit& c);
 
 qgpu_status parse_qasm(const char* text, size_t len, Circuit* out, std::string* err);
 // Lower a gate name: fills the arity and the target matrix; false if the name is unknown.
@@ -126,6 +128,7 @@ struct Pass {
   int nswap = 0;
   int swap_global[8], swap_local[8];
   int kg_from = 0;              // activation pass
+  mutable void* jit_fn = nullptr;  // specialised kernel, resolved at the first launch
   uint64_t unfused_bytes = 0;   // bytes the pass's gates would move one gate per pass
 };
 

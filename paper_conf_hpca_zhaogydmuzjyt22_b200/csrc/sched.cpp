@@ -107,6 +107,24 @@ std::vector<int> reorder(const std::vector<Gate>& gates, int mode) {
   return out;
 }
 
+uint64_t circuit_hash(const Circuit& c) {
+  uint64_t h = 1469598103934665603ull ^ uint64_t(c.n);
+  auto mix = [&](const void* p, size_t n) {
+    const unsigned char* b = static_cast<const unsigned char*>(p);
+    for (size_t i = 0; i < n; ++i) {
+      h ^= b[i];
+      h *= 1099511628211ull;
+    }
+  };
+  for (const Gate& g : c.gates) {
+    mix(&g.nt, sizeof(g.nt));
+    mix(g.t, sizeof(g.t));
+    mix(&g.cmask, sizeof(g.cmask));
+    mix(g.U, sizeof(cplx) * (1 << (2 * g.nt)));
+  }
+  return h;
+}
+
 // ----------------------------------------------------------------------------------- a3
 void QubitMap::init(int n_, int m_) {
   n = n_;

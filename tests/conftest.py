@@ -17,3 +17,7 @@ def pytest_configure(config):
 def rng():
     import numpy as np
     return np.random.default_rng(12345)
+
+# Specialise (NVRTC) only passes of >= 2^20 amplitudes in the test suite, to keep its compile
+# time bounded; the JIT path itself is covered by the jit=2 tests and the full-size tests.
+os.environ.setdefault("QGPU_JIT_MIN_BITS", "20")
