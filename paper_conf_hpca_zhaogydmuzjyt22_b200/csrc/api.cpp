@@ -931,7 +931,7 @@ qgpu_status qgpu_probabilities(qgpu_state* st, int mq, const int* qubits, double
     pa.L = active ? live(st, st->map.kl) : 0;
     pa.out = i == 0 ? acc : tmp;
     CK(launch_probs(st->stream, pa, part));
-    st->stats.kernels_launched += (mq <= 12) ? 2 : 1;
+    st->stats.kernels_launched += 1;
     if (i > 0) CK(launch_add(st->stream, acc, tmp, B));
   }
   if (st->comm) {

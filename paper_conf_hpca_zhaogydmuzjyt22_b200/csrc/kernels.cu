@@ -265,39 +265,98 @@ __global__ void gather_kernel(GatherArgs a) {
   }
 }
 
-// per-CTA buckets in shared memory (2^m <= 4096), partial sums per CTA, then a fixed-order
-// second pass (deterministic given the grid).
-__global__ void __launch_bounds__(kThreads) probs_block_kernel(ProbArgs a) {
-  extern __shared__ double hist[];
+// a11 probabilities. Each warp owns a contiguous range of the live prefix and walks it 32
+// amplitudes at a time (lane bits = index bits 0..4). The bucket index splits into a part
+// given by requested positions < 5 (per lane) and a part given by positions >= 5 (uniform over
+// the warp, changing only every 2^(p-5) steps): |psi|^2 accumulates in a register while the
+// uniform part is unchanged; on a change the lanes are reduced over the non-requested lane bits
+// (butterfly) and one lane per lane-pattern adds into the histogram (shared memory for
+// 2^m <= 4096 buckets, then one atomic per bucket and CTA into the output; global otherwise).
+__device__ __forceinline__ void probs_flush(double acc, int lane, uint32_t lowreq, uint32_t ylow, uint64_t hi,
+                                            double* hist, bool private_hist) {
+  // sum over the lane bits that are not requested
+#pragma unroll
+  for (int b = 0; b < 5; ++b)
+    if (!((lowreq >> b) & 1)) acc += __shfl_xor_sync(0xffffffffu, acc, 1 << b);
+  // representatives (lanes whose non-requested bits are 0) hold distinct buckets
+  if ((uint32_t(lane) & ~lowreq & 31u) == 0 && acc != 0.0) {
+    const uint64_t y = hi | ylow;
+    if (private_hist) hist[y] += acc;  // this warp's own histogram: no other writer
+    else atomicAdd(&hist[y], acc);
+  }
+}
+
+// mode 0: per-warp private histograms in shared memory (2^m <= 1024), mode 1: one shared
+// histogram per CTA with atomics (2^m <= 4096), mode 2: global atomics. The bucket of an
+// index is assembled from five byte tables (bits 8k..8k+7 of the index -> bucket bits).
+__global__ void __launch_bounds__(kThreads) probs_kernel(ProbArgs a, int mode) {
+  extern __shared__ double shist[];
+  __shared__ uint32_t btab[5][256];
   const uint32_t B = 1u << a.m;
-  for (uint32_t y = threadIdx.x; y < B; y += blockDim.x) hist[y] = 0.0;
-  __syncthreads();
-  const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
-  for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < a.L; i += stride) {
-    const double2 v = a.psi[i];
-    uint32_t y = uint32_t(a.yfixed);
-    for (int j = 0; j < a.m; ++j) y |= uint32_t((i >> a.ppos[j]) & 1) << j;
-    atomicAdd(&hist[y], v.x * v.x + v.y * v.y);
+  const int lane = threadIdx.x & 31, wib = threadIdx.x >> 5, nwb = blockDim.x >> 5;
+  double* hist = mode == 0 ? shist + size_t(wib) * B : (mode == 1 ? shist : a.out);
+  for (int e = threadIdx.x; e < 5 * 256; e += blockDim.x) {
+    const int k = e >> 8, byte = e & 255;
+    uint32_t y = 0;
+    for (int j = 0; j < a.m; ++j) {
+      const int p = a.ppos[j] - 8 * k;
+      if (p >= 0 && p < 8 && ((byte >> p) & 1)) y |= 1u << j;
+    }
+    btab[k][byte] = y;
+  }
+  if (mode < 2) {
+    const uint32_t tot = mode == 0 ? B * nwb : B;
+    for (uint32_t y = threadIdx.x; y < tot; y += blockDim.x) shist[y] = 0.0;
   }
   __syncthreads();
-  for (uint32_t y = threadIdx.x; y < B; y += blockDim.x) a.partial[uint64_t(blockIdx.x) * B + y] = hist[y];
-}
-
-__global__ void probs_reduce_kernel(const double* partial, int nblk, uint32_t B, double* out) {
-  for (uint32_t y = blockIdx.x * blockDim.x + threadIdx.x; y < B; y += gridDim.x * blockDim.x) {
-    double s = 0.0;
-    for (int k = 0; k < nblk; ++k) s += partial[uint64_t(k) * B + y];
-    out[y] = s;
+  uint32_t lowreq = 0;
+  for (int j = 0; j < a.m; ++j)
+    if (a.ppos[j] < 5) lowreq |= 1u << a.ppos[j];
+  const uint32_t ylow = btab[0][lane];  // bucket bits from the lane bits (positions 0..4)
+  const uint64_t nwarps = (uint64_t(gridDim.x) * blockDim.x) >> 5;
+  const uint64_t gw = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
+  const uint64_t steps = (a.L + 31) >> 5;
+  const uint64_t per = (steps + nwarps - 1) / nwarps;
+  const uint64_t s0 = gw * per, s1 = min(steps, s0 + per);
+  // requested positions >= 5 (uniform over the warp at each step)
+  uint64_t himask = 0;
+  for (int j = 0; j < a.m; ++j)
+    if (a.ppos[j] >= 5 && a.ppos[j] < 40) himask |= 1ull << a.ppos[j];
+  double acc = 0.0;
+  uint64_t cur = ~0ull, curbits = ~0ull;
+  constexpr int U = 8;  // loads in flight per lane
+  for (uint64_t st = s0; st < s1; st += U) {
+    double2 v[U];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint64_t i = ((st + u) << 5) | uint64_t(lane);
+      v[u] = (st + u < s1 && i < a.L) ? __ldcs(a.psi + i) : make_double2(0.0, 0.0);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      const uint64_t bits = ((st + u) << 5) & himask;
+      if (bits != curbits) {
+        const uint64_t hi = a.yfixed | btab[0][bits & 255] | btab[1][(bits >> 8) & 255] |
+                            btab[2][(bits >> 16) & 255] | btab[3][(bits >> 24) & 255] | btab[4][(bits >> 32) & 255];
+        if (cur != ~0ull) probs_flush(acc, lane, lowreq, ylow, cur, hist, mode == 0);
+        acc = 0.0;
+        cur = hi;
+        curbits = bits;
+      }
+      acc = fma(v[u].x, v[u].x, fma(v[u].y, v[u].y, acc));
+    }
   }
-}
-
-__global__ void probs_global_kernel(ProbArgs a) {
-  const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
-  for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < a.L; i += stride) {
-    const double2 v = a.psi[i];
-    uint64_t y = a.yfixed;
-    for (int j = 0; j < a.m; ++j) y |= ((i >> a.ppos[j]) & 1) << j;
-    atomicAdd(&a.out[y], v.x * v.x + v.y * v.y);
+  if (cur != ~0ull) probs_flush(acc, lane, lowreq, ylow, cur, hist, mode == 0);
+  if (mode < 2) {
+    __syncthreads();
+    for (uint32_t y = threadIdx.x; y < B; y += blockDim.x) {
+      double t = 0.0;
+      if (mode == 0)
+        for (int w = 0; w < nwb; ++w) t += shist[size_t(w) * B + y];
+      else
+        t = shist[y];
+      if (t != 0.0) atomicAdd(&a.out[y], t);
+    }
   }
 }
 
@@ -427,27 +486,21 @@ cudaError_t launch_gather(cudaStream_t st, const GatherArgs& a) {
 }
 
 // out: device buffer of 2^m doubles; scratch: >= probs_scratch_bytes(m) bytes
-size_t probs_scratch_doubles(int m) {
-  if (m > 12) return 0;
-  return size_t(num_sms()) * 2 * (size_t(1) << m);
-}
+size_t probs_scratch_doubles(int) { return 0; }
 
-cudaError_t launch_probs(cudaStream_t st, ProbArgs a, double* scratch) {
-  const uint32_t B = 1u << a.m;
-  if (a.m <= 12) {
-    const unsigned g = unsigned(num_sms()) * 2;
-    a.partial = scratch;
-    probs_block_kernel<<<g, kThreads, B * sizeof(double), st>>>(a);
-    cudaError_t e = cudaGetLastError();
-    if (e != cudaSuccess) return e;
-    probs_reduce_kernel<<<(B + 255) / 256, 256, 0, st>>>(scratch, int(g), B, a.out);
-    return cudaGetLastError();
+cudaError_t launch_probs(cudaStream_t st, ProbArgs a, double*) {
+  const size_t B = size_t(1) << a.m;
+  cudaError_t e = cudaMemsetAsync(a.out, 0, sizeof(double) * B, st);
+  if (e != cudaSuccess || a.L == 0) return e;
+  const int mode = a.m <= 10 ? 0 : (a.m <= 12 ? 1 : 2);
+  const size_t smem = mode == 0 ? B * sizeof(double) * (kThreads / 32) : (mode == 1 ? B * sizeof(double) : 0);
+  static bool configured = false;
+  if (!configured) {
+    cudaFuncSetAttribute(probs_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024);
+    configured = true;
   }
-  cudaError_t e = cudaMemsetAsync(a.out, 0, sizeof(double) * (size_t(1) << a.m), st);
-  if (e != cudaSuccess) return e;
-  if (a.L == 0) return cudaSuccess;
-  const unsigned g = grid_for(a.L, 256, 8);
-  probs_global_kernel<<<g, 256, 0, st>>>(a);
+  const unsigned g = unsigned(num_sms()) * 2;
+  probs_kernel<<<g, kThreads, smem, st>>>(a, mode);
   return cudaGetLastError();
 }
 
