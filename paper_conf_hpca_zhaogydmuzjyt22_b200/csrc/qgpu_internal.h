@@ -138,6 +138,7 @@ struct PlanOptions {
   int max_u_ops = 24;   // non-diagonal ops per fused pass (FP64 / smem budget)
   int max_ops = 256;    // all ops per fused pass
   int reg_bits = 4;     // register bits per thread (2^reg_bits amplitudes in registers)
+  bool peephole = true; // fuse CX . D . CX into a diagonal (exact)
   bool prune = true;
 };
 

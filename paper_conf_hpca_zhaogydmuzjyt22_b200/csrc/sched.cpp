@@ -258,6 +258,64 @@ int mat_class(const cplx* U, int nt) {
 //     entirely outside the tile commute with the whole pass and become the tile scalar;
 //  3. assign register bits per segment (earliest next use), encode conditions relative to
 //     the mapping, and group each run's terms into distinct patterns.
+namespace {
+
+// Peephole on the executed order (logical gates): CX(a->b) . D(b) . CX(a->b) = D'(a, b) with
+// D'(xa, xb) = d[xa xor xb] (CX is an involution, the conjugated diagonal stays diagonal).
+// Gates in between that touch neither a nor b commute with the triple. The fused form
+// multiplies every amplitude by the same entry of d the original sequence would (the CXs only
+// move amplitudes), so results are bit-identical; QAOA's cost layers (CX, RZ, CX per edge)
+// become diagonal phase terms that cost no tile bit. The involvement trace and the qubit
+// placement are still those of the original gates (the head CX touches a and b first).
+bool is_cx_gate(const Gate& g) {
+  if (g.diag || g.nt != 1 || std::popcount(g.cmask) != 1) return false;
+  const cplx* U = g.U;
+  return U[0].re == 0 && U[0].im == 0 && U[3].re == 0 && U[3].im == 0 && U[1].re == 1 && U[1].im == 0 &&
+         U[2].re == 1 && U[2].im == 0;
+}
+
+// fused[k] >= 0: order position k is the head of a fused triple (index into `out`);
+// absorbed[k]: position k was folded into an earlier head.
+void find_cx_diag_cx(const std::vector<Gate>& gates, const std::vector<int>& order, std::vector<int>* fused,
+                     std::vector<char>* absorbed, std::vector<Gate>* out) {
+  const size_t G = order.size();
+  fused->assign(G, -1);
+  absorbed->assign(G, 0);
+  for (size_t i = 0; i < G; ++i) {
+    if ((*absorbed)[i]) continue;
+    const Gate& c1 = gates[order[i]];
+    if (!is_cx_gate(c1)) continue;
+    const int a = std::countr_zero(c1.cmask), b = c1.t[0];
+    const uint64_t ab = (1ull << a) | (1ull << b);
+    size_t j = i + 1;
+    while (j < G && (gates[order[j]].qmask() & ab) == 0) ++j;
+    if (j >= G || (*absorbed)[j]) continue;
+    const Gate& d = gates[order[j]];
+    if (!(d.diag && d.nt == 1 && d.t[0] == b && d.cmask == 0)) continue;
+    size_t k = j + 1;
+    while (k < G && (gates[order[k]].qmask() & ab) == 0) ++k;
+    if (k >= G || (*absorbed)[k]) continue;
+    const Gate& c2 = gates[order[k]];
+    if (!is_cx_gate(c2) || c2.t[0] != b || c2.cmask != c1.cmask) continue;
+    Gate f;
+    f.nt = 2;
+    f.t[0] = b;  // U index bit 0
+    f.t[1] = a;  // U index bit 1
+    f.cmask = 0;
+    f.diag = true;
+    for (auto& e : f.U) e = cplx{0.0, 0.0};
+    f.U[0] = d.U[0];   // xb=0, xa=0
+    f.U[5] = d.U[3];   // xb=1, xa=0
+    f.U[10] = d.U[3];  // xb=0, xa=1
+    f.U[15] = d.U[0];  // xb=1, xa=1
+    (*fused)[i] = int(out->size());
+    out->push_back(f);
+    (*absorbed)[j] = (*absorbed)[k] = 1;
+  }
+}
+
+}  // namespace
+
 void build_tile_ops(Pass& p, int /*m*/, int reg_bits) {
   TileProgram& P = p.prog;
   P = TileProgram();
@@ -545,13 +603,23 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
   Builder B{gates, map, opt, passes};
   const bool fuse = opt.fuse_bits > 0;
   const int m = map.m;
+  std::vector<int> fused;
+  std::vector<char> absorbed;
+  std::vector<Gate> fgates;
+  if (opt.peephole) find_cx_diag_cx(gates, order, &fused, &absorbed, &fgates);
   for (int k = 0; k < int(order.size()); ++k) {
-    const Gate& g = gates[order[k]];
+    const Gate& g0 = gates[order[k]];
     const int k_before = map.kl;
     const int kg_before = map.kg;
-    const uint64_t fresh = g.qmask() & ~map.involvement;
-    map.touch(g.qmask());
+    const uint64_t fresh = g0.qmask() & ~map.involvement;
+    map.touch(g0.qmask());
     if (inv_after) inv_after->push_back(map.involvement);
+    if (opt.peephole && absorbed[k]) {  // folded into an earlier fused gate
+      if (B.open) B.cur.count++;
+      else if (!passes->empty()) passes->back().count++;
+      continue;
+    }
+    const Gate& g = (opt.peephole && fused[k] >= 0) ? fgates[fused[k]] : g0;
     if (map.kg > kg_before) {
       // sharded: a qubit was placed on a rank bit; the ranks that become active hold zeros
       B.close();

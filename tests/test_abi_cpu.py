@@ -103,7 +103,7 @@ def test_plan_invariants(q, name, fuse):
         k_prev = kout
         if fuse == 0:
             assert kind in (1, 2, 3, 4)
-            assert count == 1
+            assert count >= 1  # > 1 when CX.D.CX triples are fused into one diagonal gate
         else:
             assert kind in (0, 4)
             if kind == 0:
