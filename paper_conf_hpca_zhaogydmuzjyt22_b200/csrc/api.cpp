@@ -241,6 +241,9 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     a.nops = int(P.ops.size());
     a.npat = int(P.patterns.size());
     a.nscalar = int(P.scalar.size());
+    a.spat = P.spat;
+    a.lb = P.lb;
+    a.off_tlo = int(P.off_tlo);
     a.off_entries = int(P.off_entries);
     a.off_patterns = int(P.off_patterns);
     a.off_terms = int(P.off_terms);
@@ -267,7 +270,9 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     a.remaps = 0;
     for (size_t i = 1; i < P.ops.size(); ++i)
       if (P.ops[i].kind == OP_REMAP || P.ops[i].kind == OP_SMEM1 || P.ops[i].kind == OP_SMEM2) a.remaps = 1;
-    a.nbuf = 3;
+    // programs without remaps need one tile buffer (each thread only reads its own slots),
+    // which lets two CTAs share an SM; otherwise triple (or double) buffering
+    a.nbuf = a.remaps ? 3 : 1;
     if (tile_smem_bytes(a) > 227 * 1024) a.nbuf = 2;
     const int jit = st->cfg.jit;
     cudaError_t e = cudaErrorNotSupported;

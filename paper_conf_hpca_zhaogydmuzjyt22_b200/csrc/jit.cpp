@@ -52,6 +52,7 @@ struct JitLib {
   decltype(&cuModuleGetFunction) moduleGetFunction = nullptr;
   decltype(&cuFuncSetAttribute) funcSetAttribute = nullptr;
   decltype(&cuLaunchKernel) launchKernel = nullptr;
+  decltype(&cuOccupancyMaxActiveBlocksPerMultiprocessor) occupancy = nullptr;
   std::mutex mu;
   std::unordered_map<std::string, CUfunction> cache;
 };
@@ -101,6 +102,7 @@ bool load_driver(JitLib& L) {
   QGPU_SYM(moduleGetFunction, "cuModuleGetFunction")
   QGPU_SYM(funcSetAttribute, "cuFuncSetAttribute")
   QGPU_SYM(launchKernel, "cuLaunchKernel")
+  QGPU_SYM(occupancy, "cuOccupancyMaxActiveBlocksPerMultiprocessor")
 #undef QGPU_SYM
   return true;
 }
@@ -358,7 +360,7 @@ std::string tile_jit_source(const Pass& p) {
   }
   o << "  }\n};\n";
   o << "extern \"C\" __global__ void __launch_bounds__(" << (NR >= 4 ? 256 : 512)
-    << ", 1) qgpu_tile_pass(const TileArgs a) {\n";
+    << ", 1) qgpu_tile_pass(const TileArgs a) {\n";  // 1 or 2 CTAs/SM by registers and buffers
   o << "  JitBody body;\n  tile_driver<" << NR << ">(a, body);\n}\n";
   return o.str();
 }
@@ -495,7 +497,9 @@ cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, s
   }
   p.jit_fn = fn;
   const unsigned threads = 32u << a.nw;
-  const unsigned grid = unsigned(std::min<uint64_t>(a.ntiles, uint64_t(num_sms)));
+  int bps = 1;
+  if (L.occupancy(&bps, fn, int(threads), smem) != CUDA_SUCCESS || bps < 1) bps = 1;
+  const unsigned grid = unsigned(std::min<uint64_t>(a.ntiles, uint64_t(num_sms) * uint64_t(bps)));
   TileArgs args = a;
   void* params[] = {&args};
   const CUresult r = L.launchKernel(fn, grid, 1, 1, threads, 1, 1, unsigned(smem), reinterpret_cast<CUstream>(st),

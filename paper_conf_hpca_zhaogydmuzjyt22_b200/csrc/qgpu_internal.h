@@ -89,9 +89,13 @@ struct TileProgram {
   std::vector<PhaseTerm> terms;
   std::vector<PhaseTerm> scalar;   // tile-uniform diagonal terms (commute with the whole pass)
   std::vector<cplx> pool;          // U matrices
+  std::vector<cplx> tlo;           // [pattern][2^lb] products of the low-tile-index-bit terms
   int nr = 0, nw = 0;
+  int lb = 0;                      // tile-index bits covered by tlo
+  int spat = -1;                   // pattern of the scalar terms (-1: none)
   // byte offsets of each region inside the blob (all multiples of 16)
-  size_t off_entries = 0, off_patterns = 0, off_terms = 0, off_scalar = 0, off_pool = 0, bytes = 0;
+  size_t off_entries = 0, off_patterns = 0, off_terms = 0, off_scalar = 0, off_pool = 0, off_tlo = 0,
+         bytes = 0;
   void layout();
   void pack(unsigned char* dst) const;
 };

@@ -212,6 +212,8 @@ void TileProgram::layout() {
   o += scalar.size() * sizeof(PhaseTerm);
   off_pool = o;
   o += pool.size() * sizeof(cplx);
+  off_tlo = o;
+  o += tlo.size() * sizeof(cplx);
   bytes = o;
 }
 
@@ -222,6 +224,7 @@ void TileProgram::pack(unsigned char* dst) const {
   std::memcpy(dst + off_terms, terms.data(), terms.size() * sizeof(PhaseTerm));
   std::memcpy(dst + off_scalar, scalar.data(), scalar.size() * sizeof(PhaseTerm));
   std::memcpy(dst + off_pool, pool.data(), pool.size() * sizeof(cplx));
+  std::memcpy(dst + off_tlo, tlo.data(), tlo.size() * sizeof(cplx));
 }
 
 namespace {
@@ -316,7 +319,70 @@ void find_cx_diag_cx(const std::vector<Gate>& gates, const std::vector<int>& ord
 
 }  // namespace
 
-void build_tile_ops(Pass& p, int /*m*/, int reg_bits) {
+namespace {
+
+cplx cmul_h(cplx a, cplx b) { return cplx{a.re * b.re - a.im * b.im, a.re * b.im + a.im * b.re}; }
+
+// Split each pattern's tile-uniform terms by the tile index (bits of the tile index fill the
+// non-tile local positions in ascending order, see tile_base): terms whose condition lies on the
+// lowest lb of those positions are tabulated per pattern (Tlo), terms that avoid them are
+// evaluated once per chunk of 2^lb consecutive tiles, the rest per tile. The scalar terms become
+// one more pattern. lb depends only on the pass (never on prune or the launch), so every
+// execution mode rounds identically; it is the largest lb <= 4 whose tables still let three
+// tile buffers fit in shared memory.
+void split_patterns(TileProgram& P, const Pass& p, int m) {
+  P.spat = -1;
+  if (!P.scalar.empty()) {
+    P.spat = int(P.patterns.size());
+    P.patterns.push_back(Pattern{uint32_t(P.terms.size()), uint32_t(P.scalar.size()), 0, 0});
+    for (const PhaseTerm& t : P.scalar) P.terms.push_back(t);
+  }
+  uint64_t smask = 0;
+  for (int i = 0; i < p.b; ++i) smask |= 1ull << p.spos[i];
+  int lopos[4], nlo = 0;
+  for (int q = 0; q < m && nlo < 4; ++q)
+    if (!(smask >> q & 1)) lopos[nlo++] = q;
+  const size_t npat = P.patterns.size();
+  P.layout();
+  const size_t fixed = 3 * (size_t(16) << p.b) + ((size_t(1) << (p.b - p.l)) + 2) * 8 + P.bytes +
+                       2 * (size_t(1) << P.nw) * npat * 16 + 16;
+  int lb = nlo;
+  while (lb > 0 && fixed + npat * (size_t(16) << lb) > 227 * 1024) --lb;
+  P.lb = lb;
+  uint64_t lom = 0;
+  for (int i = 0; i < lb; ++i) lom |= 1ull << lopos[i];
+  std::vector<PhaseTerm> terms;
+  P.tlo.assign(npat << lb, cplx{1.0, 0.0});
+  for (size_t pi = 0; pi < npat; ++pi) {
+    Pattern& pt = P.patterns[pi];
+    std::vector<PhaseTerm> hi, loose, lo;
+    for (uint32_t q = pt.first; q < pt.first + pt.count; ++q) {
+      const PhaseTerm& t = P.terms[q];
+      if ((t.omask & lom) == 0) hi.push_back(t);
+      else if ((t.omask & ~lom) == 0) lo.push_back(t);
+      else loose.push_back(t);
+    }
+    for (uint32_t v = 0; v < (1u << lb); ++v) {
+      uint64_t g = 0;
+      for (int i = 0; i < lb; ++i)
+        if (v >> i & 1) g |= 1ull << lopos[i];
+      cplx c{1.0, 0.0};
+      for (const PhaseTerm& t : lo)
+        if ((g & t.omask) == t.omatch) c = cmul_h(c, cplx{t.re, t.im});
+      P.tlo[(pi << lb) + v] = c;
+    }
+    pt.first = uint32_t(terms.size());
+    pt.nhi = uint32_t(hi.size());
+    pt.count = uint32_t(hi.size() + loose.size());
+    for (const PhaseTerm& t : hi) terms.push_back(t);
+    for (const PhaseTerm& t : loose) terms.push_back(t);
+  }
+  P.terms.swap(terms);
+}
+
+}  // namespace
+
+void build_tile_ops(Pass& p, int m, int reg_bits) {
   TileProgram& P = p.prog;
   P = TileProgram();
   std::vector<RawOp> raw;
@@ -525,6 +591,7 @@ void build_tile_ops(Pass& p, int /*m*/, int reg_bits) {
     P.ops.push_back(op);
     ++i;
   }
+  split_patterns(P, p, m);
   P.layout();
   if (std::getenv("QGPU_DEBUG_PLAN")) {
     int cnt[7] = {0, 0, 0, 0, 0, 0, 0}, groups = 0;
@@ -532,10 +599,10 @@ void build_tile_ops(Pass& p, int /*m*/, int reg_bits) {
     for (const RunEntry& e : P.entries) groups += e.gend;
     std::fprintf(stderr,
                  "tile pass k %d->%d b=%d nr=%d nw=%d gates=%zu ops=%zu remap=%d u1r=%d u1l=%d u2r=%d smem=%d "
-                 "runs=%d entries=%zu groups=%d patterns=%zu terms=%zu scalar=%zu S=",
+                 "runs=%d entries=%zu groups=%d patterns=%zu terms=%zu scalar=%zu lb=%d S=",
                  p.k_in, p.k_out, p.b, nr, nw, p.gates.size(), P.ops.size(), cnt[0], cnt[1], cnt[2], cnt[3],
                  cnt[4] + cnt[5], cnt[6], P.entries.size(), groups, P.patterns.size(), P.terms.size(),
-                 P.scalar.size());
+                 P.scalar.size(), P.lb);
     for (int i = 0; i < p.b; ++i) std::fprintf(stderr, "%d%s", p.spos[i], i + 1 < p.b ? "," : "\n");
   }
 }

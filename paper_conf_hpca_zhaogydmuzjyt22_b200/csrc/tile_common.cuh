@@ -62,8 +62,12 @@ struct PhaseTerm {
   uint64_t omask, omatch;  // tile-uniform condition
   double re, im;           // phase factor
 };
+// Per-tile pattern constant = Chi(tile >> lb) * Tlo[pattern][tile & (2^lb - 1)] * loose terms:
+// terms[first, first + nhi) depend only on tile-index bits >= lb (recomputed once per chunk of
+// 2^lb consecutive tiles), terms[first + nhi, first + count) straddle both (evaluated per tile),
+// and the terms on the low lb tile-index bits are folded into the host-built table Tlo.
 struct Pattern {
-  uint32_t first, count, pad0, pad1;  // range of PhaseTerms
+  uint32_t first, count, nhi, pad;
 };
 
 #if defined(__CUDACC__)
@@ -73,7 +77,9 @@ struct TileArgs {
   const void* blob;        // TileProgram blob (ops | entries | patterns | terms | scalar | pool)
   int blob_bytes;
   int nops, npat, nscalar;
-  int off_entries, off_patterns, off_terms, off_scalar, off_pool;
+  int spat;                // pattern holding the tile-uniform (scalar) terms, -1: none
+  int lb;                  // low tile-index bits covered by the Tlo tables
+  int off_entries, off_patterns, off_terms, off_scalar, off_pool, off_tlo;
   int nr, nw;              // register / warp bits of the thread mapping
   int b, l;
   int spos[kMaxTileBits];
@@ -604,9 +610,10 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   const RunEntry* ents = reinterpret_cast<const RunEntry*>(blob + a.off_entries);
   const Pattern* pats = reinterpret_cast<const Pattern*>(blob + a.off_patterns);
   const PhaseTerm* terms = reinterpret_cast<const PhaseTerm*>(blob + a.off_terms);
-  const PhaseTerm* scal = reinterpret_cast<const PhaseTerm*>(blob + a.off_scalar);
   const double2* pool = reinterpret_cast<const double2*>(blob + a.off_pool);
+  const double2* tlo = reinterpret_cast<const double2*>(blob + a.off_tlo);
   double2* Cw = reinterpret_cast<double2*>(blob + a.blob_bytes);  // per-warp pattern constants
+  double2* Chw = Cw + (size_t(nthr) >> 5) * a.npat;               // per-warp high-bit parts
 
   {
     const int4* src = reinterpret_cast<const int4*>(a.blob);
@@ -640,16 +647,30 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   const unsigned zm0 = wzero ? 0xffffu : Body::kZM0;
   (void)nwarps;
 
-  uint64_t tile = blockIdx.x;
+  // Tile order: rounds of G CTAs x 2^lb consecutive tiles (CTA i takes chunk i of each round),
+  // so a CTA walks runs of 2^lb tiles that share the high tile-index bits; the tiles left over
+  // after the full rounds are dealt out one at a time.
+  const uint64_t G = gridDim.x, CH = 1ull << a.lb;
+  const uint64_t nfull = (a.ntiles / (G * CH)) * CH;  // tiles per CTA in full rounds
+  const uint64_t rem0 = nfull * G;
+  auto tile_at = [&](uint64_t it) -> uint64_t {
+    if (it < nfull) return ((it >> a.lb) * G + blockIdx.x) * CH + (it & (CH - 1));
+    return rem0 + blockIdx.x + (it - nfull) * G;
+  };
+  uint64_t tile = tile_at(0);
   if (tile < a.ntiles) issue_own_loads<NR, Body>(bufs, a, mp0, sa0, tile_base(tile, a), zm0, c.own);
   int k = 0;
-  for (int it = 0; tile < a.ntiles; tile += gridDim.x, ++it) {
+  uint64_t cur_hi = ~0ull;
+  for (uint64_t it = 0; tile < a.ntiles; ++it) {
     double2* s = bufs + k * T;
     const int kn = (k + 1 == nbuf) ? 0 : k + 1;
     const uint64_t base = tile_base(tile, a);
     const uint64_t gbase = a.rank_base | base;
-    const bool more = tile + gridDim.x < a.ntiles;
-    if (more) issue_own_loads<NR, Body>(bufs + kn * T, a, mp0, sa0, tile_base(tile + gridDim.x, a), zm0, c.own);
+    const uint64_t next = tile_at(it + 1);
+    const bool more = next < a.ntiles;
+    // nbuf >= 2: prefetch into the next buffer now; nbuf == 1 (programs without remaps, every
+    // thread reads only its own slots): prefetch into the same buffer right after the reload
+    if (more && nbuf > 1) issue_own_loads<NR, Body>(bufs + kn * T, a, mp0, sa0, tile_base(next, a), zm0, c.own);
     if (base >= a.L_in) {
       // the whole tile lies in the zero region of a first-touch expansion and no op of the pass
       // targets its non-tile bits: it stays zero -> store zeros, skip the program
@@ -657,34 +678,45 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
 #pragma unroll
         for (int r = 0; r < (1 << NR); ++r) st_stream(a.psi + (base | sa0.at(r)), make_double2(0.0, 0.0));
       }
+      if (more && nbuf == 1) {
+        cp_async_wait_all();
+        issue_own_loads<NR, Body>(s, a, mp0, sa0, tile_base(next, a), zm0, c.own);
+      }
       k = kn;
+      tile = next;
       if (nbuf < 3 && a.remaps) __syncthreads();
       continue;
     }
-    // pattern constants of this tile, per warp (lane-strided)
-    for (int pi = lane; pi < a.npat; pi += 32) {
-      double2 cc = make_double2(1.0, 0.0);
-      const Pattern pt = pats[pi];
-      for (uint32_t q = pt.first; q < pt.first + pt.count; ++q)
-        if ((gbase & terms[q].omask) == terms[q].omatch) cc = cmul(cc, make_double2(terms[q].re, terms[q].im));
-      Cw[size_t(warp) * a.npat + pi] = cc;
-    }
-    // tile-uniform phase, per lane (lane-strided product, then butterfly)
-    double2 sc = make_double2(1.0, 0.0);
-    if (Body::kHasScalar && a.nscalar) {
-      for (int q = lane; q < a.nscalar; q += 32)
-        if ((gbase & scal[q].omask) == scal[q].omatch) sc = cmul(sc, make_double2(scal[q].re, scal[q].im));
-#pragma unroll
-      for (int o = 16; o > 0; o >>= 1) {
-        double2 t;
-        t.x = __shfl_xor_sync(0xffffffffu, sc.x, o);
-        t.y = __shfl_xor_sync(0xffffffffu, sc.y, o);
-        sc = cmul(sc, t);
+    // pattern constants of this tile, per warp (lane-strided; each lane owns the same patterns
+    // in Chw and Cw): high-bit part once per run of 2^lb tiles, then table x loose terms
+    {
+      const uint64_t hi = tile >> a.lb;
+      const uint32_t lo = uint32_t(tile) & uint32_t(CH - 1);
+      double2* cw = Cw + size_t(warp) * a.npat;
+      double2* chw = Chw + size_t(warp) * a.npat;
+      if (hi != cur_hi) {
+        cur_hi = hi;
+        for (int pi = lane; pi < a.npat; pi += 32) {
+          double2 cc = make_double2(1.0, 0.0);
+          const Pattern pt = pats[pi];
+          for (uint32_t q = pt.first; q < pt.first + pt.nhi; ++q)
+            if ((gbase & terms[q].omask) == terms[q].omatch) cc = cmul(cc, make_double2(terms[q].re, terms[q].im));
+          chw[pi] = cc;
+        }
+      }
+      for (int pi = lane; pi < a.npat; pi += 32) {
+        double2 cc = cmul(chw[pi], tlo[(size_t(pi) << a.lb) + lo]);
+        const Pattern pt = pats[pi];
+        for (uint32_t q = pt.first + pt.nhi; q < pt.first + pt.count; ++q)
+          if ((gbase & terms[q].omask) == terms[q].omatch) cc = cmul(cc, make_double2(terms[q].re, terms[q].im));
+        cw[pi] = cc;
       }
     }
-    if (more) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
+    if (more && nbuf > 1) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
     else cp_async_wait_all();
     __syncwarp();
+    // tile-uniform phase (the scalar pattern)
+    const double2 sc = (Body::kHasScalar && a.spat >= 0) ? Cw[size_t(warp) * a.npat + a.spat] : make_double2(1.0, 0.0);
     c.s = s;
     c.gbase = gbase;
     double2 v[kRegAmps];
@@ -696,6 +728,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       else j = mp0.j(r);
       v[r] = (c.own && !((zm0 >> r) & 1)) ? s[j] : make_double2(0.0, 0.0);
     }
+    if (more && nbuf == 1) issue_own_loads<NR, Body>(s, a, mp0, sa0, tile_base(next, a), zm0, c.own);
     body(v, mp, c);
     if (Body::kHasScalar && !(sc.x == 1.0 && sc.y == 0.0)) {
 #pragma unroll
@@ -713,6 +746,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       }
     }
     k = kn;
+    tile = next;
     // the lanes of this warp are done reading this tile's pattern constants before the next
     // tile's constants are written
     __syncwarp();
