@@ -43,6 +43,17 @@ struct CachedPlan {
 
 namespace {
 
+// QGPU_BSTORE: 0 (default) per-thread stores from registers, 1 bulk stores for programs with
+// remaps, 2 bulk stores for every tile pass. Measured on B200 (profiles/r01/README.md): bulk
+// stores of 1-8 KiB runs are 1.5-1.8x slower than the per-thread stores, so they stay off.
+int bstore_mode() {
+  static const int v = [] {
+    const char* ev = std::getenv("QGPU_BSTORE");
+    return ev ? std::atoi(ev) : 0;
+  }();
+  return v;
+}
+
 // jit=1: specialise fused passes whose live range is >= 2^jit_min_bits amplitudes
 int jit_min_bits() {
   static const int v = [] {
@@ -273,7 +284,11 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     // programs without remaps need one tile buffer (each thread only reads its own slots),
     // which lets two CTAs share an SM; otherwise triple (or double) buffering
     a.nbuf = a.remaps ? 3 : 1;
+    // optional bulk stores (staged tile, async copies per run; QGPU_BSTORE)
+    const int bs = bstore_mode();
+    if (bs == 2 || (bs == 1 && a.remaps)) a.nbuf = 3;
     if (tile_smem_bytes(a) > 227 * 1024) a.nbuf = 2;
+    a.bstore = (a.nbuf == 3 && (bs == 2 || (bs == 1 && a.remaps))) ? 1 : 0;
     const int jit = st->cfg.jit;
     cudaError_t e = cudaErrorNotSupported;
     if (jit == 2 || (jit == 1 && p.k_out >= jit_min_bits())) {

@@ -252,6 +252,7 @@ std::string tile_jit_source(const Pass& p) {
   o << "  static constexpr uint32_t kJ0[kRegAmps] = " << jtab(R) << ";\n";
   o << "  static constexpr uint64_t kP0[kRegAmps] = " << ptab(R) << ";\n";
   o << "  static constexpr uint64_t kPF[kRegAmps] = " << ptab(RF) << ";\n";
+  o << "  static constexpr uint32_t kJF[kRegAmps] = " << jtab(RF) << ";\n";
   o << "  __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c) const {\n";
   o << "    const TileOp* ops = c.ops;\n";
   {
@@ -359,8 +360,9 @@ std::string tile_jit_source(const Pass& p) {
     o << "    }\n";
   }
   o << "  }\n};\n";
-  o << "extern \"C\" __global__ void __launch_bounds__(" << (NR >= 4 ? 256 : 512)
-    << ", 1) qgpu_tile_pass(const TileArgs a) {\n";  // 1 or 2 CTAs/SM by registers and buffers
+  // one CTA per SM with up to 255 registers: measured faster than 2 CTAs/SM at <= 128
+  // registers even for the single-buffer (remap-free) programs
+  o << "extern \"C\" __global__ void __launch_bounds__(" << (NR >= 4 ? 256 : 512) << ", 1) qgpu_tile_pass(const TileArgs a) {\n";
   o << "  JitBody body;\n  tile_driver<" << NR << ">(a, body);\n}\n";
   return o.str();
 }
@@ -390,6 +392,7 @@ bool jit_compile_cubin(const std::string& src, std::string* cubin, std::string* 
   L.getLogSize(prog, &n);
   log->assign(n, '\0');
   if (n) L.getLog(prog, &(*log)[0]);
+  if (std::getenv("QGPU_JIT_LOG") && n > 1) std::fprintf(stderr, "qgpu: NVRTC log:\n%s\n", log->c_str());
   bool ok = rc == NVRTC_SUCCESS;
   if (ok) {
     size_t cn = 0;

@@ -171,6 +171,7 @@ struct InterpBody {
   static constexpr uint32_t kJ0[kRegAmps] = {};
   static constexpr uint64_t kP0[kRegAmps] = {};
   static constexpr uint64_t kPF[kRegAmps] = {};
+  static constexpr uint32_t kJF[kRegAmps] = {};
   int nops;
   __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c) const {
     for (int i = 1; i < nops; ++i) {

@@ -90,7 +90,8 @@ struct TileArgs {
   uint64_t rank_base;      // rank << m (global bits for tile-uniform conditions)
   const double2* zero;     // >= 2^kMaxTileBits zero amplitudes (source of the expanded region)
   int nbuf;                // tile buffers in shared memory (2 or 3)
-  int bulk;                // 1: bulk async copies (runs of >= 2^7 amplitudes), 0: per-thread
+  int bstore;              // 1: results staged in the tile buffer and written by bulk async
+                           // copies (needs nbuf == 3), 0: per-thread stores from registers
   int remaps;              // the program contains REMAP / shared-memory ops
 };
 
@@ -588,6 +589,23 @@ __device__ __forceinline__ void issue_own_loads(double2* buf, const TileArgs& a,
   asm volatile("cp.async.commit_group;\n" ::: "memory");
 }
 
+// Bulk store of a staged tile: the tile buffer holds the results at their tile index; runs of
+// 2^l consecutive tile indices are contiguous in HBM. The lanes of warp 0 first wait until the
+// previous tile's bulk reads of shared memory are done (that buffer is the next prefetch target),
+// then the barrier publishes both facts to the CTA, then they issue one copy per run.
+__device__ __forceinline__ void bulk_store_tile(double2* s, const TileArgs& a, uint64_t base, const uint64_t* hiOff,
+                                                int warp, int lane) {
+  fence_proxy_async();
+  if (warp == 0) asm volatile("cp.async.bulk.wait_group.read 0;\n" ::: "memory");
+  __syncthreads();
+  if (warp == 0) {
+    const int nh = 1 << (a.b - a.l);
+    const uint32_t run = 16u << a.l;
+    for (int h = lane; h < nh; h += 32) bulk_s2g(a.psi + (base | hiOff[h]), s + (size_t(h) << a.l), run);
+    bulk_commit();
+  }
+}
+
 // The persistent tile loop shared by the interpreted and the JIT kernels: one CTA per SM, nbuf
 // tile buffers (3; 2 when the program blob is large). Tile i+1 is prefetched into the slots its
 // threads will own while tile i is computed in registers; stores go straight from registers
@@ -674,6 +692,16 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     if (base >= a.L_in) {
       // the whole tile lies in the zero region of a first-touch expansion and no op of the pass
       // targets its non-tile bits: it stays zero -> store zeros, skip the program
+      if (a.bstore) {
+        if (c.own) {
+#pragma unroll
+          for (int r = 0; r < (1 << NR); ++r) s[mp0.j(r)] = make_double2(0.0, 0.0);
+        }
+        bulk_store_tile(s, a, base, hiOff, warp, lane);
+        k = kn;
+        tile = next;
+        continue;
+      }
       if (c.own) {
 #pragma unroll
         for (int r = 0; r < (1 << NR); ++r) st_stream(a.psi + (base | sa0.at(r)), make_double2(0.0, 0.0));
@@ -734,7 +762,18 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
 #pragma unroll
       for (int r = 0; r < (1 << NR); ++r) v[r] = cmul(v[r], sc);
     }
-    if (c.own) {
+    if (a.bstore) {
+      if (c.own) {
+        if constexpr (Body::kStatic) {
+#pragma unroll
+          for (int r = 0; r < (1 << NR); ++r) s[mp.base + Body::kJF[r]] = v[r];
+        } else {
+#pragma unroll
+          for (int r = 0; r < (1 << NR); ++r) s[mp.j(r)] = v[r];
+        }
+      }
+      bulk_store_tile(s, a, base, hiOff, warp, lane);
+    } else if (c.own) {
       if constexpr (Body::kStatic) {
         const uint64_t pb = base | (mp.base & lowmask) | hiOff[mp.base >> l];
 #pragma unroll
@@ -753,6 +792,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     // with two buffers the next prefetch refills the buffer other warps read during remaps
     if (nbuf < 3 && a.remaps) __syncthreads();
   }
+  if (a.bstore && warp == 0) bulk_wait_all();  // shared memory must outlive the bulk reads
 }
 
 #endif  // __CUDACC__
