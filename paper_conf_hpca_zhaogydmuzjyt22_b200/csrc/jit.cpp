@@ -163,6 +163,10 @@ void cache_write(const std::string& key, const std::string& cubin) {
 
 bool jit_cubin_cached(const std::string& src, std::string* cubin, std::string* log, bool* hit) {
   const std::string key = cache_key(src);
+  if (const char* dir = std::getenv("QGPU_JIT_DUMP")) {  // generated sources, for inspection
+    std::ofstream f(std::string(dir) + "/qgpu_pass_" + key + ".cu");
+    f << src;
+  }
   if (cache_read(key, cubin)) {
     if (hit) *hit = true;
     return true;
@@ -281,37 +285,55 @@ std::string tile_jit_source(const Pass& p) {
         const char* acc[5] = {"t0", "e0", "e1", "e2", "e3"};
         uint32_t e = op.moff;
         o << "      const uint32_t tb = mp.base; (void)tb;\n";
-        o << "      double2 t0 = make_double2(1.0, 0.0), e0 = t0, e1 = t0, e2 = t0, e3 = t0;\n";
+        o << "      const double2 one = make_double2(1.0, 0.0); (void)one;\n";
+        // the product of a list of entries: entries with equal tmask have distinct tmatch, so at
+        // most one of them matches a thread -> one select per tmask group, one cmul per extra
+        // group, and an unconditional entry is a plain load
+        auto product = [&](const char* name, uint32_t e0, uint32_t e1) {
+          std::vector<uint32_t> masks;
+          for (uint32_t q = e0; q < e1; ++q)
+            if (std::find(masks.begin(), masks.end(), P.entries[q].tmask) == masks.end())
+              masks.push_back(P.entries[q].tmask);
+          for (size_t gi = 0; gi < masks.size(); ++gi) {
+            const uint32_t m = masks[gi];
+            const std::string f = gi == 0 ? std::string(name) : std::string("f");
+            o << "      { double2 f;\n" + std::string(gi == 0 ? "" : "");
+            if (m == 0) {
+              for (uint32_t q = e0; q < e1; ++q)
+                if (P.entries[q].tmask == 0) o << "        f = c.C[" << P.entries[q].pat << "];\n";
+            } else {
+              o << "        f = one;\n";
+              for (uint32_t q = e0; q < e1; ++q)
+                if (P.entries[q].tmask == m)
+                  o << "        if ((tb & " << m << "u) == " << P.entries[q].tmatch << "u) f = c.C["
+                    << P.entries[q].pat << "];\n";
+            }
+            if (gi == 0) o << "        " << name << " = f; }\n";
+            else o << "        " << name << " = cmul(" << name << ", f); }\n";
+            (void)f;
+          }
+        };
+        o << "      double2 t0 = one, e0 = one, e1 = one, e2 = one, e3 = one;\n";
         int used = 0;
         for (int sl = 0; sl < 5; ++sl) {
-          for (int k = 0; k < ns[sl]; ++k, ++e) {
-            const RunEntry& en = P.entries[e];
-            used |= 1 << sl;
-            o << "      ";
-            if (en.tmask) o << "if ((tb & " << en.tmask << "u) == " << en.tmatch << "u) ";
-            o << acc[sl] << " = cmul(" << acc[sl] << ", c.C[" << en.pat << "]);\n";
-          }
+          if (ns[sl]) used |= 1 << sl;
+          product(acc[sl], e, e + uint32_t(ns[sl]));
+          e += uint32_t(ns[sl]);
         }
         if (used)
-          o << "      run_apply_table_z<" << NR << ", " << ((used >> 1) & 1 ? "true" : "false") << ", "
-            << ((used >> 2) & 1 ? "true" : "false") << ", " << ((used >> 3) & 1 ? "true" : "false") << ", "
-            << ((used >> 4) & 1 ? "true" : "false") << ", " << zm << "u>(v, t0, e0, e1, e2, e3);\n";
+          o << "      run_apply_ptab_z<" << NR << ", " << (used & 1 ? "true" : "false") << ", "
+            << ((used >> 1) & 1 ? "true" : "false") << ", " << ((used >> 2) & 1 ? "true" : "false") << ", "
+            << ((used >> 3) & 1 ? "true" : "false") << ", " << ((used >> 4) & 1 ? "true" : "false") << ", " << zm
+            << "u>(v, t0, e0, e1, e2, e3);\n";
         const uint32_t end = op.moff + op.cnt;
-        bool open_group = false;
-        for (; e < end; ++e) {
-          const RunEntry& en = P.entries[e];
-          if (!open_group) {
-            o << "      { double2 acc = make_double2(1.0, 0.0);\n";
-            open_group = true;
-          }
-          o << "        ";
-          if (en.tmask) o << "if ((tb & " << en.tmask << "u) == " << en.tmatch << "u) ";
-          o << "acc = cmul(acc, c.C[" << en.pat << "]);\n";
-          if (en.gend) {
-            o << "        run_apply_group_z<" << NR << ", " << en.rmask << "u, " << en.rmatch << "u, " << zm
-              << "u>(v, acc); }\n";
-            open_group = false;
-          }
+        for (uint32_t g0 = e; g0 < end;) {
+          uint32_t g1 = g0;
+          while (!P.entries[g1].gend) ++g1;
+          o << "      { double2 acc;\n";
+          product("acc", g0, g1 + 1);
+          o << "        run_apply_group_z<" << NR << ", " << P.entries[g0].rmask << "u, " << P.entries[g0].rmatch << "u, "
+            << zm << "u>(v, acc); }\n";
+          g0 = g1 + 1;
         }
         break;
       }

@@ -400,9 +400,33 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
       const int dim = 1 << g.nt;
       uint64_t tmask = 1ull << g.p[0];
       if (g.nt == 2) tmask |= 1ull << g.p[1];
+      // Controls (if any) outside the tile: factor the most frequent diagonal entry out as a
+      // tile-uniform term, so that only the amplitudes whose entry differs get a multiply
+      // (e.g. ZZ = diag(d0,d1,d1,d0) -> d0 * diag(1,r,r,1), RZ -> d0 * diag(1,r)).
+      cplx ref{1.0, 0.0};
+      if (to_local(g.pc, p) == 0) {
+        int best = 0, bestn = 0;
+        for (int v = 0; v < dim; ++v) {
+          const cplx d = g.U[v * (dim + 1)];
+          int cnt = 0;
+          for (int w = 0; w < dim; ++w) {
+            const cplx e = g.U[w * (dim + 1)];
+            cnt += (e.re == d.re && e.im == d.im) ? 1 : 0;
+          }
+          if (cnt > bestn) best = v, bestn = cnt;
+        }
+        const cplx d = g.U[best * (dim + 1)];
+        if (bestn > 1 && !(d.re == 1.0 && d.im == 0.0)) {
+          ref = d;
+          P.scalar.push_back(PhaseTerm{outside(g.pc, p), outside(g.pc, p), d.re, d.im});
+        }
+      }
+      const double rn = ref.re * ref.re + ref.im * ref.im;
       for (int v = 0; v < dim; ++v) {
-        const cplx d = g.U[v * (dim + 1)];
-        if (d.re == 1.0 && d.im == 0.0) continue;
+        cplx d = g.U[v * (dim + 1)];
+        if (d.re == ref.re && d.im == ref.im) continue;  // also skips exact 1 when ref = 1
+        if (!(ref.re == 1.0 && ref.im == 0.0))
+          d = cplx{(d.re * ref.re + d.im * ref.im) / rn, (d.im * ref.re - d.re * ref.im) / rn};
         uint64_t match = g.pc;
         for (int j = 0; j < g.nt; ++j)
           if (v >> j & 1) match |= 1ull << g.p[j];

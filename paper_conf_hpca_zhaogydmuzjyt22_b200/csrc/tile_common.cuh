@@ -472,6 +472,37 @@ __device__ __forceinline__ void run_apply_table_z(double2 (&v)[kRegAmps], double
   for (int r = 0; r < (1 << NR); ++r)
     if (!((ZM >> r) & 1)) v[r] = cmul(v[r], P[r]);
 }
+// As run_apply_table_z with compile-time identity tracking: T0 = false means t0 == 1, so the
+// table entries that are products of identities are neither formed nor applied.
+template <int NR, bool T0, bool E0, bool E1, bool E2, bool E3, unsigned ZM>
+__device__ __forceinline__ void run_apply_ptab_z(double2 (&v)[kRegAmps], double2 t0, double2 e0, double2 e1,
+                                                 double2 e2, double2 e3) {
+  double2 P[kRegAmps];
+  bool id[kRegAmps];
+  P[0] = t0;
+  id[0] = !T0;
+  const double2 ek[4] = {e0, e1, e2, e3};
+  const bool has[4] = {E0, E1, E2, E3};
+#pragma unroll
+  for (int k = 0; k < NR; ++k)
+#pragma unroll
+    for (int r = 0; r < (1 << k); ++r) {
+      const int q = r | (1 << k);
+      if (!has[k]) {
+        P[q] = P[r];
+        id[q] = id[r];
+      } else if (id[r]) {
+        P[q] = ek[k];
+        id[q] = false;
+      } else {
+        P[q] = cmul(P[r], ek[k]);
+        id[q] = false;
+      }
+    }
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r)
+    if (!((ZM >> r) & 1) && !id[r]) v[r] = cmul(v[r], P[r]);
+}
 template <int NR, unsigned RM, unsigned RT, unsigned ZM>
 __device__ __forceinline__ void run_apply_group_z(double2 (&v)[kRegAmps], double2 acc) {
 #pragma unroll
