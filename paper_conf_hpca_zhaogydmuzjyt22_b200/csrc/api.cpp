@@ -545,6 +545,7 @@ uint64_t plan_key(const qgpu_state* st, const qgpu_circuit* c) {
   for (int q = 0; q < st->n; ++q) mix(uint64_t(uint32_t(st->map.pos[q])));
   if (const char* ev = std::getenv("QGPU_REGBITS")) mix(uint64_t(std::atoi(ev)) << 32);
   if (const char* ev = std::getenv("QGPU_MAX_UOPS")) mix(uint64_t(std::atoi(ev)) << 40);
+  if (const char* ev = std::getenv("QGPU_LOOKAHEAD")) mix(uint64_t(std::atoi(ev)) << 48);
   return h;
 }
 
@@ -583,11 +584,17 @@ void prepare_jit(qgpu_state* st, const std::vector<Pass>& passes) {
   st->stats.jit_ms += ms;
 }
 
+// experiment overrides of the planner defaults (also part of the plan-cache key)
+void plan_env(PlanOptions* o) {
+  if (const char* ev = std::getenv("QGPU_REGBITS")) o->reg_bits = std::atoi(ev);
+  if (const char* ev = std::getenv("QGPU_MAX_UOPS")) o->max_u_ops = std::atoi(ev);
+  if (const char* ev = std::getenv("QGPU_LOOKAHEAD")) o->lookahead = std::atoi(ev);
+}
+
 PlanOptions plan_options(const qgpu_config& cfg, bool fuse) {
   PlanOptions o;
   o.fuse_bits = fuse ? cfg.fuse_bits : 0;
-  if (const char* ev = std::getenv("QGPU_REGBITS")) o.reg_bits = std::atoi(ev);
-  if (const char* ev = std::getenv("QGPU_MAX_UOPS")) o.max_u_ops = std::atoi(ev);
+  plan_env(&o);
   o.prune = cfg.prune != 0;
   return o;
 }
@@ -1027,6 +1034,7 @@ qgpu_status qgpu_circuit_plan(const qgpu_circuit* c, int n, int world, int reord
     map.init(n, n - g);
     PlanOptions o;
     o.fuse_bits = fuse_bits;
+    plan_env(&o);
     std::vector<Pass> passes;
     plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode), map, o, &passes, nullptr);
     if (n_passes) *n_passes = passes.size();
@@ -1057,6 +1065,7 @@ qgpu_status qgpu_circuit_plan_text(const qgpu_circuit* c, int n, int world, int 
     map.init(n, n - g);
     PlanOptions o;
     o.fuse_bits = fuse_bits;
+    plan_env(&o);
     std::vector<Pass> passes;
     plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode), map, o, &passes, nullptr);
     std::string t;
@@ -1105,6 +1114,7 @@ qgpu_status qgpu_circuit_jit_check(const qgpu_circuit* c, int n, int reorder_mod
     map.init(n, n);
     PlanOptions o;
     o.fuse_bits = fuse_bits;
+    plan_env(&o);
     std::vector<Pass> passes;
     plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode), map, o, &passes, nullptr);
     std::string cubin, log;

@@ -143,11 +143,14 @@ struct PlanOptions {
   int max_ops = 256;    // all ops per fused pass
   int reg_bits = 4;     // register bits per thread (2^reg_bits amplitudes in registers)
   bool peephole = true; // fuse CX . D . CX into a diagonal (exact)
+  int lookahead = 192;  // fusion lookahead window (gates); 0: passes are runs of `order`
   bool prune = true;
 };
 
-// Cut `order` of `gates` into passes, updating `map` (involvement, placement) exactly as the
-// execution will. inv_after[k] = involvement after the k-th executed gate.
+// Cut `gates` into passes, updating `map` (involvement, placement) exactly as the execution
+// will. The execution order is `order` with fusion lookahead (later commuting gates that join
+// the open tile pass are pulled forward); passes are consecutive runs of that execution order.
+// inv_after[k] = involvement after the k-th gate of `order` (the paper's trace).
 void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order, QubitMap& map,
                   const PlanOptions& opt, std::vector<Pass>* passes,
                   std::vector<uint64_t>* inv_after);

@@ -12,6 +12,7 @@
 // a4  pass planner: cuts the executed order into CONSECUTIVE runs (the per-gate involvement
 //     trace is unchanged); each run is one fused HBM pass over tiles of 2^b amplitudes.
 #include <algorithm>
+#include <array>
 #include <bit>
 #include <cstdio>
 #include <cstdlib>
@@ -280,7 +281,7 @@ bool is_cx_gate(const Gate& g) {
 // fused[k] >= 0: order position k is the head of a fused triple (index into `out`);
 // absorbed[k]: position k was folded into an earlier head.
 void find_cx_diag_cx(const std::vector<Gate>& gates, const std::vector<int>& order, std::vector<int>* fused,
-                     std::vector<char>* absorbed, std::vector<Gate>* out) {
+                     std::vector<char>* absorbed, std::vector<Gate>* out, std::vector<std::array<int, 2>>* parts) {
   const size_t G = order.size();
   fused->assign(G, -1);
   absorbed->assign(G, 0);
@@ -313,6 +314,7 @@ void find_cx_diag_cx(const std::vector<Gate>& gates, const std::vector<int>& ord
     f.U[15] = d.U[0];  // xb=1, xa=1
     (*fused)[i] = int(out->size());
     out->push_back(f);
+    parts->push_back({int(j), int(k)});
     (*absorbed)[j] = (*absorbed)[k] = 1;
   }
 }
@@ -694,27 +696,41 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
   Builder B{gates, map, opt, passes};
   const bool fuse = opt.fuse_bits > 0;
   const int m = map.m;
+  const int G = int(order.size());
   std::vector<int> fused;
   std::vector<char> absorbed;
   std::vector<Gate> fgates;
-  if (opt.peephole) find_cx_diag_cx(gates, order, &fused, &absorbed, &fgates);
-  for (int k = 0; k < int(order.size()); ++k) {
+  std::vector<std::array<int, 2>> parts;
+  if (opt.peephole) find_cx_diag_cx(gates, order, &fused, &absorbed, &fgates, &parts);
+  // the paper's involvement trace follows `order` (Alg.1 l.11), whatever the execution order
+  if (inv_after) {
+    uint64_t inv = map.involvement;
+    for (int k = 0; k < G; ++k) inv_after->push_back(inv |= gates[order[k]].qmask());
+  }
+  auto gate_at = [&](int k) -> const Gate& {
+    return (opt.peephole && fused[k] >= 0) ? fgates[fused[k]] : gates[order[k]];
+  };
+  int xi = 0;  // execution index: passes are consecutive runs of the execution order
+
+  // execute order position k: placement, sharded activation / swaps, then the gate joins the
+  // open fused pass or opens a new one
+  auto emit = [&](int k) {
     const Gate& g0 = gates[order[k]];
     const int k_before = map.kl;
     const int kg_before = map.kg;
     const uint64_t fresh = g0.qmask() & ~map.involvement;
     map.touch(g0.qmask());
-    if (inv_after) inv_after->push_back(map.involvement);
     if (opt.peephole && absorbed[k]) {  // folded into an earlier fused gate
       if (B.open) B.cur.count++;
       else if (!passes->empty()) passes->back().count++;
-      continue;
+      ++xi;
+      return;
     }
-    const Gate& g = (opt.peephole && fused[k] >= 0) ? fgates[fused[k]] : g0;
+    const Gate& g = gate_at(k);
     if (map.kg > kg_before) {
       // sharded: a qubit was placed on a rank bit; the ranks that become active hold zeros
       B.close();
-      B.start(PK_ACTIVATE, k, k_before);
+      B.start(PK_ACTIVATE, xi, k_before);
       B.cur.kg_from = kg_before;
       B.cur.kg = map.kg;
       B.cur.k_out = map.kl;
@@ -727,15 +743,17 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
         map.swap_positions(pa, pb);
         B.cur.k_out = map.kl;
         B.cur.count++;
-        continue;
+        ++xi;
+        return;
       }
       B.close();
-      B.start(PK_RELABEL, k, k_before);
+      B.start(PK_RELABEL, xi, k_before);
       map.swap_positions(pa, pb);
       B.cur.k_out = map.kl;
       B.cur.count = 1;
       B.close();
-      continue;
+      ++xi;
+      return;
     }
     if (!g.diag) {
       // a non-diagonal target on a rank bit: swap it with a local position first (a10).
@@ -749,7 +767,7 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
       }
       if (ng) {
         B.close();
-        B.start(PK_SWAP, k, map.kl);
+        B.start(PK_SWAP, xi, map.kl);
         B.cur.count = 0;
         int victim = m - 1;
         for (int j = 0; j < ng; ++j) {
@@ -782,7 +800,7 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
       int n_new_ops = g.diag ? (1 << g.nt) : 1;
       if (!(B.open && B.cur.kind == PK_TILE && B.fits(need, n_new_ops))) {
         B.close();
-        B.start(PK_TILE, k, k_before);
+        B.start(PK_TILE, xi, k_before);
       }
       B.used |= need;
       if (need) B.n_u++;
@@ -793,13 +811,74 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
       B.cur.unfused_bytes += unfused_gate_bytes(pg, k_before, map.kl);
     } else {
       B.close();
-      B.start(g.diag ? PK_DIAG : (g.nt == 1 ? PK_PAIR : PK_QUAD), k, k_before);
+      B.start(g.diag ? PK_DIAG : (g.nt == 1 ? PK_PAIR : PK_QUAD), xi, k_before);
       B.cur.gates.push_back(pg);
       B.cur.count = 1;
       B.cur.k_out = map.kl;
       B.cur.unfused_bytes = unfused_gate_bytes(pg, k_before, map.kl);
       B.close();
     }
+    ++xi;
+  };
+
+  // Does order position k join the open tile pass as it stands? Only for gates that place no
+  // new qubit, move no data (no relabel, no rank-bit target) and fit the tile's budget.
+  auto joins_open_pass = [&](int k) {
+    if (!(fuse && B.open && B.cur.kind == PK_TILE)) return false;
+    const Gate& g = gate_at(k);
+    if (g.relabel || (g.qmask() & ~map.involvement)) return false;
+    uint64_t need = 0;
+    if (!g.diag) {
+      for (int j = 0; j < g.nt; ++j) {
+        const int p = map.pos[g.t[j]];
+        if (p >= m) return false;
+        need |= 1ull << p;
+      }
+    }
+    return B.fits(need, g.diag ? (1 << g.nt) : 1);
+  };
+
+  // Fusion lookahead: when the next gate in order cannot join the open tile pass, a later gate
+  // that commutes with everything it would overtake (shares no qubit with any gate still
+  // pending ahead of it) and joins the pass is executed first. Gates that place new qubits are
+  // never moved, so the delayed involvement of Alg.3's order is kept.
+  std::vector<int> pend;
+  pend.reserve(size_t(G));
+  for (int k = 0; k < G; ++k)
+    if (!(opt.peephole && absorbed[k])) pend.push_back(k);
+  std::vector<std::array<int, 2>> part_of(size_t(G), {-1, -1});
+  for (int k = 0; k < G; ++k)
+    if (opt.peephole && fused[k] >= 0) part_of[size_t(k)] = parts[size_t(fused[k])];
+  const int W = fuse ? opt.lookahead : 0;
+  size_t head = 0;
+  std::vector<char> done(size_t(G), 0);
+  while (head < pend.size()) {
+    size_t pick = head;
+    if (W > 0 && B.open && B.cur.kind == PK_TILE && !joins_open_pass(pend[head])) {
+      const Gate& g = gate_at(pend[head]);
+      if (!g.relabel && !(g.qmask() & ~map.involvement)) {
+        uint64_t blocked = g.qmask();
+        int seen = 0;
+        for (size_t i = head + 1; i < pend.size() && seen < W; ++i) {
+          if (done[size_t(pend[i])]) continue;
+          ++seen;
+          const uint64_t qm = gate_at(pend[i]).qmask();
+          if (!(qm & blocked) && joins_open_pass(pend[i])) {
+            pick = i;
+            break;
+          }
+          blocked |= qm;
+        }
+      }
+    }
+    const int k = pend[pick];
+    done[size_t(k)] = 1;
+    emit(k);
+    if (part_of[size_t(k)][0] >= 0) {
+      emit(part_of[size_t(k)][0]);
+      emit(part_of[size_t(k)][1]);
+    }
+    while (head < pend.size() && done[size_t(pend[head])]) ++head;
   }
   B.close();
 }

@@ -163,3 +163,21 @@ def test_jit_sources_compile_without_gpu(q):
             raise
         n_tile = sum(1 for r in qc.plan(c.n, 1, 2, 7) if r[2] == 0)
         assert k == n_tile
+
+
+def test_fusion_lookahead_cuts_hbm_passes(q, monkeypatch):
+    """Fusion lookahead (planner): commuting later gates join the open tile pass, so a depth-20
+    random circuit needs far fewer full-state passes than cutting the reordered list in runs;
+    the partition stays a sequence of consecutive runs of the execution order."""
+    c = wc.rqc(30, 20, seed=3)
+
+    def traffic(la):
+        monkeypatch.setenv("QGPU_LOOKAHEAD", str(la))
+        plan = q.Circuit(c.qasm()).plan(c.n, 1, 2, 12)
+        pos = 0
+        for first, count, *_ in plan:
+            assert first == pos
+            pos += count
+        return sum(2.0 ** r[3] + 2.0 ** r[4] for r in plan if r[2] == 0) / 2 ** (c.n + 1)
+
+    assert traffic(192) < 0.6 * traffic(0)
