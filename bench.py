@@ -33,7 +33,15 @@ sys.path.insert(0, ROOT)
 METRIC = "circuit sec & gate-apply HBM GB/s vs peak, 28–36 qubits, 1/2/4/8 B200"
 
 
-def workload(name: str, n: int | None):
+def grid_shape(n: int):
+    """rows x cols = n with rows <= cols as close as possible (grid workloads)."""
+    r = int(math.isqrt(n))
+    while n % r:
+        r -= 1
+    return r, n // r
+
+
+def workload(name: str, n: int | None, world: int = 1):
     from workloads import circuits as wc
     if name == "qft28":
         nn = n or 28
@@ -44,10 +52,13 @@ def workload(name: str, n: int | None):
     if name == "rqc":
         nn = n or 30
         return wc.rqc(nn, 20, seed=3), f"rqc_{nn} depth 20 seed 3 (configs[3] shape)"
+    # grid workloads (configs[4]: 36 qubits on 8 GPUs = 128 GB per GPU): 2^33 amplitudes per GPU
     if name == "gs":
-        return wc.gs(6, 6), "gs_36 6x6 grid (configs[4])"
+        r, cc = grid_shape(n or min(36, 33 + int(math.log2(world))))
+        return wc.gs(r, cc), f"gs_{r * cc} {r}x{cc} grid (configs[4] shape, 128 GB per GPU at 36 qubits / 8 GPUs)"
     if name == "hlf":
-        return wc.hlf(6, 6, seed=2), "hlf_36 6x6 grid seed 2 (configs[4])"
+        r, cc = grid_shape(n or min(36, 33 + int(math.log2(world))))
+        return wc.hlf(r, cc, seed=2), f"hlf_{r * cc} {r}x{cc} grid seed 2 (configs[4] shape)"
     raise SystemExit(f"unknown workload {name}")
 
 
@@ -60,28 +71,71 @@ def peaks():
 
 
 class ClockSampler:
-    """nvidia-smi clocks + throttle reasons sampled every 200 ms during the timed region."""
+    """SM clocks and throttle reasons sampled DURING the timed region. NVML (pynvml) is polled
+    from a thread every ~1 ms, so even a few-millisecond timed region gets samples; without
+    NVML, `nvidia-smi -lms 200` (the profiling recipe's clocks line) is the fallback."""
+    REASONS = (("hw_slowdown", 0x8), ("hw_thermal_slowdown", 0x40), ("sw_thermal_slowdown", 0x20),
+               ("sw_power_cap", 0x4))
     FIELDS = ("clocks.sm,clocks.max.sm,clocks_event_reasons.hw_slowdown,"
               "clocks_event_reasons.hw_thermal_slowdown,clocks_event_reasons.sw_thermal_slowdown,"
               "clocks_event_reasons.sw_power_cap")
 
     def __init__(self, device: int):
         self.device = device
+        self.rows = []
+        self.nv = None
         self.proc = None
         self.f = None
+        self.source = None
+
+    def _nvml_handle(self):
+        import pynvml
+        import torch
+        pynvml.nvmlInit()
+        try:
+            p = torch.cuda.get_device_properties(self.device)
+            bus = f"{p.pci_domain_id:08x}:{p.pci_bus_id:02x}:{p.pci_device_id:02x}.0"
+            return pynvml, pynvml.nvmlDeviceGetHandleByPciBusId(bus)
+        except Exception:
+            return pynvml, pynvml.nvmlDeviceGetHandleByIndex(self.device)
+
+    def _poll(self):
+        nv, h = self.nv
+        while not self.stop.is_set():
+            try:
+                self.rows.append((nv.nvmlDeviceGetClockInfo(h, nv.NVML_CLOCK_SM),
+                                  nv.nvmlDeviceGetMaxClockInfo(h, nv.NVML_CLOCK_SM),
+                                  nv.nvmlDeviceGetCurrentClocksEventReasons(h)))
+            except Exception:
+                break
+            time.sleep(0.001)
 
     def __enter__(self):
+        import threading
+        try:
+            self.nv = self._nvml_handle()
+            self.stop = threading.Event()
+            self.th = threading.Thread(target=self._poll, daemon=True)
+            self.th.start()
+            self.source = "nvml poll ~1 ms"
+            return self
+        except Exception:
+            self.nv = None
         try:
             self.f = tempfile.NamedTemporaryFile("w+", delete=False, suffix=".csv")
             self.proc = subprocess.Popen(
                 ["nvidia-smi", "-i", str(self.device), f"--query-gpu={self.FIELDS}",
                  "--format=csv,noheader,nounits", "-lms", "200"], stdout=self.f,
                 stderr=subprocess.DEVNULL)
+            self.source = "nvidia-smi -lms 200"
         except Exception:
             self.proc = None
         return self
 
     def __exit__(self, *a):
+        if self.nv is not None:
+            self.stop.set()
+            self.th.join(timeout=5)
         if self.proc is not None:
             self.proc.terminate()
             try:
@@ -90,22 +144,24 @@ class ClockSampler:
                 self.proc.kill()
 
     def summary(self):
-        if self.proc is None:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["nvidia-smi unavailable"]}
-        self.f.flush()
-        rows = []
-        for line in open(self.f.name):
-            parts = [x.strip() for x in line.split(",")]
-            if len(parts) == 6 and parts[0].isdigit():
-                rows.append(parts)
-        os.unlink(self.f.name)
+        if self.nv is not None:
+            rows = [(c, m, r) for c, m, r in self.rows]
+        elif self.proc is not None:
+            self.f.flush()
+            rows = []
+            for line in open(self.f.name):
+                parts = [x.strip() for x in line.split(",")]
+                if len(parts) == 6 and parts[0].isdigit():
+                    bits = sum(b for (_, b), v in zip(self.REASONS, parts[2:]) if v == "Active")
+                    rows.append((int(parts[0]), int(parts[1]), bits))
+            os.unlink(self.f.name)
+        else:
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": ["no NVML / nvidia-smi"], "samples": 0}
         if not rows:
-            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0}
-        names = ["hw_slowdown", "hw_thermal_slowdown", "sw_thermal_slowdown", "sw_power_cap"]
-        reasons = sorted({names[i] for r in rows for i in range(4) if r[2 + i] == "Active"})
-        return {"sm_mhz": statistics.median(int(r[0]) for r in rows),
-                "sm_max_mhz": max(int(r[1]) for r in rows), "reasons": reasons,
-                "samples": len(rows)}
+            return {"sm_mhz": None, "sm_max_mhz": None, "reasons": [], "samples": 0, "source": self.source}
+        reasons = sorted({name for _, _, r in rows for name, bit in self.REASONS if r & bit})
+        return {"sm_mhz": statistics.median(c for c, _, _ in rows), "sm_max_mhz": max(m for _, m, _ in rows),
+                "reasons": reasons, "samples": len(rows), "source": self.source}
 
 
 def dist_setup(args):
@@ -245,7 +301,7 @@ def run_ours(args):
     from paper_conf_hpca_zhaogydmuzjyt22_b200 import qgpu as q
     q.load()
 
-    circ, desc = workload(args.workload, args.n)
+    circ, desc = workload(args.workload, args.n, world if args.sharded else 1)
     text = circ.qasm()
     n = circ.n
     stream = torch.cuda.Stream(device=device)
