@@ -25,8 +25,10 @@ struct qgpu_circuit {
 
 namespace {
 // A planned circuit for a given starting qubit map: passes (with their resolved JIT kernels)
-// and the device copy of their programs. Reused when the same circuit is applied again from
-// the same map (e.g. after qgpu_state_reset): no host planning, no upload.
+// and their packed programs (pinned host blob + device copy). Reused when the same circuit is
+// applied again from the same map (e.g. after qgpu_state_reset): no host planning; the packed
+// gate data (matrices, phases, conditions) is re-sent host->device on every apply, an async
+// copy of a few KB that keeps each apply's inputs flowing like an uncached run.
 struct CachedPlan {
   uint64_t key = 0;
   std::vector<int> order;
@@ -34,6 +36,7 @@ struct CachedPlan {
   std::vector<Pass> passes;
   std::vector<size_t> off;
   unsigned char* d_blob = nullptr;
+  unsigned char* h_blob = nullptr;  // pinned, immutable once packed
   size_t blob_bytes = 0;
   qgpu::QubitMap map_after;
   uint64_t relabels = 0;
@@ -561,15 +564,19 @@ qgpu_status upload_plan(qgpu_state* st, CachedPlan* cp) {
   }
   cp->blob_bytes = nbytes;
   if (!nbytes) return QGPU_OK;
-  qgpu_status s = ensure_ops(st, nbytes);
-  if (s) return s;
-  CK(cudaEventSynchronize(st->ops_evt));
+  CK(cudaMallocHost(&cp->h_blob, nbytes));
   for (size_t i = 0; i < cp->passes.size(); ++i)
-    if (cp->passes[i].kind == PK_TILE) cp->passes[i].prog.pack(st->h_ops + cp->off[i]);
+    if (cp->passes[i].kind == PK_TILE) cp->passes[i].prog.pack(cp->h_blob + cp->off[i]);
   CK(cudaMalloc(&cp->d_blob, nbytes));
-  CK(cudaMemcpyAsync(cp->d_blob, st->h_ops, nbytes, cudaMemcpyHostToDevice, st->stream));
-  st->stats.h2d_bytes += nbytes;
-  CK(cudaEventRecord(st->ops_evt, st->stream));
+  return QGPU_OK;
+}
+
+// Send a plan's packed programs to its device blob, ordered on the state's stream after every
+// earlier pass that read the blob.
+qgpu_status send_plan(qgpu_state* st, CachedPlan* cp) {
+  if (!cp->blob_bytes) return QGPU_OK;
+  CK(cudaMemcpyAsync(cp->d_blob, cp->h_blob, cp->blob_bytes, cudaMemcpyHostToDevice, st->stream));
+  st->stats.h2d_bytes += cp->blob_bytes;
   return QGPU_OK;
 }
 
@@ -733,8 +740,10 @@ qgpu_status qgpu_state_destroy(qgpu_state* st) {
   if (st->h_ops) cudaFreeHost(st->h_ops);
   if (st->d_scratch) cudaFree(st->d_scratch);
   if (st->d_zero) cudaFree(st->d_zero);
-  for (CachedPlan& cp : st->plans)
+  for (CachedPlan& cp : st->plans) {
     if (cp.d_blob) cudaFree(cp.d_blob);
+    if (cp.h_blob) cudaFreeHost(cp.h_blob);
+  }
   if (st->ops_evt) cudaEventDestroy(st->ops_evt);
   if (st->own_stream && st->stream) cudaStreamDestroy(st->stream);
   delete st;
@@ -843,12 +852,14 @@ qgpu_status qgpu_apply_circuit(qgpu_state* st, const qgpu_circuit* c) {
           if (st->plans[i].last_use < st->plans[lru].last_use) lru = i;
         CK(cudaStreamSynchronize(st->stream));
         if (st->plans[lru].d_blob) cudaFree(st->plans[lru].d_blob);
+        if (st->plans[lru].h_blob) cudaFreeHost(st->plans[lru].h_blob);
         st->plans.erase(st->plans.begin() + lru);
       }
       st->plans.push_back(std::move(cp));
       hit = &st->plans.back();
       prepare_jit(st, hit->passes);
     }
+    if (qgpu_status s = send_plan(st, hit)) return s;
     hit->last_use = ++st->plan_clock;
     record_trace(st, hit->order, hit->inv, 0);
     st->stats.relabels += hit->relabels;
