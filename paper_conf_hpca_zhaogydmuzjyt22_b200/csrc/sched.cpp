@@ -445,21 +445,52 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
       }
     }
   }
-  // 2. sink phase terms
-  std::vector<RawOp> seq, pending;
-  for (const RawOp& o : raw) {
-    if (o.kind == 2) {
-      pending.push_back(o);
-      continue;
+  // 2. place phase terms. A term commutes with every U op that does not target one of its tile
+  //    bits, so it may sit in any slot between the last U op before it and the first U op after
+  //    it that targets one of its bits (slot s = just before U op s). Each distinct slot used is
+  //    one run, so the slots are chosen by interval stabbing (fewest points hitting every
+  //    interval: greedy by right end), which gathers the terms into the fewest runs.
+  std::vector<RawOp> seq;
+  {
+    std::vector<const RawOp*> us, ts;
+    std::vector<int> tpos;  // number of U ops before each term in program order
+    for (const RawOp& o : raw) {
+      if (o.kind == 2) {
+        ts.push_back(&o);
+        tpos.push_back(int(us.size()));
+      } else {
+        us.push_back(&o);
+      }
     }
-    uint32_t tb = 1u << o.t[0];
-    if (o.kind == 1) tb |= 1u << o.t[1];
-    std::vector<RawOp> keep;
-    for (const RawOp& ph : pending) (ph.lmask & tb ? seq : keep).push_back(ph);
-    pending.swap(keep);
-    seq.push_back(o);
+    auto tbits = [](const RawOp& o) {
+      uint32_t tb = 1u << o.t[0];
+      if (o.kind == 1) tb |= 1u << o.t[1];
+      return tb;
+    };
+    const int K = int(us.size());
+    std::vector<int> lo(ts.size()), hi(ts.size()), slot(ts.size());
+    for (size_t q = 0; q < ts.size(); ++q) {
+      int e = tpos[q];
+      while (e > 0 && !(tbits(*us[e - 1]) & ts[q]->lmask)) --e;
+      int l = tpos[q];
+      while (l < K && !(tbits(*us[l]) & ts[q]->lmask)) ++l;
+      lo[q] = e;
+      hi[q] = l;
+    }
+    std::vector<size_t> byhi(ts.size());
+    for (size_t q = 0; q < ts.size(); ++q) byhi[q] = q;
+    std::stable_sort(byhi.begin(), byhi.end(), [&](size_t x, size_t y) { return hi[x] < hi[y]; });
+    int point = -1;
+    for (size_t q : byhi) {
+      if (point < lo[q]) point = hi[q];
+      slot[q] = point;
+    }
+    for (int s = 0; s <= K; ++s) {
+      for (size_t q = 0; q < ts.size(); ++q)
+        if (slot[q] == s) seq.push_back(*ts[q]);
+      if (s < K) seq.push_back(*us[s]);
+    }
   }
-  for (const RawOp& ph : pending) seq.push_back(ph);
 
   // 3. mapping
   const int b = p.b;
