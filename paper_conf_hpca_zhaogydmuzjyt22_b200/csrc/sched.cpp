@@ -14,6 +14,7 @@
 #include <algorithm>
 #include <array>
 #include <bit>
+#include <cmath>
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
@@ -251,6 +252,32 @@ int mat_class(const cplx* U, int nt) {
   return MAT_GENERIC;
 }
 
+// Split a generic unitary U (row-major 2x2) as U = p0 diag(1, r1) R diag(1, q1) with R =
+// [[c, -s], [s, c]] real (c = |U00|, s = |U10|) and |p0| = |r1| = |q1| = 1 (a ZYZ-type
+// factorisation). Refused (false) when c or s is small or the recomposition is not within a few
+// ulps of U, so the split never costs accuracy beyond rounding.
+bool split_real(const cplx* U, cplx* p0, cplx* r1, cplx* R, cplx* q1) {
+  const double c = std::hypot(U[0].re, U[0].im), s = std::hypot(U[2].re, U[2].im);
+  if (c < 1e-3 || s < 1e-3) return false;
+  const cplx a{U[0].re / c, U[0].im / c};  // p0
+  const cplx b{U[2].re / s, U[2].im / s};  // p1 = p0 r1
+  // q1 = U11 / (p1 c)
+  const cplx q{(U[3].re * b.re + U[3].im * b.im) / c, (U[3].im * b.re - U[3].re * b.im) / c};
+  const cplx r{b.re * a.re + b.im * a.im, b.im * a.re - b.re * a.im};  // p1 / p0
+  const cplx Rm[4] = {{c, 0.0}, {-s, 0.0}, {s, 0.0}, {c, 0.0}};
+  // recompose: U' = p0 * diag(1, r) * R * diag(1, q)
+  auto mul = [](cplx x, cplx y) { return cplx{x.re * y.re - x.im * y.im, x.re * y.im + x.im * y.re}; };
+  const cplx V[4] = {mul(a, Rm[0]), mul(mul(a, Rm[1]), q), mul(mul(mul(a, r), Rm[2]), cplx{1.0, 0.0}),
+                     mul(mul(mul(a, r), Rm[3]), q)};
+  for (int i = 0; i < 4; ++i)
+    if (std::fabs(V[i].re - U[i].re) > 4e-16 || std::fabs(V[i].im - U[i].im) > 4e-16) return false;
+  *p0 = a;
+  *r1 = r;
+  *q1 = q;
+  for (int i = 0; i < 4; ++i) R[i] = Rm[i];
+  return true;
+}
+
 }  // namespace
 
 // Build the device program of a tile pass (a9). Steps:
@@ -388,7 +415,44 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
   TileProgram& P = p.prog;
   P = TileProgram();
   std::vector<RawOp> raw;
+  // a phase term multiplying the amplitudes whose tile-local bits match (lm, lt) and whose
+  // outside bits match (om, ot) by ph (lm == 0: tile-uniform -> the scalar)
+  auto phase_term = [&](uint32_t lm, uint32_t lt, uint64_t om, uint64_t ot, cplx ph) {
+    if (ph.re == 1.0 && ph.im == 0.0) return;
+    if (lm == 0) {
+      P.scalar.push_back(PhaseTerm{om, ot, ph.re, ph.im});
+      return;
+    }
+    RawOp o{};
+    o.kind = 2;
+    o.lmask = lm;
+    o.lmatch = lt;
+    o.omask = om;
+    o.omatch = ot;
+    o.ph = ph;
+    raw.push_back(o);
+  };
   for (const PhysGate& g : p.gates) {
+    cplx p0, r1, q1, R[4];
+    if (!g.diag && g.nt == 1 && mat_class(g.U, 1) == MAT_GENERIC && split_real(g.U, &p0, &r1, R, &q1)) {
+      // U = p0 diag(1, r1) R diag(1, q1), R real: the U op costs 8 instead of 16 FP64 per pair,
+      // the diagonal factors join the neighbouring phase runs (placed by step 2) and p0 is
+      // tile-uniform unless the gate has controls inside the tile
+      const int t = local_bit(g.p[0], p);
+      const uint32_t lc = to_local(g.pc, p), tb = lc | (1u << t);
+      const uint64_t oc = outside(g.pc, p);
+      phase_term(tb, tb, oc, oc, q1);
+      RawOp o{};
+      o.kind = 0;
+      o.t[0] = t;
+      o.lmask = o.lmatch = lc;
+      o.omask = o.omatch = oc;
+      std::memcpy(o.U, R, sizeof(R));
+      raw.push_back(o);
+      phase_term(lc, lc, oc, oc, p0);
+      phase_term(tb, tb, oc, oc, r1);
+      continue;
+    }
     if (!g.diag) {
       RawOp o{};
       o.kind = g.nt == 1 ? 0 : 1;
