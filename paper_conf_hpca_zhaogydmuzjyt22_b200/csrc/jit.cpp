@@ -229,10 +229,16 @@ std::string tile_jit_source(const Pass& p) {
     return zm;
   };
   uint32_t Wmask = 0;  // tile bits that are warp bits in the current mapping
+  int W[3] = {0, 0, 0};  // warp-bit index -> tile bit
   auto decode_w = [&](const TileOp& op) {
     Wmask = 0;
-    for (int k = 0; k < P.nw; ++k) Wmask |= 1u << ((op.a1 >> (4 * k)) & 15);
+    for (int k = 0; k < P.nw; ++k) {
+      W[k] = (op.a1 >> (4 * k)) & 15;
+      Wmask |= 1u << W[k];
+    }
   };
+  // warp-group remaps: (mbarrier base index, number of changed warp-bit indices)
+  std::vector<std::pair<int, int>> groups;
   decode(P.ops[0]);
   decode_w(P.ops[0]);
   std::ostringstream o;
@@ -248,15 +254,17 @@ std::string tile_jit_source(const Pass& p) {
   for (const TileOp& op : P.ops)
     if (op.kind == OP_REMAP)
       for (int k = 0; k < 4; ++k) RF[k] = (op.a0 >> (4 * k)) & 15;
-  o << "struct JitBody {\n";
-  o << "  static constexpr unsigned kZM0 = " << zm_start << "u;\n";
-  o << "  static constexpr uint32_t kZW0 = " << zw_start << "u;\n";
-  o << "  static constexpr bool kStatic = true;\n";
-  o << "  static constexpr bool kHasScalar = " << (P.scalar.empty() ? "false" : "true") << ";\n";
-  o << "  static constexpr uint32_t kJ0[kRegAmps] = " << jtab(R) << ";\n";
-  o << "  static constexpr uint64_t kP0[kRegAmps] = " << ptab(R) << ";\n";
-  o << "  static constexpr uint64_t kPF[kRegAmps] = " << ptab(RF) << ";\n";
-  o << "  static constexpr uint32_t kJF[kRegAmps] = " << jtab(RF) << ";\n";
+  std::ostringstream body, hdr;
+  {
+    std::ostringstream& o = body;  // the program body is generated first (it fixes the barriers)
+  hdr << "  static constexpr unsigned kZM0 = " << zm_start << "u;\n";
+  hdr << "  static constexpr uint32_t kZW0 = " << zw_start << "u;\n";
+  hdr << "  static constexpr bool kStatic = true;\n";
+  hdr << "  static constexpr bool kHasScalar = " << (P.scalar.empty() ? "false" : "true") << ";\n";
+  hdr << "  static constexpr uint32_t kJ0[kRegAmps] = " << jtab(R) << ";\n";
+  hdr << "  static constexpr uint64_t kP0[kRegAmps] = " << ptab(R) << ";\n";
+  hdr << "  static constexpr uint64_t kPF[kRegAmps] = " << ptab(RF) << ";\n";
+  hdr << "  static constexpr uint32_t kJF[kRegAmps] = " << jtab(RF) << ";\n";
   o << "  __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c) const {\n";
   o << "    const TileOp* ops = c.ops;\n";
   {
@@ -356,10 +364,29 @@ std::string tile_jit_source(const Pass& p) {
         zpos &= ~((1u << R[op.a0]) | (1u << R[op.a1]));
         break;
       case OP_REMAP: {
+        int Wold[3] = {W[0], W[1], W[2]};
         o << "      { constexpr uint32_t Jo[kRegAmps] = " << jtab(R) << ";\n";
-        o << "        tile_spill_j<" << NR << ">(v, c, mp.base, Jo); }\n";
+        o << "        tile_store_j<" << NR << ">(v, c, mp.base, Jo); }\n";
         decode(op);
         decode_w(op);
+        {
+          int nchg = 0;
+          std::string gexpr = "0";
+          int gi = 0;
+          for (int k = 0; k < P.nw; ++k) {
+            if (W[k] != Wold[k]) {
+              ++nchg;
+            } else {
+              gexpr += " | (((c.warp >> " + std::to_string(k) + ") & 1) << " + std::to_string(gi) + ")";
+              ++gi;
+            }
+          }
+          if (nchg > 0) {  // nchg == 0: the thread's own slots, a register permutation
+            const int base = int(groups.size()) * 4;
+            groups.push_back({base, nchg});
+            o << "      group_sync(c, " << base << " + (" << gexpr << "));\n";
+          }
+        }
         o << "      mp.base = " << base_expr(op) << ";\n";
         o << "      { constexpr uint32_t Jn[kRegAmps] = " << jtab(R) << ";\n";
         o << "        tile_reload_j<" << NR << ">(v, c, mp.base, Jn); }\n";
@@ -381,7 +408,16 @@ std::string tile_jit_source(const Pass& p) {
     if (wguard) o << "      }\n";
     o << "    }\n";
   }
-  o << "  }\n};\n";
+  o << "  }\n";
+  }
+  o << "struct JitBody {\n" << hdr.str();
+  o << "  static constexpr bool kGroupRemap = true;\n";
+  o << "  __device__ static void init_mbar(uint64_t* mb) {\n";
+  for (const auto& g : groups)
+    for (int q = 0; q < (1 << (P.nw - g.second)); ++q)
+      o << "    mbar_init(mb + " << (g.first + q) << ", " << (32 << g.second) << "u);\n";
+  o << "  }\n";
+  o << body.str() << "};\n";
   // one CTA per SM with up to 255 registers: measured faster than 2 CTAs/SM at <= 128
   // registers even for the single-buffer (remap-free) programs
   o << "extern \"C\" __global__ void __launch_bounds__(" << (NR >= 4 ? 256 : 512) << ", 1) qgpu_tile_pass(const TileArgs a) {\n";

@@ -168,6 +168,8 @@ struct InterpBody {
   static constexpr uint32_t kZW0 = 0u;
   static constexpr bool kStatic = false;  // mappings read from the program at run time
   static constexpr bool kHasScalar = true;
+  static constexpr bool kGroupRemap = false;  // remaps use CTA barriers
+  __device__ static void init_mbar(uint64_t*) {}
   static constexpr uint32_t kJ0[kRegAmps] = {};
   static constexpr uint64_t kP0[kRegAmps] = {};
   static constexpr uint64_t kPF[kRegAmps] = {};
@@ -415,7 +417,7 @@ size_t tile_smem_bytes(const TileArgs& a) {
   const size_t nh = size_t(1) << (a.b - a.l);
   const size_t nwarps = size_t(1) << a.nw;
   return size_t(a.nbuf) * (size_t(1) << a.b) * 16 + ((nh + 1) & ~size_t(1)) * 8 + size_t(a.blob_bytes) +
-         2 * nwarps * size_t(a.npat) * 16 + 16;
+         2 * nwarps * size_t(a.npat) * 16 + size_t(a.nmbar) * 8 + 16;
 }
 
 cudaError_t launch_pair(cudaStream_t st, const PairArgs& a, bool shfl) {

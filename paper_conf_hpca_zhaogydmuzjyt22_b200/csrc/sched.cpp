@@ -373,8 +373,10 @@ void split_patterns(TileProgram& P, const Pass& p, int m) {
     if (!(smask >> q & 1)) lopos[nlo++] = q;
   const size_t npat = P.patterns.size();
   P.layout();
+  size_t nremap = 0;
+  for (size_t i = 1; i < P.ops.size(); ++i) nremap += P.ops[i].kind == OP_REMAP;
   const size_t fixed = 3 * (size_t(16) << p.b) + ((size_t(1) << (p.b - p.l)) + 2) * 8 + P.bytes +
-                       2 * (size_t(1) << P.nw) * npat * 16 + 16;
+                       2 * (size_t(1) << P.nw) * npat * 16 + 4 * nremap * 8 + 16;
   int lb = nlo;
   while (lb > 0 && fixed + npat * (size_t(16) << lb) > 227 * 1024) --lb;
   P.lb = lb;
@@ -586,7 +588,22 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
     for (int k = 0; k < nr; ++k) R[k] = cand[k];
     std::vector<int> w(cand.begin() + nr, cand.end());
     std::sort(w.begin(), w.end());
-    for (int k = 0; k < nw; ++k) W[k] = w[k];
+    if (P.ops.empty()) {
+      for (int k = 0; k < nw; ++k) W[k] = w[k];
+    } else {
+      // a position that stays a warp bit keeps its warp-bit index, so a remap only moves data
+      // between the warps that differ in the changed indices (warp-group remap, jit.cpp)
+      int nwk[3] = {-1, -1, -1};
+      for (int k = 0; k < nw; ++k)
+        if (std::find(w.begin(), w.end(), W[k]) != w.end()) nwk[k] = W[k];
+      size_t next = 0;
+      for (int k = 0; k < nw; ++k) {
+        if (nwk[k] >= 0) continue;
+        while (std::find(nwk, nwk + 3, w[next]) != nwk + 3) ++next;
+        nwk[k] = w[next++];
+      }
+      for (int k = 0; k < nw; ++k) W[k] = nwk[k];
+    }
     TileOp op{};
     op.kind = OP_REMAP;
     for (int k = 0; k < nr; ++k) op.a0 |= R[k] << (4 * k);

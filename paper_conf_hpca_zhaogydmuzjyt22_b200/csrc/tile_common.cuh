@@ -93,6 +93,7 @@ struct TileArgs {
   int bstore;              // 1: results staged in the tile buffer and written by bulk async
                            // copies (needs nbuf == 3), 0: per-thread stores from registers
   int remaps;              // the program contains REMAP / shared-memory ops
+  int nmbar;               // mbarriers for warp-group remaps (JIT programs), 8 B each in smem
 };
 
 __device__ __forceinline__ double2 cmul(double2 a, double2 b) {
@@ -146,6 +147,9 @@ __device__ __forceinline__ void mbar_wait(uint64_t* bar, uint32_t parity) {
     asm volatile("{\n.reg .pred p;\nmbarrier.try_wait.parity.shared::cta.b64 p, [%1], %2;\nselp.u32 %0, 1, 0, p;\n}\n"
                  : "=r"(done) : "r"(smem_u32(bar)), "r"(parity) : "memory");
   } while (!done);
+}
+__device__ __forceinline__ void mbar_arrive(uint64_t* bar) {
+  asm volatile("{\n.reg .b64 st;\nmbarrier.arrive.shared::cta.b64 st, [%0];\n}\n" ::"r"(smem_u32(bar)) : "memory");
 }
 __device__ __forceinline__ void bulk_g2s(void* dst, const void* src, uint32_t bytes, uint64_t* bar) {
   asm volatile("cp.async.bulk.shared::cluster.global.mbarrier::complete_tx::bytes [%0], [%1], %2, [%3];\n"
@@ -218,6 +222,8 @@ struct TileCtx {
   uint32_t T;
   int nthr, tid, lane, warp, nw;
   bool own;              // this lane owns amplitudes (b >= 5 always)
+  uint64_t* mbar;        // warp-group remap barriers (JIT), one per (remap, group)
+  uint32_t mpar;         // their phase parity for this tile
 };
 
 template <int NR>
@@ -250,6 +256,25 @@ __device__ __forceinline__ void tile_reload_j(double2 (&v)[kRegAmps], const Tile
                                               const uint32_t (&J)[kRegAmps]) {
 #pragma unroll
   for (int r = 0; r < (1 << NR); ++r) v[r] = c.own ? c.s[base + J[r]] : make_double2(0, 0);
+}
+
+// Warp-group remap (JIT): a remap that turns register bits into warp bits and back only moves
+// amplitudes between the warps that differ in the warp-bit indices it changes (the warp-bit
+// indices of unchanged positions are kept), so instead of two CTA-wide barriers the group
+// (2, 4 or 8 warps) meets at an mbarrier: every thread stores its slots under the old mapping,
+// arrives, waits for the group's phase, then reloads under the new mapping. No WAR hazard: a
+// thread's old slots are disjoint from every other thread's old slots, and the tile loop keeps
+// one CTA barrier per tile, so the warps of a CTA are never a tile apart.
+template <int NR>
+__device__ __forceinline__ void tile_store_j(const double2 (&v)[kRegAmps], const TileCtx& c, uint32_t base,
+                                             const uint32_t (&J)[kRegAmps]) {
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r)
+    if (c.own) c.s[base + J[r]] = v[r];
+}
+__device__ __forceinline__ void group_sync(const TileCtx& c, int idx) {
+  mbar_arrive(c.mbar + idx);
+  mbar_wait(c.mbar + idx, c.mpar);
 }
 
 __device__ __forceinline__ bool op_active(const TileOp& op, uint64_t gbase) {
@@ -663,6 +688,8 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   const double2* tlo = reinterpret_cast<const double2*>(blob + a.off_tlo);
   double2* Cw = reinterpret_cast<double2*>(blob + a.blob_bytes);  // per-warp pattern constants
   double2* Chw = Cw + (size_t(nthr) >> 5) * a.npat;               // per-warp high-bit parts
+  uint64_t* mbar = reinterpret_cast<uint64_t*>(Chw + (size_t(nthr) >> 5) * a.npat);
+  if (threadIdx.x == 0) Body::init_mbar(mbar);
 
   {
     const int4* src = reinterpret_cast<const int4*>(a.blob);
@@ -690,6 +717,9 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   c.warp = warp;
   c.nw = nw;
   c.own = lane < int(T);
+  c.mbar = mbar;
+  c.mpar = 0;
+  uint32_t nexec = 0;  // tiles whose program ran (the remap barriers' phase)
   const Mapping mp0 = make_mapping<NR>(ops[0], nw, lane, warp);  // ops[0] is always OP_REMAP
   const SlotAddr sa0 = slot_addr<NR>(mp0, hiOff, lowmask, l);
   const bool wzero = (mp0.base & Body::kZW0) != 0u;  // this warp's slots start in the zero region
@@ -743,7 +773,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       }
       k = kn;
       tile = next;
-      if (nbuf < 3 && a.remaps) __syncthreads();
+      if ((nbuf < 3 || Body::kGroupRemap) && a.remaps) __syncthreads();
       continue;
     }
     // pattern constants of this tile, per warp (lane-strided; each lane owns the same patterns
@@ -788,6 +818,8 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       v[r] = (c.own && !((zm0 >> r) & 1)) ? s[j] : make_double2(0.0, 0.0);
     }
     if (more && nbuf == 1) issue_own_loads<NR, Body>(s, a, mp0, sa0, tile_base(next, a), zm0, c.own);
+    c.mpar = nexec & 1u;
+    ++nexec;
     body(v, mp, c);
     if (Body::kHasScalar && !(sc.x == 1.0 && sc.y == 0.0)) {
 #pragma unroll
@@ -820,8 +852,9 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     // the lanes of this warp are done reading this tile's pattern constants before the next
     // tile's constants are written
     __syncwarp();
-    // with two buffers the next prefetch refills the buffer other warps read during remaps
-    if (nbuf < 3 && a.remaps) __syncthreads();
+    // with two buffers the next prefetch refills the buffer other warps read during remaps;
+    // with warp-group remaps this is the one CTA barrier per tile that bounds warp drift
+    if ((nbuf < 3 || Body::kGroupRemap) && a.remaps) __syncthreads();
   }
   if (a.bstore && warp == 0) bulk_wait_all();  // shared memory must outlive the bulk reads
 }
