@@ -14,6 +14,8 @@ Modules
   statevector.py ctypes wrapper around sv.c, program-order simulation
   schedule.py    Alg.1 pruning replay, Alg.2 greedy and Alg.3 forward-looking reorder,
                  chunk bitmap, Table II statistic
+  gfc.py         GFC-style lossless compression of amplitude doubles, segment/micro-chunk
+                 residual coding with 4-bit sign + leading-zero-byte prefixes
 
 Parity status: every function is pinned by tests in tests/test_oracle_*.py (closed forms,
 brute-force unitaries, the paper's worked examples); see DESIGN.md "Oracle pins".
