@@ -234,6 +234,38 @@ qgpu_status qgpu_reset_stats(qgpu_state* st);
  * torch.distributed). UNSUPPORTED if libnccl.so.2 cannot be loaded ($QGPU_NCCL_LIB). */
 qgpu_status qgpu_nccl_unique_id(void* out, size_t len);
 
+/* ---- GFC lossless compression of amplitude data ----------
+ * The paper compresses every state chunk on the GPU before it crosses the host link: segments
+ * of `seg_len` doubles are compressed independently, one warp per segment, as micro-chunks of
+ * 32 doubles whose residual against the previous micro-chunk is stored as a 4-bit prefix (sign
+ * + count of leading zero bytes) plus the remaining bytes. Byte format (readings
+ * G1-G5): residual = w - prev on the 64-bit patterns (mod 2^64), prev = 0 for a
+ * segment's first micro-chunk; nibble = sign << 3 | min(7, leading zero bytes of |residual|),
+ * payload = the 8 - count low-order bytes of |residual|, little-endian; a micro-chunk of cnt
+ * values = ceil(cnt/2) nibble bytes (value i in byte i/2, low nibble for even i) followed by the
+ * payloads in order; a segment stream is zero-padded to a multiple of 16 bytes; the output is
+ * the segment streams in order and offsets[s] = byte offset of segment s (offsets[0] = 0,
+ * offsets[n_seg] = total). Lossless for every bit pattern (NaN payloads, -0.0).
+ * All pointers except `out_bytes` / `max_bytes` are DEVICE memory owned by the caller; `d_out`
+ * and `d_in` must be 16-byte aligned; `stream` is a cudaStream_t (NULL = legacy default).
+ * seg_len must be a positive multiple of 32; n = number of doubles (2 per amplitude). */
+
+/* Host: the largest possible compressed size of n doubles (every value 8 payload bytes). */
+qgpu_status qgpu_gfc_max_bytes(uint64_t n, uint32_t seg_len, uint64_t* max_bytes);
+
+/* Compress d_in[0..n) into d_out (capacity out_cap bytes) and d_offsets[0..n_seg], n_seg =
+ * ceil(n / seg_len). Synchronises `stream` (the size is data dependent) and returns the total
+ * in *out_bytes. If out_cap is too small: QGPU_ERR_INVALID_ARG, *out_bytes = the size needed,
+ * d_offsets valid, d_out untouched. */
+qgpu_status qgpu_gfc_compress(const double* d_in, uint64_t n, uint32_t seg_len, void* d_out,
+                              uint64_t out_cap, uint64_t* d_offsets, uint64_t* out_bytes,
+                              void* stream);
+
+/* Inverse: d_out[0..n) from the stream d_in and d_offsets produced by qgpu_gfc_compress with
+ * the same n and seg_len. Asynchronous on `stream`. */
+qgpu_status qgpu_gfc_decompress(const void* d_in, const uint64_t* d_offsets, uint64_t n,
+                                uint32_t seg_len, double* d_out, void* stream);
+
 /* Thread-local detail of the last error on this thread (valid until the next call). */
 const char* qgpu_last_error(void);
 

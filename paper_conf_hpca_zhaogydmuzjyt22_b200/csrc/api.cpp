@@ -615,6 +615,61 @@ extern "C" {
 
 const char* qgpu_last_error(void) { return g_err.c_str(); }
 
+qgpu_status qgpu_gfc_max_bytes(uint64_t n, uint32_t seg_len, uint64_t* max_bytes) {
+  if (!max_bytes) return fail(QGPU_ERR_INVALID_ARG, "max_bytes is NULL");
+  if (seg_len == 0 || seg_len % 32) return fail(QGPU_ERR_INVALID_ARG, "seg_len %u is not a positive multiple of 32", seg_len);
+  uint64_t total = 0;
+  for (uint64_t s = 0; s < n; s += seg_len) {
+    const uint64_t c = std::min<uint64_t>(seg_len, n - s);
+    const uint64_t b = 8 * c + (c / 32) * 16 + ((c % 32) + 1) / 2;
+    total += (b + 15) & ~15ull;
+  }
+  *max_bytes = total;
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_gfc_compress(const double* d_in, uint64_t n, uint32_t seg_len, void* d_out, uint64_t out_cap,
+                              uint64_t* d_offsets, uint64_t* out_bytes, void* stream) {
+  if (!out_bytes || !d_offsets) return fail(QGPU_ERR_INVALID_ARG, "out_bytes/d_offsets is NULL");
+  if (seg_len == 0 || seg_len % 32) return fail(QGPU_ERR_INVALID_ARG, "seg_len %u is not a positive multiple of 32", seg_len);
+  if (n && (!d_in || !d_out)) return fail(QGPU_ERR_INVALID_ARG, "d_in/d_out is NULL");
+  if ((reinterpret_cast<uintptr_t>(d_in) | reinterpret_cast<uintptr_t>(d_out)) % 16)
+    return fail(QGPU_ERR_INVALID_ARG, "d_in and d_out must be 16-byte aligned");
+  cudaStream_t cs = static_cast<cudaStream_t>(stream);
+  const uint64_t nseg = (n + seg_len - 1) / seg_len;
+  CK0(cudaMemsetAsync(d_offsets, 0, sizeof(uint64_t), cs));
+  *out_bytes = 0;
+  if (nseg == 0) {
+    CK0(cudaStreamSynchronize(cs));
+    return QGPU_OK;
+  }
+  uint64_t* scratch = nullptr;
+  CK0(cudaMallocAsync(reinterpret_cast<void**>(&scratch), gfc_scan_scratch_elems(nseg) * sizeof(uint64_t), cs));
+  cudaError_t e = launch_gfc_sizes(cs, d_in, n, seg_len, d_offsets + 1);
+  if (e == cudaSuccess) e = launch_scan_u64(cs, d_offsets + 1, nseg, scratch);
+  uint64_t total = 0;
+  if (e == cudaSuccess) e = cudaMemcpyAsync(&total, d_offsets + nseg, sizeof(uint64_t), cudaMemcpyDeviceToHost, cs);
+  cudaFreeAsync(scratch, cs);
+  CK0(e);
+  CK0(cudaStreamSynchronize(cs));
+  *out_bytes = total;
+  if (total > out_cap)
+    return fail(QGPU_ERR_INVALID_ARG, "out_cap %llu < compressed size %llu", (unsigned long long)out_cap,
+                (unsigned long long)total);
+  CK0(launch_gfc_encode(cs, d_in, n, seg_len, d_offsets, d_out));
+  CK0(cudaStreamSynchronize(cs));
+  return QGPU_OK;
+}
+
+qgpu_status qgpu_gfc_decompress(const void* d_in, const uint64_t* d_offsets, uint64_t n, uint32_t seg_len,
+                                double* d_out, void* stream) {
+  if (seg_len == 0 || seg_len % 32) return fail(QGPU_ERR_INVALID_ARG, "seg_len %u is not a positive multiple of 32", seg_len);
+  if (n && (!d_in || !d_offsets || !d_out)) return fail(QGPU_ERR_INVALID_ARG, "NULL pointer");
+  if (reinterpret_cast<uintptr_t>(d_in) % 16) return fail(QGPU_ERR_INVALID_ARG, "d_in must be 16-byte aligned");
+  CK0(launch_gfc_decode(static_cast<cudaStream_t>(stream), d_in, d_offsets, n, seg_len, d_out));
+  return QGPU_OK;
+}
+
 const char* qgpu_version(void) {
   return "qgpu abi " "1" " sm_100a (B200) complex128";
 }

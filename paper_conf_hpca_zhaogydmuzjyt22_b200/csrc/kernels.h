@@ -81,4 +81,14 @@ cudaError_t launch_unpack_half(cudaStream_t st, double2* psi, const double2* buf
                                uint64_t count);
 cudaError_t launch_add(cudaStream_t st, double* out, const double* in, uint64_t count);
 
+// GFC compression (gfc.cu): per-segment padded sizes, encode at scanned offsets,
+// decode; in-place inclusive scan of uint64 (scratch: gfc_scan_scratch_elems(n) elements)
+cudaError_t launch_gfc_sizes(cudaStream_t st, const double* in, uint64_t n, uint32_t seg, uint64_t* sizes);
+cudaError_t launch_gfc_encode(cudaStream_t st, const double* in, uint64_t n, uint32_t seg, const uint64_t* offsets,
+                              void* out);
+cudaError_t launch_gfc_decode(cudaStream_t st, const void* in, const uint64_t* offsets, uint64_t n, uint32_t seg,
+                              double* out);
+uint64_t gfc_scan_scratch_elems(uint64_t n);
+cudaError_t launch_scan_u64(cudaStream_t st, uint64_t* a, uint64_t n, uint64_t* scratch);
+
 }  // namespace qgpu

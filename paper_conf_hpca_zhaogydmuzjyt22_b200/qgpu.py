@@ -26,7 +26,8 @@ EXPORTS = [
     "qgpu_probabilities", "qgpu_circuit_from_qasm", "qgpu_circuit_info", "qgpu_circuit_destroy",
     "qgpu_circuit_reorder", "qgpu_circuit_plan", "qgpu_circuit_plan_text", "qgpu_circuit_jit_check", "qgpu_get_involvement", "qgpu_get_chunk_bitmap",
     "qgpu_get_schedule", "qgpu_get_qubit_map", "qgpu_get_stats", "qgpu_reset_stats",
-    "qgpu_nccl_unique_id", "qgpu_last_error", "qgpu_version",
+    "qgpu_nccl_unique_id", "qgpu_gfc_max_bytes", "qgpu_gfc_compress", "qgpu_gfc_decompress",
+    "qgpu_last_error", "qgpu_version",
 ]
 
 
@@ -89,6 +90,9 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
         "qgpu_get_schedule": [P, P, P, U64, P], "qgpu_get_qubit_map": [P, P],
         "qgpu_get_stats": [P, P], "qgpu_reset_stats": [P],
         "qgpu_nccl_unique_id": [P, ctypes.c_size_t],
+        "qgpu_gfc_max_bytes": [U64, ctypes.c_uint32, P],
+        "qgpu_gfc_compress": [P, U64, ctypes.c_uint32, P, U64, P, P, P],
+        "qgpu_gfc_decompress": [P, P, U64, ctypes.c_uint32, P, P],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -310,6 +314,28 @@ def nccl_unique_id() -> bytes:
     buf = ctypes.create_string_buffer(128)
     _check(load().qgpu_nccl_unique_id(buf, 128))
     return buf.raw
+
+
+def gfc_max_bytes(n: int, seg_len: int) -> int:
+    """Largest compressed size of n doubles (qgpu_gfc_max_bytes)."""
+    out = ctypes.c_uint64()
+    _check(load().qgpu_gfc_max_bytes(n, seg_len, ctypes.byref(out)))
+    return out.value
+
+
+def gfc_compress(d_in: int, n: int, seg_len: int, d_out: int, out_cap: int, d_offsets: int,
+                 stream: int = 0) -> int:
+    """GFC-compress n doubles at device address d_in into d_out / d_offsets (device
+    addresses); returns the compressed size in bytes (qgpu_gfc_compress, synchronising)."""
+    out = ctypes.c_uint64()
+    _check(load().qgpu_gfc_compress(d_in, n, seg_len, d_out, out_cap, d_offsets, ctypes.byref(out),
+                                    stream or None))
+    return out.value
+
+
+def gfc_decompress(d_in: int, d_offsets: int, n: int, seg_len: int, d_out: int, stream: int = 0) -> None:
+    """Inverse of gfc_compress (device addresses; asynchronous on `stream`)."""
+    _check(load().qgpu_gfc_decompress(d_in, d_offsets, n, seg_len, d_out, stream or None))
 
 
 def version() -> str:
