@@ -288,6 +288,43 @@ def single_qubit_sweep(q, torch, n: int, reps: int = 3):
     return res
 
 
+def gfc_measure(q, torch, st, seg: int = 4096):
+    """NEXT-3: GFC compression of the state left by the workload (the physical
+    buffer, as a host-link or swap transfer would send it): ratio and device throughput of
+    qgpu_gfc_compress / qgpu_gfc_decompress (CUDA events, best of 3), lossless check."""
+    _, n_loc, dev = st.info()
+    n = 2 << n_loc
+    cap = q.gfc_max_bytes(n, seg)
+    if 16 * (1 << n_loc) + cap + 8 * n > 0.8 * torch.cuda.mem_get_info()[0] + 16 * (1 << n_loc):
+        return {"skipped": "state too large for a compressed copy + decompressed copy"}
+    out = torch.empty(cap, dtype=torch.uint8, device="cuda")
+    off = torch.empty((n + seg - 1) // seg + 1, dtype=torch.int64, device="cuda")
+    back = torch.empty(n, dtype=torch.int64, device="cuda")
+    best_c = best_d = float("inf")
+    nb = 0
+    for _ in range(3):
+        torch.cuda.synchronize()
+        e0, e1, e2 = (torch.cuda.Event(enable_timing=True) for _ in range(3))
+        e0.record()
+        nb = q.gfc_compress(dev, n, seg, out.data_ptr(), cap, off.data_ptr())
+        e1.record()
+        q.gfc_decompress(out.data_ptr(), off.data_ptr(), n, seg, back.data_ptr())
+        e2.record()
+        torch.cuda.synchronize()
+        best_c, best_d = min(best_c, e0.elapsed_time(e1)), min(best_d, e1.elapsed_time(e2))
+    out2 = torch.empty_like(out)
+    off2 = torch.empty_like(off)
+    nb2 = q.gfc_compress(back.data_ptr(), n, seg, out2.data_ptr(), cap, off2.data_ptr())
+    lossless = bool(nb2 == nb and torch.equal(out[:nb], out2[:nb]))
+    res = {"seg_len": seg, "doubles": n, "compressed_bytes": nb, "ratio": 8.0 * n / nb,
+           "compress_ms": best_c, "decompress_ms": best_d,
+           "compress_GBps_in": 8.0 * n / best_c / 1e6, "decompress_GBps_out": 8.0 * n / best_d / 1e6,
+           "lossless": lossless}
+    del out, off, back, out2, off2
+    torch.cuda.empty_cache()
+    return res
+
+
 def run_ours(args):
     import numpy as np
     import torch
@@ -389,6 +426,7 @@ def run_ours(args):
     e2e_val = allreduce_max(statistics.mean(e2e_times), world, device)
     assert abs(p.sum() - 1) < 1e-9, "e2e readout not normalised"
 
+    gfc = gfc_measure(q, torch, st) if (args.gfc and not sharded) else None
     launches = s0["kernels_launched"]
     line = {
         "metric": METRIC, "value": ms / 1e3, "unit": "s", "n_gpus": world, "steps": args.steps,
@@ -421,6 +459,8 @@ def run_ours(args):
         "gpu_launches_per_step": launches,
         "clocks": clocks,
     }
+    if gfc is not None:
+        line["gfc_compression"] = gfc
     st.close()
 
     if args.micro and rank == 0:
@@ -461,6 +501,7 @@ def main():
     ap.add_argument("--cpu-seconds", type=float, default=20.0)
     ap.add_argument("--ref-step-seconds", type=float, default=8.0)
     ap.add_argument("--ref-gates", type=int, default=None)
+    ap.add_argument("--gfc", type=int, default=1, help="1: also measure GFC compression of the final state")
     ap.add_argument("--sharded", action="store_true",
                     help="N>1: shard one state over the ranks (NCCL swaps) instead of N replicas")
     args = ap.parse_args()

@@ -95,7 +95,8 @@ __global__ void __launch_bounds__(kWarps * 32) gfc_size_kernel(const uint64_t* _
   }
 }
 
-// Pass 2: encode each segment at its offset.
+// Pass 2: encode each segment at its offset (byte stores into the ring: measured faster than
+// 64-bit shared atomics, which serialise when many 1-byte payloads share a word).
 __global__ void __launch_bounds__(kWarps * 32) gfc_encode_kernel(const uint64_t* __restrict__ in, uint64_t n,
                                                                  uint32_t seg, uint64_t nseg,
                                                                  const uint64_t* __restrict__ offsets,
@@ -154,13 +155,16 @@ __global__ void __launch_bounds__(kWarps * 32) gfc_encode_kernel(const uint64_t*
   }
 }
 
+// Decode: the stream is staged in the ring in 512-byte blocks; a lane reads its nibble and its
+// payload as two aligned 64-bit words and a funnel shift.
 __global__ void __launch_bounds__(kWarps * 32) gfc_decode_kernel(const unsigned char* __restrict__ in,
                                                                  const uint64_t* __restrict__ offsets, uint64_t n,
                                                                  uint32_t seg, uint64_t nseg,
                                                                  uint64_t* __restrict__ out) {
-  __shared__ __align__(16) unsigned char rings[kWarps][kRing];
+  constexpr uint32_t kW = kRing / 8;
+  __shared__ __align__(16) unsigned long long rings[kWarps][kW];
   const int lane = threadIdx.x & 31, wid = threadIdx.x >> 5;
-  unsigned char* ring = rings[wid];
+  unsigned long long* ring = rings[wid];
   const uint64_t gw = (uint64_t(blockIdx.x) * blockDim.x + threadIdx.x) >> 5;
   const uint64_t nw = (uint64_t(gridDim.x) * blockDim.x) >> 5;
   constexpr uint64_t kMaxChunk = 16 + 32 * 8;
@@ -174,20 +178,29 @@ __global__ void __launch_bounds__(kWarps * 32) gfc_decode_kernel(const unsigned 
       while (loaded < sbytes && loaded - pos < kMaxChunk) {
         const uint64_t off = loaded + 16 * uint64_t(lane);
         if (off < sbytes)
-          reinterpret_cast<int4*>(ring + off % kRing)[0] = __ldcs(reinterpret_cast<const int4*>(src + off));
+          reinterpret_cast<int4*>(ring)[(off % kRing) / 16] = __ldcs(reinterpret_cast<const int4*>(src + off));
         loaded += kBlock;
         __syncwarp();
       }
       const int c = int(cnt - k < 32 ? cnt - k : 32);
       const bool valid = lane < c;
       const int npre = (c + 1) / 2;
-      const uint32_t nib = valid ? (ring[(pos + uint64_t(lane >> 1)) % kRing] >> (4 * (lane & 1))) & 15u : 0u;
+      uint32_t nib = 0;
+      if (valid) {
+        const uint64_t bp = pos + uint64_t(lane >> 1);
+        nib = uint32_t(ring[(bp >> 3) % kW] >> (8 * (bp & 7) + 4 * (lane & 1))) & 15u;
+      }
       const int nb = valid ? 8 - int(nib & 7u) : 0;
       const int incl = warp_incl_scan(nb, lane);
       const int total = __shfl_sync(kFull, incl, 31);
-      const uint64_t q = pos + uint64_t(npre) + uint64_t(incl - nb);
       uint64_t mag = 0;
-      for (int b = 0; b < nb; ++b) mag |= uint64_t(ring[(q + uint64_t(b)) % kRing]) << (8 * b);
+      if (nb) {
+        const uint64_t q = pos + uint64_t(npre) + uint64_t(incl - nb);
+        const uint32_t wi = uint32_t(q >> 3) % kW, sh = uint32_t(q & 7) * 8;
+        uint64_t v = ring[wi] >> sh;
+        if (sh) v |= uint64_t(ring[(wi + 1) % kW]) << (64 - sh);
+        mag = nb == 8 ? v : (v & ((1ull << (8 * nb)) - 1));
+      }
       const uint64_t w = prev + ((nib & 8u) ? (0ull - mag) : mag);
       if (valid) __stcs(reinterpret_cast<unsigned long long*>(dst + k + uint64_t(lane)), (unsigned long long)w);
       prev = w;
