@@ -1,0 +1,103 @@
+"""The paper's version ablation (Fig.12-13: Pruning, Reorder on top of the baseline),
+re-done on one B200 for every synthetic family, plus the B200-specific fusion ablation.
+
+For each family at n qubits, circuit seconds (device CUDA events around qgpu_state_reset +
+qgpu_apply_circuit on the state's stream, median of --reps after one warm-up) for:
+  base      prune=0 reorder=0   every pass over the full 2^n state, program order
+  prune     prune=1 reorder=0   Alg.1 pruning / delayed involvement, program order
+  greedy    prune=1 reorder=1   + Alg.2 greedy reorder
+  forward   prune=1 reorder=2   + Alg.3 forward-looking reorder (the default)
+  unfused   prune=1 reorder=2 fuse_bits=0   one gate per HBM pass (the paper's granularity)
+with the pruning statistics (live amplitudes processed / full, Table II "ops before full
+involvement"). Writes one JSON object per family to --out (JSON lines) and prints a table.
+
+    python scripts/ablation.py [--n 30] [--families qft,qaoa,gs,hlf,iqp,bv,rqc] [--out f.jsonl]
+"""
+import argparse
+import json
+import os
+import statistics
+import sys
+
+sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
+
+VERSIONS = [("base", dict(prune=0, reorder=0)), ("prune", dict(prune=1, reorder=0)),
+            ("greedy", dict(prune=1, reorder=1)), ("forward", dict(prune=1, reorder=2)),
+            ("unfused", dict(prune=1, reorder=2, fuse_bits=0))]
+
+
+def family(name, n):
+    from workloads import circuits as wc
+    if name == "qft":
+        return wc.qft(n)
+    if name == "qaoa":
+        return wc.qaoa(n, 2, seed=1)
+    if name == "rqc":
+        return wc.rqc(n, 20, seed=3)
+    if name in ("gs", "hlf"):
+        r = 1
+        for k in range(1, int(n ** 0.5) + 1):
+            if n % k == 0:
+                r = k
+        return wc.gs(r, n // r) if name == "gs" else wc.hlf(r, n // r, seed=2)
+    if name == "iqp":
+        return wc.iqp(n)
+    if name == "bv":
+        return wc.bv(n, (0b1011 * 0x11111111) & ((1 << (n - 1)) - 1))
+    raise SystemExit(f"unknown family {name}")
+
+
+def main():
+    ap = argparse.ArgumentParser()
+    ap.add_argument("--n", type=int, default=30)
+    ap.add_argument("--families", default="qft,qaoa,gs,hlf,iqp,bv,rqc")
+    ap.add_argument("--reps", type=int, default=3)
+    ap.add_argument("--unfused-max-gates", type=int, default=1200)
+    ap.add_argument("--out", default=None)
+    args = ap.parse_args()
+    import torch
+    from paper_conf_hpca_zhaogydmuzjyt22_b200 import qgpu as q
+    q.load()
+    stream = torch.cuda.Stream()
+    rows = []
+    for fam in args.families.split(","):
+        c = family(fam, args.n)
+        circ = q.Circuit(c.qasm())
+        ngates = circ.info()[1]
+        res = {"family": fam, "n": args.n, "gates": ngates}
+        for vname, cfg in VERSIONS:
+            if vname == "unfused" and ngates > args.unfused_max_gates:
+                continue
+            st = q.State(args.n, stream=stream.cuda_stream, **cfg)
+            times = []
+            for it in range(1 + args.reps):
+                e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+                e0.record(stream)
+                st.reset()
+                st.apply_circuit(circ)
+                e1.record(stream)
+                e1.synchronize()
+                if it:
+                    times.append(e0.elapsed_time(e1))
+            s = st.stats()
+            st.close()
+            res[vname] = {"ms": statistics.median(times), "passes": s["passes"],
+                          "live_frac": s["amps_processed"] / max(s["amps_full"], 1),
+                          "ops_before_full_involvement": s["ops_before_full_involvement"]}
+        rows.append(res)
+        print(json.dumps(res), flush=True)
+    if args.out:
+        with open(args.out, "w") as f:
+            for r in rows:
+                f.write(json.dumps(r) + "\n")
+    print(f"\n{'family':8} {'gates':>6} " + " ".join(f"{v:>10}" for v, _ in VERSIONS) +
+          "   prune/base forward/prune live%(fwd) TableII(prog->fwd)")
+    for r in rows:
+        ms = [r[v]["ms"] if v in r else float("nan") for v, _ in VERSIONS]
+        print(f"{r['family']:8} {r['gates']:6d} " + " ".join(f"{m:10.3f}" for m in ms) +
+              f"   {ms[1] / ms[0]:10.3f} {ms[3] / ms[1]:12.3f} {100 * r['forward']['live_frac']:9.1f}"
+              f"   {r['prune']['ops_before_full_involvement']}->{r['forward']['ops_before_full_involvement']}")
+
+
+if __name__ == "__main__":
+    main()
