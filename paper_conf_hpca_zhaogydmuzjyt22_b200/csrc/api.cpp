@@ -285,7 +285,7 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     a.nmbar = 0;
     for (size_t i = 1; i < P.ops.size(); ++i) {
       if (P.ops[i].kind == OP_REMAP || P.ops[i].kind == OP_SMEM1 || P.ops[i].kind == OP_SMEM2) a.remaps = 1;
-      if (P.ops[i].kind == OP_REMAP) a.nmbar += 4;  // one per warp group (<= 4) of each remap
+      if (P.ops[i].kind == OP_REMAP) a.nmbar += 1 << P.nw;  // one per warp group of each remap
     }
     // programs without remaps need one tile buffer (each thread only reads its own slots),
     // which lets two CTAs share an SM; otherwise triple (or double) buffering

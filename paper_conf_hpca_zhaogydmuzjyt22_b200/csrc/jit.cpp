@@ -14,6 +14,7 @@
 #include <nvrtc.h>
 
 #include <algorithm>
+#include <bit>
 #include <atomic>
 #include <chrono>
 #include <fstream>
@@ -229,7 +230,7 @@ std::string tile_jit_source(const Pass& p) {
     return zm;
   };
   uint32_t Wmask = 0;  // tile bits that are warp bits in the current mapping
-  int W[3] = {0, 0, 0};  // warp-bit index -> tile bit
+  int W[4] = {0, 0, 0, 0};  // warp-bit index -> tile bit
   auto decode_w = [&](const TileOp& op) {
     Wmask = 0;
     for (int k = 0; k < P.nw; ++k) {
@@ -328,20 +329,67 @@ std::string tile_jit_source(const Pass& p) {
           product(acc[sl], e, e + uint32_t(ns[sl]));
           e += uint32_t(ns[sl]);
         }
+        // general groups (compile-time r condition). Phase factors have modulus 1, so a factor
+        // a on "r bit k clear" is a on all slots times conj(a) on "r bit k set" (two doubling
+        // factors of the P-table instead of 8 multiplies), and a pair a on (r_i, r_j) = (1, 0),
+        // b on (0, 1) is e_i *= a, e_j *= b and conj(a b) on (1, 1) (4 multiplies instead of 8)
+        struct Grp {
+          uint32_t g0, g1, rm, rt;
+          bool done;
+        };
+        std::vector<Grp> grps;
+        const uint32_t end = op.moff + op.cnt;
+        for (uint32_t g0 = e; g0 < end;) {
+          uint32_t g1 = g0;
+          while (!P.entries[g1].gend) ++g1;
+          grps.push_back({g0, g1 + 1, P.entries[g0].rmask, P.entries[g0].rmatch, false});
+          g0 = g1 + 1;
+        }
+        std::vector<std::pair<uint32_t, std::string>> late;  // (r mask, factor) applied on r & mask == mask
+        int nfac = 0;
+        for (Grp& g : grps) {
+          if (std::popcount(g.rm) == 1 && g.rt == 0) {
+            const int k = std::countr_zero(g.rm);
+            o << "      { double2 acc;\n";
+            product("acc", g.g0, g.g1);
+            o << "        t0 = cmul(t0, acc); " << acc[1 + k] << " = cmul(" << acc[1 + k]
+              << ", make_double2(acc.x, -acc.y)); }\n";
+            used |= 1 | (2 << k);
+            g.done = true;
+          }
+        }
+        for (size_t x = 0; x < grps.size(); ++x) {
+          Grp& A = grps[x];
+          if (A.done || std::popcount(A.rm) != 2 || std::popcount(A.rt) != 1) continue;
+          for (size_t y = x + 1; y < grps.size(); ++y) {
+            Grp& B = grps[y];
+            if (B.done || B.rm != A.rm || B.rt != (A.rm & ~A.rt)) continue;
+            const int i = std::countr_zero(A.rt), j = std::countr_zero(B.rt);
+            const std::string fn = "fac" + std::to_string(nfac++);
+            o << "      double2 " << fn << ";\n      { double2 fa, fb;\n";
+            product("fa", A.g0, A.g1);
+            product("fb", B.g0, B.g1);
+            o << "        " << acc[1 + i] << " = cmul(" << acc[1 + i] << ", fa); " << acc[1 + j] << " = cmul("
+              << acc[1 + j] << ", fb);\n        " << fn << " = cmul(fa, fb); " << fn << ".y = -" << fn << ".y; }\n";
+            used |= (2 << i) | (2 << j);
+            late.push_back({A.rm, fn});
+            A.done = B.done = true;
+            break;
+          }
+        }
         if (used)
           o << "      run_apply_ptab_z<" << NR << ", " << (used & 1 ? "true" : "false") << ", "
             << ((used >> 1) & 1 ? "true" : "false") << ", " << ((used >> 2) & 1 ? "true" : "false") << ", "
             << ((used >> 3) & 1 ? "true" : "false") << ", " << ((used >> 4) & 1 ? "true" : "false") << ", " << zm
             << "u>(v, t0, e0, e1, e2, e3);\n";
-        const uint32_t end = op.moff + op.cnt;
-        for (uint32_t g0 = e; g0 < end;) {
-          uint32_t g1 = g0;
-          while (!P.entries[g1].gend) ++g1;
+        for (const auto& lf : late)
+          o << "      run_apply_group_z<" << NR << ", " << lf.first << "u, " << lf.first << "u, " << zm << "u>(v, "
+            << lf.second << ");\n";
+        for (const Grp& g : grps) {
+          if (g.done) continue;
           o << "      { double2 acc;\n";
-          product("acc", g0, g1 + 1);
-          o << "        run_apply_group_z<" << NR << ", " << P.entries[g0].rmask << "u, " << P.entries[g0].rmatch << "u, "
-            << zm << "u>(v, acc); }\n";
-          g0 = g1 + 1;
+          product("acc", g.g0, g.g1);
+          o << "        run_apply_group_z<" << NR << ", " << g.rm << "u, " << g.rt << "u, " << zm << "u>(v, acc); }\n";
         }
         break;
       }
@@ -364,7 +412,7 @@ std::string tile_jit_source(const Pass& p) {
         zpos &= ~((1u << R[op.a0]) | (1u << R[op.a1]));
         break;
       case OP_REMAP: {
-        int Wold[3] = {W[0], W[1], W[2]};
+        int Wold[4] = {W[0], W[1], W[2], W[3]};
         o << "      { constexpr uint32_t Jo[kRegAmps] = " << jtab(R) << ";\n";
         o << "        tile_store_j<" << NR << ">(v, c, mp.base, Jo); }\n";
         decode(op);
@@ -382,7 +430,7 @@ std::string tile_jit_source(const Pass& p) {
             }
           }
           if (nchg > 0) {  // nchg == 0: the thread's own slots, a register permutation
-            const int base = int(groups.size()) * 4;
+            const int base = int(groups.size()) << P.nw;
             groups.push_back({base, nchg});
             o << "      group_sync(c, " << base << " + (" << gexpr << "));\n";
           }

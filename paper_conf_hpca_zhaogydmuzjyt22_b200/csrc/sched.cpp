@@ -376,7 +376,7 @@ void split_patterns(TileProgram& P, const Pass& p, int m) {
   size_t nremap = 0;
   for (size_t i = 1; i < P.ops.size(); ++i) nremap += P.ops[i].kind == OP_REMAP;
   const size_t fixed = 3 * (size_t(16) << p.b) + ((size_t(1) << (p.b - p.l)) + 2) * 8 + P.bytes +
-                       2 * (size_t(1) << P.nw) * npat * 16 + 4 * nremap * 8 + 16;
+                       2 * (size_t(1) << P.nw) * npat * 16 + (size_t(1) << P.nw) * nremap * 8 + 16;
   int lb = nlo;
   while (lb > 0 && fixed + npat * (size_t(16) << lb) > 227 * 1024) --lb;
   P.lb = lb;
@@ -574,7 +574,7 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
     }
     return INF;
   };
-  int R[4] = {0, 0, 0, 0}, W[3] = {0, 0, 0};
+  int R[4] = {0, 0, 0, 0}, W[4] = {0, 0, 0, 0};
   auto choose = [&](uint32_t need, size_t from) {
     std::vector<int> cand;
     for (int t = lanes; t < b; ++t) cand.push_back(t);
@@ -593,13 +593,13 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
     } else {
       // a position that stays a warp bit keeps its warp-bit index, so a remap only moves data
       // between the warps that differ in the changed indices (warp-group remap, jit.cpp)
-      int nwk[3] = {-1, -1, -1};
+      int nwk[4] = {-1, -1, -1, -1};
       for (int k = 0; k < nw; ++k)
         if (std::find(w.begin(), w.end(), W[k]) != w.end()) nwk[k] = W[k];
       size_t next = 0;
       for (int k = 0; k < nw; ++k) {
         if (nwk[k] >= 0) continue;
-        while (std::find(nwk, nwk + 3, w[next]) != nwk + 3) ++next;
+        while (std::find(nwk, nwk + 4, w[next]) != nwk + 4) ++next;
         nwk[k] = w[next++];
       }
       for (int k = 0; k < nw; ++k) W[k] = nwk[k];
