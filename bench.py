@@ -491,7 +491,7 @@ def main():
     ap.add_argument("--warmup", type=int, default=3)
     ap.add_argument("--impl", default="ours", choices=["ours", "reference"])
     ap.add_argument("--workload", default="qft28")
-    ap.add_argument("--n", type=int, default=None)
+    ap.add_argument("--n", "--qubits", dest="n", type=int, default=None)
     ap.add_argument("--fuse-bits", type=int, default=12)
     ap.add_argument("--reorder", type=int, default=2)
     ap.add_argument("--no-prune", action="store_true")
