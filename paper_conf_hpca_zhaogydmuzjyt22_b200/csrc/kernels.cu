@@ -11,6 +11,9 @@
 //                     of the pass applied, one HBM read + one HBM write per amplitude
 //   gather/probs  a11 readout
 #include <cuda_runtime.h>
+#include <cstdlib>
+#include <bit>
+#include <vector>
 
 #include <algorithm>
 #include <cstdio>
@@ -363,6 +366,129 @@ __global__ void __launch_bounds__(kThreads) probs_kernel(ProbArgs a, int mode) {
   }
 }
 
+// a11 probabilities, mapped form: the index bits are dealt to the thread so that requested
+// positions are lane bits (0..4), warp bits or CTA-id bits wherever possible; then a thread's
+// bucket is fixed over its whole loop except for the <= 3 requested positions left in the loop
+// (the innermost loop bits, one register accumulator each). No histogram, no atomics in the
+// loop: every warp reads 512 contiguous bytes per step; at the end the lanes are reduced over the
+// non-requested lane bits and one atomic per bucket and warp adds into the output. Needs the
+// live range to be a power of two (it always is) and >= 2^5.
+struct ProbMap {
+  int wbits, cbits, ebits;
+  int wpos[4], cpos[16], epos[3];
+  int nfrun;                      // runs of fixed (non-loop) positions, ascending
+  int frun_pos[40], frun_len[40];
+  int obits;                      // loop bits
+};
+
+template <int E>
+__global__ void __launch_bounds__(512) probs_mapped_kernel(ProbArgs a, ProbMap mp) {
+  const int lane = threadIdx.x & 31, warp = threadIdx.x >> 5;
+  uint64_t tb = uint64_t(lane);
+  for (int k = 0; k < mp.wbits; ++k)
+    if ((warp >> k) & 1) tb |= 1ull << mp.wpos[k];
+  for (int k = 0; k < mp.cbits; ++k)
+    if ((blockIdx.x >> k) & 1) tb |= 1ull << mp.cpos[k];
+  auto bucket = [&](uint64_t idx) {
+    uint64_t y = a.yfixed;
+    for (int j = 0; j < a.m; ++j)
+      if (a.ppos[j] < 63 && ((idx >> a.ppos[j]) & 1)) y |= 1ull << j;
+    return y;
+  };
+  constexpr int NE = 1 << E;
+  uint64_t eoff[NE];
+#pragma unroll
+  for (int e = 0; e < NE; ++e) {
+    eoff[e] = 0;
+    for (int k = 0; k < E; ++k)
+      if ((e >> k) & 1) eoff[e] |= 1ull << mp.epos[k];
+  }
+  double acc[NE];
+#pragma unroll
+  for (int e = 0; e < NE; ++e) acc[e] = 0.0;
+  constexpr int U = NE >= 8 ? 1 : 8 / NE;  // loads in flight per thread: U * NE = 8
+  const uint64_t nouter = 1ull << mp.obits;
+  for (uint64_t o = 0; o < nouter; o += U) {
+    double2 v[U][NE];
+#pragma unroll
+    for (int u = 0; u < U; ++u) {
+      uint64_t t = o + u;
+      for (int i = 0; i < mp.nfrun; ++i) {
+        const int p = mp.frun_pos[i];
+        t = ((t >> p) << (p + mp.frun_len[i])) | (t & ((1ull << p) - 1));
+      }
+      const bool ok = o + u < nouter;
+#pragma unroll
+      for (int e = 0; e < NE; ++e) v[u][e] = ok ? __ldcs(a.psi + (tb | t | eoff[e])) : make_double2(0.0, 0.0);
+    }
+#pragma unroll
+    for (int u = 0; u < U; ++u)
+#pragma unroll
+      for (int e = 0; e < NE; ++e) acc[e] = fma(v[u][e].x, v[u][e].x, fma(v[u][e].y, v[u][e].y, acc[e]));
+  }
+  uint32_t lowreq = 0;
+  for (int j = 0; j < a.m; ++j)
+    if (a.ppos[j] < 5) lowreq |= 1u << a.ppos[j];
+#pragma unroll
+  for (int e = 0; e < NE; ++e) {
+    double x = acc[e];
+#pragma unroll
+    for (int b = 0; b < 5; ++b)
+      if (!((lowreq >> b) & 1)) x += __shfl_xor_sync(0xffffffffu, x, 1 << b);
+    if ((uint32_t(lane) & ~lowreq & 31u) == 0 && x != 0.0) atomicAdd(&a.out[bucket(tb | eoff[e])], x);
+  }
+}
+
+// Deal the live index bits (k = log2 L) to lanes / warps / CTAs / loop for probs_mapped_kernel;
+// false if more than 3 requested positions would be left in the loop.
+bool plan_probs_map(const ProbArgs& a, int k, ProbMap* mp) {
+  if (k < 5) return false;
+  std::vector<int> req;
+  uint64_t reqmask = 0;
+  for (int j = 0; j < a.m; ++j)
+    if (a.ppos[j] >= 5 && a.ppos[j] < k) req.push_back(a.ppos[j]), reqmask |= 1ull << a.ppos[j];
+  std::sort(req.begin(), req.end());
+  std::vector<int> other;  // non-requested positions >= 5, highest first
+  for (int p = k - 1; p >= 5; --p)
+    if (!((reqmask >> p) & 1)) other.push_back(p);
+  size_t ri = 0, oi = 0;
+  uint64_t fixed = 31;
+  *mp = ProbMap{};
+  mp->wbits = std::min(4, k - 5);
+  for (int i = 0; i < mp->wbits; ++i) {
+    const int p = ri < req.size() ? req[ri++] : other[oi++];
+    mp->wpos[i] = p;
+    fixed |= 1ull << p;
+  }
+  mp->cbits = std::min(10, k - 5 - mp->wbits);
+  for (int i = 0; i < mp->cbits; ++i) {
+    const int p = ri < req.size() ? req[ri++] : other[oi++];
+    mp->cpos[i] = p;
+    fixed |= 1ull << p;
+  }
+  mp->ebits = int(req.size() - ri);
+  if (mp->ebits > 3) return false;
+  for (int i = 0; i < mp->ebits; ++i) {
+    mp->epos[i] = req[ri + i];
+    fixed |= 1ull << mp->epos[i];
+  }
+  mp->obits = k - 5 - mp->wbits - mp->cbits - mp->ebits;
+  mp->nfrun = 0;
+  for (int p = 0; p < k;) {
+    if (!((fixed >> p) & 1)) {
+      ++p;
+      continue;
+    }
+    int q = p;
+    while (q + 1 < k && ((fixed >> (q + 1)) & 1)) ++q;
+    mp->frun_pos[mp->nfrun] = p;
+    mp->frun_len[mp->nfrun] = q - p + 1;
+    mp->nfrun++;
+    p = q + 1;
+  }
+  return true;
+}
+
 __global__ void set_amp_kernel(double2* psi, uint64_t i, double2 v) { psi[i] = v; }
 
 // a10 (virtual ranks): exchange the lp=1 half of shard a with the lp=0 half of shard b
@@ -495,6 +621,18 @@ cudaError_t launch_probs(cudaStream_t st, ProbArgs a, double*) {
   const size_t B = size_t(1) << a.m;
   cudaError_t e = cudaMemsetAsync(a.out, 0, sizeof(double) * B, st);
   if (e != cudaSuccess || a.L == 0) return e;
+  const int k = std::countr_zero(a.L);
+  ProbMap mp;
+  if ((a.L & (a.L - 1)) == 0 && std::getenv("QGPU_PROBS_HIST") == nullptr && plan_probs_map(a, k, &mp)) {
+    const unsigned grid = 1u << mp.cbits, threads = 32u << mp.wbits;
+    switch (mp.ebits) {
+      case 0: probs_mapped_kernel<0><<<grid, threads, 0, st>>>(a, mp); break;
+      case 1: probs_mapped_kernel<1><<<grid, threads, 0, st>>>(a, mp); break;
+      case 2: probs_mapped_kernel<2><<<grid, threads, 0, st>>>(a, mp); break;
+      default: probs_mapped_kernel<3><<<grid, threads, 0, st>>>(a, mp); break;
+    }
+    return cudaGetLastError();
+  }
   const int mode = a.m <= 10 ? 0 : (a.m <= 12 ? 1 : 2);
   const size_t smem = mode == 0 ? B * sizeof(double) * (kThreads / 32) : (mode == 1 ? B * sizeof(double) : 0);
   static bool configured = false;

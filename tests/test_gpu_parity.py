@@ -239,6 +239,28 @@ def test_probabilities_vs_oracle(q):
             assert np.abs(p - osv.probabilities(ref, n, qs)).max() <= 1e-12
 
 
+@pytest.mark.parametrize("hist", [0, 1])
+def test_probabilities_mapped_and_histogram_kernels(q, hist, monkeypatch):
+    """Both readout kernels (mapped: requested positions dealt to lanes/warps/CTAs; histogram:
+    QGPU_PROBS_HIST=1) on fully and partially involved states, many qubit subsets."""
+    if hist:
+        monkeypatch.setenv("QGPU_PROBS_HIST", "1")
+    rng = np.random.default_rng(77)
+    n = 16
+    for nq_involved in (16, 11):
+        c = wc.random_circuit(nq_involved, 160, seed=40 + nq_involved)
+        text = c.qasm().replace(f"qreg q[{nq_involved}];", f"qreg q[{n}];")
+        ref = oracle_run(text)
+        with q.State(n) as s:
+            s.apply_circuit(q.Circuit(text))
+            subsets = [[], [0], list(range(n)), [15, 3], list(range(10)), list(range(6, 16))]
+            subsets += [list(rng.choice(n, size=int(rng.integers(1, 13)), replace=False)) for _ in range(10)]
+            for qs in subsets:
+                qs = [int(x) for x in qs]
+                p = s.probabilities(qs)
+                assert np.abs(p - osv.probabilities(ref, n, qs)).max() <= 1e-12, qs
+
+
 def test_bv_large(q):
     n, sec = 24, 0b10110011100011110000101
     with q.State(n) as s:
