@@ -5,6 +5,7 @@
 #include <cctype>
 #include <cmath>
 #include <cstdlib>
+#include <cstring>
 #include <map>
 #include <string>
 #include <vector>
@@ -33,6 +34,7 @@ class Lexer {
   Lexer(const char* t, size_t n) : p_(t), e_(t + n) {}
   std::vector<Tok> run() {
     std::vector<Tok> out;
+    out.reserve(size_t(e_ - p_) / 3 + 16);
     for (;;) {
       skip();
       Tok t{T_EOF, "", 0, line_, col()};
@@ -62,12 +64,12 @@ class Lexer {
         t.k = T_STR; t.s.assign(s, p_); ++p_;
       } else if (c == '-' && p_ + 1 < e_ && p_[1] == '>') {
         t.k = T_ARROW; t.s = "->"; p_ += 2;
-      } else if (std::string(";,[](){}+-*/^").find(c) != std::string::npos) {
+      } else if (c != '\0' && std::strchr(";,[](){}+-*/^", c) != nullptr) {
         t.k = T_SYM; t.s = std::string(1, c); ++p_;
       } else {
         throw ParseError{QGPU_ERR_PARSE, at(t) + "unexpected character '" + std::string(1, c) + "'"};
       }
-      out.push_back(t);
+      out.push_back(std::move(t));
     }
   }
   static std::string at(const Tok& t) {
@@ -102,17 +104,17 @@ class Parser {
       expect(";");
     }
     while (peek().k != T_EOF) {
-      Tok t = next();
+      const Tok& t = next();
       if (t.k != T_ID) fail(t, "unexpected token '" + t.s + "'");
       if (t.s == "include") {
         if (peek().k != T_STR) fail(peek(), "expected file name");
         next();
         expect(";");
       } else if (t.s == "qreg" || t.s == "creg") {
-        Tok name = next();
+        const Tok& name = next();
         if (name.k != T_ID) fail(name, "expected register name");
         expect("[");
-        Tok sz = next();
+        const Tok& sz = next();
         if (sz.k != T_NUM) fail(sz, "expected register size");
         expect("]");
         expect(";");
@@ -136,7 +138,7 @@ class Parser {
 
  private:
   const Tok& peek() const { return t_[i_]; }
-  Tok next() { return t_[i_ < t_.size() - 1 ? i_++ : i_]; }
+  const Tok& next() { return t_[i_ < t_.size() - 1 ? i_++ : i_]; }
   bool is(const char* s) const { return peek().k == T_SYM && peek().s == s; }
   void expect(const char* s) {
     if (!is(s)) fail(peek(), std::string("expected '") + s + "', got '" + peek().s + "'");
@@ -177,7 +179,7 @@ class Parser {
     return b;
   }
   double primary() {
-    Tok t = next();
+    const Tok& t = next();
     if (t.k == T_NUM) return t.v;
     if (t.k == T_ID) {
       if (t.s == "pi") return M_PI;
@@ -201,12 +203,12 @@ class Parser {
   }
 
   std::vector<int> operand() {
-    Tok t = next();
+    const Tok& t = next();
     if (t.k != T_ID || !regs_.count(t.s)) fail(t, "unknown register '" + t.s + "'");
     auto r = regs_[t.s];
     if (is("[")) {
       next();
-      Tok i = next();
+      const Tok& i = next();
       if (i.k != T_NUM) fail(i, "expected index");
       expect("]");
       const int idx = int(i.v);
