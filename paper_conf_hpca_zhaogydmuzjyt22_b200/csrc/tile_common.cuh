@@ -773,7 +773,9 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       }
       k = kn;
       tile = next;
-      if ((nbuf < 3 || Body::kGroupRemap) && a.remaps) __syncthreads();
+      // no barrier: a zero tile neither reads nor fills its buffer (its loads were skipped), so
+      // running ahead through zero tiles cannot overwrite a buffer another warp still reads --
+      // the barrier after each live tile already orders every reuse of a buffer
       continue;
     }
     // pattern constants of this tile, per warp (lane-strided; each lane owns the same patterns
