@@ -6,7 +6,7 @@ and pruning (reorder=2, prune=1, fused passes b=12). A step = qgpu_state_reset +
 qgpu_apply_circuit of the whole circuit (every gate, the state resident in HBM); the metric
 is circuit seconds (lower is better). See DESIGN.md §7 for the byte model and peaks.
 
-    python bench.py [--gpus N --steps K --warmup W] [--workload qft28|qaoa32|rqc|gs|hlf]
+    python bench.py [--gpus N --steps K --warmup W] [--workload qft28|qaoa32|rqc|gs|hlf|grqc|iqp|bv]
     python bench.py --impl reference ...     # the oracle (plain CPU simulator) as the baseline arm
 
 N > 1 (torchrun): each rank runs its own replica of the workload (weak scaling, no data-path
@@ -52,6 +52,17 @@ def workload(name: str, n: int | None, world: int = 1):
     if name == "rqc":
         nn = n or 30
         return wc.rqc(nn, 20, seed=3), f"rqc_{nn} depth 20 seed 3 (configs[3] shape)"
+    if name == "grqc":
+        # Table III's deep Google circuit: 4x8 grid, 7238 operations at 32 qubits
+        nn = n or 32
+        r, cc = grid_shape(nn)
+        return wc.grqc(r, cc, 473, seed=5), f"grqc_{nn} {r}x{cc} grid depth 473 seed 5 (Table III deep circuit)"
+    if name == "iqp":
+        nn = n or 30
+        return wc.iqp(nn), f"iqp_{nn} seed 4"
+    if name == "bv":
+        nn = n or 30
+        return wc.bv(nn, (0b1011 * 0x11111111) & ((1 << (nn - 1)) - 1)), f"bv_{nn}"
     # grid workloads (configs[4]: 36 qubits on 8 GPUs = 128 GB per GPU): 2^33 amplitudes per GPU
     if name == "gs":
         r, cc = grid_shape(n or min(36, 33 + int(math.log2(world))))

@@ -92,6 +92,18 @@ def test_rqc30_mirror(q):
     assert abs(p[0] - 1) <= 1e-12
 
 
+def test_grqc30_deep_mirror(q):
+    """The paper's deep-circuit case (Table III): a 5x6 grid Google-style circuit of
+    ~2200 operations and its mirror (~4400 operations) returns |0...0> at 30 qubits."""
+    c = wc.grqc(5, 6, 120, seed=5)
+    with q.State(c.n) as s:
+        s.apply_circuit(q.Circuit(wc.mirror(c).qasm()))
+        a = s.amplitudes(0, 4096)
+        p = s.probabilities([])
+    assert abs(a[0] - 1) <= TOL and np.abs(a[1:]).max() <= TOL
+    assert abs(p[0] - 1) <= 1e-12
+
+
 def test_graph_state_30_sampled_ranges(q):
     c = wc.gs(5, 6)
     n, edges = c.n, c.meta["edges"]

@@ -69,13 +69,14 @@ def test_random_circuit_fuzz(q, n, G, seed, cfg):
     assert abs(1 - np.vdot(got, got).real) <= NORM_TOL
 
 
-@pytest.mark.parametrize("fam", ["qft", "qaoa", "rqc", "gs", "hlf", "iqp", "bv"])
+@pytest.mark.parametrize("fam", ["qft", "qaoa", "rqc", "gs", "hlf", "iqp", "bv", "grqc"])
 @pytest.mark.parametrize("fuse", [0, 12])
 def test_families_vs_oracle(q, fam, fuse):
     c = {"qft": lambda: wc.qft(18, x=12345), "qaoa": lambda: wc.qaoa(16, 2, seed=1),
          "rqc": lambda: wc.rqc(18, 12, seed=3), "gs": lambda: wc.gs(4, 4),
          "hlf": lambda: wc.hlf(4, 4, seed=2), "iqp": lambda: wc.iqp(14),
-         "bv": lambda: wc.bv(15, 0b101101110110101)}[fam]()
+         "bv": lambda: wc.bv(15, 0b101101110110101),
+         "grqc": lambda: wc.grqc(4, 4, 60, seed=5)}[fam]()
     text = c.qasm()
     got = gpu_run(q, text, fuse_bits=fuse)
     ref = oracle_run(text)

@@ -30,6 +30,7 @@ CIRCS = {
     "rqc": lambda: wc.rqc(12, 8, seed=3),
     "qaoa": lambda: wc.qaoa(12, 2, seed=5),
     "hlf": lambda: wc.hlf(3, 4, seed=2),
+    "grqc": lambda: wc.grqc(3, 4, 48, seed=5),  # deep 2-D circuit: many global-local swaps
 }
 
 

@@ -241,11 +241,12 @@ def test_grover_success_probability(n, w, k):
     assert abs(abs(psi[w]) ** 2 - math.sin((2 * k + 1) * th) ** 2) < 1e-12
 
 
-@pytest.mark.parametrize("fam", ["qaoa", "rqc", "random", "iqp"])
+@pytest.mark.parametrize("fam", ["qaoa", "rqc", "random", "iqp", "grqc"])
 def test_norm_and_mirror(fam):
     """norm conserved; U U^dagger returns e_0."""
     c = {"qaoa": lambda: wc.qaoa(10, 2, seed=1), "rqc": lambda: wc.rqc(10, 8, seed=3),
-         "random": lambda: wc.random_circuit(9, 200, seed=5), "iqp": lambda: wc.iqp(9)}[fam]()
+         "random": lambda: wc.random_circuit(9, 200, seed=5), "iqp": lambda: wc.iqp(9),
+         "grqc": lambda: wc.grqc(3, 3, 40, seed=5)}[fam]()
     psi = osv.simulate(c.qasm())
     assert abs(1 - np.vdot(psi, psi).real) < 1e-12
     m = osv.simulate(wc.mirror(c).qasm())

@@ -146,12 +146,13 @@ def q():
 
 
 @pytest.mark.parametrize("world", [2, 4])
-@pytest.mark.parametrize("name", ["random", "qft", "rqc", "ghz"])
+@pytest.mark.parametrize("name", ["random", "qft", "rqc", "ghz", "grqc"])
 def test_sharded_protocol_vs_oracle(q, world, name):
     c = {"random": lambda: wc.random_circuit(8, 90, seed=world),
          "qft": lambda: wc.qft(8, x=171),
          "rqc": lambda: wc.rqc(8, 6, seed=3),
-         "ghz": lambda: wc.ghz(9)}[name]()
+         "ghz": lambda: wc.ghz(9),
+         "grqc": lambda: wc.grqc(2, 4, 40, seed=5)}[name]()
     got, text = _run_sharded(q, c, world, fuse=12)
     ref = osv.simulate(c.qasm())
     assert np.abs(got - ref).max() <= 1e-12

@@ -178,6 +178,51 @@ def rqc(n: int, depth: int = 20, seed: int = 3) -> Circuit:
     return c
 
 
+def grqc(rows: int, cols: int, depth: int, seed: int = 5) -> Circuit:
+    """Google-style deep random circuit on a 2-D grid (the paper's "grqc", Table III,
+    generated "under rules defined in [9]"; the exact rules are not given, reading in DESIGN.md):
+    H on all; cycle t = 1..depth applies CZ on the couplers of class (t - 1) mod 8 (horizontal
+    couplers split by (row mod 2, col mod 2), then vertical ones likewise), then on every qubit
+    that was in a CZ in the previous cycle and is not in one now a single-qubit gate: T if it
+    has had none yet, else one of {sqrt X, sqrt Y, T} different from its previous one. A 4x8
+    grid with depth 473 gives 7238 operations, the size of Table III's grqc_32 (7241)."""
+    rng = np.random.default_rng(seed)
+    n = rows * cols
+    c = Circuit(n, meta={"family": "grqc", "rows": rows, "cols": cols, "depth": depth, "seed": seed})
+    for q in range(n):
+        c.add("h", [q])
+    classes: List[List[Tuple[int, int]]] = [[] for _ in range(8)]
+    for r in range(rows):
+        for cc in range(cols):
+            q = r * cols + cc
+            if cc + 1 < cols:
+                classes[2 * (r % 2) + (cc % 2)].append((q, q + 1))
+            if r + 1 < rows:
+                classes[4 + 2 * (r % 2) + (cc % 2)].append((q, q + cols))
+    gates = [("rx", ("pi/2",)), ("ry", ("pi/2",)), ("t", ())]
+    last = [-1] * n
+    prev_cz: set = set()
+    for t in range(1, depth + 1):
+        cur = classes[(t - 1) % 8]
+        busy = set()
+        for u, v in cur:
+            c.add("cz", [u, v])
+            busy.update((u, v))
+        for q in range(n):
+            if q in prev_cz and q not in busy:
+                if last[q] < 0:
+                    k = 2
+                else:
+                    k = int(rng.integers(0, 3))
+                    while k == last[q]:
+                        k = int(rng.integers(0, 3))
+                last[q] = k
+                name, ps = gates[k]
+                c.add(name, [q], ps)
+        prev_cz = busy
+    return c
+
+
 def grid_edges(rows: int, cols: int) -> List[Tuple[int, int]]:
     e = []
     for r in range(rows):
