@@ -35,7 +35,7 @@
 extern "C" {
 #endif
 
-#define QGPU_ABI_VERSION 1
+#define QGPU_ABI_VERSION 2
 
 typedef enum {
   QGPU_OK = 0,
@@ -75,6 +75,16 @@ typedef struct {
   int jit;                    /* fused passes: 0 = generic tile kernel only; 1 (default) = NVRTC-
                                  specialised kernel for passes of >= 2^20 amplitudes; 2 = always.
                                  Falls back to the generic kernel if NVRTC is unavailable   */
+  int host_slice_bits;        /* h: host-memory tier (the paper's setting,
+                                 P:185-191). 0 (default) = state resident in HBM. h > 0
+                                 (world_size = 1 only): the 2^n amplitudes live in pinned host
+                                 memory as 2^h slices of 2^(n-h); the circuit is planned as
+                                 for 2^h virtual ranks (slice index = top h physical bits) and
+                                 each run of passes between global-local swaps streams the
+                                 active slices through device slots (H2D, passes, D2H on three
+                                 streams, double-buffered). Pruning skips never-active slices
+                                 and moves only each slice's live prefix across the link.
+                                 Device memory: 4-8 slots of 16 * 2^(n-h) bytes              */
 } qgpu_config;
 
 typedef struct {
@@ -101,6 +111,13 @@ typedef struct {
   uint64_t jit_launches;       /* fused passes run by an NVRTC-specialised kernel            */
   uint64_t jit_compiles;       /* kernels compiled (cache misses)                            */
   double jit_ms;               /* host time spent compiling                                  */
+  /* host-memory tier (host_slice_bits > 0) */
+  uint64_t host_h2d_bytes;     /* slice bytes copied host -> device (live prefixes only)      */
+  uint64_t host_d2h_bytes;     /* slice bytes copied device -> host                           */
+  uint64_t host_slice_loads;   /* slices streamed through the device                         */
+  uint64_t host_slice_skips;   /* slice visits skipped because the slice is all zero  */
+  uint64_t host_runs;          /* runs of passes (one streaming sweep over the slices each)  */
+  double host_ms;              /* timing=1: CUDA-event time of the streaming sweeps          */
 } qgpu_stats;
 
 /* ---- configuration and state ---------------------------------------------------------- */
@@ -126,13 +143,15 @@ qgpu_status qgpu_state_reset(qgpu_state* st);
 
 /* Overwrite the full logical state from host memory: amps = 2 * 2^n doubles (re, im) in
  * logical index order. Marks every qubit involved (nothing left to prune). Synchronises.
- * Single-GPU only (UNSUPPORTED when sharded). */
+ * Single-GPU or host tier (UNSUPPORTED when sharded over ranks). */
 qgpu_status qgpu_set_amplitudes(qgpu_state* st, const double* amps);
 
 /* Block until all work enqueued on the state's stream is done; reports async errors. */
 qgpu_status qgpu_synchronize(qgpu_state* st);
 
-/* Number of qubits, local qubits (n - log2 world) and device pointer of the local buffer. */
+/* Number of qubits, local qubits (n - log2 world, or n - host_slice_bits) and the pointer of
+ * the local buffer (device memory; with the host tier: the pinned host state, which is also
+ * device-accessible through unified addressing). */
 qgpu_status qgpu_state_info(const qgpu_state* st, int* n_qubits, int* n_local, void** dev_ptr);
 
 /* ---- gate application (the hot path) --------------------------------------------------- */

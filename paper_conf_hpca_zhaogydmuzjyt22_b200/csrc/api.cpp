@@ -78,6 +78,8 @@ qgpu_status fail(qgpu_status s, const char* fmt, ...) {
   return s;
 }
 
+constexpr int kHostSweep = 100;  // TimedLaunch kind of a host-tier streaming sweep
+
 struct TimedLaunch {
   cudaEvent_t a, b;
   int kind;
@@ -122,6 +124,16 @@ struct qgpu_state {
   Comm* comm = nullptr;
   std::vector<CachedPlan> plans;  // small LRU (kMaxPlans)
   uint64_t plan_clock = 0;
+  // host-memory tier (cfg.host_slice_bits = h > 0, NEXT-2): 2^h slices of 2^m amplitudes in
+  // pinned, device-mapped host memory (shards[r].psi = slice r), streamed through device slots
+  bool host = false;
+  double2* h_state = nullptr;
+  std::vector<uint64_t> hlive;       // slice r: amplitudes [0, hlive[r]) valid, the rest zero
+  std::vector<double2*> slots;       // device slot buffers, 2^m amplitudes each
+  int unit_cap = 0;                  // slices per slot group (slots.size() / groups)
+  cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
+  cudaEvent_t ev_loaded[2] = {}, ev_computed[2] = {}, ev_stored[2] = {}, ev_join = nullptr;
+  bool group_used[2] = {false, false};
 };
 
 namespace {
@@ -161,6 +173,8 @@ qgpu_status drain_timing(qgpu_state* st) {
     CK(cudaEventElapsedTime(&ms, t.a, t.b));
     if (t.kind == PK_SWAP) {
       st->stats.swap_ms += ms;
+    } else if (t.kind == kHostSweep) {
+      st->stats.host_ms += ms;
     } else {
       st->stats.kernel_ms += ms;
       if (t.kind == PK_TILE) {
@@ -320,7 +334,11 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     } else if (p.kind == PK_PAIR || p.kind == PK_QUAD) {
       const bool full = g.expands_target || !st->cfg.prune;
       const int krun = full ? kout : kin;
-      if (!full) {
+      // the kernel writes only the pairs whose controls are satisfied: the rest of an expanded
+      // region [L_in, L_out) must be written as zeros here (the buffer may hold stale data
+      // from before a reset, or another slice's in a host-tier slot)
+      const bool zero_new = !full || (lc != 0 && L_out > L_in);
+      if (zero_new) {
         qgpu_status s = zero_fill(st, psi, L_in, L_out);
         if (s) return s;
       }
@@ -338,7 +356,7 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
         a.L_in = L_in;
         const bool shfl = g.p[0] < 5 && krun >= 5 && (lc & 31) == 0;
         CK(launch_pair(st->stream, a, shfl));
-        bytes = 32 * a.npairs + (full ? 0 : 16 * (L_out - L_in));
+        bytes = 32 * a.npairs + (zero_new ? 16 * (L_out - L_in) : 0);
       } else {
         QuadArgs a{};
         a.psi = psi;
@@ -350,7 +368,7 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
         a.nquads = ctl_in_range ? (1ull << (krun - 2 - nlc)) : 0;
         a.L_in = L_in;
         CK(launch_quad(st->stream, a));
-        bytes = 64 * a.nquads + (full ? 0 : 16 * (L_out - L_in));
+        bytes = 64 * a.nquads + (zero_new ? 16 * (L_out - L_in) : 0);
       }
       st->stats.kernels_launched++;
     } else {  // PK_DIAG: the expanded region stays zero under a diagonal gate
@@ -464,6 +482,235 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops)
   return QGPU_OK;
 }
 
+// ------------------------------------------------------------ host-memory tier (NEXT-2)
+// The paper keeps the state in host memory and moves chunks to the GPU and back for every
+// gate, overlapping the transfers on two streams and skipping all-zero chunks
+// (Alg.1). B200 form: the circuit is planned for 2^h virtual ranks (slice index = the
+// top h physical bits), so between two global-local swaps every pass works on one slice at a
+// time. Such a run of passes becomes ONE streaming sweep over the active slices: per unit of
+// slices, H2D of their live prefixes (s_h2d), every pass of the run (the state's stream), D2H
+// (s_d2h); two slot groups let the copies of one unit overlap the compute of the other. A swap
+// is folded into the next sweep: a unit is the set of slices that differ in the swapped rank
+// bits, exchanged on the device right after loading. Never-active slices (all zero) are
+// skipped, and only the live prefix [0, 2^kl) of a slice crosses the link.
+
+struct HostSwap {
+  int j, lp;  // rank bit j <-> local position lp
+};
+
+// Ensure two groups of `unit` device slots (one group if memory runs out).
+qgpu_status ensure_slots(qgpu_state* st, int unit, int* ngroups) {
+  const size_t bytes = (size_t(1) << st->m) * sizeof(double2);
+  while (st->slots.size() < size_t(2 * unit)) {
+    double2* p = nullptr;
+    cudaError_t e = cudaMalloc(&p, bytes);
+    if (e != cudaSuccess) {
+      cudaGetLastError();
+      if (st->slots.size() >= size_t(unit)) break;
+      return fail(QGPU_ERR_OUT_OF_MEMORY, "host tier: cudaMalloc of a %llu-byte slot: %s",
+                  (unsigned long long)bytes, cudaGetErrorString(e));
+    }
+    st->slots.push_back(p);
+  }
+  *ngroups = st->slots.size() >= size_t(2 * unit) ? 2 : 1;
+  return QGPU_OK;
+}
+
+// One streaming sweep: swaps `sw` (made while 2^kg_sw ranks were active), then the passes `run`.
+qgpu_status host_sweep(qgpu_state* st, const std::vector<const Pass*>& run,
+                       const std::vector<const unsigned char*>& ops, const std::vector<HostSwap>& sw,
+                       int kg_sw) {
+  const int m = st->m;
+  const uint64_t full = 1ull << m;
+  int kg = sw.empty() ? 0 : kg_sw;
+  for (const Pass* p : run) kg = std::max(kg, p->kg);
+  const uint64_t nact = 1ull << kg;
+  int ubit[8], nub = 0;
+  uint64_t ubits = 0;
+  for (const HostSwap& x : sw)
+    if (!(ubits >> x.j & 1)) {
+      ubits |= 1ull << x.j;
+      ubit[nub++] = x.j;
+    }
+  const int unit = 1 << nub;
+  int ngroups = 1;
+  if (qgpu_status s = ensure_slots(st, unit, &ngroups)) return s;
+  // every earlier use of the slices: work on the state's stream and earlier sweeps' stores
+  CK(cudaEventRecord(st->ev_join, st->stream));
+  CK(cudaStreamWaitEvent(st->s_h2d, st->ev_join, 0));
+  for (int gi = 0; gi < 2; ++gi)
+    if (st->group_used[gi]) CK(cudaStreamWaitEvent(st->s_h2d, st->ev_stored[gi], 0));
+  const bool timing = st->cfg.timing != 0;
+  TimedLaunch sweep{};
+  if (timing) {
+    sweep.a = get_event(st);
+    sweep.b = get_event(st);
+    sweep.kind = kHostSweep;
+    CK(cudaEventRecord(sweep.a, st->s_h2d));
+  }
+  const uint64_t L_end = run.empty() ? full : live(st, run.back()->k_out);
+  std::vector<char> accounted(run.size(), 0);
+  uint64_t moved = 0;
+  int u = 0;
+  for (uint64_t base = 0; base < nact; ++base) {
+    if (base & ubits) continue;
+    const int gi = (ngroups == 2) ? (u & 1) : 0;
+    ++u;
+    double2** slot = &st->slots[size_t(gi) * size_t(unit)];
+    uint64_t rs[1 << 8];
+    for (int x = 0; x < unit; ++x) {
+      rs[x] = base;
+      for (int i = 0; i < nub; ++i)
+        if (x >> i & 1) rs[x] |= 1ull << ubit[i];
+    }
+    const bool swap_here = !sw.empty() && base < (1ull << kg_sw);
+    // load: the live prefix from host memory, zeros up to what the first pass reads
+    if (st->group_used[gi]) CK(cudaStreamWaitEvent(st->s_h2d, st->ev_stored[gi], 0));
+    for (int x = 0; x < unit; ++x) {
+      const uint64_t r = rs[x];
+      uint64_t need = 0;
+      if (swap_here) {
+        need = full;
+      } else {
+        for (const Pass* p : run)
+          if (r < (1ull << p->kg)) {
+            need = live(st, p->k_in);
+            break;
+          }
+      }
+      const uint64_t copy = std::min(st->hlive[r], need);
+      if (copy)
+        CK(cudaMemcpyAsync(slot[x], st->shards[r].psi, copy * sizeof(double2), cudaMemcpyHostToDevice,
+                           st->s_h2d));
+      if (need > copy)
+        CK(cudaMemsetAsync(slot[x] + copy, 0, (need - copy) * sizeof(double2), st->s_h2d));
+      st->stats.host_h2d_bytes += copy * sizeof(double2);
+      st->stats.h2d_bytes += copy * sizeof(double2);
+      st->stats.host_slice_loads++;
+    }
+    CK(cudaEventRecord(st->ev_loaded[gi], st->s_h2d));
+    // compute: swaps, then every pass of the run on every slice active at that pass
+    CK(cudaStreamWaitEvent(st->stream, st->ev_loaded[gi], 0));
+    if (swap_here) {
+      for (const HostSwap& x : sw) {
+        int bi = 0;
+        while (ubit[bi] != x.j) ++bi;
+        for (int xi = 0; xi < unit; ++xi) {
+          if (xi >> bi & 1) continue;
+          CK(launch_swap_halves(st->stream, slot[xi], slot[xi | (1 << bi)], x.lp, full / 2));
+          st->stats.kernels_launched++;
+        }
+      }
+    }
+    for (size_t i = 0; i < run.size(); ++i) {
+      const Pass& p = *run[i];
+      const uint64_t L_in = live(st, p.k_in), L_out = live(st, p.k_out);
+      for (int x = 0; x < unit; ++x) {
+        const uint64_t r = rs[x];
+        if (r >= (1ull << p.kg)) continue;
+        uint64_t b = 0;
+        if (p.kind == PK_RELABEL) {
+          if (L_out <= L_in) continue;
+          if (qgpu_status s = zero_fill(st, slot[x], L_in, L_out)) return s;
+          st->stats.kernels_launched++;
+          b = 16 * (L_out - L_in);
+        } else {
+          TimedLaunch tl{};
+          if (timing) {
+            tl.a = get_event(st);
+            tl.b = get_event(st);
+            tl.kind = p.kind;
+            CK(cudaEventRecord(tl.a, st->stream));
+          }
+          if (qgpu_status s = exec_compute(st, p, ops[i], slot[x], r, &b)) return s;
+          if (timing) {
+            CK(cudaEventRecord(tl.b, st->stream));
+            tl.bytes = b;
+            st->pending.push_back(tl);
+          }
+        }
+        if (!accounted[i]) {
+          accounted[i] = 1;
+          account(st, L_out, b);
+          st->stats.unfused_bytes += p.unfused_bytes;
+        }
+      }
+    }
+    CK(cudaEventRecord(st->ev_computed[gi], st->stream));
+    // store the live prefix back
+    CK(cudaStreamWaitEvent(st->s_d2h, st->ev_computed[gi], 0));
+    for (int x = 0; x < unit; ++x) {
+      const uint64_t r = rs[x];
+      CK(cudaMemcpyAsync(st->shards[r].psi, slot[x], L_end * sizeof(double2), cudaMemcpyDeviceToHost,
+                         st->s_d2h));
+      st->hlive[r] = L_end;
+      st->stats.host_d2h_bytes += L_end * sizeof(double2);
+      st->stats.d2h_bytes += L_end * sizeof(double2);
+      moved += L_end;
+    }
+    CK(cudaEventRecord(st->ev_stored[gi], st->s_d2h));
+    st->group_used[gi] = true;
+  }
+  (void)moved;
+  st->stats.host_slice_skips += (1ull << st->g) - nact;
+  for (const HostSwap& x : sw) {
+    (void)x;
+    st->stats.swaps++;
+    st->stats.swap_bytes += 16 * (full / 2) * (nact >> 1);
+  }
+  st->stats.host_runs++;
+  if (timing) {
+    CK(cudaEventRecord(sweep.b, st->s_d2h));
+    st->pending.push_back(sweep);
+  }
+  // later work on the state's stream (readout, the next apply) sees the stored slices
+  CK(cudaEventRecord(st->ev_join, st->s_d2h));
+  CK(cudaStreamWaitEvent(st->stream, st->ev_join, 0));
+  return QGPU_OK;
+}
+
+// Execute planned passes: resident state pass by pass; host tier as streaming sweeps, one per
+// run of passes between global-local swaps (consecutive swaps join one sweep, <= 2 rank bits).
+qgpu_status exec_passes(qgpu_state* st, const std::vector<Pass>& passes,
+                        const std::vector<const unsigned char*>& ops) {
+  if (!st->host) {
+    for (size_t i = 0; i < passes.size(); ++i)
+      if (qgpu_status s = exec_pass(st, passes[i], ops[i])) return s;
+    return QGPU_OK;
+  }
+  std::vector<const Pass*> run;
+  std::vector<const unsigned char*> run_ops;
+  std::vector<HostSwap> sw;
+  int kg_sw = 0;
+  auto flush = [&]() -> qgpu_status {
+    if (run.empty() && sw.empty()) return QGPU_OK;
+    qgpu_status s = host_sweep(st, run, run_ops, sw, kg_sw);
+    run.clear();
+    run_ops.clear();
+    sw.clear();
+    return s;
+  };
+  for (size_t i = 0; i < passes.size(); ++i) {
+    const Pass& p = passes[i];
+    if (p.kind == PK_ACTIVATE) continue;  // newly active slices are all zero (hlive = 0)
+    if (p.kind == PK_SWAP) {
+      if (!run.empty())
+        if (qgpu_status s = flush()) return s;
+      uint64_t bits = 0;
+      for (const HostSwap& x : sw) bits |= 1ull << x.j;
+      for (int k = 0; k < p.nswap; ++k) bits |= 1ull << (p.swap_global[k] - st->m);
+      if (std::popcount(bits) > 2)
+        if (qgpu_status s = flush()) return s;
+      for (int k = 0; k < p.nswap; ++k) sw.push_back(HostSwap{p.swap_global[k] - st->m, p.swap_local[k]});
+      kg_sw = p.kg;
+      continue;
+    }
+    run.push_back(&p);
+    run_ops.push_back(ops[i]);
+  }
+  return flush();
+}
+
 qgpu_status ensure_ops(qgpu_state* st, size_t n) {
   if (n <= st->ops_cap) return QGPU_OK;
   size_t cap = std::max<size_t>(n, 2 * st->ops_cap);
@@ -500,11 +747,9 @@ qgpu_status run_plan(qgpu_state* st, const std::vector<Pass>& passes) {
     CK(cudaEventRecord(st->ops_evt, st->stream));
   }
   prepare_jit(st, passes);
-  for (size_t i = 0; i < passes.size(); ++i) {
-    qgpu_status s = exec_pass(st, passes[i], st->d_ops + off[i]);
-    if (s) return s;
-  }
-  return QGPU_OK;
+  std::vector<const unsigned char*> ops(passes.size());
+  for (size_t i = 0; i < passes.size(); ++i) ops[i] = st->d_ops + off[i];
+  return exec_passes(st, passes, ops);
 }
 
 void record_trace(qgpu_state* st, const std::vector<int>& order, const std::vector<uint64_t>& inv,
@@ -526,6 +771,16 @@ qgpu_status check_state(qgpu_state* st) {
 }
 
 qgpu_status init_amplitudes(qgpu_state* st) {
+  if (st->host) {
+    // host tier: |0...0> = slice 0 holds psi[0] = 1, every other amplitude reads as zero
+    // through hlive (the host pages beyond hlive are never read)
+    CK(cudaStreamSynchronize(st->stream));
+    CK(cudaStreamSynchronize(st->s_d2h));
+    st->h_state[0] = make_double2(1.0, 0.0);
+    std::fill(st->hlive.begin(), st->hlive.end(), 0);
+    st->hlive[0] = 1;
+    return QGPU_OK;
+  }
   for (Shard& sh : st->shards) {
     if (!st->cfg.prune) CK(cudaMemsetAsync(sh.psi, 0, (1ull << st->m) * sizeof(double2), st->stream));
     if (sh.rank == 0) {
@@ -671,7 +926,9 @@ qgpu_status qgpu_gfc_decompress(const void* d_in, const uint64_t* d_offsets, uin
 }
 
 const char* qgpu_version(void) {
-  return "qgpu abi " "1" " sm_100a (B200) complex128";
+#define QGPU_STR2(x) #x
+#define QGPU_STR(x) QGPU_STR2(x)
+  return "qgpu abi " QGPU_STR(QGPU_ABI_VERSION) " sm_100a (B200) complex128";
 }
 
 qgpu_status qgpu_config_init(qgpu_config* cfg) {
@@ -705,8 +962,12 @@ qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out
       return fail(QGPU_ERR_INVALID_ARG, "world_size %d is not a power of two", cfg.world_size);
     if (cfg.rank < 0 || cfg.rank >= cfg.world_size)
       return fail(QGPU_ERR_INVALID_ARG, "rank %d out of range", cfg.rank);
-    const int g = std::countr_zero(unsigned(cfg.world_size));
-    if (n - g < 5) return fail(QGPU_ERR_INVALID_ARG, "need n - log2(world_size) >= 5");
+    if (cfg.host_slice_bits < 0 || cfg.host_slice_bits > 16)
+      return fail(QGPU_ERR_INVALID_ARG, "host_slice_bits %d out of [0, 16]", cfg.host_slice_bits);
+    if (cfg.host_slice_bits > 0 && (cfg.world_size != 1 || cfg.state_buffer))
+      return fail(QGPU_ERR_UNSUPPORTED, "the host tier needs world_size 1 and no state_buffer");
+    const int g = cfg.host_slice_bits > 0 ? cfg.host_slice_bits : std::countr_zero(unsigned(cfg.world_size));
+    if (n - g < 5) return fail(QGPU_ERR_INVALID_ARG, "need n - log2(world_size) - host_slice_bits >= 5");
     if (cfg.fuse_bits < 0 || cfg.fuse_bits > kMaxTileBits - 1)
       return fail(QGPU_ERR_INVALID_ARG, "fuse_bits %d out of [0, %d]", cfg.fuse_bits, kMaxTileBits - 1);
     if (cfg.fuse_bits > 0 && cfg.fuse_bits < 7)
@@ -740,9 +1001,37 @@ qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out
     // world_size > 1 without an NCCL id: "virtual ranks", every shard in this process on this
     // GPU (exercises the sharded path -- rank-bit conditions, activation, swaps -- on one GPU)
     st->virt = cfg.world_size > 1 && cfg.nccl_unique_id == nullptr;
-    const int nshard = st->virt ? cfg.world_size : 1;
+    st->host = cfg.host_slice_bits > 0;
+    const int nshard = st->host ? (1 << g) : st->virt ? cfg.world_size : 1;
     if (st->virt && cfg.state_buffer) return bail(fail(QGPU_ERR_UNSUPPORTED, "virtual ranks allocate their own shards"));
-    for (int r = 0; r < nshard; ++r) {
+    if (st->host) {
+      // pinned, device-mapped host memory: slices stream through device slots; readout kernels
+      // read it in place (zero-copy) through unified addressing
+      const size_t hbytes = (size_t(1) << n) * sizeof(double2);
+      e = cudaHostAlloc(&st->h_state, hbytes, cudaHostAllocMapped | cudaHostAllocPortable);
+      if (e != cudaSuccess) {
+        cudaGetLastError();
+        st->h_state = nullptr;
+        return bail(fail(QGPU_ERR_OUT_OF_MEMORY, "host tier: cudaHostAlloc(%zu): %s", hbytes, cudaGetErrorString(e)));
+      }
+      double2* dev = nullptr;
+      e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&dev), st->h_state, 0);
+      if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaHostGetDevicePointer: %s", cudaGetErrorString(e)));
+      for (int r = 0; r < nshard; ++r) st->shards.push_back(Shard{r, dev + (size_t(r) << st->m), false});
+      st->hlive.assign(size_t(nshard), 0);
+      for (cudaStream_t* sp : {&st->s_h2d, &st->s_d2h}) {
+        e = cudaStreamCreateWithFlags(sp, cudaStreamNonBlocking);
+        if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaStreamCreate: %s", cudaGetErrorString(e)));
+      }
+      for (int i = 0; i < 2 && e == cudaSuccess; ++i) {
+        e = cudaEventCreateWithFlags(&st->ev_loaded[i], cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&st->ev_computed[i], cudaEventDisableTiming);
+        if (e == cudaSuccess) e = cudaEventCreateWithFlags(&st->ev_stored[i], cudaEventDisableTiming);
+      }
+      if (e == cudaSuccess) e = cudaEventCreateWithFlags(&st->ev_join, cudaEventDisableTiming);
+      if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e)));
+    }
+    for (int r = 0; r < nshard && !st->host; ++r) {
       Shard sh;
       sh.rank = st->virt ? r : cfg.rank;
       if (cfg.state_buffer) {
@@ -792,6 +1081,16 @@ qgpu_status qgpu_state_destroy(qgpu_state* st) {
   }
   for (auto e : st->event_pool) cudaEventDestroy(e);
   if (st->comm) comm_destroy(st->comm);
+  if (st->s_h2d) cudaStreamSynchronize(st->s_h2d);
+  if (st->s_d2h) cudaStreamSynchronize(st->s_d2h);
+  for (double2* p : st->slots) cudaFree(p);
+  if (st->h_state) cudaFreeHost(st->h_state);
+  for (int i = 0; i < 2; ++i)
+    for (cudaEvent_t e : {st->ev_loaded[i], st->ev_computed[i], st->ev_stored[i]})
+      if (e) cudaEventDestroy(e);
+  if (st->ev_join) cudaEventDestroy(st->ev_join);
+  if (st->s_h2d) cudaStreamDestroy(st->s_h2d);
+  if (st->s_d2h) cudaStreamDestroy(st->s_d2h);
   for (Shard& sh : st->shards)
     if (sh.own && sh.psi) cudaFree(sh.psi);
   if (st->d_ops) cudaFree(st->d_ops);
@@ -823,16 +1122,24 @@ qgpu_status qgpu_state_reset(qgpu_state* st) {
 qgpu_status qgpu_set_amplitudes(qgpu_state* st, const double* amps) {
   if (qgpu_status s = check_state(st)) return s;
   if (!amps) return fail(QGPU_ERR_INVALID_ARG, "amps is NULL");
-  if (st->g > 0) return fail(QGPU_ERR_UNSUPPORTED, "set_amplitudes is single-GPU only");
-  st->psi = st->shards[0].psi;
-  CK(cudaMemcpyAsync(st->psi, amps, (1ull << st->n) * sizeof(double2), cudaMemcpyHostToDevice, st->stream));
-  CK(cudaStreamSynchronize(st->stream));
+  if (st->g > 0 && !st->host) return fail(QGPU_ERR_UNSUPPORTED, "set_amplitudes is single-GPU only");
+  if (st->host) {
+    CK(cudaStreamSynchronize(st->stream));
+    CK(cudaStreamSynchronize(st->s_d2h));
+    std::memcpy(st->h_state, amps, (size_t(1) << st->n) * sizeof(double2));
+    std::fill(st->hlive.begin(), st->hlive.end(), 1ull << st->m);
+  } else {
+    st->psi = st->shards[0].psi;
+    CK(cudaMemcpyAsync(st->psi, amps, (1ull << st->n) * sizeof(double2), cudaMemcpyHostToDevice, st->stream));
+    CK(cudaStreamSynchronize(st->stream));
+  }
   st->map.init(st->n, st->m);
   for (int q = 0; q < st->n; ++q) {
     st->map.pos[q] = q;
     st->map.lq[q] = q;
   }
-  st->map.kl = st->n;
+  st->map.kl = st->m;
+  st->map.kg = st->n - st->m;
   st->map.involvement = (st->n >= 64) ? ~0ull : ((1ull << st->n) - 1);
   return QGPU_OK;
 }
@@ -922,11 +1229,9 @@ qgpu_status qgpu_apply_circuit(qgpu_state* st, const qgpu_circuit* c) {
     record_trace(st, hit->order, hit->inv, 0);
     st->stats.relabels += hit->relabels;
     st->map = hit->map_after;
-    for (size_t i = 0; i < hit->passes.size(); ++i) {
-      qgpu_status s = exec_pass(st, hit->passes[i], hit->d_blob ? hit->d_blob + hit->off[i] : nullptr);
-      if (s) return s;
-    }
-    return QGPU_OK;
+    std::vector<const unsigned char*> ops(hit->passes.size());
+    for (size_t i = 0; i < hit->passes.size(); ++i) ops[i] = hit->d_blob ? hit->d_blob + hit->off[i] : nullptr;
+    return exec_passes(st, hit->passes, ops);
   } catch (const std::exception& ex) {
     return fail(QGPU_ERR_OUT_OF_MEMORY, "exception: %s", ex.what());
   }
@@ -957,6 +1262,7 @@ qgpu_status qgpu_get_amplitudes_device(qgpu_state* st, uint64_t start, uint64_t 
       if (st->map.pos[q] < 0) a.unassigned |= 1ull << q;
     }
     a.L = live(st, st->map.kl);
+    if (st->host) a.L = std::min(a.L, st->hlive[size_t(sh.rank)]);  // zero-copy read of the slice
     CK(launch_gather(st->stream, a));
     st->stats.kernels_launched++;
   }
@@ -1025,6 +1331,7 @@ qgpu_status qgpu_probabilities(qgpu_state* st, int mq, const int* qubits, double
     }
     const bool active = st->g == 0 || (uint64_t(sh.rank) >> st->map.kg) == 0;
     pa.L = active ? live(st, st->map.kl) : 0;
+    if (st->host) pa.L = std::min(pa.L, st->hlive[i]);  // zero-copy read of the slice
     pa.out = i == 0 ? acc : tmp;
     CK(launch_probs(st->stream, pa, part));
     st->stats.kernels_launched += 1;

@@ -45,7 +45,7 @@ class Config(ctypes.Structure):
         ("rank", ctypes.c_int), ("world_size", ctypes.c_int), ("nccl_unique_id", ctypes.c_void_p),
         ("chunk_bits", ctypes.c_int), ("prune", ctypes.c_int), ("reorder", ctypes.c_int),
         ("fuse_bits", ctypes.c_int), ("timing", ctypes.c_int), ("swap_slab_bytes", ctypes.c_uint64),
-        ("jit", ctypes.c_int),
+        ("jit", ctypes.c_int), ("host_slice_bits", ctypes.c_int),
     ]
 
 
@@ -57,7 +57,10 @@ class Stats(ctypes.Structure):
         ("tile_kernel_ms", ctypes.c_double), ("tile_kernel_launches", ctypes.c_uint64),
         ("tile_algo_bytes", ctypes.c_uint64), ("swap_ms", ctypes.c_double),
         ("h2d_bytes", ctypes.c_uint64), ("d2h_bytes", ctypes.c_uint64),
-        ("jit_launches", ctypes.c_uint64), ("jit_compiles", ctypes.c_uint64), ("jit_ms", ctypes.c_double)]
+        ("jit_launches", ctypes.c_uint64), ("jit_compiles", ctypes.c_uint64), ("jit_ms", ctypes.c_double),
+        ("host_h2d_bytes", ctypes.c_uint64), ("host_d2h_bytes", ctypes.c_uint64),
+        ("host_slice_loads", ctypes.c_uint64), ("host_slice_skips", ctypes.c_uint64),
+        ("host_runs", ctypes.c_uint64), ("host_ms", ctypes.c_double)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
