@@ -134,6 +134,10 @@ struct qgpu_state {
   cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
   cudaEvent_t ev_loaded[2] = {}, ev_computed[2] = {}, ev_stored[2] = {}, ev_join = nullptr;
   bool group_used[2] = {false, false};
+  std::vector<cudaEvent_t> ev_slice;   // slice r: its last D2H (host copy valid after it)
+  std::vector<uint64_t> slice_seq;     // order of the slices' last D2H (0 = never stored)
+  uint64_t store_seq = 0, unit_seq = 0;
+  int last_unit = 0;                   // slices per slot group in the previous sweep
 };
 
 namespace {
@@ -535,37 +539,49 @@ qgpu_status host_sweep(qgpu_state* st, const std::vector<const Pass*>& run,
   const int unit = 1 << nub;
   int ngroups = 1;
   if (qgpu_status s = ensure_slots(st, unit, &ngroups)) return s;
-  // every earlier use of the slices: work on the state's stream and earlier sweeps' stores
+  // earlier work on the state's stream (reset, readout, the previous sweep's compute); the
+  // previous sweep's stores are waited for per slice and per slot group below, so this sweep's
+  // first loads overlap the previous sweep's last stores
   CK(cudaEventRecord(st->ev_join, st->stream));
   CK(cudaStreamWaitEvent(st->s_h2d, st->ev_join, 0));
-  for (int gi = 0; gi < 2; ++gi)
-    if (st->group_used[gi]) CK(cudaStreamWaitEvent(st->s_h2d, st->ev_stored[gi], 0));
-  const bool timing = st->cfg.timing != 0;
-  TimedLaunch sweep{};
-  if (timing) {
-    sweep.a = get_event(st);
-    sweep.b = get_event(st);
-    sweep.kind = kHostSweep;
-    CK(cudaEventRecord(sweep.a, st->s_h2d));
+  if (unit != st->last_unit) {  // the slot groups are re-cut: drain every earlier store
+    for (int gi = 0; gi < 2; ++gi)
+      if (st->group_used[gi]) CK(cudaStreamWaitEvent(st->s_h2d, st->ev_stored[gi], 0));
+    st->last_unit = unit;
   }
+  const bool timing = st->cfg.timing != 0;
   const uint64_t L_end = run.empty() ? full : live(st, run.back()->k_out);
   std::vector<char> accounted(run.size(), 0);
-  uint64_t moved = 0;
-  int u = 0;
+  auto unit_slice = [&](uint64_t base, int x) {
+    uint64_t r = base;
+    for (int i = 0; i < nub; ++i)
+      if (x >> i & 1) r |= 1ull << ubit[i];
+    return r;
+  };
+  // units in the order their slices were last stored (earliest first): the first loads of this
+  // sweep need only the previous sweep's first stores
+  std::vector<std::pair<uint64_t, uint64_t>> units;  // (latest store among the unit's slices, base)
   for (uint64_t base = 0; base < nact; ++base) {
     if (base & ubits) continue;
-    const int gi = (ngroups == 2) ? (u & 1) : 0;
-    ++u;
+    uint64_t last = 0;
+    for (int x = 0; x < unit; ++x) last = std::max(last, st->slice_seq[unit_slice(base, x)]);
+    units.emplace_back(last, base);
+  }
+  std::stable_sort(units.begin(), units.end(),
+                   [](const auto& a, const auto& b) { return a.first < b.first; });
+  for (const auto& ub : units) {
+    const uint64_t base = ub.second;
+    const int gi = (ngroups == 2) ? int(st->unit_seq & 1) : 0;
+    ++st->unit_seq;
     double2** slot = &st->slots[size_t(gi) * size_t(unit)];
     uint64_t rs[1 << 8];
-    for (int x = 0; x < unit; ++x) {
-      rs[x] = base;
-      for (int i = 0; i < nub; ++i)
-        if (x >> i & 1) rs[x] |= 1ull << ubit[i];
-    }
+    for (int x = 0; x < unit; ++x) rs[x] = unit_slice(base, x);
     const bool swap_here = !sw.empty() && base < (1ull << kg_sw);
-    // load: the live prefix from host memory, zeros up to what the first pass reads
+    // load: the live prefix from host memory, zeros up to what the first pass reads; the slot
+    // group must be drained and each slice's previous store complete
     if (st->group_used[gi]) CK(cudaStreamWaitEvent(st->s_h2d, st->ev_stored[gi], 0));
+    for (int x = 0; x < unit; ++x)
+      if (st->slice_seq[rs[x]]) CK(cudaStreamWaitEvent(st->s_h2d, st->ev_slice[rs[x]], 0));
     for (int x = 0; x < unit; ++x) {
       const uint64_t r = rs[x];
       uint64_t need = 0;
@@ -646,12 +662,12 @@ qgpu_status host_sweep(qgpu_state* st, const std::vector<const Pass*>& run,
       st->hlive[r] = L_end;
       st->stats.host_d2h_bytes += L_end * sizeof(double2);
       st->stats.d2h_bytes += L_end * sizeof(double2);
-      moved += L_end;
+      CK(cudaEventRecord(st->ev_slice[r], st->s_d2h));
+      st->slice_seq[r] = ++st->store_seq;
     }
     CK(cudaEventRecord(st->ev_stored[gi], st->s_d2h));
     st->group_used[gi] = true;
   }
-  (void)moved;
   st->stats.host_slice_skips += (1ull << st->g) - nact;
   for (const HostSwap& x : sw) {
     (void)x;
@@ -659,11 +675,11 @@ qgpu_status host_sweep(qgpu_state* st, const std::vector<const Pass*>& run,
     st->stats.swap_bytes += 16 * (full / 2) * (nact >> 1);
   }
   st->stats.host_runs++;
-  if (timing) {
-    CK(cudaEventRecord(sweep.b, st->s_d2h));
-    st->pending.push_back(sweep);
-  }
-  // later work on the state's stream (readout, the next apply) sees the stored slices
+  return QGPU_OK;
+}
+
+// Later work on the state's stream (readout, host writes after a sync) sees the stored slices.
+qgpu_status host_join(qgpu_state* st) {
   CK(cudaEventRecord(st->ev_join, st->s_d2h));
   CK(cudaStreamWaitEvent(st->stream, st->ev_join, 0));
   return QGPU_OK;
@@ -682,6 +698,14 @@ qgpu_status exec_passes(qgpu_state* st, const std::vector<Pass>& passes,
   std::vector<const unsigned char*> run_ops;
   std::vector<HostSwap> sw;
   int kg_sw = 0;
+  // timing=1: one interval from the first load to the last store (sweeps overlap)
+  TimedLaunch span{};
+  if (st->cfg.timing) {
+    span.a = get_event(st);
+    span.b = get_event(st);
+    span.kind = kHostSweep;
+    CK(cudaEventRecord(span.a, st->stream));
+  }
   auto flush = [&]() -> qgpu_status {
     if (run.empty() && sw.empty()) return QGPU_OK;
     qgpu_status s = host_sweep(st, run, run_ops, sw, kg_sw);
@@ -708,7 +732,13 @@ qgpu_status exec_passes(qgpu_state* st, const std::vector<Pass>& passes,
     run.push_back(&p);
     run_ops.push_back(ops[i]);
   }
-  return flush();
+  if (qgpu_status s = flush()) return s;
+  if (qgpu_status s = host_join(st)) return s;
+  if (st->cfg.timing) {
+    CK(cudaEventRecord(span.b, st->stream));
+    st->pending.push_back(span);
+  }
+  return QGPU_OK;
 }
 
 qgpu_status ensure_ops(qgpu_state* st, size_t n) {
@@ -1029,6 +1059,10 @@ qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out
         if (e == cudaSuccess) e = cudaEventCreateWithFlags(&st->ev_stored[i], cudaEventDisableTiming);
       }
       if (e == cudaSuccess) e = cudaEventCreateWithFlags(&st->ev_join, cudaEventDisableTiming);
+      st->ev_slice.assign(size_t(nshard), nullptr);
+      st->slice_seq.assign(size_t(nshard), 0);
+      for (int r = 0; r < nshard && e == cudaSuccess; ++r)
+        e = cudaEventCreateWithFlags(&st->ev_slice[size_t(r)], cudaEventDisableTiming);
       if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaEventCreate: %s", cudaGetErrorString(e)));
     }
     for (int r = 0; r < nshard && !st->host; ++r) {
@@ -1089,6 +1123,8 @@ qgpu_status qgpu_state_destroy(qgpu_state* st) {
     for (cudaEvent_t e : {st->ev_loaded[i], st->ev_computed[i], st->ev_stored[i]})
       if (e) cudaEventDestroy(e);
   if (st->ev_join) cudaEventDestroy(st->ev_join);
+  for (cudaEvent_t e : st->ev_slice)
+    if (e) cudaEventDestroy(e);
   if (st->s_h2d) cudaStreamDestroy(st->s_h2d);
   if (st->s_d2h) cudaStreamDestroy(st->s_d2h);
   for (Shard& sh : st->shards)
