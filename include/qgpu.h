@@ -85,6 +85,14 @@ typedef struct {
                                  streams, double-buffered). Pruning skips never-active slices
                                  and moves only each slice's live prefix across the link.
                                  Device memory: 4-8 slots of 16 * 2^(n-h) bytes              */
+  int involve_rule;           /* which qubits a gate involves:
+                                 0 (default) = the paper's rule, every operand (P:229 l.11);
+                                 1 = refined: a gate with a control on a never-involved qubit
+                                 is the identity on the current state and is skipped; a
+                                 diagonal gate on a never-involved target is restricted to that
+                                 bit = 0 (a global phase becomes a scalar on the live part);
+                                 neither involves anything. Exact. Also changes the
+                                 Alg.2/3 costs (new qubits a gate would involve)            */
 } qgpu_config;
 
 typedef struct {
@@ -196,7 +204,9 @@ qgpu_status qgpu_circuit_info(const qgpu_circuit* c, int* n_qubits, uint64_t* n_
 qgpu_status qgpu_circuit_destroy(qgpu_circuit* c);
 
 /* Host-only (no GPU needed): the execution order chosen by `mode` (0 program, 1 greedy
- * Alg.2, 2 forward-looking Alg.3) as gate indices into order[cap]. *n = number of gates. */
+ * Alg.2, 2 forward-looking Alg.3; + 4 = costs under the refined involvement rule, see
+ * qgpu_config.involve_rule) as gate indices into order[cap]. *n = number of gates. The
+ * `reorder` argument of the plan / plan_text / jit_check diagnostics takes the same +4 flag. */
 qgpu_status qgpu_circuit_reorder(const qgpu_circuit* c, int mode, uint64_t* order, uint64_t cap,
                                  uint64_t* n);
 

@@ -12,13 +12,20 @@ Written step by step in the paper's order and notation (§IV-B, §IV-C)
   (the paper breaks ties at random) and the +inf initialisation of Q3.
 * Table II statistic: number of operations strictly before all qubits are involved (Q17).
 
-"Involve" uses the paper's rule (reading Q7): every operand qubit, targets and controls,
-of every gate, diagonal or not (P:223, P:229 l.11).
+"Involve" uses the paper's rule (reading Q7) by default: every operand qubit, targets and
+controls, of every gate, diagonal or not (P:223, P:229 l.11). ``rule=1`` is the refined rule of
+SURVEY §8f NEXT-1, read off P:221 ("if a qubit is not involved ... the amplitudes with that bit
+set are zero"): on such a state a gate with a control on an uninvolved qubit is the identity,
+and a diagonal gate maps every zero amplitude to zero, so neither involves anything; every other
+gate involves all its operands. Alg.2/3 then count the new qubits a gate would involve under
+the same rule.
 """
 from __future__ import annotations
 
 import math
 from typing import List, Optional, Sequence, Set, Tuple
+
+import numpy as np
 
 
 def gate_qubits(g) -> Tuple[int, ...]:
@@ -63,6 +70,26 @@ def alg1_chunks(involvement: int, n: int) -> Tuple[int, List[int]]:
     return chunk_size, processed
 
 
+def is_diagonal(U) -> bool:
+    """Every off-diagonal entry exactly zero."""
+    U = np.asarray(U)
+    return bool(np.all(U[~np.eye(U.shape[0], dtype=bool)] == 0))
+
+
+def involved_by(g, involvement: int, rule: int = 0) -> Tuple[int, ...]:
+    """The qubits gate g involves when executed after ``involvement`` (bit mask).
+    rule 0: all operands (Q7). rule 1 (NEXT-1): none if a control is uninvolved or g is
+    diagonal, else all operands."""
+    qs = gate_qubits(g)
+    if rule == 0:
+        return qs
+    if any(not (involvement >> c) & 1 for c in g.controls):
+        return ()
+    if is_diagonal(g.U):
+        return ()
+    return qs
+
+
 def update_involvement(involvement: int, qubits: Sequence[int]) -> int:
     """Algorithm 1 line 11: set the bits of the qubits this operation involves."""
     for q in qubits:
@@ -86,22 +113,23 @@ def bitmap_words(bits: Sequence[int]) -> List[int]:
     return words
 
 
-def involvement_trace(gates: Sequence, order: Optional[Sequence[int]] = None) -> List[int]:
+def involvement_trace(gates: Sequence, order: Optional[Sequence[int]] = None,
+                      rule: int = 0) -> List[int]:
     """involvement after each executed operation (P:229 l.11)."""
     order = range(len(gates)) if order is None else order
     inv, out = 0, []
     for i in order:
-        inv = update_involvement(inv, gate_qubits(gates[i]))
+        inv = update_involvement(inv, involved_by(gates[i], inv, rule))
         out.append(inv)
     return out
 
 
 def ops_before_full_involvement(gates: Sequence, n: int,
-                                order: Optional[Sequence[int]] = None) -> int:
+                                order: Optional[Sequence[int]] = None, rule: int = 0) -> int:
     """Table II, reading Q17: number of operations strictly before the first op
     after which all n qubits are involved (len(order) if never)."""
     full = (1 << n) - 1
-    for k, inv in enumerate(involvement_trace(gates, order)):
+    for k, inv in enumerate(involvement_trace(gates, order, rule)):
         if inv == full:
             return k
     return len(gates) if order is None else len(order)
@@ -139,7 +167,14 @@ def _new_qubits(qs: Sequence[int], involved: Set[int]) -> int:
     return sum(1 for q in set(qs) if q not in involved)
 
 
-def reorder_greedy(gates: Sequence, forced: Sequence[int] = ()) -> List[int]:
+def _involves(gates: Sequence, g: int, involved: Set[int], rule: int) -> Tuple[int, ...]:
+    """Operands gate g would involve given the involved set (rule 0: all of them)."""
+    if rule == 0:
+        return tuple(gate_qubits(gates[g]))
+    return involved_by(gates[g], qubit_mask(involved), rule)
+
+
+def reorder_greedy(gates: Sequence, forced: Sequence[int] = (), rule: int = 0) -> List[int]:
     """Algorithm 2. Cost = number of new qubits the gate involves. Ties: first in
     exeList (reading Q4). ``forced`` pins the first picks (to reproduce the paper's random
     picks g1,g3,g5,g2 in the gs_5 walk-through)."""
@@ -156,12 +191,12 @@ def reorder_greedy(gates: Sequence, forced: Sequence[int] = ()) -> List[int]:
             assert next_gate in exe_list, "forced pick must be ready"
         else:
             for g in exe_list:                               # line 11
-                cost = _new_qubits(dag.qubits[g], involved)  # line 12
+                cost = _new_qubits(_involves(gates, g, involved, rule), involved)  # line 12
                 if cost < min_cost:                          # line 13
                     min_cost, next_gate = cost, g            # lines 14-15
         exe_list.remove(next_gate)                           # line 16
         gates_list.append(next_gate)                         # line 17
-        involved.update(dag.qubits[next_gate])
+        involved.update(_involves(gates, next_gate, involved, rule))
         for g in dag.desc[next_gate]:                        # line 18
             npred[g] -= 1                                    # line 19
             if npred[g] == 0:                                # line 20
@@ -170,13 +205,15 @@ def reorder_greedy(gates: Sequence, forced: Sequence[int] = ()) -> List[int]:
 
 
 def forward_cost(g: int, dag: DAG, npred: List[int], exe_list: List[int],
-                 involved: Set[int]) -> Tuple[int, int]:
+                 involved: Set[int], gates: Sequence = (), rule: int = 0) -> Tuple[int, int]:
     """Algorithm 3 on copies of exeList / involvedQubits. Returns
-    (cost, costCurrent)."""
+    (cost, costCurrent). Under rule 1 a gate's qubits are those it would involve."""
+    qubits = (lambda h, inv: dag.qubits[h]) if rule == 0 else \
+        (lambda h, inv: _involves(gates, h, inv, rule))
     involved = set(involved)                      # copies (P:336)
     exe_list = list(exe_list)
     cost_current, cost_look_ahead = 0, math.inf   # line 1 (Q3: look-ahead starts at +inf)
-    for q in dag.qubits[g]:                       # lines 3-6
+    for q in set(qubits(g, involved)):            # lines 3-6
         if q not in involved:
             cost_current += 1
             involved.add(q)
@@ -186,7 +223,7 @@ def forward_cost(g: int, dag: DAG, npred: List[int], exe_list: List[int],
             exe_list.append(d)
     for g2 in exe_list:                           # lines 12-18
         cur = 0
-        for q in dag.qubits[g2]:
+        for q in set(qubits(g2, involved)):
             if q not in involved:
                 cur += 1
         if cur < cost_look_ahead:
@@ -196,7 +233,7 @@ def forward_cost(g: int, dag: DAG, npred: List[int], exe_list: List[int],
     return cost_current + cost_look_ahead, cost_current   # line 19
 
 
-def reorder_forward(gates: Sequence) -> List[int]:
+def reorder_forward(gates: Sequence, rule: int = 0) -> List[int]:
     """Forward-looking reorder: Algorithm 2's traversal with Algorithm 3's cost; the
     minimum of the key (cost, costCurrent, position in exeList) wins (reading Q4)."""
     dag = DAG(gates)
@@ -207,13 +244,13 @@ def reorder_forward(gates: Sequence) -> List[int]:
     while exe_list:
         best, best_key = None, None
         for pos, g in enumerate(exe_list):
-            cost, cur = forward_cost(g, dag, npred, exe_list, involved)
+            cost, cur = forward_cost(g, dag, npred, exe_list, involved, gates, rule)
             key = (cost, cur, pos)
             if best_key is None or key < best_key:
                 best, best_key = g, key
         exe_list.remove(best)
         gates_list.append(best)
-        involved.update(dag.qubits[best])
+        involved.update(_involves(gates, best, involved, rule))
         for d in dag.desc[best]:
             npred[d] -= 1
             if npred[d] == 0:
@@ -221,14 +258,14 @@ def reorder_forward(gates: Sequence) -> List[int]:
     return gates_list
 
 
-def reorder(gates: Sequence, mode: int) -> List[int]:
+def reorder(gates: Sequence, mode: int, rule: int = 0) -> List[int]:
     """mode 0: program order, 1: greedy (Alg.2), 2: forward-looking (Alg.3)."""
     if mode == 0:
         return list(range(len(gates)))
     if mode == 1:
-        return reorder_greedy(gates)
+        return reorder_greedy(gates, rule=rule)
     if mode == 2:
-        return reorder_forward(gates)
+        return reorder_forward(gates, rule)
     raise ValueError(mode)
 
 

@@ -828,7 +828,7 @@ uint64_t plan_key(const qgpu_state* st, const qgpu_circuit* c) {
   auto mix = [&](uint64_t v) {
     h ^= v + 0x9e3779b97f4a7c15ull + (h << 6) + (h >> 2);
   };
-  mix(uint64_t(st->cfg.reorder));
+  mix(uint64_t(st->cfg.reorder) | uint64_t(st->cfg.involve_rule) << 4);
   mix(uint64_t(st->cfg.fuse_bits));
   mix(uint64_t(st->m));
   mix(st->map.involvement);
@@ -891,6 +891,7 @@ PlanOptions plan_options(const qgpu_config& cfg, bool fuse) {
   o.fuse_bits = fuse ? cfg.fuse_bits : 0;
   plan_env(&o);
   o.prune = cfg.prune != 0;
+  o.rule = cfg.involve_rule;
   return o;
 }
 
@@ -1003,6 +1004,7 @@ qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out
     if (cfg.fuse_bits > 0 && cfg.fuse_bits < 7)
       return fail(QGPU_ERR_INVALID_ARG, "fuse_bits must be 0 or >= 7");
     if (cfg.reorder < 0 || cfg.reorder > 2) return fail(QGPU_ERR_INVALID_ARG, "reorder must be 0, 1 or 2");
+    if (cfg.involve_rule < 0 || cfg.involve_rule > 1) return fail(QGPU_ERR_INVALID_ARG, "involve_rule must be 0 or 1");
     cfg.chunk_bits = std::min(std::max(cfg.chunk_bits, 0), n - g);
     if (const char* ev = std::getenv("QGPU_JIT")) cfg.jit = std::atoi(ev);
     if (cfg.jit < 0 || cfg.jit > 2) return fail(QGPU_ERR_INVALID_ARG, "jit must be 0, 1 or 2");
@@ -1241,7 +1243,7 @@ qgpu_status qgpu_apply_circuit(qgpu_state* st, const qgpu_circuit* c) {
     if (!hit) {
       CachedPlan cp;
       cp.key = key;
-      cp.order = reorder(c->c.gates, st->cfg.reorder);
+      cp.order = reorder(c->c.gates, st->cfg.reorder, st->cfg.involve_rule);
       QubitMap map = st->map;
       plan_circuit(c->c.gates, cp.order, map, plan_options(st->cfg, st->cfg.fuse_bits > 0), &cp.passes, &cp.inv);
       cp.map_after = map;
@@ -1424,8 +1426,8 @@ qgpu_status qgpu_circuit_destroy(qgpu_circuit* c) {
 qgpu_status qgpu_circuit_reorder(const qgpu_circuit* c, int mode, uint64_t* order, uint64_t cap, uint64_t* n) {
   try {
     if (!c) return fail(QGPU_ERR_INVALID_ARG, "circuit is NULL");
-    if (mode < 0 || mode > 2) return fail(QGPU_ERR_INVALID_ARG, "mode must be 0, 1 or 2");
-    std::vector<int> o = reorder(c->c.gates, mode);
+    if ((mode & 3) > 2 || (mode & ~7)) return fail(QGPU_ERR_INVALID_ARG, "mode must be 0, 1 or 2 (+4: refined rule)");
+    std::vector<int> o = reorder(c->c.gates, mode & 3, mode >> 2 & 1);
     if (n) *n = o.size();
     if (order)
       for (uint64_t i = 0; i < std::min<uint64_t>(cap, o.size()); ++i) order[i] = uint64_t(o[i]);
@@ -1447,8 +1449,9 @@ qgpu_status qgpu_circuit_plan(const qgpu_circuit* c, int n, int world, int reord
     PlanOptions o;
     o.fuse_bits = fuse_bits;
     plan_env(&o);
+    o.rule = reorder_mode >> 2 & 1;
     std::vector<Pass> passes;
-    plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode), map, o, &passes, nullptr);
+    plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode & 3, o.rule), map, o, &passes, nullptr);
     if (n_passes) *n_passes = passes.size();
     for (uint64_t i = 0; info && i < std::min<uint64_t>(cap, passes.size()); ++i) {
       const Pass& p = passes[i];
@@ -1478,8 +1481,9 @@ qgpu_status qgpu_circuit_plan_text(const qgpu_circuit* c, int n, int world, int 
     PlanOptions o;
     o.fuse_bits = fuse_bits;
     plan_env(&o);
+    o.rule = reorder_mode >> 2 & 1;
     std::vector<Pass> passes;
-    plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode), map, o, &passes, nullptr);
+    plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode & 3, o.rule), map, o, &passes, nullptr);
     std::string t;
     char line[512];
     for (const Pass& p : passes) {
@@ -1527,8 +1531,9 @@ qgpu_status qgpu_circuit_jit_check(const qgpu_circuit* c, int n, int reorder_mod
     PlanOptions o;
     o.fuse_bits = fuse_bits;
     plan_env(&o);
+    o.rule = reorder_mode >> 2 & 1;
     std::vector<Pass> passes;
-    plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode), map, o, &passes, nullptr);
+    plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode & 3, o.rule), map, o, &passes, nullptr);
     std::string cubin, log;
     for (const Pass& p : passes) {
       if (p.kind != PK_TILE) continue;

@@ -59,7 +59,18 @@ bool is_diagonal(const cplx* U, int nt);
 bool is_swap_matrix(const cplx* U, int nt);
 
 // ------------------------------------------------------------------------------ schedule
-std::vector<int> reorder(const std::vector<Gate>& gates, int mode);  // 0, 1 (Alg.2), 2 (Alg.3)
+// Qubits a gate involves when executed with involvement I (logical masks).
+//   rule 0 (the paper, reading Q7): every operand, P:229 l.11;
+//   rule 1 (refined; exact by P:221): a gate with a control outside I acts
+//   as the identity (every amplitude has that bit 0) and a diagonal gate maps the zero
+//   amplitudes to zero, so neither involves anything; other gates involve every operand.
+inline uint64_t involving(const Gate& g, uint64_t I, int rule) {
+  if (rule == 0) return g.qmask();
+  if ((g.cmask & ~I) || g.diag) return 0;
+  return g.qmask();
+}
+// mode 0 program order, 1 greedy (Alg.2), 2 forward-looking (Alg.3); costs use `rule`
+std::vector<int> reorder(const std::vector<Gate>& gates, int mode, int rule = 0);
 
 // Qubit map + involvement (a3). Physical positions 0..m-1 are local index bits, m..n-1 are
 // global (rank) bits when sharded. Positions are handed out in first-touch order, local ones
@@ -145,6 +156,7 @@ struct PlanOptions {
   bool peephole = true; // fuse CX . D . CX into a diagonal (exact)
   int lookahead = 192;  // fusion lookahead window (gates); 0: passes are runs of `order`
   bool prune = true;
+  int rule = 0;         // involvement rule (see involving()); 1 disables the peephole
 };
 
 // Cut `gates` into passes, updating `map` (involvement, placement) exactly as the execution

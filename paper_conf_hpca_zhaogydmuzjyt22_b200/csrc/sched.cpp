@@ -61,7 +61,7 @@ inline int newq(uint64_t q, uint64_t involved) { return std::popcount(q & ~invol
 
 }  // namespace
 
-std::vector<int> reorder(const std::vector<Gate>& gates, int mode) {
+std::vector<int> reorder(const std::vector<Gate>& gates, int mode, int rule) {
   const int G = int(gates.size());
   std::vector<int> out;
   out.reserve(G);
@@ -80,15 +80,16 @@ std::vector<int> reorder(const std::vector<Gate>& gates, int mode) {
     long best_cost = std::numeric_limits<long>::max(), best_cur = best_cost;
     for (int pos = 0; pos < int(exe.size()); ++pos) {
       const int g = exe[pos];
-      const long cur = newq(d.q[g], involved);          // Alg.3 l.3-6 (= Alg.2 cost)
+      const uint64_t ig = involving(gates[g], involved, rule);
+      const long cur = newq(ig, involved);                 // Alg.3 l.3-6 (= Alg.2 cost)
       long cost = cur;
       if (mode == 2) {
-        const uint64_t inv2 = involved | d.q[g];
+        const uint64_t inv2 = involved | ig;
         long la = std::numeric_limits<long>::max();       // Q3: +inf
         for (int h : exe)                                   // Alg.3 l.7, l.12-18
-          if (h != g) la = std::min<long>(la, newq(d.q[h], inv2));
+          if (h != g) la = std::min<long>(la, newq(involving(gates[h], inv2, rule), inv2));
         for (int h : d.desc[g])                             // Alg.3 l.8-10
-          if (d.npred[h] == 1) la = std::min<long>(la, newq(d.q[h], inv2));
+          if (d.npred[h] == 1) la = std::min<long>(la, newq(involving(gates[h], inv2, rule), inv2));
         if (la == std::numeric_limits<long>::max()) la = 0;
         cost = cur + la;                                    // Alg.3 l.19
       }
@@ -102,7 +103,7 @@ std::vector<int> reorder(const std::vector<Gate>& gates, int mode) {
     const int next = exe[best_pos];
     exe.erase(exe.begin() + best_pos);                      // Alg.2 l.16
     out.push_back(next);                                    // Alg.2 l.17
-    involved |= d.q[next];
+    involved |= involving(gates[next], involved, rule);
     for (int h : d.desc[next])                              // Alg.2 l.18-21
       if (--d.npred[h] == 0) exe.push_back(h);
   }
@@ -747,6 +748,52 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
 
 namespace {
 
+// Refined rule (NEXT-1): restrict a diagonal gate (controls all involved) to the entries whose
+// uninvolved target bits are 0. Output: a diagonal gate on the involved targets; a controlled
+// scalar s becomes diag(1, s) on one control; an uncontrolled scalar comes back as nt = 1,
+// t[0] = -1, U = diag(s, s) (the caller places it). false: the restriction is the identity.
+bool restrict_diag(const Gate& g, uint64_t I, Gate* out) {
+  const int dim = 1 << g.nt;
+  int keep[2], nk = 0;
+  for (int j = 0; j < g.nt; ++j)
+    if (I >> g.t[j] & 1) keep[nk++] = j;
+  cplx d[4];
+  for (int w = 0; w < (1 << nk); ++w) {
+    int v = 0;
+    for (int q = 0; q < nk; ++q)
+      if (w >> q & 1) v |= 1 << keep[q];
+    d[w] = g.U[v * (dim + 1)];
+  }
+  bool identity = true;
+  for (int w = 0; w < (1 << nk); ++w) identity = identity && d[w].re == 1.0 && d[w].im == 0.0;
+  if (identity) return false;
+  Gate r;
+  r.diag = true;
+  r.relabel = false;
+  r.line = g.line;
+  for (auto& u : r.U) u = cplx{0, 0};
+  r.cmask = g.cmask;
+  if (nk > 0) {
+    r.nt = nk;
+    for (int q = 0; q < nk; ++q) r.t[q] = g.t[keep[q]];
+    for (int w = 0; w < (1 << nk); ++w) r.U[w * ((1 << nk) + 1)] = d[w];
+  } else if (g.cmask) {
+    const int c0 = std::countr_zero(g.cmask);
+    r.nt = 1;
+    r.t[0] = c0;
+    r.cmask = g.cmask & ~(1ull << c0);
+    r.U[0] = cplx{1, 0};
+    r.U[3] = d[0];
+  } else {
+    r.nt = 1;
+    r.t[0] = -1;
+    r.U[0] = d[0];
+    r.U[3] = d[0];
+  }
+  *out = r;
+  return true;
+}
+
 struct Builder {
   const std::vector<Gate>& gates;
   QubitMap& map;
@@ -813,32 +860,81 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
   std::vector<char> absorbed;
   std::vector<Gate> fgates;
   std::vector<std::array<int, 2>> parts;
-  if (opt.peephole) find_cx_diag_cx(gates, order, &fused, &absorbed, &fgates, &parts);
+  const bool peephole = opt.peephole && opt.rule == 0;
+  if (peephole) find_cx_diag_cx(gates, order, &fused, &absorbed, &fgates, &parts);
   // the paper's involvement trace follows `order` (Alg.1 l.11), whatever the execution order
+  // (the fusion lookahead only moves gates past gates that share none of their qubits, so the
+  // involvement each gate sees is the same)
   if (inv_after) {
     uint64_t inv = map.involvement;
-    for (int k = 0; k < G; ++k) inv_after->push_back(inv |= gates[order[k]].qmask());
+    for (int k = 0; k < G; ++k) inv_after->push_back(inv |= involving(gates[order[k]], inv, opt.rule));
   }
   auto gate_at = [&](int k) -> const Gate& {
-    return (opt.peephole && fused[k] >= 0) ? fgates[fused[k]] : gates[order[k]];
+    return (peephole && fused[k] >= 0) ? fgates[fused[k]] : gates[order[k]];
   };
   int xi = 0;  // execution index: passes are consecutive runs of the execution order
 
   // execute order position k: placement, sharded activation / swaps, then the gate joins the
   // open fused pass or opens a new one
+  Gate restricted;  // refined rule: a diagonal gate restricted to its involved operands
   auto emit = [&](int k) {
     const Gate& g0 = gates[order[k]];
     const int k_before = map.kl;
     const int kg_before = map.kg;
-    const uint64_t fresh = g0.qmask() & ~map.involvement;
-    map.touch(g0.qmask());
-    if (opt.peephole && absorbed[k]) {  // folded into an earlier fused gate
-      if (B.open) B.cur.count++;
-      else if (!passes->empty()) passes->back().count++;
+    const uint64_t inv_g = involving(g0, map.involvement, opt.rule);
+    const uint64_t fresh = inv_g & ~map.involvement;
+    auto skip = [&]() {
+      if (B.open) {
+        B.cur.count++;
+      } else if (!passes->empty()) {
+        passes->back().count++;
+      } else {  // nothing planned yet: an empty relabel pass keeps the runs consecutive
+        B.start(PK_RELABEL, xi, k_before);
+        B.cur.count = 1;
+        B.close();
+      }
+      ++xi;
+    };
+    const Gate* gp = nullptr;
+    bool scalar_at_origin = false;  // global phase while nothing is involved (live size 1)
+    if (opt.rule == 1 && ((g0.cmask & ~map.involvement) ||
+                          (g0.diag && (g0.tmask() & ~map.involvement)))) {
+      // refined rule (NEXT-1): an unsatisfiable control makes the gate the identity; a diagonal
+      // gate on a target that is |0> everywhere reduces to its entries with that bit 0
+      if (g0.cmask & ~map.involvement) return skip();
+      if (!restrict_diag(g0, map.involvement, &restricted)) return skip();  // identity
+      if (restricted.nt == 1 && restricted.t[0] < 0) {  // uncontrolled global phase
+        if (map.involvement) {
+          restricted.t[0] = std::countr_zero(map.involvement);
+        } else {
+          scalar_at_origin = true;
+          restricted.t[0] = 0;
+        }
+      }
+      gp = &restricted;
+    }
+    map.touch(inv_g);
+    if (peephole && absorbed[k]) return skip();  // folded into an earlier fused gate
+    const Gate& g = gp ? *gp : gate_at(k);
+    if (scalar_at_origin) {
+      // nothing involved: the state is psi[0] |0...0>; one diagonal kernel scales psi[0]
+      B.close();
+      B.start(PK_DIAG, xi, k_before);
+      PhysGate pg;
+      pg.gate = order[k];
+      pg.nt = 1;
+      pg.p[0] = 0;
+      pg.pc = 0;
+      std::memcpy(pg.U, g.U, sizeof(g.U));
+      pg.diag = true;
+      B.cur.gates.push_back(pg);
+      B.cur.count = 1;
+      B.cur.k_out = map.kl;
+      B.cur.unfused_bytes = 32;
+      B.close();
       ++xi;
       return;
     }
-    const Gate& g = gate_at(k);
     if (map.kg > kg_before) {
       // sharded: a qubit was placed on a rank bit; the ranks that become active hold zeros
       B.close();
@@ -938,6 +1034,7 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
   auto joins_open_pass = [&](int k) {
     if (!(fuse && B.open && B.cur.kind == PK_TILE)) return false;
     const Gate& g = gate_at(k);
+    // (refined rule: gates on uninvolved qubits are rewritten at emission, never moved)
     if (g.relabel || (g.qmask() & ~map.involvement)) return false;
     uint64_t need = 0;
     if (!g.diag) {
@@ -957,10 +1054,10 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
   std::vector<int> pend;
   pend.reserve(size_t(G));
   for (int k = 0; k < G; ++k)
-    if (!(opt.peephole && absorbed[k])) pend.push_back(k);
+    if (!(peephole && absorbed[k])) pend.push_back(k);
   std::vector<std::array<int, 2>> part_of(size_t(G), {-1, -1});
   for (int k = 0; k < G; ++k)
-    if (opt.peephole && fused[k] >= 0) part_of[size_t(k)] = parts[size_t(fused[k])];
+    if (peephole && fused[k] >= 0) part_of[size_t(k)] = parts[size_t(fused[k])];
   const int W = fuse ? opt.lookahead : 0;
   size_t head = 0;
   std::vector<char> done(size_t(G), 0);

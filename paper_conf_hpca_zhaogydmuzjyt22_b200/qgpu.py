@@ -45,7 +45,7 @@ class Config(ctypes.Structure):
         ("rank", ctypes.c_int), ("world_size", ctypes.c_int), ("nccl_unique_id", ctypes.c_void_p),
         ("chunk_bits", ctypes.c_int), ("prune", ctypes.c_int), ("reorder", ctypes.c_int),
         ("fuse_bits", ctypes.c_int), ("timing", ctypes.c_int), ("swap_slab_bytes", ctypes.c_uint64),
-        ("jit", ctypes.c_int), ("host_slice_bits", ctypes.c_int),
+        ("jit", ctypes.c_int), ("host_slice_bits", ctypes.c_int), ("involve_rule", ctypes.c_int),
     ]
 
 

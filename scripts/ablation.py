@@ -25,6 +25,17 @@ VERSIONS = [("base", dict(prune=0, reorder=0)), ("prune", dict(prune=1, reorder=
             ("greedy", dict(prune=1, reorder=1)), ("forward", dict(prune=1, reorder=2)),
             ("unfused", dict(prune=1, reorder=2, fuse_bits=0))]
 
+# --host-slice-bits h: the paper's own setting (state in host memory) on the host tier
+# (NEXT-2). The paper applies one gate per traversal of the chunks, so its versions are unfused:
+#   base_u    prune=0 reorder=0 fuse_bits=0   every gate streams the whole state (Baseline+Overlap)
+#   prune_u   prune=1 reorder=0 fuse_bits=0   + pruning / delayed involvement (Pruning)
+#   forward_u prune=1 reorder=2 fuse_bits=0   + Alg.3 reorder (Reorder)
+#   forward   prune=1 reorder=2               + B200 fusion: one sweep per run of passes
+HOST_VERSIONS = [("base_u", dict(prune=0, reorder=0, fuse_bits=0)),
+                 ("prune_u", dict(prune=1, reorder=0, fuse_bits=0)),
+                 ("forward_u", dict(prune=1, reorder=2, fuse_bits=0)),
+                 ("forward", dict(prune=1, reorder=2))]
+
 
 def family(name, n):
     from workloads import circuits as wc
@@ -54,7 +65,12 @@ def main():
     ap.add_argument("--reps", type=int, default=3)
     ap.add_argument("--unfused-max-gates", type=int, default=1200)
     ap.add_argument("--out", default=None)
+    ap.add_argument("--host-slice-bits", type=int, default=0)
     args = ap.parse_args()
+    global VERSIONS
+    host = args.host_slice_bits
+    if host:
+        VERSIONS = HOST_VERSIONS
     import torch
     from paper_conf_hpca_zhaogydmuzjyt22_b200 import qgpu as q
     q.load()
@@ -64,11 +80,11 @@ def main():
         c = family(fam, args.n)
         circ = q.Circuit(c.qasm())
         ngates = circ.info()[1]
-        res = {"family": fam, "n": args.n, "gates": ngates}
+        res = {"family": fam, "n": args.n, "gates": ngates, "host_slice_bits": host}
         for vname, cfg in VERSIONS:
-            if vname == "unfused" and ngates > args.unfused_max_gates:
+            if vname.startswith("unfused") and ngates > args.unfused_max_gates:
                 continue
-            st = q.State(args.n, stream=stream.cuda_stream, **cfg)
+            st = q.State(args.n, stream=stream.cuda_stream, host_slice_bits=host, timing=1 if host else 0, **cfg)
             times = []
             for it in range(1 + args.reps):
                 e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
@@ -84,12 +100,22 @@ def main():
             res[vname] = {"ms": statistics.median(times), "passes": s["passes"],
                           "live_frac": s["amps_processed"] / max(s["amps_full"], 1),
                           "ops_before_full_involvement": s["ops_before_full_involvement"]}
+            if host:
+                res[vname].update(sweeps=s["host_runs"], slice_loads=s["host_slice_loads"],
+                                  slice_skips=s["host_slice_skips"],
+                                  link_GB=(s["host_h2d_bytes"] + s["host_d2h_bytes"]) / 1e9)
         rows.append(res)
         print(json.dumps(res), flush=True)
     if args.out:
         with open(args.out, "w") as f:
             for r in rows:
                 f.write(json.dumps(r) + "\n")
+    if host:
+        print(f"\nhost tier 2^{host} slices, n={args.n}: circuit ms (link GB, sweeps)")
+        for r in rows:
+            print(f"{r['family']:8} {r['gates']:6d} " + " ".join(
+                f"{v}={r[v]['ms']:.0f}ms({r[v]['link_GB']:.0f}GB,{r[v]['sweeps']})" for v, _ in VERSIONS if v in r))
+        return
     print(f"\n{'family':8} {'gates':>6} " + " ".join(f"{v:>10}" for v, _ in VERSIONS) +
           "   prune/base forward/prune live%(fwd) TableII(prog->fwd)")
     for r in rows:

@@ -75,6 +75,21 @@ def test_reorder_bit_exact_vs_oracle(q, name, mode):
     assert list(got) == list(ref)
 
 
+@pytest.mark.parametrize("name", sorted(CIRCS) + ["randdiag"])
+@pytest.mark.parametrize("mode", [0, 1, 2])
+def test_reorder_refined_rule_bit_exact_vs_oracle(q, name, mode):
+    """NEXT-1: with the refined involvement rule (mode + 4) the Alg.2/Alg.3 costs count only the
+    qubits a gate would involve; library and oracle schedules stay identical."""
+    c = CIRCS[name]() if name in CIRCS else wc.random_circuit(
+        9, 120, seed=13, names=["cp", "cz", "rz", "cx", "crx", "ccx", "t", "h", "rzz", "cswap", "x"])
+    text = c.qasm()
+    _, gates = oq.parse(text)
+    ref = osch.reorder(gates, mode, rule=1)
+    got = q.Circuit(text).reorder(mode + 4)
+    assert list(got) == list(ref)
+    assert osch.is_topological(gates, list(got))
+
+
 def test_reorder_gs5_walkthrough(q):
     """forward-looking reorder of the gs_5 example gives 1,2,2,3,3,4,4,4,5."""
     text = ('OPENQASM 2.0;\ninclude "qelib1.inc";\nqreg q[5];\nh q[0];\nh q[1];\nh q[2];\nh q[3];\n'
@@ -115,6 +130,29 @@ def test_plan_invariants(q, name, fuse):
                 assert S >> kout == 0
     assert pos == ng
     assert k_prev == n or ng == 0 or k_prev == bin(osch.involvement_trace(oq.parse(c.qasm())[1])[-1]).count("1")
+
+
+@pytest.mark.parametrize("name", ["qft12", "qft9x", "rand10", "hlf3x4", "ghz_qft5"])
+@pytest.mark.parametrize("fuse", [0, 9, 12])
+def test_plan_invariants_refined_rule(q, name, fuse):
+    """NEXT-1 plans (reorder + 4): still consecutive runs covering every gate (skipped gates are
+    counted in the pass they fall in), live sizes never shrink, and the final live size is the
+    refined involvement of the oracle replay."""
+    c = CIRCS[name]()
+    text = c.qasm()
+    qc = q.Circuit(text)
+    n, ng = qc.info()
+    _, gates = oq.parse(text)
+    plan = qc.plan(n, 1, 6, fuse)
+    pos, k_prev = 0, 0
+    for first, count, kind, kin, kout, b, slo, shi in plan:
+        assert first == pos and count >= 1
+        pos += count
+        assert kin == k_prev and kout >= kin
+        k_prev = kout
+    assert pos == ng
+    inv = osch.involvement_trace(gates, osch.reorder(gates, 2, rule=1), rule=1)[-1]
+    assert k_prev == bin(inv).count("1")
 
 
 def test_fused_qft28_is_few_passes(q):

@@ -121,3 +121,75 @@ def test_forward_reorder_delays_involvement_on_qft():
     base = os_.ops_before_full_involvement(gates, n)
     fw = os_.ops_before_full_involvement(gates, n, os_.reorder_forward(gates))
     assert fw > base
+
+
+# ------------------------------------------------------------- refined involvement (NEXT-1)
+
+def _g(name, qubits, params=()):
+    text = 'OPENQASM 2.0;\ninclude "qelib1.inc";\nqreg q[4];\n'
+    p = f"({','.join(str(x) for x in params)})" if params else ""
+    text += f"{name}{p} " + ",".join(f"q[{q}]" for q in qubits) + ";\n"
+    return oq.parse(text)[1][0]
+
+
+def test_refined_rule_hand_cases():
+    """NEXT-1 / P:221: on a state where qubit q is |0> everywhere, a gate controlled by q is the
+    identity and a diagonal gate leaves the zeros zero: neither involves anything."""
+    assert os_.involved_by(_g("cp", [0, 1], [0.3]), 0, 1) == ()        # both uninvolved
+    assert os_.involved_by(_g("cx", [0, 1]), 0, 1) == ()               # control uninvolved
+    assert set(os_.involved_by(_g("cx", [0, 1]), 0b01, 1)) == {0, 1}   # control involved: X moves
+    assert os_.involved_by(_g("rz", [2], [0.7]), 0, 1) == ()           # diagonal: a phase
+    assert os_.involved_by(_g("cz", [0, 1]), 0b11, 1) == ()            # diagonal on involved
+    assert set(os_.involved_by(_g("h", [3]), 0, 1)) == {3}
+    assert set(os_.involved_by(_g("swap", [0, 1]), 0, 1)) == {0, 1}    # non-diagonal: all
+    for g in (_g("cp", [0, 1], [0.3]), _g("cx", [0, 1]), _g("rz", [2], [0.7])):
+        assert set(os_.involved_by(g, 0, 0)) == set(g.qubits)          # the paper's rule Q7
+
+
+def test_refined_rule_qft_on_zero_is_hadamards_only():
+    """QFT|0...0> = H^n up to the final SWAP layer: every CP meets an uninvolved control or
+    target-side |0>, so under rule 1 only the H gates (and SWAPs of involved qubits) involve."""
+    n, gates = oq.parse(wc.qft(8).qasm())
+    trace = os_.involvement_trace(gates, rule=1)
+    inv = 0
+    for g, t in zip(gates, trace):
+        if g.name == "h":
+            inv |= 1 << g.targets[0]
+        assert t == inv
+    assert os_.ops_before_full_involvement(gates, n, rule=1) < len(gates)
+
+
+@pytest.mark.parametrize("fam", ["qft0", "random", "randdiag", "qaoa"])
+def test_refined_rule_pruning_soundness(fam):
+    """P:221 under the refined rule: after every step of a schedule (program order and the
+    refined Alg.2/3 orders), every bitmap-0 chunk is exactly zero in the unpruned state evolved
+    along that schedule. A rule that skipped involving a qubit a gate can make non-zero fails."""
+    c = {"qft0": lambda: wc.qft(8), "random": lambda: wc.random_circuit(8, 60, seed=3),
+         "randdiag": lambda: wc.random_circuit(8, 60, seed=4,
+                                               names=["cp", "cz", "rz", "cx", "crx", "ccx", "t", "h", "rzz", "cswap"]),
+         "qaoa": lambda: wc.qaoa(8, 1, seed=2)}[fam]()
+    n, gates = oq.parse(c.qasm())
+    ref = osv.simulate_gates(n, gates)
+    for mode in (0, 1, 2):
+        order = os_.reorder(gates, mode, rule=1)
+        assert os_.is_topological(gates, order)
+        psi = osv.zero_state(n)
+        inv = 0
+        for i in order:
+            g = gates[i]
+            osv.apply_gate(psi, n, g.U, g.targets, g.controls)
+            inv = os_.update_involvement(inv, os_.involved_by(g, inv, 1))
+            for cb in (0, 2, 4):
+                bm = np.array(os_.chunk_bitmap(inv, n, cb), dtype=bool)
+                z = osv.zero_map(psi, n, cb)
+                assert np.all(z[~bm])
+        assert np.abs(psi - ref).max() < 1e-12
+
+
+def test_refined_rule_delays_involvement_at_least_as_much():
+    """The refined involved set is a subset of the paper's after every step of the same order."""
+    for seed in range(4):
+        n, gates = oq.parse(wc.random_circuit(9, 80, seed=seed).qasm())
+        a = os_.involvement_trace(gates, rule=0)
+        b = os_.involvement_trace(gates, rule=1)
+        assert all((y & ~x) == 0 for x, y in zip(a, b))
