@@ -57,6 +57,13 @@ int bstore_mode() {
   return v;
 }
 
+// QGPU_HOST_SWEEP_PER_PASS=1 (ablation): the host tier streams the slices once per pass, as the
+// paper traverses every chunk once per gate, instead of once per run of passes
+bool host_sweep_per_pass() {
+  const char* ev = std::getenv("QGPU_HOST_SWEEP_PER_PASS");  // read per call: ablations flip it
+  return ev && std::atoi(ev) != 0;
+}
+
 // jit=1: specialise fused passes whose live range is >= 2^jit_min_bits amplitudes
 int jit_min_bits() {
   static const int v = [] {
@@ -731,6 +738,8 @@ qgpu_status exec_passes(qgpu_state* st, const std::vector<Pass>& passes,
     }
     run.push_back(&p);
     run_ops.push_back(ops[i]);
+    if (host_sweep_per_pass())
+      if (qgpu_status s = flush()) return s;
   }
   if (qgpu_status s = flush()) return s;
   if (qgpu_status s = host_join(st)) return s;

@@ -108,7 +108,7 @@ bool load_driver(JitLib& L) {
   return true;
 }
 
-// ---- on-disk cubin cache: <dir>/<fnv1a64(source|options)>.cubin
+// ---- on-disk cubin cache: <dir>/<fnv1a64(source|tile_common.cuh|options)>.cubin
 // dir = $QGPU_JIT_CACHE, else <directory of libqgpu.so>/build/jitcache
 std::string cache_dir() {
   if (const char* ev = std::getenv("QGPU_JIT_CACHE")) return ev;
@@ -130,6 +130,7 @@ std::string cache_key(const std::string& src) {
     }
   };
   mix(src);
+  mix(kTileCommonSrc);  // the included device code: a change to it must not hit stale cubins
   mix("|sm_100a|-std=c++17|-lineinfo|");
   if (const char* ev = std::getenv("QGPU_JIT_OPTS")) mix(ev);
   char buf[32];
@@ -261,6 +262,24 @@ std::string tile_jit_source(const Pass& p) {
   hdr << "  static constexpr unsigned kZM0 = " << zm_start << "u;\n";
   hdr << "  static constexpr uint32_t kZW0 = " << zw_start << "u;\n";
   hdr << "  static constexpr bool kStatic = true;\n";
+  {  // tile positions as runs of consecutive bits (tile index -> base address at compile time)
+    std::vector<int> rp, rl;
+    for (int i = 0; i < p.b;) {
+      int j = i;
+      while (j + 1 < p.b && p.spos[j + 1] == p.spos[j] + 1) ++j;
+      rp.push_back(p.spos[i]);
+      rl.push_back(j - i + 1);
+      i = j + 1;
+    }
+    auto arr = [](const std::vector<int>& v) {
+      std::string t = "{";
+      for (size_t i = 0; i < v.size(); ++i) t += (i ? ", " : "") + std::to_string(v[i]);
+      return t + "}";
+    };
+    hdr << "  static constexpr int kNsrun = " << rp.size() << ";\n";
+    hdr << "  static constexpr int kSrunPos[" << rp.size() << "] = " << arr(rp) << ";\n";
+    hdr << "  static constexpr int kSrunLen[" << rl.size() << "] = " << arr(rl) << ";\n";
+  }
   hdr << "  static constexpr bool kHasScalar = " << (P.scalar.empty() ? "false" : "true") << ";\n";
   hdr << "  static constexpr uint32_t kJ0[kRegAmps] = " << jtab(R) << ";\n";
   hdr << "  static constexpr uint64_t kP0[kRegAmps] = " << ptab(R) << ";\n";

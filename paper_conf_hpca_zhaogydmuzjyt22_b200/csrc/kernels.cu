@@ -170,6 +170,9 @@ struct InterpBody {
   static constexpr unsigned kZM0 = 0u;
   static constexpr uint32_t kZW0 = 0u;
   static constexpr bool kStatic = false;  // mappings read from the program at run time
+  static constexpr int kNsrun = -1;       // tile positions read from the arguments
+  static constexpr int kSrunPos[1] = {0};
+  static constexpr int kSrunLen[1] = {0};
   static constexpr bool kHasScalar = true;
   static constexpr bool kGroupRemap = false;  // remaps use CTA barriers
   __device__ static void init_mbar(uint64_t*) {}

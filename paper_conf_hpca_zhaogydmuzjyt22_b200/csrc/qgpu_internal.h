@@ -156,7 +156,7 @@ struct PlanOptions {
   bool peephole = true; // fuse CX . D . CX into a diagonal (exact)
   int lookahead = 192;  // fusion lookahead window (gates); 0: passes are runs of `order`
   bool prune = true;
-  int rule = 0;         // involvement rule (see involving()); 1 disables the peephole
+  int rule = 0;         // involvement rule (see involving())
 };
 
 // Cut `gates` into passes, updating `map` (involvement, placement) exactly as the execution

@@ -308,8 +308,12 @@ bool is_cx_gate(const Gate& g) {
 
 // fused[k] >= 0: order position k is the head of a fused triple (index into `out`);
 // absorbed[k]: position k was folded into an earlier head.
+// inv_before (refined rule only): involvement before each order position; a triple is fused only
+// if both of its qubits are already involved, where the fused diagonal and the three gates
+// involve the same (nothing new)
 void find_cx_diag_cx(const std::vector<Gate>& gates, const std::vector<int>& order, std::vector<int>* fused,
-                     std::vector<char>* absorbed, std::vector<Gate>* out, std::vector<std::array<int, 2>>* parts) {
+                     std::vector<char>* absorbed, std::vector<Gate>* out, std::vector<std::array<int, 2>>* parts,
+                     const std::vector<uint64_t>* inv_before = nullptr) {
   const size_t G = order.size();
   fused->assign(G, -1);
   absorbed->assign(G, 0);
@@ -319,6 +323,7 @@ void find_cx_diag_cx(const std::vector<Gate>& gates, const std::vector<int>& ord
     if (!is_cx_gate(c1)) continue;
     const int a = std::countr_zero(c1.cmask), b = c1.t[0];
     const uint64_t ab = (1ull << a) | (1ull << b);
+    if (inv_before && ((*inv_before)[i] & ab) != ab) continue;
     size_t j = i + 1;
     while (j < G && (gates[order[j]].qmask() & ab) == 0) ++j;
     if (j >= G || (*absorbed)[j]) continue;
@@ -860,8 +865,18 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
   std::vector<char> absorbed;
   std::vector<Gate> fgates;
   std::vector<std::array<int, 2>> parts;
-  const bool peephole = opt.peephole && opt.rule == 0;
-  if (peephole) find_cx_diag_cx(gates, order, &fused, &absorbed, &fgates, &parts);
+  const bool peephole = opt.peephole;
+  if (peephole) {
+    std::vector<uint64_t> before;
+    if (opt.rule == 1) {  // refined rule: only triples on already involved qubits (see above)
+      uint64_t inv = map.involvement;
+      for (int k = 0; k < G; ++k) {
+        before.push_back(inv);
+        inv |= involving(gates[order[k]], inv, 1);
+      }
+    }
+    find_cx_diag_cx(gates, order, &fused, &absorbed, &fgates, &parts, opt.rule == 1 ? &before : nullptr);
+  }
   // the paper's involvement trace follows `order` (Alg.1 l.11), whatever the execution order
   // (the fusion lookahead only moves gates past gates that share none of their qubits, so the
   // involvement each gate sees is the same)

@@ -123,6 +123,21 @@ __device__ __forceinline__ uint64_t tile_base(uint64_t t, const TileArgs& a) {
   return t;
 }
 
+// same with the runs fixed at compile time (NVRTC-specialised passes: Body::kNsrun >= 0)
+template <class Body>
+__device__ __forceinline__ uint64_t tile_base_t(uint64_t t, const TileArgs& a) {
+  if constexpr (Body::kNsrun >= 0) {
+#pragma unroll
+    for (int i = 0; i < Body::kNsrun; ++i) {
+      const int p = Body::kSrunPos[i];
+      t = ((t >> p) << (p + Body::kSrunLen[i])) | (t & ((1ull << p) - 1));
+    }
+    return t;
+  } else {
+    return tile_base(t, a);
+  }
+}
+
 __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src_bytes) {
   const unsigned sa = static_cast<unsigned>(__cvta_generic_to_shared(smem));
   asm volatile("cp.async.cg.shared.global [%0], [%1], 16, %2;\n" ::"r"(sa), "l"(gmem), "r"(src_bytes)
@@ -737,19 +752,21 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     return rem0 + blockIdx.x + (it - nfull) * G;
   };
   uint64_t tile = tile_at(0);
-  if (tile < a.ntiles) issue_own_loads<NR, Body>(bufs, a, mp0, sa0, tile_base(tile, a), zm0, c.own);
+  uint64_t base_next = tile_base_t<Body>(tile, a);  // base of `tile`, carried across iterations
+  if (tile < a.ntiles) issue_own_loads<NR, Body>(bufs, a, mp0, sa0, base_next, zm0, c.own);
   int k = 0;
   uint64_t cur_hi = ~0ull;
   for (uint64_t it = 0; tile < a.ntiles; ++it) {
     double2* s = bufs + k * T;
     const int kn = (k + 1 == nbuf) ? 0 : k + 1;
-    const uint64_t base = tile_base(tile, a);
+    const uint64_t base = base_next;
     const uint64_t gbase = a.rank_base | base;
     const uint64_t next = tile_at(it + 1);
     const bool more = next < a.ntiles;
+    base_next = tile_base_t<Body>(next, a);
     // nbuf >= 2: prefetch into the next buffer now; nbuf == 1 (programs without remaps, every
     // thread reads only its own slots): prefetch into the same buffer right after the reload
-    if (more && nbuf > 1) issue_own_loads<NR, Body>(bufs + kn * T, a, mp0, sa0, tile_base(next, a), zm0, c.own);
+    if (more && nbuf > 1) issue_own_loads<NR, Body>(bufs + kn * T, a, mp0, sa0, base_next, zm0, c.own);
     if (base >= a.L_in) {
       // the whole tile lies in the zero region of a first-touch expansion and no op of the pass
       // targets its non-tile bits: it stays zero -> store zeros, skip the program
@@ -769,7 +786,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       }
       if (more && nbuf == 1) {
         cp_async_wait_all();
-        issue_own_loads<NR, Body>(s, a, mp0, sa0, tile_base(next, a), zm0, c.own);
+        issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
       }
       k = kn;
       tile = next;
@@ -819,7 +836,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       else j = mp0.j(r);
       v[r] = (c.own && !((zm0 >> r) & 1)) ? s[j] : make_double2(0.0, 0.0);
     }
-    if (more && nbuf == 1) issue_own_loads<NR, Body>(s, a, mp0, sa0, tile_base(next, a), zm0, c.own);
+    if (more && nbuf == 1) issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
     c.mpar = nexec & 1u;
     ++nexec;
     body(v, mp, c);

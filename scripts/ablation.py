@@ -24,6 +24,7 @@ sys.path.insert(0, os.path.dirname(os.path.dirname(os.path.abspath(__file__))))
 VERSIONS = [("base", dict(prune=0, reorder=0)), ("prune", dict(prune=1, reorder=0)),
             ("greedy", dict(prune=1, reorder=1)), ("forward", dict(prune=1, reorder=2)),
             ("unfused", dict(prune=1, reorder=2, fuse_bits=0))]
+REFINED = ("refined", dict(prune=1, reorder=2, involve_rule=1))  # NEXT-1 (--refined)
 
 # --host-slice-bits h: the paper's own setting (state in host memory) on the host tier
 # (NEXT-2). The paper applies one gate per traversal of the chunks, so its versions are unfused:
@@ -31,10 +32,15 @@ VERSIONS = [("base", dict(prune=0, reorder=0)), ("prune", dict(prune=1, reorder=
 #   prune_u   prune=1 reorder=0 fuse_bits=0   + pruning / delayed involvement (Pruning)
 #   forward_u prune=1 reorder=2 fuse_bits=0   + Alg.3 reorder (Reorder)
 #   forward   prune=1 reorder=2               + B200 fusion: one sweep per run of passes
-HOST_VERSIONS = [("base_u", dict(prune=0, reorder=0, fuse_bits=0)),
+# paper_*: one sweep of the slices per gate (QGPU_HOST_SWEEP_PER_PASS=1), the paper's traversal
+HOST_VERSIONS = [("paper_base", dict(prune=0, reorder=0, fuse_bits=0, per_pass=1)),
+                 ("paper_prune", dict(prune=1, reorder=0, fuse_bits=0, per_pass=1)),
+                 ("paper_reorder", dict(prune=1, reorder=2, fuse_bits=0, per_pass=1)),
+                 ("base_u", dict(prune=0, reorder=0, fuse_bits=0)),
                  ("prune_u", dict(prune=1, reorder=0, fuse_bits=0)),
                  ("forward_u", dict(prune=1, reorder=2, fuse_bits=0)),
-                 ("forward", dict(prune=1, reorder=2))]
+                 ("forward", dict(prune=1, reorder=2)),
+                 ("refined", dict(prune=1, reorder=2, involve_rule=1))]
 
 
 def family(name, n):
@@ -66,11 +72,16 @@ def main():
     ap.add_argument("--unfused-max-gates", type=int, default=1200)
     ap.add_argument("--out", default=None)
     ap.add_argument("--host-slice-bits", type=int, default=0)
+    ap.add_argument("--paper-max-gates", type=int, default=500,
+                    help="host tier: skip the one-sweep-per-gate versions above this many gates")
+    ap.add_argument("--refined", action="store_true", help="also the refined involvement rule (NEXT-1)")
     args = ap.parse_args()
     global VERSIONS
     host = args.host_slice_bits
     if host:
         VERSIONS = HOST_VERSIONS
+    elif args.refined:
+        VERSIONS = VERSIONS + [REFINED]
     import torch
     from paper_conf_hpca_zhaogydmuzjyt22_b200 import qgpu as q
     q.load()
@@ -83,6 +94,10 @@ def main():
         res = {"family": fam, "n": args.n, "gates": ngates, "host_slice_bits": host}
         for vname, cfg in VERSIONS:
             if vname.startswith("unfused") and ngates > args.unfused_max_gates:
+                continue
+            cfg = dict(cfg)
+            os.environ["QGPU_HOST_SWEEP_PER_PASS"] = str(cfg.pop("per_pass", 0))
+            if cfg.get("per_pass_skip") or (host and "paper" in vname and ngates > args.paper_max_gates):
                 continue
             st = q.State(args.n, stream=stream.cuda_stream, host_slice_bits=host, timing=1 if host else 0, **cfg)
             times = []
