@@ -304,6 +304,8 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     }
     a.ntiles = 1ull << (kout - p.b);
     a.L_in = L_in;
+    a.zin = st->cfg.prune ? p.zin : 0;
+    a.zout = st->cfg.prune ? p.zout : 0;
     a.rank_base = rank << m;
     a.zero = st->d_zero;
     a.remaps = 0;
@@ -331,7 +333,12 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     if (e == cudaErrorNotSupported) e = launch_tile(st->stream, a);
     CK(e);
     st->stats.kernels_launched++;
-    bytes = 16 * (L_in + L_out);
+    // live input / output amplitudes: a skipped zero position halves the part that moves
+    bytes = 16 * ((L_in >> std::popcount(a.zin & (L_in - 1))) + (L_out >> std::popcount(a.zout & (L_out - 1))));
+  } else if (p.kind == PK_ZERO) {
+    CK(launch_zero_where(st->stream, psi, L_out, p.zmask));
+    st->stats.kernels_launched++;
+    bytes = 16 * (L_out - (L_out >> std::popcount(p.zmask & (L_out - 1))));
   } else {
     const PhysGate& g = p.gates[0];
     const uint64_t gpc = g.pc & ~lmask;                  // controls on rank bits
@@ -846,6 +853,7 @@ uint64_t plan_key(const qgpu_state* st, const qgpu_circuit* c) {
   if (const char* ev = std::getenv("QGPU_REGBITS")) mix(uint64_t(std::atoi(ev)) << 32);
   if (const char* ev = std::getenv("QGPU_MAX_UOPS")) mix(uint64_t(std::atoi(ev)) << 40);
   if (const char* ev = std::getenv("QGPU_LOOKAHEAD")) mix(uint64_t(std::atoi(ev)) << 48);
+  if (const char* ev = std::getenv("QGPU_ZSKIP")) mix(uint64_t(std::atoi(ev) + 1) << 56);
   return h;
 }
 
@@ -890,6 +898,7 @@ void prepare_jit(qgpu_state* st, const std::vector<Pass>& passes) {
 
 // experiment overrides of the planner defaults (also part of the plan-cache key)
 void plan_env(PlanOptions* o) {
+  if (const char* ev = std::getenv("QGPU_ZSKIP")) o->zskip = std::atoi(ev) != 0;
   if (const char* ev = std::getenv("QGPU_REGBITS")) o->reg_bits = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_MAX_UOPS")) o->max_u_ops = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_LOOKAHEAD")) o->lookahead = std::atoi(ev);

@@ -218,7 +218,7 @@ std::string tile_jit_source(const Pass& p) {
   // is >= k_in hold zeros until a non-diagonal op targets them
   uint32_t zpos = 0;
   for (int i = 0; i < p.b; ++i)
-    if (p.spos[i] >= p.k_in) zpos |= 1u << i;
+    if (p.spos[i] >= p.k_in || (p.zin >> p.spos[i] & 1)) zpos |= 1u << i;
   int R[4] = {0, 0, 0, 0};
   auto decode = [&](const TileOp& op) {
     for (int k = 0; k < 4; ++k) R[k] = (op.a0 >> (4 * k)) & 15;

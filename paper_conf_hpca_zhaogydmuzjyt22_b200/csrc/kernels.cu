@@ -668,6 +668,18 @@ cudaError_t launch_add(cudaStream_t st, double* out, const double* in, uint64_t 
   return cudaGetLastError();
 }
 
+// zero-position skipping: materialise the zero halves, psi[i] = 0 for i < L with (i & mask) != 0
+__global__ void zero_where_kernel(double2* psi, uint64_t L, uint64_t mask) {
+  const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+  for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < L; i += stride)
+    if (i & mask) __stcs(psi + i, make_double2(0.0, 0.0));
+}
+cudaError_t launch_zero_where(cudaStream_t st, double2* psi, uint64_t L, uint64_t mask) {
+  if (!L || !mask) return cudaSuccess;
+  zero_where_kernel<<<grid_for(L, 256 * 4, 8), 256, 0, st>>>(psi, L, mask);
+  return cudaGetLastError();
+}
+
 cudaError_t launch_set_amp(cudaStream_t st, double2* psi, uint64_t i, double re, double im) {
   set_amp_kernel<<<1, 1, 0, st>>>(psi, i, make_double2(re, im));
   return cudaGetLastError();

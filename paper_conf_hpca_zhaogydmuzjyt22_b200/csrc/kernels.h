@@ -73,6 +73,7 @@ cudaError_t launch_tile(cudaStream_t st, const TileArgs& a);
 cudaError_t launch_gather(cudaStream_t st, const GatherArgs& a);
 cudaError_t launch_probs(cudaStream_t st, ProbArgs a, double* scratch);
 cudaError_t launch_set_amp(cudaStream_t st, double2* psi, uint64_t i, double re, double im);
+cudaError_t launch_zero_where(cudaStream_t st, double2* psi, uint64_t L, uint64_t mask);
 // sharded swaps (a10)
 cudaError_t launch_swap_halves(cudaStream_t st, double2* a, double2* b, int lp, uint64_t half);
 cudaError_t launch_pack_half(cudaStream_t st, const double2* psi, double2* buf, int lp, int bit, uint64_t t0,

@@ -125,7 +125,8 @@ struct PhysGate {
 
 enum PassKind : int {
   PK_TILE = 0, PK_PAIR = 1, PK_QUAD = 2, PK_DIAG = 3, PK_RELABEL = 4, PK_SWAP = 5,
-  PK_ACTIVATE = 6  // ranks [2^kg_from, 2^kg) become active (their buffers are zeroed)
+  PK_ACTIVATE = 6,  // ranks [2^kg_from, 2^kg) become active (their buffers are zeroed)
+  PK_ZERO = 7       // write zeros over the live amplitudes that have a bit of `zmask` set
 };
 
 struct Pass {
@@ -145,6 +146,10 @@ struct Pass {
   int kg_from = 0;              // activation pass
   mutable void* jit_fn = nullptr;  // specialised kernel, resolved at the first launch
   uint64_t unfused_bytes = 0;   // bytes the pass's gates would move one gate per pass
+  // zero-position skipping (tile passes): physical positions p whose bit-p = 1 half of the live
+  // state is exactly zero and NOT materialised in memory -- on input (zin: loads read zeros
+  // instead) and on output (zout: those amplitudes are not stored); PK_ZERO materialises zmask
+  uint64_t zin = 0, zout = 0, zmask = 0;
 };
 
 struct PlanOptions {
@@ -157,6 +162,9 @@ struct PlanOptions {
   int lookahead = 192;  // fusion lookahead window (gates); 0: passes are runs of `order`
   bool prune = true;
   int rule = 0;         // involvement rule (see involving())
+  // skip the halves of positions that a first touch left zero (placed by a diagonal gate or as
+  // a control) until a non-diagonal op targets them; single resident state, fused passes only
+  bool zskip = true;
 };
 
 // Cut `gates` into passes, updating `map` (involvement, placement) exactly as the execution

@@ -743,10 +743,10 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
     for (const RunEntry& e : P.entries) groups += e.gend;
     std::fprintf(stderr,
                  "tile pass k %d->%d b=%d nr=%d nw=%d gates=%zu ops=%zu remap=%d u1r=%d u1l=%d u2r=%d smem=%d "
-                 "runs=%d entries=%zu groups=%d patterns=%zu terms=%zu scalar=%zu lb=%d S=",
+                 "runs=%d entries=%zu groups=%d patterns=%zu terms=%zu scalar=%zu lb=%d zin=%llx zout=%llx S=",
                  p.k_in, p.k_out, p.b, nr, nw, p.gates.size(), P.ops.size(), cnt[0], cnt[1], cnt[2], cnt[3],
                  cnt[4] + cnt[5], cnt[6], P.entries.size(), groups, P.patterns.size(), P.terms.size(),
-                 P.scalar.size(), P.lb);
+                 P.scalar.size(), P.lb, (unsigned long long)p.zin, (unsigned long long)p.zout);
     for (int i = 0; i < p.b; ++i) std::fprintf(stderr, "%d%s", p.spos[i], i + 1 < p.b ? "," : "\n");
   }
 }
@@ -808,6 +808,7 @@ struct Builder {
   Pass cur;
   uint64_t used = 0;   // physical positions that must be tile bits (non-diagonal targets)
   int n_u = 0;
+  uint64_t zpos = 0;   // zero-position skipping: positions whose 1-half is zero, not in memory
 
   void close() {
     if (!open) return;
@@ -817,6 +818,9 @@ struct Builder {
       const int b = std::min(opt.fuse_bits, kt);
       uint64_t S = used;
       for (int pos = 0; pos < kt && std::popcount(S) < b; ++pos) S |= 1ull << pos;
+      // tile bits are stored in full (a diagonal-only one as computed zeros): they leave zpos
+      p.zout = zpos & ~S;
+      zpos = p.zout;
       p.b = std::popcount(S);
       int i = 0;
       for (uint64_t r = S; r; r &= r - 1) p.spos[i++] = std::countr_zero(r);
@@ -838,9 +842,23 @@ struct Builder {
     cur.k_in = k_in;
     cur.k_out = k_in;
     cur.kg = map.kg;
+    cur.zin = kind == PK_TILE ? zpos : 0;
     open = true;
     used = 0;
     n_u = 0;
+  }
+
+  // materialise the skipped halves (before a pass that is not a tile pass, and at the end)
+  void materialise(int first) {
+    if (!zpos) return;
+    close();
+    start(PK_ZERO, first, map.kl);
+    cur.zmask = zpos;
+    cur.count = 0;
+    zpos = 0;
+    out->push_back(std::move(cur));
+    cur = Pass();
+    open = false;
   }
 
   bool fits(uint64_t need, int n_ops_new) const {
@@ -860,6 +878,7 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
   Builder B{gates, map, opt, passes};
   const bool fuse = opt.fuse_bits > 0;
   const int m = map.m;
+  const bool zskip = opt.zskip && fuse && opt.prune && map.m == map.n;
   const int G = int(order.size());
   std::vector<int> fused;
   std::vector<char> absorbed;
@@ -929,10 +948,20 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
       gp = &restricted;
     }
     map.touch(inv_g);
-    if (peephole && absorbed[k]) return skip();  // folded into an earlier fused gate
     const Gate& g = gp ? *gp : gate_at(k);
+    if (zskip && fresh) {
+      // a qubit placed by a diagonal gate, or as a control, leaves its new half zero; the
+      // half is skipped (not written, not read) until a non-diagonal op targets the position
+      const uint64_t nz = g.diag ? 0 : g.tmask();
+      for (uint64_t f = fresh & ~nz; f; f &= f - 1) {
+        const int pos = map.pos[std::countr_zero(f)];
+        if (pos >= 0 && pos < m) B.zpos |= 1ull << pos;
+      }
+    }
+    if (peephole && absorbed[k]) return skip();  // folded into an earlier fused gate
     if (scalar_at_origin) {
       // nothing involved: the state is psi[0] |0...0>; one diagonal kernel scales psi[0]
+      B.materialise(xi);
       B.close();
       B.start(PK_DIAG, xi, k_before);
       PhysGate pg;
@@ -989,6 +1018,7 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
         else tloc |= 1ull << p;
       }
       if (ng) {
+        B.materialise(xi);
         B.close();
         B.start(PK_SWAP, xi, map.kl);
         B.cur.count = 0;
@@ -1033,6 +1063,7 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
       B.cur.k_out = map.kl;
       B.cur.unfused_bytes += unfused_gate_bytes(pg, k_before, map.kl);
     } else {
+      B.materialise(xi);
       B.close();
       B.start(g.diag ? PK_DIAG : (g.nt == 1 ? PK_PAIR : PK_QUAD), xi, k_before);
       B.cur.gates.push_back(pg);
@@ -1105,6 +1136,7 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
     while (head < pend.size() && done[size_t(pend[head])]) ++head;
   }
   B.close();
+  B.materialise(xi);  // the state in memory is complete again at the end of every plan
 }
 
 }  // namespace qgpu

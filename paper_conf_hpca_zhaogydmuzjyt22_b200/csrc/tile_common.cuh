@@ -87,6 +87,8 @@ struct TileArgs {
   int srun_pos[kMaxTileBits], srun_len[kMaxTileBits];
   uint64_t ntiles;
   uint64_t L_in;
+  uint64_t zin, zout;      // zero-position skipping (Pass::zin / zout): amplitudes with a zin bit
+                           // read as zero; tiles with a zout bit are neither loaded nor stored
   uint64_t rank_base;      // rank << m (global bits for tile-uniform conditions)
   const double2* zero;     // >= 2^kMaxTileBits zero amplitudes (source of the expanded region)
   int nbuf;                // tile buffers in shared memory (2 or 3)
@@ -640,7 +642,7 @@ __device__ __forceinline__ SlotAddr slot_addr(const Mapping& mp, const uint64_t*
 template <int NR, class Body>
 __device__ __forceinline__ void issue_own_loads(double2* buf, const TileArgs& a, const Mapping& mp0,
                                                 const SlotAddr& sa0, uint64_t base, unsigned zm, bool own) {
-  if (own && base < a.L_in) {
+  if (own && base < a.L_in && !(base & a.zin)) {
 #pragma unroll
     for (int r = 0; r < (1 << NR); ++r) {
       if ((zm >> r) & 1) continue;
@@ -653,7 +655,7 @@ __device__ __forceinline__ void issue_own_loads(double2* buf, const TileArgs& a,
         idx = base | sa0.at(r);
         j = mp0.j(r);
       }
-      const bool live = idx < a.L_in;
+      const bool live = idx < a.L_in && !(idx & a.zin);
       cp_async16(buf + j, a.psi + (live ? idx : 0), live ? 16 : 0);
     }
   }
@@ -767,7 +769,18 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     // nbuf >= 2: prefetch into the next buffer now; nbuf == 1 (programs without remaps, every
     // thread reads only its own slots): prefetch into the same buffer right after the reload
     if (more && nbuf > 1) issue_own_loads<NR, Body>(bufs + kn * T, a, mp0, sa0, base_next, zm0, c.own);
-    if (base >= a.L_in) {
+    if (base & a.zout) {
+      // zero-position skipping: a non-tile bit of this tile selects a half that is zero and is
+      // not materialised in memory -> nothing to load, compute or store
+      if (more && nbuf == 1) {
+        cp_async_wait_all();
+        issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
+      }
+      k = kn;
+      tile = next;
+      continue;
+    }
+    if (base >= a.L_in || (base & a.zin)) {
       // the whole tile lies in the zero region of a first-touch expansion and no op of the pass
       // targets its non-tile bits: it stays zero -> store zeros, skip the program
       if (a.bstore) {
