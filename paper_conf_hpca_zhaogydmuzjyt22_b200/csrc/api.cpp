@@ -854,6 +854,7 @@ uint64_t plan_key(const qgpu_state* st, const qgpu_circuit* c) {
   if (const char* ev = std::getenv("QGPU_MAX_UOPS")) mix(uint64_t(std::atoi(ev)) << 40);
   if (const char* ev = std::getenv("QGPU_LOOKAHEAD")) mix(uint64_t(std::atoi(ev)) << 48);
   if (const char* ev = std::getenv("QGPU_ZSKIP")) mix(uint64_t(std::atoi(ev) + 1) << 56);
+  if (const char* ev = std::getenv("QGPU_LMIN")) mix(uint64_t(std::atoi(ev) + 1) << 60);
   return h;
 }
 
@@ -899,6 +900,7 @@ void prepare_jit(qgpu_state* st, const std::vector<Pass>& passes) {
 // experiment overrides of the planner defaults (also part of the plan-cache key)
 void plan_env(PlanOptions* o) {
   if (const char* ev = std::getenv("QGPU_ZSKIP")) o->zskip = std::atoi(ev) != 0;
+  if (const char* ev = std::getenv("QGPU_LMIN")) o->l_min = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_REGBITS")) o->reg_bits = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_MAX_UOPS")) o->max_u_ops = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_LOOKAHEAD")) o->lookahead = std::atoi(ev);
