@@ -8,6 +8,7 @@
 #include <cstring>
 #include <map>
 #include <string>
+#include <string_view>
 #include <vector>
 
 #include "qgpu_internal.h"
@@ -19,7 +20,7 @@ enum TokKind { T_EOF, T_ID, T_NUM, T_STR, T_SYM, T_ARROW };
 
 struct Tok {
   TokKind k;
-  std::string s;
+  std::string_view s;  // view into the source text (which outlives the parse)
   double v = 0;
   int line, col;
 };
@@ -43,7 +44,7 @@ class Lexer {
       if (std::isalpha((unsigned char)c) || c == '_') {
         const char* s = p_;
         while (p_ < e_ && (std::isalnum((unsigned char)*p_) || *p_ == '_')) ++p_;
-        t.k = T_ID; t.s.assign(s, p_);
+        t.k = T_ID; t.s = std::string_view(s, size_t(p_ - s));
       } else if (std::isdigit((unsigned char)c) || (c == '.' && p_ + 1 < e_ && std::isdigit((unsigned char)p_[1]))) {
         const char* s = p_;
         while (p_ < e_ && (std::isdigit((unsigned char)*p_) || *p_ == '.')) ++p_;
@@ -55,17 +56,17 @@ class Lexer {
             while (p_ < e_ && std::isdigit((unsigned char)*p_)) ++p_;
           }
         }
-        t.k = T_NUM; t.s.assign(s, p_);
-        t.v = std::strtod(t.s.c_str(), nullptr);
+        t.k = T_NUM; t.s = std::string_view(s, size_t(p_ - s));
+        t.v = std::strtod(std::string(t.s).c_str(), nullptr);
       } else if (c == '"') {
         const char* s = ++p_;
         while (p_ < e_ && *p_ != '"' && *p_ != '\n') ++p_;
         if (p_ >= e_ || *p_ != '"') throw ParseError{QGPU_ERR_PARSE, at(t) + "unterminated string"};
-        t.k = T_STR; t.s.assign(s, p_); ++p_;
+        t.k = T_STR; t.s = std::string_view(s, size_t(p_ - s)); ++p_;
       } else if (c == '-' && p_ + 1 < e_ && p_[1] == '>') {
-        t.k = T_ARROW; t.s = "->"; p_ += 2;
+        t.k = T_ARROW; t.s = std::string_view(p_, 2); p_ += 2;
       } else if (c != '\0' && std::strchr(";,[](){}+-*/^", c) != nullptr) {
-        t.k = T_SYM; t.s = std::string(1, c); ++p_;
+        t.k = T_SYM; t.s = std::string_view(p_, 1); ++p_;
       } else {
         throw ParseError{QGPU_ERR_PARSE, at(t) + "unexpected character '" + std::string(1, c) + "'"};
       }
@@ -101,34 +102,34 @@ class Parser {
       next();
       if (peek().k != T_NUM) fail(peek(), "expected version");
       next();
-      expect(";");
+      expect(';');
     }
     while (peek().k != T_EOF) {
       const Tok& t = next();
-      if (t.k != T_ID) fail(t, "unexpected token '" + t.s + "'");
+      if (t.k != T_ID) fail(t, "unexpected token '" + std::string(t.s) + "'");
       if (t.s == "include") {
         if (peek().k != T_STR) fail(peek(), "expected file name");
         next();
-        expect(";");
+        expect(';');
       } else if (t.s == "qreg" || t.s == "creg") {
         const Tok& name = next();
         if (name.k != T_ID) fail(name, "expected register name");
-        expect("[");
+        expect('[');
         const Tok& sz = next();
         if (sz.k != T_NUM) fail(sz, "expected register size");
-        expect("]");
-        expect(";");
+        expect(']');
+        expect(';');
         if (t.s == "qreg") {
           if (regs_.count(name.s)) fail(name, "duplicate register", QGPU_ERR_INVALID_ARG);
-          regs_[name.s] = {n_, int(sz.v)};
+          regs_[std::string(name.s)] = {n_, int(sz.v)};
           n_ += int(sz.v);
           if (n_ > kMaxQubits) fail(sz, "too many qubits", QGPU_ERR_UNSUPPORTED);
         }
       } else if (t.s == "measure" || t.s == "barrier") {
-        while (peek().k != T_EOF && !(peek().k == T_SYM && peek().s == ";")) next();
-        expect(";");
+        while (peek().k != T_EOF && !is(';')) next();
+        expect(';');
       } else if (t.s == "gate" || t.s == "opaque" || t.s == "reset" || t.s == "if") {
-        fail(t, "'" + t.s + "' is not supported", QGPU_ERR_UNSUPPORTED);
+        fail(t, "'" + std::string(t.s) + "' is not supported", QGPU_ERR_UNSUPPORTED);
       } else {
         gate(t, c);
       }
@@ -139,9 +140,9 @@ class Parser {
  private:
   const Tok& peek() const { return t_[i_]; }
   const Tok& next() { return t_[i_ < t_.size() - 1 ? i_++ : i_]; }
-  bool is(const char* s) const { return peek().k == T_SYM && peek().s == s; }
-  void expect(const char* s) {
-    if (!is(s)) fail(peek(), std::string("expected '") + s + "', got '" + peek().s + "'");
+  bool is(char ch) const { return peek().k == T_SYM && peek().s[0] == ch; }  // symbols: 1 char
+  void expect(char ch) {
+    if (!is(ch)) fail(peek(), std::string("expected '") + ch + "', got '" + std::string(peek().s) + "'");
     next();
   }
   [[noreturn]] void fail(const Tok& t, const std::string& m, qgpu_status c = QGPU_ERR_PARSE) {
@@ -152,8 +153,8 @@ class Parser {
   // unary := ('-'|'+') unary | power; power := primary ('^' unary)?
   double expr() {
     double v = term();
-    while (is("+") || is("-")) {
-      const bool add = next().s == "+";
+    while (is('+') || is('-')) {
+      const bool add = next().s[0] == '+';
       const double r = term();
       v = add ? v + r : v - r;
     }
@@ -161,21 +162,21 @@ class Parser {
   }
   double term() {
     double v = unary();
-    while (is("*") || is("/")) {
-      const bool mul = next().s == "*";
+    while (is('*') || is('/')) {
+      const bool mul = next().s[0] == '*';
       const double r = unary();
       v = mul ? v * r : v / r;
     }
     return v;
   }
   double unary() {
-    if (is("-")) { next(); return -unary(); }
-    if (is("+")) { next(); return unary(); }
+    if (is('-')) { next(); return -unary(); }
+    if (is('+')) { next(); return unary(); }
     return power();
   }
   double power() {
     const double b = primary();
-    if (is("^")) { next(); return std::pow(b, unary()); }
+    if (is('^')) { next(); return std::pow(b, unary()); }
     return b;
   }
   double primary() {
@@ -183,34 +184,35 @@ class Parser {
     if (t.k == T_NUM) return t.v;
     if (t.k == T_ID) {
       if (t.s == "pi") return M_PI;
-      static const std::map<std::string, double (*)(double)> f = {
+      static const std::map<std::string, double (*)(double), std::less<>> f = {
           {"sin", [](double x) { return std::sin(x); }},  {"cos", [](double x) { return std::cos(x); }},
           {"tan", [](double x) { return std::tan(x); }},  {"exp", [](double x) { return std::exp(x); }},
           {"ln", [](double x) { return std::log(x); }},   {"sqrt", [](double x) { return std::sqrt(x); }}};
       auto it = f.find(t.s);
-      if (it == f.end()) fail(t, "unknown identifier '" + t.s + "' in expression");
-      expect("(");
+      if (it == f.end()) fail(t, "unknown identifier '" + std::string(t.s) + "' in expression");
+      expect('(');
       const double v = expr();
-      expect(")");
+      expect(')');
       return it->second(v);
     }
-    if (t.k == T_SYM && t.s == "(") {
+    if (t.k == T_SYM && t.s[0] == '(') {
       const double v = expr();
-      expect(")");
+      expect(')');
       return v;
     }
-    fail(t, "unexpected token '" + t.s + "' in expression");
+    fail(t, "unexpected token '" + std::string(t.s) + "' in expression");
   }
 
   std::vector<int> operand() {
     const Tok& t = next();
-    if (t.k != T_ID || !regs_.count(t.s)) fail(t, "unknown register '" + t.s + "'");
-    auto r = regs_[t.s];
-    if (is("[")) {
+    const auto rit = t.k == T_ID ? regs_.find(t.s) : regs_.end();
+    if (rit == regs_.end()) fail(t, "unknown register '" + std::string(t.s) + "'");
+    const auto r = rit->second;
+    if (is('[')) {
       next();
       const Tok& i = next();
       if (i.k != T_NUM) fail(i, "expected index");
-      expect("]");
+      expect(']');
       const int idx = int(i.v);
       if (idx < 0 || idx >= r.second) fail(i, "index out of range", QGPU_ERR_INVALID_ARG);
       return {r.first + idx};
@@ -223,29 +225,30 @@ class Parser {
   void gate(const Tok& t, Circuit* c) {
     int np, nq, nc;
     cplx U[16];
-    if (!gate_matrix(t.s, {}, &np, &nq, &nc, U, false))
-      fail(t, "unknown gate '" + t.s + "'", QGPU_ERR_UNSUPPORTED);
+    const std::string name(t.s);
+    if (!gate_matrix(name, {}, &np, &nq, &nc, U, false))
+      fail(t, "unknown gate '" + std::string(t.s) + "'", QGPU_ERR_UNSUPPORTED);
     std::vector<double> p;
-    if (is("(")) {
+    if (is('(')) {
       next();
-      if (!is(")")) {
+      if (!is(')')) {
         p.push_back(expr());
-        while (is(",")) { next(); p.push_back(expr()); }
+        while (is(',')) { next(); p.push_back(expr()); }
       }
-      expect(")");
+      expect(')');
     }
     if (int(p.size()) != np)
-      fail(t, t.s + " takes " + std::to_string(np) + " parameters", QGPU_ERR_INVALID_ARG);
+      fail(t, std::string(t.s) + " takes " + std::to_string(np) + " parameters", QGPU_ERR_INVALID_ARG);
     std::vector<std::vector<int>> ops{operand()};
-    while (is(",")) { next(); ops.push_back(operand()); }
-    expect(";");
+    while (is(',')) { next(); ops.push_back(operand()); }
+    expect(';');
     if (int(ops.size()) != nq)
-      fail(t, t.s + " takes " + std::to_string(nq) + " qubits", QGPU_ERR_INVALID_ARG);
+      fail(t, std::string(t.s) + " takes " + std::to_string(nq) + " qubits", QGPU_ERR_INVALID_ARG);
     size_t width = 1;
     for (auto& o : ops) width = std::max(width, o.size());
     for (auto& o : ops)
       if (o.size() != 1 && o.size() != width) fail(t, "register size mismatch", QGPU_ERR_INVALID_ARG);
-    gate_matrix(t.s, p, &np, &nq, &nc, U, true);
+    gate_matrix(name, p, &np, &nq, &nc, U, true);
     const int nt = nq - nc;
     for (size_t k = 0; k < width; ++k) {
       Gate g;
@@ -269,7 +272,7 @@ class Parser {
   std::vector<Tok> t_;
   size_t i_ = 0;
   int n_ = 0;
-  std::map<std::string, std::pair<int, int>> regs_;
+  std::map<std::string, std::pair<int, int>, std::less<>> regs_;
 };
 
 }  // namespace

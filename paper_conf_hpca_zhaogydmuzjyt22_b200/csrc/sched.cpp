@@ -111,19 +111,21 @@ std::vector<int> reorder(const std::vector<Gate>& gates, int mode, int rule) {
 }
 
 uint64_t circuit_hash(const Circuit& c) {
-  uint64_t h = 1469598103934665603ull ^ uint64_t(c.n);
-  auto mix = [&](const void* p, size_t n) {
-    const unsigned char* b = static_cast<const unsigned char*>(p);
-    for (size_t i = 0; i < n; ++i) {
-      h ^= b[i];
-      h *= 1099511628211ull;
-    }
+  // content hash (plan-cache key): 64-bit words, multiply-xorshift mixing
+  uint64_t h = 0x9e3779b97f4a7c15ull ^ uint64_t(c.n);
+  auto mix = [&](uint64_t w) {
+    h = (h ^ w) * 0xff51afd7ed558ccdull;
+    h ^= h >> 32;
   };
   for (const Gate& g : c.gates) {
-    mix(&g.nt, sizeof(g.nt));
-    mix(g.t, sizeof(g.t));
-    mix(&g.cmask, sizeof(g.cmask));
-    mix(g.U, sizeof(cplx) * (1 << (2 * g.nt)));
+    mix(uint64_t(uint32_t(g.nt)) | uint64_t(uint32_t(g.t[0])) << 8 | uint64_t(uint32_t(g.t[1])) << 32);
+    mix(g.cmask);
+    const uint64_t* u = reinterpret_cast<const uint64_t*>(g.U);
+    for (int i = 0, e = 2 << (2 * g.nt); i < e; ++i) {
+      uint64_t w;
+      std::memcpy(&w, u + i, sizeof(w));
+      mix(w);
+    }
   }
   return h;
 }
