@@ -855,6 +855,7 @@ uint64_t plan_key(const qgpu_state* st, const qgpu_circuit* c) {
   if (const char* ev = std::getenv("QGPU_LOOKAHEAD")) mix(uint64_t(std::atoi(ev)) << 48);
   if (const char* ev = std::getenv("QGPU_ZSKIP")) mix(uint64_t(std::atoi(ev) + 1) << 56);
   if (const char* ev = std::getenv("QGPU_LMIN")) mix(uint64_t(std::atoi(ev) + 1) << 60);
+  if (const char* ev = std::getenv("QGPU_LRELAX")) mix(uint64_t(std::atoi(ev) + 1) << 52);
   return h;
 }
 
@@ -901,6 +902,7 @@ void prepare_jit(qgpu_state* st, const std::vector<Pass>& passes) {
 void plan_env(PlanOptions* o) {
   if (const char* ev = std::getenv("QGPU_ZSKIP")) o->zskip = std::atoi(ev) != 0;
   if (const char* ev = std::getenv("QGPU_LMIN")) o->l_min = std::atoi(ev);
+  if (const char* ev = std::getenv("QGPU_LRELAX")) o->l_relax = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_REGBITS")) o->reg_bits = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_MAX_UOPS")) o->max_u_ops = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_LOOKAHEAD")) o->lookahead = std::atoi(ev);

@@ -866,9 +866,14 @@ struct Builder {
   bool fits(uint64_t need, int n_ops_new) const {
     if (cur.n_est + n_ops_new > opt.max_ops) return false;
     if (need && n_u + 1 > opt.max_u_ops) return false;
-    const int lm = std::min(opt.l_min, std::max(cur.k_out, 0));
-    uint64_t S = used | need | ((lm > 0) ? ((1ull << lm) - 1) : 0);
-    return std::popcount(S) <= opt.fuse_bits;
+    auto fits_l = [&](int lmin) {
+      const int lm = std::min(lmin, std::max(cur.k_out, 0));
+      const uint64_t S = used | need | ((lm > 0) ? ((1ull << lm) - 1) : 0);
+      return std::popcount(S) <= opt.fuse_bits;
+    };
+    // l_relax (experiment): a gate that does not fit with l_min contiguous low tile positions may
+    // join with l_relax of them (shorter contiguous runs per warp access) instead of a new pass
+    return fits_l(opt.l_min) || (opt.l_relax > 0 && fits_l(opt.l_relax));
   }
 };
 

@@ -17,15 +17,25 @@ from workloads import circuits as wc  # noqa: E402
 ap = argparse.ArgumentParser()
 ap.add_argument("--jit", type=int, default=0)
 ap.add_argument("--big", action="store_true", help="multi-tile-per-CTA cases (buffer reuse)")
+ap.add_argument("--new", action="store_true",
+                help="zero halves (QFT|0>), host tier with swaps, refined involvement rule")
 args = ap.parse_args()
 cases = [(wc.random_circuit(13, 120, seed=1), 12, 1), (wc.qft(14, x=99), 12, 1), (wc.qaoa(12, 1, seed=2), 9, 1),
          (wc.rqc(13, 4, seed=3), 12, 2), (wc.random_circuit(12, 80, seed=4), 0, 1)]
 if args.big:  # > 3 tiles per CTA: exercises the prefetch / triple-buffer reuse and remaps
     cases = [(wc.random_circuit(21, 60, seed=7), 12, 1), (wc.qaoa(20, 1, seed=3), 12, 1),
              (wc.qft(21, x=12345), 12, 1)]
+extra = [{}] * len(cases)
+if args.new:
+    cases = [(wc.qft(17), 12, 1), (wc.qft(15), 9, 1), (wc.random_circuit(13, 120, seed=5), 9, 1),
+             (wc.qaoa(14, 1, seed=2), 9, 1), (wc.qft(14), 12, 1)]
+    extra = [{}, {}, dict(host_slice_bits=2), dict(host_slice_bits=3), dict(involve_rule=1)]
 worst = 0.0
-for c, fuse, world in cases:
-    with q.State(c.n, fuse_bits=fuse, jit=args.jit, world_size=world) as s:
+for (c, fuse, world), kw in zip(cases, extra):
+    with q.State(c.n, fuse_bits=fuse, jit=args.jit, world_size=world, **kw) as s:
+        if args.new:  # stale non-zero data under the skipped halves
+            s.apply_circuit(q.Circuit(wc.random_circuit(c.n, 40, seed=9).qasm()))
+            s.reset()
         s.apply_circuit(q.Circuit(c.qasm()))
         got = s.amplitudes()
         s.probabilities([0, 3, 5])

@@ -110,8 +110,8 @@ def _shard_main(rank, world, port, text, n, out):
     dist.destroy_process_group()
 
 
-def _run_sharded(q, circ, world, fuse):
-    text = q.Circuit(circ.qasm()).plan_text(circ.n, world, 2, fuse)
+def _run_sharded(q, circ, world, fuse, mode=2):
+    text = q.Circuit(circ.qasm()).plan_text(circ.n, world, mode, fuse)
     ctx = mp.get_context("spawn")
     out = ctx.SimpleQueue()
     port = _free_port()
@@ -158,3 +158,16 @@ def test_sharded_protocol_vs_oracle(q, world, name):
     assert np.abs(got - ref).max() <= 1e-12
     if name in ("random", "rqc", "ghz"):
         assert "\nP 5 " in "\n" + text  # the plan exercised at least one global-local swap
+
+
+@pytest.mark.parametrize("world", [2, 4])
+@pytest.mark.parametrize("name", ["qft0", "randdiag"])
+def test_sharded_protocol_refined_rule(q, world, name):
+    """NEXT-1 plans (reorder mode 2 + 4) through the same shard executor: skipped and restricted
+    gates, rank-bit diagonal restrictions and swaps stay exact."""
+    c = {"qft0": lambda: wc.qft(8),
+         "randdiag": lambda: wc.random_circuit(8, 90, seed=5, names=["cp", "cz", "rz", "cx", "crx", "ccx",
+                                                                      "h", "rzz", "x", "crz", "swap"])}[name]()
+    got, text = _run_sharded(q, c, world, fuse=12, mode=6)
+    assert np.abs(got - osv.simulate(c.qasm())).max() <= 1e-12
+
