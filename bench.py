@@ -393,7 +393,8 @@ def run_ours(args):
     n = circ.n
     stream = torch.cuda.Stream(device=device)
     cfg = dict(device=local, stream=stream.cuda_stream, fuse_bits=args.fuse_bits, reorder=args.reorder,
-               prune=int(not args.no_prune), timing=1, host_slice_bits=args.host_slice_bits)
+               prune=int(not args.no_prune), timing=1, host_slice_bits=args.host_slice_bits,
+               host_compress=args.host_compress)
     sharded = args.sharded and world > 1
     if sharded:
         # one state sharded over the ranks: top log2(N) qubits on rank bits, global-local swaps
@@ -526,6 +527,7 @@ def run_ours(args):
         line["config"]["state_location"] = "host (pinned), streamed through device slots"
         line["host_tier"] = {
             "slice_bits": args.host_slice_bits, "slice_bytes": 16 << (n - args.host_slice_bits),
+            "compressed": bool(args.host_compress),
             "h2d_bytes_per_step": statistics.mean(s["host_h2d_bytes"] for s in stats),
             "d2h_bytes_per_step": statistics.mean(s["host_d2h_bytes"] for s in stats),
             "full_state_bytes": 16 << n,
@@ -582,6 +584,8 @@ def main():
     ap.add_argument("--gfc", type=int, default=1, help="1: also measure GFC compression of the final state")
     ap.add_argument("--host-slice-bits", type=int, default=0,
                     help="h > 0: host-memory tier, state in pinned host memory as 2^h slices (NEXT-2)")
+    ap.add_argument("--host-compress", type=int, default=0,
+                    help="1: host tier slices cross the link GFC-compressed (NEXT-3 on the NEXT-2 link)")
     ap.add_argument("--sharded", action="store_true",
                     help="N>1: shard one state over the ranks (NCCL swaps) instead of N replicas")
     args = ap.parse_args()

@@ -93,6 +93,12 @@ typedef struct {
                                  bit = 0 (a global phase becomes a scalar on the live part);
                                  neither involves anything. Exact. Also changes the
                                  Alg.2/3 costs (new qubits a gate would involve)            */
+  int host_compress;          /* host tier only: 1 = slices cross the host link GFC-compressed
+                                 (SURVEY §8f NEXT-3 on the NEXT-2 link): each stored
+                                 live prefix is compressed on the device and written straight
+                                 into pinned host memory, and decompressed on the device when
+                                 it is loaded again. Lossless (bit-exact). Host memory: 2^h
+                                 slices of gfc_max_bytes(2 * 2^(n-h), 4096) bytes            */
 } qgpu_config;
 
 typedef struct {

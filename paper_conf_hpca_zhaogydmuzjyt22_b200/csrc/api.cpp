@@ -57,6 +57,18 @@ int bstore_mode() {
   return v;
 }
 
+// host_compress loads: by default the host waits for the slice's store, copies the exact
+// compressed size and decodes from device memory; QGPU_HOST_ZC_DECODE=1 (measured slower: the
+// decoder reading host memory occupies SMs the concurrent tile passes need) decodes straight
+// from pinned host memory without a host wait
+bool host_zc_decode() {
+  static const bool v = [] {
+    const char* ev = std::getenv("QGPU_HOST_ZC_DECODE");
+    return ev && std::atoi(ev) != 0;
+  }();
+  return v;
+}
+
 // QGPU_HOST_SWEEP_PER_PASS=1 (ablation): the host tier streams the slices once per pass, as the
 // paper traverses every chunk once per gate, instead of once per run of passes
 bool host_sweep_per_pass() {
@@ -141,6 +153,23 @@ struct qgpu_state {
   cudaStream_t s_h2d = nullptr, s_d2h = nullptr;
   cudaEvent_t ev_loaded[2] = {}, ev_computed[2] = {}, ev_stored[2] = {}, ev_join = nullptr;
   bool group_used[2] = {false, false};
+  // host_compress: slice r is stored GFC-compressed (hraw[r] = 0) in its own buffer of hcap
+  // bytes (raw slices use the same buffer); hoff[r] = its segment offsets (pinned host)
+  bool hcomp = false;
+  uint32_t hseg = 4096;
+  uint64_t hcap = 0, hnseg = 0;
+  std::vector<char> hraw;
+  std::vector<uint64_t*> hoff;
+  uint64_t* hoff_base = nullptr;
+  // link statistics of compressed transfers: each store also copies its total size into a pinned
+  // ring entry; stores and zero-copy loads are counted from the ring at synchronisation points
+  uint64_t* hsz = nullptr;
+  size_t hsz_n = 0;
+  static constexpr size_t kSzRing = 1 << 16;
+  std::vector<size_t> store_k;          // slice r: ring entry of its last compressed store
+  std::vector<std::pair<size_t, uint64_t>> cnt_d2h, cnt_h2d;  // (ring entry, segments)
+  std::vector<uint64_t*> doff, dscan;   // per device slot: offsets, scan scratch
+  std::vector<unsigned char*> dstage;   // per device slot: compressed input of a load
   std::vector<cudaEvent_t> ev_slice;   // slice r: its last D2H (host copy valid after it)
   std::vector<uint64_t> slice_seq;     // order of the slices' last D2H (0 = never stored)
   uint64_t store_seq = 0, unit_seq = 0;
@@ -529,9 +558,135 @@ qgpu_status ensure_slots(qgpu_state* st, int unit, int* ngroups) {
                   (unsigned long long)bytes, cudaGetErrorString(e));
     }
     st->slots.push_back(p);
+    if (st->hcomp) {
+      uint64_t* o = nullptr;
+      uint64_t* sc = nullptr;
+      unsigned char* stg = nullptr;
+      cudaError_t e2 = cudaMalloc(&o, (st->hnseg + 1) * sizeof(uint64_t));
+      if (e2 == cudaSuccess) e2 = cudaMalloc(&sc, std::max<uint64_t>(1, gfc_scan_scratch_elems(st->hnseg)) * sizeof(uint64_t));
+      if (e2 == cudaSuccess) e2 = cudaMalloc(&stg, st->hcap);
+      if (e2 != cudaSuccess) {
+        cudaGetLastError();
+        return fail(QGPU_ERR_OUT_OF_MEMORY, "host tier: compression scratch: %s", cudaGetErrorString(e2));
+      }
+      st->doff.push_back(o);
+      st->dscan.push_back(sc);
+      st->dstage.push_back(stg);
+    }
   }
   *ngroups = st->slots.size() >= size_t(2 * unit) ? 2 : 1;
   return QGPU_OK;
+}
+
+// Load slice r (its valid prefix hlive[r]; raw or GFC-compressed) into device buffer `dst` on
+// stream `s`, zero-filling [hlive, need). Compressed: the host waits for the slice's last store
+// (its size is data dependent), copies the compressed bytes and offsets, decodes on the device.
+qgpu_status host_load_slice(qgpu_state* st, uint64_t r, double2* dst, size_t slot, uint64_t need, cudaStream_t s) {
+  const uint64_t have = st->hlive[r];
+  const uint64_t copy = std::max(std::min(have, need), st->hcomp && !st->hraw[r] ? have : 0);
+  if (copy && (!st->hcomp || st->hraw[r])) {
+    CK(cudaMemcpyAsync(dst, st->shards[r].psi, copy * sizeof(double2), cudaMemcpyHostToDevice, s));
+    st->stats.host_h2d_bytes += copy * sizeof(double2);
+    st->stats.h2d_bytes += copy * sizeof(double2);
+  } else if (copy) {
+    const uint64_t nd = 2 * copy, ns = (nd + st->hseg - 1) / st->hseg;
+    if (host_zc_decode()) {
+      // zero-copy: the decoder reads the compressed stream and its offsets straight from pinned
+      // host memory; only a stream dependency on the slice's last store, no host wait
+      CK(cudaStreamWaitEvent(s, st->ev_slice[r], 0));
+      CK(launch_gfc_decode(s, st->shards[r].psi, st->hoff[r], nd, st->hseg, reinterpret_cast<double*>(dst)));
+      st->stats.kernels_launched++;
+      st->cnt_h2d.push_back({st->store_k[r], ns});  // bytes counted at the next sync point
+    } else {
+      CK(cudaEventSynchronize(st->ev_slice[r]));
+      const uint64_t total = st->hoff[r][ns];
+      CK(cudaMemcpyAsync(st->dstage[slot], st->shards[r].psi, total, cudaMemcpyHostToDevice, s));
+      CK(cudaMemcpyAsync(st->doff[slot], st->hoff[r], (ns + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice, s));
+      CK(launch_gfc_decode(s, st->dstage[slot], st->doff[slot], nd, st->hseg, reinterpret_cast<double*>(dst)));
+      st->stats.kernels_launched++;
+      st->stats.host_h2d_bytes += total + (ns + 1) * sizeof(uint64_t);
+      st->stats.h2d_bytes += total + (ns + 1) * sizeof(uint64_t);
+    }
+  }
+  if (need > copy) CK(cudaMemsetAsync(dst + copy, 0, (need - copy) * sizeof(double2), s));
+  return QGPU_OK;
+}
+
+void host_account_stores(qgpu_state* st);
+
+// Store the prefix [0, L) of device buffer `src` as slice r on stream `s` (after its compute).
+// Compressed: size pass, scan, then the encoder writes the stream straight into the slice's
+// pinned host buffer (zero-copy, so no host round trip for the data-dependent size); the
+// offsets follow with one D2H copy.
+qgpu_status host_store_slice(qgpu_state* st, uint64_t r, const double2* src, size_t slot, uint64_t L, cudaStream_t s) {
+  if (!st->hcomp) {
+    CK(cudaMemcpyAsync(st->shards[r].psi, src, L * sizeof(double2), cudaMemcpyDeviceToHost, s));
+    st->stats.host_d2h_bytes += L * sizeof(double2);
+    st->stats.d2h_bytes += L * sizeof(double2);
+  } else if (L) {
+    const uint64_t nd = 2 * L, ns = (nd + st->hseg - 1) / st->hseg;
+    if (st->hsz_n == qgpu_state::kSzRing) {  // ring full: count what it holds first
+      CK(cudaStreamSynchronize(s));
+      host_account_stores(st);
+    }
+    const double* in = reinterpret_cast<const double*>(src);
+    CK(cudaMemsetAsync(st->doff[slot], 0, sizeof(uint64_t), s));
+    CK(launch_gfc_sizes(s, in, nd, st->hseg, st->doff[slot] + 1));
+    CK(launch_scan_u64(s, st->doff[slot] + 1, ns, st->dscan[slot]));
+    CK(launch_gfc_encode(s, in, nd, st->hseg, st->doff[slot], st->shards[r].psi));
+    CK(cudaMemcpyAsync(st->hoff[r], st->doff[slot], (ns + 1) * sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    const size_t k = st->hsz_n++;
+    CK(cudaMemcpyAsync(st->hsz + k, st->doff[slot] + ns, sizeof(uint64_t), cudaMemcpyDeviceToHost, s));
+    st->store_k[r] = k;
+    st->cnt_d2h.push_back({k, ns});
+    st->stats.kernels_launched += 3;
+    st->hraw[r] = 0;
+  }
+  st->hlive[r] = L;
+  return QGPU_OK;
+}
+
+// Readout of slice r: raw slices are read in place (zero-copy); a compressed one is decoded into
+// device slot 0 first (on the state's stream, so the next slice waits for this readout)
+qgpu_status host_readable(qgpu_state* st, size_t r, const double2** psi) {
+  if (!st->host || !st->hcomp || st->hraw[r] || !st->hlive[r]) return QGPU_OK;
+  int ng = 1;
+  if (qgpu_status s = ensure_slots(st, 1, &ng)) return s;
+  if (qgpu_status s = host_load_slice(st, r, st->slots[0], 0, st->hlive[r], st->stream)) return s;
+  *psi = st->slots[0];
+  return QGPU_OK;
+}
+
+// host_compress: add the compressed bytes of stores and zero-copy loads to the link statistics
+// (the ring entries are final once s_d2h has drained: callers synchronise it first)
+void host_account_stores(qgpu_state* st) {
+  if (!st->hcomp) return;
+  for (auto [k, ns] : st->cnt_d2h) {
+    const uint64_t b = st->hsz[k] + (ns + 1) * sizeof(uint64_t);
+    st->stats.host_d2h_bytes += b;
+    st->stats.d2h_bytes += b;
+  }
+  for (auto [k, ns] : st->cnt_h2d) {
+    const uint64_t b = st->hsz[k] + (ns + 1) * sizeof(uint64_t);
+    st->stats.host_h2d_bytes += b;
+    st->stats.h2d_bytes += b;
+  }
+  st->cnt_d2h.clear();
+  st->cnt_h2d.clear();
+  // ring entries still referenced by slices are kept: compact them to the front
+  std::vector<std::pair<size_t, size_t>> keep;  // (old k, slice)
+  for (size_t r = 0; r < st->store_k.size(); ++r)
+    if (!st->hraw[r]) keep.push_back({st->store_k[r], r});
+  std::sort(keep.begin(), keep.end());
+  size_t nk = 0, last = ~size_t(0);
+  for (auto [k, r] : keep) {
+    if (k != last) {
+      st->hsz[nk++] = st->hsz[k];
+      last = k;
+    }
+    st->store_k[r] = nk - 1;
+  }
+  st->hsz_n = nk;
 }
 
 // One streaming sweep: swaps `sw` (made while 2^kg_sw ranks were active), then the passes `run`.
@@ -608,14 +763,8 @@ qgpu_status host_sweep(qgpu_state* st, const std::vector<const Pass*>& run,
             break;
           }
       }
-      const uint64_t copy = std::min(st->hlive[r], need);
-      if (copy)
-        CK(cudaMemcpyAsync(slot[x], st->shards[r].psi, copy * sizeof(double2), cudaMemcpyHostToDevice,
-                           st->s_h2d));
-      if (need > copy)
-        CK(cudaMemsetAsync(slot[x] + copy, 0, (need - copy) * sizeof(double2), st->s_h2d));
-      st->stats.host_h2d_bytes += copy * sizeof(double2);
-      st->stats.h2d_bytes += copy * sizeof(double2);
+      if (qgpu_status s = host_load_slice(st, r, slot[x], size_t(gi) * size_t(unit) + size_t(x), need, st->s_h2d))
+        return s;
       st->stats.host_slice_loads++;
     }
     CK(cudaEventRecord(st->ev_loaded[gi], st->s_h2d));
@@ -671,11 +820,8 @@ qgpu_status host_sweep(qgpu_state* st, const std::vector<const Pass*>& run,
     CK(cudaStreamWaitEvent(st->s_d2h, st->ev_computed[gi], 0));
     for (int x = 0; x < unit; ++x) {
       const uint64_t r = rs[x];
-      CK(cudaMemcpyAsync(st->shards[r].psi, slot[x], L_end * sizeof(double2), cudaMemcpyDeviceToHost,
-                         st->s_d2h));
-      st->hlive[r] = L_end;
-      st->stats.host_d2h_bytes += L_end * sizeof(double2);
-      st->stats.d2h_bytes += L_end * sizeof(double2);
+      if (qgpu_status s = host_store_slice(st, r, slot[x], size_t(gi) * size_t(unit) + size_t(x), L_end, st->s_d2h))
+        return s;
       CK(cudaEventRecord(st->ev_slice[r], st->s_d2h));
       st->slice_seq[r] = ++st->store_seq;
     }
@@ -822,8 +968,10 @@ qgpu_status init_amplitudes(qgpu_state* st) {
     // through hlive (the host pages beyond hlive are never read)
     CK(cudaStreamSynchronize(st->stream));
     CK(cudaStreamSynchronize(st->s_d2h));
-    st->h_state[0] = make_double2(1.0, 0.0);
+    host_account_stores(st);
+    st->shards[0].psi[0] = make_double2(1.0, 0.0);
     std::fill(st->hlive.begin(), st->hlive.end(), 0);
+    std::fill(st->hraw.begin(), st->hraw.end(), 1);
     st->hlive[0] = 1;
     return QGPU_OK;
   }
@@ -1058,10 +1206,21 @@ qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out
     st->host = cfg.host_slice_bits > 0;
     const int nshard = st->host ? (1 << g) : st->virt ? cfg.world_size : 1;
     if (st->virt && cfg.state_buffer) return bail(fail(QGPU_ERR_UNSUPPORTED, "virtual ranks allocate their own shards"));
+    if (cfg.host_compress && !cfg.host_slice_bits)
+      return bail(fail(QGPU_ERR_INVALID_ARG, "host_compress needs host_slice_bits > 0"));
     if (st->host) {
       // pinned, device-mapped host memory: slices stream through device slots; readout kernels
       // read it in place (zero-copy) through unified addressing
-      const size_t hbytes = (size_t(1) << n) * sizeof(double2);
+      size_t hbytes = (size_t(1) << n) * sizeof(double2);
+      size_t sstride = (size_t(1) << st->m);  // slice stride in amplitudes
+      if (cfg.host_compress) {  // each slice holds its worst-case compressed size (>= raw)
+        st->hcomp = true;
+        const uint64_t nd = 2ull << st->m;
+        qgpu_gfc_max_bytes(nd, st->hseg, &st->hcap);
+        st->hnseg = (nd + st->hseg - 1) / st->hseg;
+        sstride = st->hcap / sizeof(double2);
+        hbytes = size_t(st->hcap) << g;
+      }
       e = cudaHostAlloc(&st->h_state, hbytes, cudaHostAllocMapped | cudaHostAllocPortable);
       if (e != cudaSuccess) {
         cudaGetLastError();
@@ -1071,8 +1230,17 @@ qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out
       double2* dev = nullptr;
       e = cudaHostGetDevicePointer(reinterpret_cast<void**>(&dev), st->h_state, 0);
       if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaHostGetDevicePointer: %s", cudaGetErrorString(e)));
-      for (int r = 0; r < nshard; ++r) st->shards.push_back(Shard{r, dev + (size_t(r) << st->m), false});
+      for (int r = 0; r < nshard; ++r) st->shards.push_back(Shard{r, dev + size_t(r) * sstride, false});
       st->hlive.assign(size_t(nshard), 0);
+      st->hraw.assign(size_t(nshard), 1);
+      if (st->hcomp) {
+        e = cudaMallocHost(&st->hoff_base, size_t(nshard) * (st->hnseg + 1) * sizeof(uint64_t));
+        if (e != cudaSuccess) return bail(fail(QGPU_ERR_OUT_OF_MEMORY, "host tier offsets: %s", cudaGetErrorString(e)));
+        for (int r = 0; r < nshard; ++r) st->hoff.push_back(st->hoff_base + size_t(r) * (st->hnseg + 1));
+        e = cudaMallocHost(&st->hsz, qgpu_state::kSzRing * sizeof(uint64_t));
+        if (e != cudaSuccess) return bail(fail(QGPU_ERR_OUT_OF_MEMORY, "host tier size ring: %s", cudaGetErrorString(e)));
+        st->store_k.assign(size_t(nshard), 0);
+      }
       for (cudaStream_t* sp : {&st->s_h2d, &st->s_d2h}) {
         e = cudaStreamCreateWithFlags(sp, cudaStreamNonBlocking);
         if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaStreamCreate: %s", cudaGetErrorString(e)));
@@ -1142,6 +1310,11 @@ qgpu_status qgpu_state_destroy(qgpu_state* st) {
   if (st->s_h2d) cudaStreamSynchronize(st->s_h2d);
   if (st->s_d2h) cudaStreamSynchronize(st->s_d2h);
   for (double2* p : st->slots) cudaFree(p);
+  for (uint64_t* p : st->doff) cudaFree(p);
+  for (uint64_t* p : st->dscan) cudaFree(p);
+  for (unsigned char* p : st->dstage) cudaFree(p);
+  if (st->hoff_base) cudaFreeHost(st->hoff_base);
+  if (st->hsz) cudaFreeHost(st->hsz);
   if (st->h_state) cudaFreeHost(st->h_state);
   for (int i = 0; i < 2; ++i)
     for (cudaEvent_t e : {st->ev_loaded[i], st->ev_computed[i], st->ev_stored[i]})
@@ -1174,6 +1347,10 @@ qgpu_status qgpu_state_reset(qgpu_state* st) {
   st->trace_inv.clear();
   st->gate_counter = 0;
   if (qgpu_status s = drain_timing(st)) return s;
+  if (st->hcomp) {  // link bytes of the work before the reset belong to the old statistics
+    CK(cudaStreamSynchronize(st->s_d2h));
+    host_account_stores(st);
+  }
   std::memset(&st->stats, 0, sizeof(st->stats));
   st->stats.ops_before_full_involvement = -1;
   return init_amplitudes(st);
@@ -1186,8 +1363,11 @@ qgpu_status qgpu_set_amplitudes(qgpu_state* st, const double* amps) {
   if (st->host) {
     CK(cudaStreamSynchronize(st->stream));
     CK(cudaStreamSynchronize(st->s_d2h));
-    std::memcpy(st->h_state, amps, (size_t(1) << st->n) * sizeof(double2));
+    host_account_stores(st);
+    for (size_t r = 0; r < st->shards.size(); ++r)
+      std::memcpy(st->shards[r].psi, amps + 2 * (r << st->m), (size_t(1) << st->m) * sizeof(double2));
     std::fill(st->hlive.begin(), st->hlive.end(), 1ull << st->m);
+    std::fill(st->hraw.begin(), st->hraw.end(), 1);
   } else {
     st->psi = st->shards[0].psi;
     CK(cudaMemcpyAsync(st->psi, amps, (1ull << st->n) * sizeof(double2), cudaMemcpyHostToDevice, st->stream));
@@ -1310,6 +1490,7 @@ qgpu_status qgpu_get_amplitudes_device(qgpu_state* st, uint64_t start, uint64_t 
     if (sharded && (uint64_t(sh.rank) >> st->map.kg) != 0) continue;  // inactive: all zero
     GatherArgs a{};
     a.psi = sh.psi;
+    if (qgpu_status s = host_readable(st, size_t(sh.rank), &a.psi)) return s;
     a.out = reinterpret_cast<double2*>(dev_out);
     a.start = start;
     a.count = count;
@@ -1384,6 +1565,8 @@ qgpu_status qgpu_probabilities(qgpu_state* st, int mq, const int* qubits, double
     const Shard& sh = st->shards[i];
     ProbArgs pa = a;
     pa.psi = sh.psi;
+    if (st->host && (uint64_t(sh.rank) >> st->map.kg) == 0)
+      if (qgpu_status s = host_readable(st, i, &pa.psi)) return s;
     pa.yfixed = 0;
     for (int j = 0; j < mq; ++j) {  // requested qubits on rank bits: fixed by this rank
       const int p = st->map.pos[qubits[j]];
@@ -1612,6 +1795,10 @@ qgpu_status qgpu_get_stats(qgpu_state* st, qgpu_stats* out) {
   if (!st || !out) return fail(QGPU_ERR_INVALID_ARG, "NULL argument");
   if (!st->pending.empty()) {
     if (qgpu_status s = drain_timing(st)) return s;
+  }
+  if (st->hcomp) {  // compressed link bytes are known once the stores have completed
+    CK(cudaStreamSynchronize(st->s_d2h));
+    host_account_stores(st);
   }
   *out = st->stats;
   return QGPU_OK;

@@ -46,6 +46,7 @@ class Config(ctypes.Structure):
         ("chunk_bits", ctypes.c_int), ("prune", ctypes.c_int), ("reorder", ctypes.c_int),
         ("fuse_bits", ctypes.c_int), ("timing", ctypes.c_int), ("swap_slab_bytes", ctypes.c_uint64),
         ("jit", ctypes.c_int), ("host_slice_bits", ctypes.c_int), ("involve_rule", ctypes.c_int),
+        ("host_compress", ctypes.c_int),
     ]
 
 

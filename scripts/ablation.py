@@ -32,6 +32,7 @@ REFINED = ("refined", dict(prune=1, reorder=2, involve_rule=1))  # NEXT-1 (--ref
 #   prune_u   prune=1 reorder=0 fuse_bits=0   + pruning / delayed involvement (Pruning)
 #   forward_u prune=1 reorder=2 fuse_bits=0   + Alg.3 reorder (Reorder)
 #   forward   prune=1 reorder=2               + B200 fusion: one sweep per run of passes
+#   compressed                                + GFC on the host link (the paper's Compression)
 # paper_*: one sweep of the slices per gate (QGPU_HOST_SWEEP_PER_PASS=1), the paper's traversal
 HOST_VERSIONS = [("paper_base", dict(prune=0, reorder=0, fuse_bits=0, per_pass=1)),
                  ("paper_prune", dict(prune=1, reorder=0, fuse_bits=0, per_pass=1)),
@@ -40,7 +41,8 @@ HOST_VERSIONS = [("paper_base", dict(prune=0, reorder=0, fuse_bits=0, per_pass=1
                  ("prune_u", dict(prune=1, reorder=0, fuse_bits=0)),
                  ("forward_u", dict(prune=1, reorder=2, fuse_bits=0)),
                  ("forward", dict(prune=1, reorder=2)),
-                 ("refined", dict(prune=1, reorder=2, involve_rule=1))]
+                 ("refined", dict(prune=1, reorder=2, involve_rule=1)),
+                 ("compressed", dict(prune=1, reorder=2, host_compress=1))]  # + GFC on the link
 
 
 def family(name, n):

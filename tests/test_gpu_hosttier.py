@@ -38,14 +38,15 @@ CIRCS = {
 }
 
 
+@pytest.mark.parametrize("comp", [0, 1])
 @pytest.mark.parametrize("h", [1, 2, 3])
 @pytest.mark.parametrize("name", sorted(CIRCS))
 @pytest.mark.parametrize("fuse", [0, 9])
-def test_host_tier_vs_oracle(q, h, name, fuse):
+def test_host_tier_vs_oracle(q, h, name, fuse, comp):
     c = CIRCS[name]()
     text = c.qasm()
     qs = list(range(c.n))[::-1][:6]
-    with q.State(c.n, host_slice_bits=h, fuse_bits=fuse, timing=1) as s:
+    with q.State(c.n, host_slice_bits=h, fuse_bits=fuse, timing=1, host_compress=comp) as s:
         s.apply_circuit(q.Circuit(text))
         got = s.amplitudes()
         st = s.stats()
@@ -145,3 +146,47 @@ def test_host_tier_argument_errors(q):
     with pytest.raises(q.QgpuError) as e:
         q.State(12, host_slice_bits=2, world_size=2)
     assert e.value.kind == "UNSUPPORTED"
+
+
+@pytest.mark.parametrize("name", ["qft0", "gs", "qaoa", "grqc", "random"])
+def test_host_compress_bit_identical_and_smaller_link(q, name):
+    """GFC on the host link (P:344-362 on the NEXT-2 link) is lossless: the compressed host tier
+    gives the same bits as the raw one; structured states (QFT of |0>, graph states) cross the
+    link in fewer bytes."""
+    c = CIRCS[name]()
+    text = c.qasm()
+    out = {}
+    for comp in (0, 1):
+        with q.State(c.n, host_slice_bits=2, fuse_bits=9, host_compress=comp) as s:
+            s.apply_circuit(q.Circuit(text))
+            s.apply_circuit(q.Circuit(text))  # loads compressed slices written by the first apply
+            out[comp] = (s.amplitudes(), s.stats(), s.probabilities([0, 1, 2]))
+    assert np.array_equal(out[0][0], out[1][0])
+    assert np.abs(out[0][2] - out[1][2]).max() <= 1e-15  # (reduction order of the readout)
+    if name in ("qft0", "gs"):
+        assert out[1][1]["host_d2h_bytes"] < 0.5 * out[0][1]["host_d2h_bytes"]
+
+
+def test_host_compress_gate_stream_and_set_amplitudes(q):
+    n = 11
+    c = wc.random_circuit(n, 60, seed=19)
+    _, gates = oq.parse(c.qasm())
+    ref = osv.zero_state(n)
+    with q.State(n, host_slice_bits=2, host_compress=1) as s:
+        for g in gates:
+            s.apply_gate(g.U, list(g.targets), list(g.controls))
+            osv.apply_gate(ref, n, g.U, g.targets, g.controls)
+        assert np.abs(s.amplitudes() - ref).max() <= TOL
+        rng = np.random.default_rng(5)
+        psi = rng.normal(size=1 << n) + 1j * rng.normal(size=1 << n)
+        psi /= np.linalg.norm(psi)
+        s.set_amplitudes(psi)  # raw slices again
+        assert np.array_equal(s.amplitudes(), psi)
+        text = wc.random_circuit(n, 40, seed=20).qasm()
+        s.apply_circuit(q.Circuit(text))
+        got = s.amplitudes()
+    _, g2 = oq.parse(text)
+    for g in g2:
+        osv.apply_gate(psi, n, g.U, g.targets, g.controls)
+    assert np.abs(got - psi).max() <= TOL
+
