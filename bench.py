@@ -299,6 +299,44 @@ def single_qubit_sweep(q, torch, n: int, reps: int = 3):
     return res
 
 
+def gate_sweep(q, torch, n: int, reps: int = 3):
+    """SURVEY §8d microbenchmark, the other gate kinds: for every position t on a fully involved
+    2^n state, a generic 2-qubit gate on (t, t+1), CX (control t, target t+1) and CP (t, t+1).
+    Algorithmic bytes per gate: 2q generic 32 * 2^n (every quad read and written), CX 16 * 2^n
+    (the half with the control set), CP 8 * 2^n (the quarter whose phase is not 1).
+    Returns {kind: [GB/s per t]}."""
+    import numpy as np
+    stream = torch.cuda.Stream()
+    s = q.State(n, stream=stream.cuda_stream, fuse_bits=0)
+    H = np.array([[1, 1], [1, -1]], dtype=complex) / math.sqrt(2)
+    for t in range(n):
+        s.apply_gate(H, [t])
+    s.synchronize()
+    rng = np.random.default_rng(2)
+    U4 = np.linalg.qr(rng.normal(size=(4, 4)) + 1j * rng.normal(size=(4, 4)))[0]
+    X = np.array([[0, 1], [1, 0]], dtype=complex)
+    P = np.diag([1, np.exp(0.7j)])
+    kinds = {"u2q": (lambda t: s.apply_gate(U4, [t, (t + 1) % n]), 32.0),
+             "cx": (lambda t: s.apply_gate(X, [(t + 1) % n], [t]), 16.0),
+             "cp": (lambda t: s.apply_gate(P, [(t + 1) % n], [t]), 8.0)}
+    out = {}
+    for kind, (fn, bpa) in kinds.items():
+        res = []
+        for t in range(n):
+            fn(t)
+            e0, e1 = torch.cuda.Event(enable_timing=True), torch.cuda.Event(enable_timing=True)
+            e0.record(stream)
+            for _ in range(reps):
+                fn(t)
+            e1.record(stream)
+            e1.synchronize()
+            ms = e0.elapsed_time(e1) / reps
+            res.append(bpa * (1 << n) / (ms * 1e-3) / 1e9)
+        out[kind] = res
+    s.close()
+    return out
+
+
 def gfc_measure(q, torch, st, seg: int = 4096):
     """NEXT-3: GFC compression of the state left by the workload (the physical
     buffer, as a host-link or swap transfer would send it): ratio and device throughput of
@@ -550,6 +588,11 @@ def run_ours(args):
                                      "GBps_per_target": [round(x, 1) for x in gbs],
                                      "frac_min": min(gbs) / peak, "frac_median": statistics.median(gbs) / peak,
                                      "frac_min_of_8TBs": min(gbs) / 8000.0}
+        for kind, g in gate_sweep(q, torch, nm).items():
+            line["single_qubit_gate"]["other_gates"] = line["single_qubit_gate"].get("other_gates", {})
+            line["single_qubit_gate"]["other_gates"][kind] = {
+                "GBps_min": min(g), "GBps_median": statistics.median(g), "frac_min": min(g) / peak,
+                "GBps_per_target": [round(x, 1) for x in g]}
 
     if rank == 0 and world == 1 and not args.no_cpu_baseline:
         v, smp = oracle_sample(text, args.cpu_seconds)
