@@ -116,3 +116,25 @@ def test_graph_state_30_sampled_ranges(q):
             for u, v in edges:
                 par ^= ((xs >> u) & 1) & ((xs >> v) & 1)
             assert np.abs(got - (1 - 2 * par) / math.sqrt(1 << n)).max() <= TOL
+
+
+@pytest.mark.parametrize("comp", [0, 1])
+def test_host_tier_qft30_basis_state_sampled(q, comp):
+    """NEXT-2 (+ NEXT-3 on the link) at 30 qubits (16 GiB in pinned host memory, 2^2 slices):
+    QFT|x> sampled ranges in every slice vs e^{2 pi i x y / 2^n} / 2^{n/2}, and the norm."""
+    n = 30
+    x = 0x2A5F3C1B & ((1 << n) - 1)
+    c = wc.qft(n, x=x)
+    with q.State(n, host_slice_bits=2, host_compress=comp) as s:
+        s.apply_circuit(q.Circuit(c.qasm()))
+        worst = 0.0
+        for start in [0, (1 << 28) - 4096, 1 << 28, 3 << 28, (1 << n) - (1 << 16)]:
+            got = s.amplitudes(start, 1 << 16)
+            y = np.arange(start, start + (1 << 16), dtype=np.int64)
+            ph = ((x * y) % (1 << n)).astype(np.float64) / (1 << n)
+            worst = max(worst, float(np.abs(got - np.exp(2j * np.pi * ph) / math.sqrt(1 << n)).max()))
+        p = s.probabilities([])
+        st = s.stats()
+    assert worst <= TOL
+    assert abs(p[0] - 1) <= 1e-12
+    assert st["host_runs"] >= 1
