@@ -164,8 +164,8 @@ qgpu_status qgpu_set_amplitudes(qgpu_state* st, const double* amps);
 qgpu_status qgpu_synchronize(qgpu_state* st);
 
 /* Number of qubits, local qubits (n - log2 world, or n - host_slice_bits) and the pointer of
- * the local buffer (device memory; with the host tier: the pinned host state, which is also
- * device-accessible through unified addressing). */
+ * the local buffer (device memory; with the host tier: the pinned host state, device-accessible
+ * through unified addressing -- raw amplitudes only with host_compress = 0). */
 qgpu_status qgpu_state_info(const qgpu_state* st, int* n_qubits, int* n_local, void** dev_ptr);
 
 /* ---- gate application (the hot path) --------------------------------------------------- */
