@@ -159,6 +159,7 @@ struct qgpu_state {
   uint32_t hseg = 4096;
   uint64_t hcap = 0, hnseg = 0;
   std::vector<char> hraw;
+  std::vector<char> hpoor;              // slice r compressed poorly last time: store it raw
   std::vector<uint64_t*> hoff;
   uint64_t* hoff_base = nullptr;
   // link statistics of compressed transfers: each store also copies its total size into a pinned
@@ -621,6 +622,9 @@ qgpu_status host_load_slice(qgpu_state* st, uint64_t r, double2* dst, size_t slo
     } else {
       CK(cudaEventSynchronize(st->ev_slice[r]));
       const uint64_t total = st->hoff[r][ns];
+      // adaptive: a slice that did not shrink by a quarter is stored raw from now on (dense
+      // amplitudes have incompressible bit patterns; compression would only add passes)
+      if (4 * total > 3 * nd * sizeof(double)) st->hpoor[r] = 1;
       CK(cudaMemcpyAsync(st->dstage[slot], st->shards[r].psi, total, cudaMemcpyHostToDevice, s));
       CK(cudaMemcpyAsync(st->doff[slot], st->hoff[r], (ns + 1) * sizeof(uint64_t), cudaMemcpyHostToDevice, s));
       CK(launch_gfc_decode(s, st->dstage[slot], st->doff[slot], nd, st->hseg, reinterpret_cast<double*>(dst)));
@@ -640,7 +644,8 @@ void host_account_stores(qgpu_state* st);
 // pinned host buffer (zero-copy, so no host round trip for the data-dependent size); the
 // offsets follow with one D2H copy.
 qgpu_status host_store_slice(qgpu_state* st, uint64_t r, const double2* src, size_t slot, uint64_t L, cudaStream_t s) {
-  if (!st->hcomp) {
+  if (!st->hcomp || st->hpoor[r]) {
+    if (st->hcomp) st->hraw[r] = 1;
     CK(cudaMemcpyAsync(st->shards[r].psi, src, L * sizeof(double2), cudaMemcpyDeviceToHost, s));
     st->stats.host_d2h_bytes += L * sizeof(double2);
     st->stats.d2h_bytes += L * sizeof(double2);
@@ -993,6 +998,7 @@ qgpu_status init_amplitudes(qgpu_state* st) {
     st->shards[0].psi[0] = make_double2(1.0, 0.0);
     std::fill(st->hlive.begin(), st->hlive.end(), 0);
     std::fill(st->hraw.begin(), st->hraw.end(), 1);
+    std::fill(st->hpoor.begin(), st->hpoor.end(), 0);
     st->hlive[0] = 1;
     return QGPU_OK;
   }
@@ -1254,6 +1260,7 @@ qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out
       for (int r = 0; r < nshard; ++r) st->shards.push_back(Shard{r, dev + size_t(r) * sstride, false});
       st->hlive.assign(size_t(nshard), 0);
       st->hraw.assign(size_t(nshard), 1);
+      st->hpoor.assign(size_t(nshard), 0);
       if (st->hcomp) {
         e = cudaMallocHost(&st->hoff_base, size_t(nshard) * (st->hnseg + 1) * sizeof(uint64_t));
         if (e != cudaSuccess) return bail(fail(QGPU_ERR_OUT_OF_MEMORY, "host tier offsets: %s", cudaGetErrorString(e)));
