@@ -103,6 +103,7 @@ struct TimedLaunch {
   cudaEvent_t a, b;
   int kind;
   uint64_t bytes;
+  int count = 1;  // launches between a and b (a run of consecutive fused passes: one interval)
 };
 
 }  // namespace
@@ -220,7 +221,7 @@ qgpu_status drain_timing(qgpu_state* st) {
       st->stats.kernel_ms += ms;
       if (t.kind == PK_TILE) {
         st->stats.tile_kernel_ms += ms;
-        st->stats.tile_kernel_launches++;
+        st->stats.tile_kernel_launches += uint64_t(t.count);
         st->stats.tile_algo_bytes += t.bytes;
       }
     }
@@ -491,7 +492,8 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
 
 // Execute one planned pass: compute passes on every active local shard (ranks >= 2^kg hold
 // only zeros and skip the work), swaps through the communicator, activations as memsets.
-qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops) {
+qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops, bool own_timing = true,
+                      uint64_t* bytes_out = nullptr) {
   const int m = st->m;
   const int kin = st->cfg.prune ? p.k_in : m, kout = st->cfg.prune ? p.k_out : m;
   const uint64_t L_in = 1ull << kin, L_out = 1ull << kout;
@@ -516,7 +518,7 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops)
       }
     return QGPU_OK;
   }
-  const bool timing = st->cfg.timing != 0;
+  const bool timing = st->cfg.timing != 0 && own_timing;
   TimedLaunch tl{};
   if (timing) {
     tl.a = get_event(st);
@@ -548,6 +550,7 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops)
     account(st, L_out, bytes);
     st->stats.unfused_bytes += p.unfused_bytes;
   }
+  if (bytes_out) *bytes_out = bytes;
   return QGPU_OK;
 }
 
@@ -876,9 +879,41 @@ qgpu_status host_join(qgpu_state* st) {
 qgpu_status exec_passes(qgpu_state* st, const std::vector<Pass>& passes,
                         const std::vector<const unsigned char*>& ops) {
   if (!st->host) {
-    for (size_t i = 0; i < passes.size(); ++i)
-      if (qgpu_status s = exec_pass(st, passes[i], ops[i])) return s;
-    return QGPU_OK;
+    // timing=1: a run of consecutive fused passes on one shard is timed as ONE event interval
+    // (events between back-to-back kernels cost a launch gap each); the interval's launches and
+    // algorithmic bytes are recorded with it
+    const bool group = st->cfg.timing != 0 && st->shards.size() == 1;
+    TimedLaunch grp{};
+    bool open = false;
+    auto close_group = [&]() -> qgpu_status {
+      if (!open) return QGPU_OK;
+      CK(cudaEventRecord(grp.b, st->stream));
+      st->pending.push_back(grp);
+      open = false;
+      return QGPU_OK;
+    };
+    for (size_t i = 0; i < passes.size(); ++i) {
+      const Pass& p = passes[i];
+      if (group && p.kind == PK_TILE) {
+        if (!open) {
+          grp = TimedLaunch{};
+          grp.a = get_event(st);
+          grp.b = get_event(st);
+          grp.kind = PK_TILE;
+          grp.count = 0;
+          CK(cudaEventRecord(grp.a, st->stream));
+          open = true;
+        }
+        uint64_t b = 0;
+        if (qgpu_status s = exec_pass(st, p, ops[i], false, &b)) return s;
+        grp.bytes += b;
+        grp.count++;
+        continue;
+      }
+      if (qgpu_status s = close_group()) return s;
+      if (qgpu_status s = exec_pass(st, p, ops[i])) return s;
+    }
+    return close_group();
   }
   std::vector<const Pass*> run;
   std::vector<const unsigned char*> run_ops;
