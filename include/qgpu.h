@@ -186,6 +186,16 @@ qgpu_status qgpu_apply_gate(qgpu_state* st, const double* U, int n_targets, cons
  * Errors: INVALID_ARG, STATE, CUDA, NCCL. Asynchronous. */
 qgpu_status qgpu_apply_circuit(qgpu_state* st, const qgpu_circuit* c);
 
+/* Apply a circuit and measure at its end (marginal probabilities as in
+ * qgpu_probabilities, Eq.1): out[y] = sum over i with bits_Q(i) = y of |psi_i|^2 after the
+ * circuit, qubits[0] <-> bit 0 of y, 0 <= m <= 30, out = 2^m doubles (host). When the plan ends
+ * with a fused pass over the whole live state (single resident state, m <= 12, the histogram
+ * fits in shared memory) that pass accumulates the histogram from the amplitudes it stores
+ * (no extra read of the state); otherwise this is qgpu_apply_circuit + qgpu_probabilities.
+ * The state is left as qgpu_apply_circuit leaves it. Synchronises. Errors as both calls. */
+qgpu_status qgpu_apply_circuit_probabilities(qgpu_state* st, const qgpu_circuit* c, int m,
+                                             const int* qubits, double* out);
+
 /* ---- readout (synchronising) ------------------------------------------------------------ */
 
 /* Copy amplitudes [start, start+count) of the LOGICAL index space to host out[2*count]

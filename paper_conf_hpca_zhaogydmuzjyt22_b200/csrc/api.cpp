@@ -176,6 +176,12 @@ struct qgpu_state {
   std::vector<uint64_t> slice_seq;     // order of the slices' last D2H (0 = never stored)
   uint64_t store_seq = 0, unit_seq = 0;
   int last_unit = 0;                   // slices per slot group in the previous sweep
+  // measurement fused into the last pass (qgpu_apply_circuit_probabilities)
+  const Pass* meas_pass = nullptr;     // the pass that accumulates the histogram
+  int meas_m = 0;
+  int meas_pos[30] = {};
+  double* d_meas = nullptr;            // 2^kMeasMax doubles
+  bool meas_done = false;
 };
 
 namespace {
@@ -353,6 +359,17 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     if (bs == 2 || (bs == 1 && a.remaps)) a.nbuf = 3;
     if (tile_smem_bytes(a) > 227 * 1024) a.nbuf = 2;
     a.bstore = (a.nbuf == 3 && (bs == 2 || (bs == 1 && a.remaps))) ? 1 : 0;
+    if (st->meas_pass == &p && !a.bstore) {  // fused measurement, if its histogram fits in smem
+      TileArgs h = a;
+      h.hist = st->d_meas;
+      h.hm = st->meas_m;
+      for (int j = 0; j < st->meas_m; ++j) h.hpos[j] = st->meas_pos[j];
+      if (tile_smem_bytes(h) > 227 * 1024 && h.nbuf == 3) h.nbuf = 2;  // make room: double buffering
+      if (tile_smem_bytes(h) <= 227 * 1024) {
+        a = h;
+        st->meas_done = true;
+      }
+    }
     const int jit = st->cfg.jit;
     cudaError_t e = cudaErrorNotSupported;
     if (jit == 2 || (jit == 1 && p.k_out >= jit_min_bits())) {
@@ -1393,6 +1410,7 @@ qgpu_status qgpu_state_destroy(qgpu_state* st) {
   if (st->h_ops) cudaFreeHost(st->h_ops);
   if (st->d_scratch) cudaFree(st->d_scratch);
   if (st->d_zero) cudaFree(st->d_zero);
+  if (st->d_meas) cudaFree(st->d_meas);
   for (CachedPlan& cp : st->plans) {
     if (cp.d_blob) cudaFree(cp.d_blob);
     if (cp.h_blob) cudaFreeHost(cp.h_blob);
@@ -1496,7 +1514,13 @@ qgpu_status qgpu_apply_gate(qgpu_state* st, const double* U, int nt, const int* 
   }
 }
 
-qgpu_status qgpu_apply_circuit(qgpu_state* st, const qgpu_circuit* c) {
+}  // extern "C"
+
+namespace {
+constexpr int kMeasMax = 12;  // fused measurement: up to 2^12 buckets (32 KiB of shared memory)
+
+// qgpu_apply_circuit; meas_m >= 0 also asks the last fused pass to histogram qubits meas_q
+qgpu_status apply_circuit_impl(qgpu_state* st, const qgpu_circuit* c, int meas_m, const int* meas_q) {
   try {
     if (qgpu_status s = check_state(st)) return s;
     if (!c) return fail(QGPU_ERR_INVALID_ARG, "circuit is NULL");
@@ -1534,10 +1558,83 @@ qgpu_status qgpu_apply_circuit(qgpu_state* st, const qgpu_circuit* c) {
     st->map = hit->map_after;
     std::vector<const unsigned char*> ops(hit->passes.size());
     for (size_t i = 0; i < hit->passes.size(); ++i) ops[i] = hit->d_blob ? hit->d_blob + hit->off[i] : nullptr;
-    return exec_passes(st, hit->passes, ops);
+    // fused measurement: the last fused pass writes the final state (only zero-half
+    // materialisation may follow it), so it can histogram the amplitudes it stores
+    st->meas_pass = nullptr;
+    st->meas_done = false;
+    if (meas_m >= 0 && !st->host && st->shards.size() == 1 && meas_m <= kMeasMax) {
+      // the map at the end of the last fused pass: undo the qubit relabels (final SWAP layers)
+      // planned after it; zero-half materialisation passes do not change amplitudes either
+      QubitMap at = hit->map_after;
+      int last = -1;
+      for (int i = int(hit->passes.size()) - 1; i >= 0; --i) {
+        const Pass& pp = hit->passes[size_t(i)];
+        if (pp.kind == PK_TILE) { last = i; break; }
+        if (pp.kind == PK_RELABEL && pp.rel_a >= 0) { at.swap_positions(pp.rel_a, pp.rel_b); continue; }
+        if (pp.kind != PK_ZERO) break;
+      }
+      // fused only when every requested qubit sits on a bit that is uniform across a warp's
+      // stored amplitudes (tile-index or warp bits): then a tile adds one warp-reduced value per
+      // warp. Lane and register bits would need an add per amplitude (shared-memory f64 atomics
+      // are compare-and-swap loops) -- measured slower than re-reading the state, so those
+      // requests take the separate readout kernel.
+      if (last >= 0) {
+        const Pass& lp = hit->passes[size_t(last)];
+        uint64_t nonuni = 0;
+        for (int i = 0; i < std::min(5, lp.b); ++i) nonuni |= 1ull << lp.spos[i];  // lane bits
+        uint32_t a0 = 0;
+        for (const TileOp& op : lp.prog.ops)
+          if (op.kind == OP_REMAP) a0 = op.a0;  // the final register-bit mapping
+        for (int k = 0; k < lp.prog.nr; ++k) nonuni |= 1ull << lp.spos[(a0 >> (4 * k)) & 15];
+        for (int j = 0; j < meas_m; ++j) {
+          const int pos = at.pos[meas_q[j]];
+          if (pos >= 0 && (nonuni >> pos & 1)) last = -1;
+        }
+      }
+      if (last >= 0) {
+        if (!st->d_meas) CK(cudaMalloc(&st->d_meas, (size_t(8) << kMeasMax)));
+        CK(cudaMemsetAsync(st->d_meas, 0, size_t(8) << meas_m, st->stream));
+        st->meas_pass = &hit->passes[size_t(last)];
+        st->meas_m = meas_m;
+        for (int j = 0; j < meas_m; ++j) {
+          const int pos = at.pos[meas_q[j]];
+          st->meas_pos[j] = pos < 0 ? 63 : pos;  // never involved: the bit is 0 everywhere
+        }
+      }
+    }
+    qgpu_status s = exec_passes(st, hit->passes, ops);
+    st->meas_pass = nullptr;
+    return s;
   } catch (const std::exception& ex) {
     return fail(QGPU_ERR_OUT_OF_MEMORY, "exception: %s", ex.what());
   }
+}
+
+}  // namespace
+
+extern "C" {
+
+qgpu_status qgpu_apply_circuit(qgpu_state* st, const qgpu_circuit* c) {
+  return apply_circuit_impl(st, c, -1, nullptr);
+}
+
+qgpu_status qgpu_apply_circuit_probabilities(qgpu_state* st, const qgpu_circuit* c, int mq, const int* qubits,
+                                             double* out) {
+  if (qgpu_status s = check_state(st)) return s;
+  if (mq < 0 || mq > 30) return fail(QGPU_ERR_INVALID_ARG, "m=%d out of [0, 30]", mq);
+  if (!out || (mq > 0 && !qubits)) return fail(QGPU_ERR_INVALID_ARG, "NULL argument");
+  uint64_t seen = 0;
+  for (int j = 0; j < mq; ++j) {
+    const int q = qubits[j];
+    if (q < 0 || q >= st->n || (seen >> q & 1)) return fail(QGPU_ERR_INVALID_ARG, "bad qubit %d", q);
+    seen |= 1ull << q;
+  }
+  if (qgpu_status s = apply_circuit_impl(st, c, mq, qubits)) return s;
+  if (!st->meas_done) return qgpu_probabilities(st, mq, qubits, out);  // not fusable: read the state
+  CK(cudaMemcpyAsync(out, st->d_meas, (size_t(8) << mq), cudaMemcpyDeviceToHost, st->stream));
+  st->stats.d2h_bytes += size_t(8) << mq;
+  CK(cudaStreamSynchronize(st->stream));
+  return drain_timing(st);
 }
 
 qgpu_status qgpu_get_amplitudes_device(qgpu_state* st, uint64_t start, uint64_t count, double* dev_out) {

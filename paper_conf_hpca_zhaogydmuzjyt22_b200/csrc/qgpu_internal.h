@@ -150,6 +150,7 @@ struct Pass {
   // state is exactly zero and NOT materialised in memory -- on input (zin: loads read zeros
   // instead) and on output (zout: those amplitudes are not stored); PK_ZERO materialises zmask
   uint64_t zin = 0, zout = 0, zmask = 0;
+  int rel_a = -1, rel_b = -1;   // PK_RELABEL: the two physical positions whose qubits it swapped
 };
 
 struct PlanOptions {

@@ -1007,6 +1007,8 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
       }
       B.close();
       B.start(PK_RELABEL, xi, k_before);
+      B.cur.rel_a = pa;
+      B.cur.rel_b = pb;
       map.swap_positions(pa, pb);
       B.cur.k_out = map.kl;
       B.cur.count = 1;

@@ -96,6 +96,11 @@ struct TileArgs {
                            // copies (needs nbuf == 3), 0: per-thread stores from registers
   int remaps;              // the program contains REMAP / shared-memory ops
   int nmbar;               // mbarriers for warp-group remaps (JIT programs), 8 B each in smem
+  // measurement fused into the pass (qgpu_apply_circuit_probabilities): hist != nullptr adds
+  // |psi_i|^2 of every stored amplitude to hist[bucket(i)], bucket bit j = bit hpos[j] of i
+  double* hist;
+  int hm;
+  int hpos[30];
 };
 
 __device__ __forceinline__ double2 cmul(double2 a, double2 b) {
@@ -707,6 +712,9 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   double2* Chw = Cw + (size_t(nthr) >> 5) * a.npat;               // per-warp high-bit parts
   uint64_t* mbar = reinterpret_cast<uint64_t*>(Chw + (size_t(nthr) >> 5) * a.npat);
   if (threadIdx.x == 0) Body::init_mbar(mbar);
+  double* hsm = reinterpret_cast<double*>(mbar + a.nmbar);  // fused-measurement histogram
+  if (a.hist)
+    for (int i = threadIdx.x; i < (1 << a.hm); i += blockDim.x) hsm[i] = 0.0;
 
   {
     const int4* src = reinterpret_cast<const int4*>(a.blob);
@@ -857,6 +865,51 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
 #pragma unroll
       for (int r = 0; r < (1 << NR); ++r) v[r] = cmul(v[r], sc);
     }
+    if (a.hist && c.own) {  // fused measurement: the amplitudes are final and in registers
+      uint64_t pbh = 0;
+      SlotAddr sah{};
+      if constexpr (Body::kStatic) pbh = base | (mp.base & lowmask) | hiOff[mp.base >> l];
+      else sah = slot_addr<NR>(mp, hiOff, lowmask, l);
+      auto bucket = [&](int r) {
+        uint64_t idx;
+        if constexpr (Body::kStatic) idx = pbh + Body::kPF[r];
+        else idx = base | sah.at(r);
+        idx |= a.rank_base;
+        uint32_t bk = 0;
+        for (int j = 0; j < a.hm; ++j) bk |= uint32_t(idx >> a.hpos[j] & 1) << j;
+        return bk;
+      };
+      // Requested qubits on tile-index / warp bits only (the usual case) give one bucket per
+      // warp: sum in registers, reduce across the warp, one shared atomic. Otherwise group per
+      // slot: warp-uniform buckets reduce, mixed ones add lane by lane.
+      const uint32_t b0 = bucket(0);
+      bool same = true;
+      double acc = 0.0;
+#pragma unroll
+      for (int r = 0; r < (1 << NR); ++r) {
+        same = same && bucket(r) == b0;
+        acc += fma(v[r].x, v[r].x, v[r].y * v[r].y);
+      }
+      const uint32_t full = 0xffffffffu;
+      if (__all_sync(full, same) && __all_sync(full, b0 == __shfl_sync(full, b0, 0))) {
+#pragma unroll
+        for (int o = 16; o > 0; o >>= 1) acc += __shfl_xor_sync(full, acc, o);
+        if (c.lane == 0) atomicAdd(hsm + b0, acc);
+      } else {
+#pragma unroll
+        for (int r = 0; r < (1 << NR); ++r) {
+          const uint32_t bk = bucket(r);
+          double x = fma(v[r].x, v[r].x, v[r].y * v[r].y);
+          if (__all_sync(full, bk == __shfl_sync(full, bk, 0))) {
+#pragma unroll
+            for (int o = 16; o > 0; o >>= 1) x += __shfl_xor_sync(full, x, o);
+            if (c.lane == 0) atomicAdd(hsm + bk, x);
+          } else {
+            atomicAdd(hsm + bk, x);
+          }
+        }
+      }
+    }
     if (a.bstore) {
       if (c.own) {
         if constexpr (Body::kStatic) {
@@ -889,6 +942,11 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     if ((nbuf < 3 || Body::kGroupRemap) && a.remaps) __syncthreads();
   }
   if (a.bstore && warp == 0) bulk_wait_all();  // shared memory must outlive the bulk reads
+  if (a.hist) {
+    __syncthreads();
+    for (int i = threadIdx.x; i < (1 << a.hm); i += blockDim.x)
+      if (hsm[i] != 0.0) atomicAdd(a.hist + i, hsm[i]);
+  }
 }
 
 #endif  // __CUDACC__

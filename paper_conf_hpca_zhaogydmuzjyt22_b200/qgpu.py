@@ -22,7 +22,7 @@ STATUS = {0: "OK", 1: "INVALID_ARG", 2: "OUT_OF_MEMORY", 3: "UNSUPPORTED", 4: "P
 EXPORTS = [
     "qgpu_config_init", "qgpu_state_create", "qgpu_state_destroy", "qgpu_state_reset",
     "qgpu_set_amplitudes", "qgpu_synchronize", "qgpu_state_info", "qgpu_apply_gate",
-    "qgpu_apply_circuit", "qgpu_get_amplitudes", "qgpu_get_amplitudes_device",
+    "qgpu_apply_circuit", "qgpu_apply_circuit_probabilities", "qgpu_get_amplitudes", "qgpu_get_amplitudes_device",
     "qgpu_probabilities", "qgpu_circuit_from_qasm", "qgpu_circuit_info", "qgpu_circuit_destroy",
     "qgpu_circuit_reorder", "qgpu_circuit_plan", "qgpu_circuit_plan_text", "qgpu_circuit_jit_check", "qgpu_get_involvement", "qgpu_get_chunk_bitmap",
     "qgpu_get_schedule", "qgpu_get_qubit_map", "qgpu_get_stats", "qgpu_reset_stats",
@@ -83,7 +83,8 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
         "qgpu_config_init": [P], "qgpu_state_create": [I, P, P], "qgpu_state_destroy": [P],
         "qgpu_state_reset": [P], "qgpu_set_amplitudes": [P, P], "qgpu_synchronize": [P],
         "qgpu_state_info": [P, P, P, P], "qgpu_apply_gate": [P, P, I, P, I, P],
-        "qgpu_apply_circuit": [P, P], "qgpu_get_amplitudes": [P, U64, U64, P],
+        "qgpu_apply_circuit": [P, P], "qgpu_apply_circuit_probabilities": [P, P, I, P, P],
+        "qgpu_get_amplitudes": [P, U64, U64, P],
         "qgpu_get_amplitudes_device": [P, U64, U64, P], "qgpu_probabilities": [P, I, P, P],
         "qgpu_circuit_from_qasm": [ctypes.c_char_p, ctypes.c_size_t, P],
         "qgpu_circuit_info": [P, P, P], "qgpu_circuit_destroy": [P],
@@ -247,6 +248,15 @@ class State:
 
     def apply_circuit(self, circ: Circuit):
         _check(load().qgpu_apply_circuit(self._h, circ.handle))
+
+    def apply_circuit_probabilities(self, circ: Circuit, qubits: Sequence[int]) -> np.ndarray:
+        """Apply `circ` and return the marginal probabilities of `qubits` at its end (fused into
+        the last pass when possible; qgpu_apply_circuit_probabilities)."""
+        q = np.ascontiguousarray(qubits if len(qubits) else [0], dtype=np.int32)
+        out = np.empty(1 << len(qubits), dtype=np.float64)
+        _check(load().qgpu_apply_circuit_probabilities(self._h, circ.handle, len(qubits), q.ctypes.data,
+                                                       out.ctypes.data))
+        return out
 
     def amplitudes(self, start: int = 0, count: Optional[int] = None) -> np.ndarray:
         if count is None:
