@@ -713,8 +713,9 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   uint64_t* mbar = reinterpret_cast<uint64_t*>(Chw + (size_t(nthr) >> 5) * a.npat);
   if (threadIdx.x == 0) Body::init_mbar(mbar);
   double* hsm = reinterpret_cast<double*>(mbar + a.nmbar);  // fused-measurement histogram
-  if (a.hist)
-    for (int i = threadIdx.x; i < (1 << a.hm); i += blockDim.x) hsm[i] = 0.0;
+  if constexpr (Body::kHist)
+    if (a.hist)
+      for (int i = threadIdx.x; i < (1 << a.hm); i += blockDim.x) hsm[i] = 0.0;
 
   {
     const int4* src = reinterpret_cast<const int4*>(a.blob);
@@ -865,7 +866,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
 #pragma unroll
       for (int r = 0; r < (1 << NR); ++r) v[r] = cmul(v[r], sc);
     }
-    if (a.hist && c.own) {  // fused measurement: the amplitudes are final and in registers
+    if constexpr (Body::kHist) if (a.hist && c.own) {  // fused measurement: final amplitudes in registers
       uint64_t pbh = 0;
       SlotAddr sah{};
       if constexpr (Body::kStatic) pbh = base | (mp.base & lowmask) | hiOff[mp.base >> l];
@@ -942,10 +943,12 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     if ((nbuf < 3 || Body::kGroupRemap) && a.remaps) __syncthreads();
   }
   if (a.bstore && warp == 0) bulk_wait_all();  // shared memory must outlive the bulk reads
-  if (a.hist) {
-    __syncthreads();
-    for (int i = threadIdx.x; i < (1 << a.hm); i += blockDim.x)
-      if (hsm[i] != 0.0) atomicAdd(a.hist + i, hsm[i]);
+  if constexpr (Body::kHist) {
+    if (a.hist) {
+      __syncthreads();
+      for (int i = threadIdx.x; i < (1 << a.hm); i += blockDim.x)
+        if (hsm[i] != 0.0) atomicAdd(a.hist + i, hsm[i]);
+    }
   }
 }
 
