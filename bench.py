@@ -557,6 +557,17 @@ def run_ours(args):
     }
     if gfc is not None:
         line["gfc_compression"] = gfc
+    if sharded:
+        # global-local swap throughput per GPU (bytes this rank sent / CUDA-event time
+        # of its swap passes on the state's stream), against NVLink 5's 900 GB/s per direction
+        sb = statistics.mean(s["swap_bytes"] for s in stats)
+        sms = statistics.mean(s["swap_ms"] for s in stats)
+        sms_max = allreduce_max(sms, world, device)
+        line["swap"] = {"swaps_per_step": s0["swaps"], "bytes_sent_per_gpu_per_step": sb,
+                        "swap_ms_per_step_max_over_ranks": sms_max,
+                        "GBps_per_gpu": sb / (sms_max * 1e-3) / 1e9 if sms_max > 0 else None,
+                        "peak": 900.0, "peak_source": "NVLink 5 per direction (spec)",
+                        "frac": (sb / (sms_max * 1e-3) / 1e9) / 900.0 if sms_max > 0 else None}
     if args.host_slice_bits:
         # host-memory tier (NEXT-2): the state lives in pinned host memory; the bound is the
         # host link, so report link bytes / sweep time against the measured pinned-copy peak
