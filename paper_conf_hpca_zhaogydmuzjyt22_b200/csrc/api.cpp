@@ -1562,7 +1562,7 @@ qgpu_status apply_circuit_impl(qgpu_state* st, const qgpu_circuit* c, int meas_m
     // materialisation may follow it), so it can histogram the amplitudes it stores
     st->meas_pass = nullptr;
     st->meas_done = false;
-    if (meas_m >= 0 && !st->host && st->shards.size() == 1 && meas_m <= kMeasMax) {
+    if (meas_m >= 0 && st->g == 0 && meas_m <= kMeasMax) {  // single resident state only
       // the map at the end of the last fused pass: undo the qubit relabels (final SWAP layers)
       // planned after it; zero-half materialisation passes do not change amplitudes either
       QubitMap at = hit->map_after;
