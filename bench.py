@@ -527,6 +527,7 @@ def run_ours(args):
     line = {
         "metric": METRIC, "value": ms / 1e3, "unit": "s", "n_gpus": world, "steps": args.steps,
         "warmup": args.warmup, "ms_per_step": ms, "higher_is_better": False,
+        "ms_per_step_median": statistics.median(times), "ms_per_step_best": min(times),
         "scaling": "strong" if sharded else "weak",
         "vs_baseline": None, "dtype": "c128", "data": "synthetic (seeded generator, QASM text)",
         "config": {"workload": desc, "n_qubits": n, "gates": ngates, "reorder": args.reorder,
