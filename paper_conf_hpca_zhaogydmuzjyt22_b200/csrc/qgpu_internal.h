@@ -7,7 +7,8 @@
 //               a4  pass planner: cuts the order into consecutive fused HBM passes
 //   kernels.cu  a5-a9, a11  sm_100a kernels (pair, quad, diag, fused tile, gather, reduce)
 //   comm.cpp    a10 global-local swaps over NCCL (sharded mode)
-//   api.cpp     the C ABI (include/qgpu.h)
+//   exec.cpp    pass execution: resident passes, swaps, host-memory tier sweeps (NEXT-2/3)
+//   api.cpp     the C ABI (include/qgpu.h): state, plan cache, readout (state.h: shared types)
 #pragma once
 
 #include <cstdint>
