@@ -508,6 +508,11 @@ def run_ours(args):
     e2e_qubits = list(range(min(10, n)))
     e2e_times = []
     h2d = d2h = 0
+    for _ in range(args.warmup):  # untimed: the measurement pass's NVRTC variant compiles here
+        cc = q.Circuit(text)
+        st.reset()
+        st.apply_circuit_probabilities(cc, e2e_qubits)
+        cc.close()
     barrier(world)
     for k in range(max(1, args.steps)):
         torch.cuda.synchronize(device)

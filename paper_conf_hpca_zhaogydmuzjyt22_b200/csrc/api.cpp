@@ -556,7 +556,15 @@ qgpu_status qgpu_apply_gate(qgpu_state* st, const double* U, int nt, const int* 
 }  // extern "C"
 
 namespace {
-constexpr int kMeasMax = 12;  // fused measurement: up to 2^12 buckets (32 KiB of shared memory)
+constexpr int kMeasMax = 12;
+// QGPU_HACC=0 turns the per-slot fused measurement off (A/B against the separate readout)
+bool hacc_enabled() {
+  static const bool on = [] {
+    const char* e = std::getenv("QGPU_HACC");
+    return !(e && e[0] == '0');
+  }();
+  return on;
+}  // fused measurement: up to 2^12 buckets (32 KiB of shared memory)
 
 // qgpu_apply_circuit; meas_m >= 0 also asks the last fused pass to histogram qubits meas_q
 qgpu_status apply_circuit_impl(qgpu_state* st, const qgpu_circuit* c, int meas_m, const int* meas_q) {
@@ -612,12 +620,27 @@ qgpu_status apply_circuit_impl(qgpu_state* st, const qgpu_circuit* c, int meas_m
         if (pp.kind == PK_RELABEL && pp.rel_a >= 0) { at.swap_positions(pp.rel_a, pp.rel_b); continue; }
         if (pp.kind != PK_ZERO) break;
       }
-      // fused only when every requested qubit sits on a bit that is uniform across a warp's
-      // stored amplitudes (tile-index or warp bits): then a tile adds one warp-reduced value per
-      // warp. Lane and register bits would need an add per amplitude (shared-memory f64 atomics
-      // are compare-and-swap loops) -- measured slower than re-reading the state, so those
-      // requests take the separate readout kernel.
+      // how the last pass histograms (TileArgs::hacc): every requested qubit on a tile bit of
+      // the final mapping -> a slot's bucket is the same in every tile: per-slot register sums,
+      // one add per slot at the end of the kernel (1); all on bits uniform across a warp's
+      // stored amplitudes (tile-index or warp bits) -> one warp-reduced add per warp and tile
+      // (0); otherwise lane / register bits mixed with tile-index bits -> per-warp private
+      // histograms in shared memory, plain adds by the lanes whose buckets differ (2; shared-
+      // memory f64 atomics are compare-and-swap loops, measured slower than re-reading the
+      // state). If the private histograms do not fit in shared memory, the separate readout.
+      st->meas_hacc = 0;
       if (last >= 0) {
+        const Pass& lp = hit->passes[size_t(last)];
+        uint64_t tilebits = 0;
+        for (int i = 0; i < lp.b; ++i) tilebits |= 1ull << lp.spos[i];
+        bool on_tile = true;
+        for (int j = 0; j < meas_m; ++j) {
+          const int pos = at.pos[meas_q[j]];
+          if (pos >= 0 && !(tilebits >> pos & 1)) on_tile = false;
+        }
+        if (on_tile && meas_m > 0 && hacc_enabled()) st->meas_hacc = 1;
+      }
+      if (last >= 0 && !st->meas_hacc) {
         const Pass& lp = hit->passes[size_t(last)];
         uint64_t nonuni = 0;
         for (int i = 0; i < std::min(5, lp.b); ++i) nonuni |= 1ull << lp.spos[i];  // lane bits
@@ -625,9 +648,23 @@ qgpu_status apply_circuit_impl(qgpu_state* st, const qgpu_circuit* c, int meas_m
         for (const TileOp& op : lp.prog.ops)
           if (op.kind == OP_REMAP) a0 = op.a0;  // the final register-bit mapping
         for (int k = 0; k < lp.prog.nr; ++k) nonuni |= 1ull << lp.spos[(a0 >> (4 * k)) & 15];
+        bool uni = true;
         for (int j = 0; j < meas_m; ++j) {
           const int pos = at.pos[meas_q[j]];
-          if (pos >= 0 && (nonuni >> pos & 1)) last = -1;
+          if (pos >= 0 && (nonuni >> pos & 1)) uni = false;
+        }
+        if (!uni) {
+          if (hacc_enabled()) {  // per-warp private histograms (mode 2)
+            st->meas_hacc = 2;
+            st->meas_hlred = 0;
+            for (int k = 0; k < std::min(5, lp.b); ++k) {
+              bool req = false;
+              for (int j = 0; j < meas_m; ++j) req = req || at.pos[meas_q[j]] == lp.spos[k];
+              if (!req) st->meas_hlred |= 1u << k;
+            }
+          } else {
+            last = -1;
+          }
         }
       }
       if (last >= 0) {

@@ -161,6 +161,8 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
       TileArgs h = a;
       h.hist = st->d_meas;
       h.hm = st->meas_m;
+      h.hacc = st->meas_hacc;
+      h.hlred = st->meas_hlred;
       for (int j = 0; j < st->meas_m; ++j) h.hpos[j] = st->meas_pos[j];
       if (tile_smem_bytes(h) > 227 * 1024 && h.nbuf == 3) h.nbuf = 2;  // make room: double buffering
       if (tile_smem_bytes(h) <= 227 * 1024) {

@@ -547,7 +547,7 @@ size_t tile_smem_bytes(const TileArgs& a) {
   const size_t nh = size_t(1) << (a.b - a.l);
   const size_t nwarps = size_t(1) << a.nw;
   return size_t(a.nbuf) * (size_t(1) << a.b) * 16 + ((nh + 1) & ~size_t(1)) * 8 + size_t(a.blob_bytes) +
-         2 * nwarps * size_t(a.npat) * 16 + size_t(a.nmbar) * 8 + 16 + (a.hist ? (size_t(8) << a.hm) : 0);
+         2 * nwarps * size_t(a.npat) * 16 + size_t(a.nmbar) * 8 + 16 + (a.hist ? (size_t(8) << a.hm) * (a.hacc == 2 ? nwarps : 1) : 0);
 }
 
 cudaError_t launch_pair(cudaStream_t st, const PairArgs& a, bool shfl) {

@@ -177,6 +177,8 @@ struct qgpu_state {
   const Pass* meas_pass = nullptr;     // the pass that accumulates the histogram
   int meas_m = 0;
   int meas_pos[30] = {};
+  int meas_hacc = 0;                   // TileArgs::hacc (see apply_circuit_impl)
+  uint32_t meas_hlred = 0;             // TileArgs::hlred: lane bits not requested
   double* d_meas = nullptr;            // 2^kMeasMax doubles
   bool meas_done = false;
 };

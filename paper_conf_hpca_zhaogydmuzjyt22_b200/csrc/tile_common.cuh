@@ -101,6 +101,15 @@ struct TileArgs {
   double* hist;
   int hm;
   int hpos[30];
+  // 1: every requested qubit sits on a tile bit of the final mapping (or is never involved), so
+  // an owned slot's bucket is the same in every tile: each thread sums |psi|^2 per slot in
+  // registers across its tiles and adds to the histogram once at the end of the kernel.
+  // 2: requested qubits on lane / register bits mixed with tile-index bits: one private
+  // histogram per warp in shared memory (2^hm doubles each); per slot the lanes first sum over
+  // the unrequested lane bits (hlred) with shuffles, then the remaining lanes -- whose buckets
+  // differ -- add without atomics. 0: requested bits uniform across a warp's slots.
+  int hacc;
+  uint32_t hlred;
 };
 
 __device__ __forceinline__ double2 cmul(double2 a, double2 b) {
@@ -714,8 +723,10 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   if (threadIdx.x == 0) Body::init_mbar(mbar);
   double* hsm = reinterpret_cast<double*>(mbar + a.nmbar);  // fused-measurement histogram
   if constexpr (Body::kHist)
-    if (a.hist)
-      for (int i = threadIdx.x; i < (1 << a.hm); i += blockDim.x) hsm[i] = 0.0;
+    if (a.hist) {
+      const int hn = (a.hacc == 2 ? (blockDim.x >> 5) : 1) << a.hm;
+      for (int i = threadIdx.x; i < hn; i += blockDim.x) hsm[i] = 0.0;
+    }
 
   {
     const int4* src = reinterpret_cast<const int4*>(a.blob);
@@ -767,6 +778,14 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   if (tile < a.ntiles) issue_own_loads<NR, Body>(bufs, a, mp0, sa0, base_next, zm0, c.own);
   int k = 0;
   uint64_t cur_hi = ~0ull;
+  double hacc[1 << NR];   // fused measurement with a.hacc: per-slot sums over this thread's tiles
+  Mapping mpf = mp0;      // the final mapping (the same after every tile)
+  uint32_t hbk[1 << NR];  // fused measurement with a.hacc == 2: bucket bits of each slot (base 0)
+  bool hbk_set = false;
+  if constexpr (Body::kHist) {
+#pragma unroll
+    for (int r = 0; r < (1 << NR); ++r) hacc[r] = 0.0;
+  }
   for (uint64_t it = 0; tile < a.ntiles; ++it) {
     double2* s = bufs + k * T;
     const int kn = (k + 1 == nbuf) ? 0 : k + 1;
@@ -866,7 +885,44 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
 #pragma unroll
       for (int r = 0; r < (1 << NR); ++r) v[r] = cmul(v[r], sc);
     }
-    if constexpr (Body::kHist) if (a.hist && c.own) {  // fused measurement: final amplitudes in registers
+    if constexpr (Body::kHist) if (a.hist && c.own && a.hacc == 1) {  // buckets fixed per slot
+#pragma unroll
+      for (int r = 0; r < (1 << NR); ++r) hacc[r] += fma(v[r].x, v[r].x, v[r].y * v[r].y);
+      mpf = mp;
+    }
+    if constexpr (Body::kHist) if (a.hist && a.hacc == 2) {
+      // per-warp private histogram: a slot's bucket = its bits at base 0 (fixed per thread, the
+      // final mapping is the same in every tile) | the tile base's bits (uniform)
+      if (!hbk_set) {
+        hbk_set = true;
+        uint64_t pbh = 0;
+        SlotAddr sah{};
+        if constexpr (Body::kStatic) pbh = (mp.base & lowmask) | hiOff[mp.base >> l];
+        else sah = slot_addr<NR>(mp, hiOff, lowmask, l);
+#pragma unroll
+        for (int r = 0; r < (1 << NR); ++r) {
+          uint64_t idx;
+          if constexpr (Body::kStatic) idx = pbh + Body::kPF[r];
+          else idx = sah.at(r);
+          uint32_t bk = 0;
+          for (int j = 0; j < a.hm; ++j) bk |= uint32_t(idx >> a.hpos[j] & 1) << j;
+          hbk[r] = bk;
+        }
+      }
+      uint32_t bt = 0;
+      for (int j = 0; j < a.hm; ++j) bt |= uint32_t(gbase >> a.hpos[j] & 1) << j;
+      double* hw = hsm + (size_t(warp) << a.hm);
+      const bool writer = (uint32_t(lane) & a.hlred) == 0u;
+#pragma unroll
+      for (int r = 0; r < (1 << NR); ++r) {
+        double x = fma(v[r].x, v[r].x, v[r].y * v[r].y);
+#pragma unroll
+        for (int k = 0; k < 5; ++k)
+          if (a.hlred >> k & 1) x += __shfl_xor_sync(0xffffffffu, x, 1 << k);
+        if (writer) hw[hbk[r] | bt] += x;
+      }
+    }
+    if constexpr (Body::kHist) if (a.hist && c.own && a.hacc == 0) {  // fused measurement: final amplitudes in registers
       uint64_t pbh = 0;
       SlotAddr sah{};
       if constexpr (Body::kStatic) pbh = base | (mp.base & lowmask) | hiOff[mp.base >> l];
@@ -945,9 +1001,30 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   if (a.bstore && warp == 0) bulk_wait_all();  // shared memory must outlive the bulk reads
   if constexpr (Body::kHist) {
     if (a.hist) {
+      if (a.hacc == 1 && c.own) {
+        // bucket of slot r: its tile-local index under the final mapping (tile base bits are not
+        // requested, so base = 0); one shared-memory add per slot and thread
+        uint64_t pbh = 0;
+        SlotAddr sah{};
+        if constexpr (Body::kStatic) pbh = (mpf.base & lowmask) | hiOff[mpf.base >> l];
+        else sah = slot_addr<NR>(mpf, hiOff, lowmask, l);
+#pragma unroll
+        for (int r = 0; r < (1 << NR); ++r) {
+          uint64_t idx;
+          if constexpr (Body::kStatic) idx = pbh + Body::kPF[r];
+          else idx = sah.at(r);
+          uint32_t bk = 0;
+          for (int j = 0; j < a.hm; ++j) bk |= uint32_t(idx >> a.hpos[j] & 1) << j;
+          if (hacc[r] != 0.0) atomicAdd(hsm + bk, hacc[r]);
+        }
+      }
       __syncthreads();
-      for (int i = threadIdx.x; i < (1 << a.hm); i += blockDim.x)
-        if (hsm[i] != 0.0) atomicAdd(a.hist + i, hsm[i]);
+      const int hw = a.hacc == 2 ? int(blockDim.x >> 5) : 1;
+      for (int i = threadIdx.x; i < (1 << a.hm); i += blockDim.x) {
+        double t = 0.0;
+        for (int w = 0; w < hw; ++w) t += hsm[(size_t(w) << a.hm) + i];
+        if (t != 0.0) atomicAdd(a.hist + i, t);
+      }
     }
   }
 }

@@ -76,3 +76,40 @@ def test_fused_measurement_reads_no_state(q):
         s.probabilities([6, 7, 8])
         k_plain = s.stats()["kernels_launched"]
     assert k_fused < k_plain
+
+
+@pytest.mark.parametrize("name", ["qft0", "qftx", "qaoa", "rqc", "partial"])
+@pytest.mark.parametrize("qsel", ["low", "many", "mixed", "high"])
+def test_fused_measurement_jit_vs_oracle(q, name, qsel):
+    """jit=2: the NVRTC-specialised measurement variant (compile-time slot offsets), including
+    the per-slot register sums used when every requested qubit is a tile bit of the last pass."""
+    c = CIRCS[name]()
+    n = c.n if name != "partial" else 14
+    text = c.qasm()
+    qubits = {"low": [0, 1, 2, 3], "high": list(range(n - 1, n - 6, -1)), "mixed": [5, 0, n - 1, 3, 7],
+              "many": list(range(12))[::-1]}[qsel]
+    with q.State(n, fuse_bits=12, jit=2) as s:
+        p = s.apply_circuit_probabilities(q.Circuit(text), qubits)
+        p2 = s.probabilities(qubits)
+    psi = osv.simulate(text) if n == c.n else np.kron(np.eye(1 << (n - c.n))[:, 0], osv.simulate(text))
+    ref = osv.probabilities(psi, n, qubits)
+    assert np.abs(p - ref).max() <= 1e-12
+    assert np.abs(p - p2).max() <= 1e-12
+
+
+@pytest.mark.parametrize("jit", [0, 2])
+def test_fused_measurement_lane_register_bits_read_no_state(q, jit):
+    """Qubits 0..9 of QFT_18 sit on lane, register and tile-index bits of the last pass: per-warp
+    private histograms (or per-slot register sums) in the pass, so no readout kernel is launched."""
+    text = wc.qft(18).qasm()
+    qubits = list(range(10))
+    with q.State(18, jit=jit) as s:
+        p = s.apply_circuit_probabilities(q.Circuit(text), qubits)
+        k_fused = s.stats()["kernels_launched"]
+        s.reset()
+        s.apply_circuit(q.Circuit(text))
+        p2 = s.probabilities(qubits)
+        k_plain = s.stats()["kernels_launched"]
+    assert k_fused < k_plain
+    assert np.abs(p - p2).max() <= 1e-12
+    assert np.abs(p - 2.0 ** -10).max() <= 1e-12  # QFT|0> is uniform: every marginal is 2^-10
