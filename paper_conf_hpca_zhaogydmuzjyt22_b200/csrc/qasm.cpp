@@ -7,6 +7,7 @@
 #include <cstdlib>
 #include <cstring>
 #include <map>
+#include <unordered_map>
 #include <string>
 #include <string_view>
 #include <vector>
@@ -57,7 +58,14 @@ class Lexer {
           }
         }
         t.k = T_NUM; t.s = std::string_view(s, size_t(p_ - s));
-        t.v = std::strtod(std::string(t.s).c_str(), nullptr);
+        // plain integers (qubit indices, most numbers in a circuit) exactly, without strtod
+        bool integral = t.s.size() <= 15;
+        uint64_t iv = 0;
+        for (char ch : t.s) {
+          if (ch < '0' || ch > '9') { integral = false; break; }
+          iv = iv * 10 + uint64_t(ch - '0');
+        }
+        t.v = integral ? double(iv) : std::strtod(std::string(t.s).c_str(), nullptr);
       } else if (c == '"') {
         const char* s = ++p_;
         while (p_ < e_ && *p_ != '"' && *p_ != '\n') ++p_;
@@ -222,23 +230,54 @@ class Parser {
     return all;
   }
 
+  // One gate statement. Its matrix depends only on the gate name and the parameter text (the
+  // expressions use constants only), so statements that repeat both -- most of a generated
+  // circuit -- reuse the matrix and flags built the first time (memo_, per parse).
   void gate(const Tok& t, Circuit* c) {
     int np, nq, nc;
     cplx U[16];
-    const std::string name(t.s);
-    if (!gate_matrix(name, {}, &np, &nq, &nc, U, false))
-      fail(t, "unknown gate '" + std::string(t.s) + "'", QGPU_ERR_UNSUPPORTED);
-    std::vector<double> p;
+    // memo key: the name and the raw source text of the parameter list
+    size_t close = i_;
     if (is('(')) {
-      next();
-      if (!is(')')) {
-        p.push_back(expr());
-        while (is(',')) { next(); p.push_back(expr()); }
+      int depth = 0;
+      for (close = i_; t_[close].k != T_EOF; ++close) {
+        if (t_[close].k == T_SYM && t_[close].s[0] == '(') ++depth;
+        if (t_[close].k == T_SYM && t_[close].s[0] == ')' && --depth == 0) break;
       }
-      expect(')');
     }
-    if (int(p.size()) != np)
-      fail(t, std::string(t.s) + " takes " + std::to_string(np) + " parameters", QGPU_ERR_INVALID_ARG);
+    std::string key(t.s);
+    if (close != i_ && t_[close].k != T_EOF)
+      key.append(t_[i_].s.data(), size_t(t_[close].s.data() - t_[i_].s.data()) + 1);
+    const bool memo_ok = close == i_ || t_[close].k != T_EOF;  // an unclosed list: parse, fail
+    auto hit = memo_ok ? memo_.find(key) : memo_.end();
+    const Memo* m = nullptr;
+    if (hit != memo_.end()) {
+      m = &hit->second;
+      i_ = close == i_ ? i_ : close + 1;  // the parameter list was evaluated before
+      np = m->np; nq = m->nq; nc = m->nc;
+    } else {
+      const std::string name(t.s);
+      if (!gate_matrix(name, {}, &np, &nq, &nc, U, false))
+        fail(t, "unknown gate '" + std::string(t.s) + "'", QGPU_ERR_UNSUPPORTED);
+      std::vector<double> p;
+      if (is('(')) {
+        next();
+        if (!is(')')) {
+          p.push_back(expr());
+          while (is(',')) { next(); p.push_back(expr()); }
+        }
+        expect(')');
+      }
+      if (int(p.size()) != np)
+        fail(t, std::string(t.s) + " takes " + std::to_string(np) + " parameters", QGPU_ERR_INVALID_ARG);
+      Memo e;
+      e.np = np; e.nq = nq; e.nc = nc;
+      gate_matrix(name, p, &np, &nq, &nc, e.U, true);
+      const int nt = nq - nc;
+      e.diag = is_diagonal(e.U, nt);
+      e.swap = is_swap_matrix(e.U, nt);
+      m = &memo_.emplace(std::move(key), e).first->second;  // unordered_map: stable addresses
+    }
     std::vector<std::vector<int>> ops{operand()};
     while (is(',')) { next(); ops.push_back(operand()); }
     expect(';');
@@ -248,7 +287,7 @@ class Parser {
     for (auto& o : ops) width = std::max(width, o.size());
     for (auto& o : ops)
       if (o.size() != 1 && o.size() != width) fail(t, "register size mismatch", QGPU_ERR_INVALID_ARG);
-    gate_matrix(name, p, &np, &nq, &nc, U, true);
+    (void)U;
     const int nt = nq - nc;
     for (size_t k = 0; k < width; ++k) {
       Gate g;
@@ -262,9 +301,9 @@ class Parser {
         if (j < nc) g.cmask |= 1ull << q;
         else g.t[j - nc] = q;
       }
-      for (int i = 0; i < (1 << (2 * nt)); ++i) g.U[i] = U[i];
-      g.diag = is_diagonal(g.U, nt);
-      g.relabel = (g.cmask == 0 && is_swap_matrix(g.U, nt));
+      for (int i = 0; i < (1 << (2 * nt)); ++i) g.U[i] = m->U[i];
+      g.diag = m->diag;
+      g.relabel = (g.cmask == 0 && m->swap);
       c->gates.push_back(g);
     }
   }
@@ -273,6 +312,12 @@ class Parser {
   size_t i_ = 0;
   int n_ = 0;
   std::map<std::string, std::pair<int, int>, std::less<>> regs_;
+  struct Memo {
+    int np, nq, nc;
+    bool diag, swap;
+    cplx U[16];
+  };
+  std::unordered_map<std::string, Memo> memo_;
 };
 
 }  // namespace
@@ -282,6 +327,7 @@ qgpu_status parse_qasm(const char* text, size_t len, Circuit* out, std::string* 
     Lexer lx(text, len);
     Parser ps(lx.run());
     Circuit c;
+    c.gates.reserve(len / 12 + 16);  // a gate statement takes >= ~12 source bytes in practice
     ps.run(&c);
     *out = std::move(c);
     return QGPU_OK;

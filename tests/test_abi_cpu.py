@@ -177,6 +177,14 @@ def test_parse_errors(q):
     with pytest.raises(q.QgpuError) as e:
         q.Circuit("OPENQASM 2.0;\nqreg q[2];\ncx q[0],q[0];\n")
     assert e.value.kind == "INVALID_ARG"
+    # statements that repeat a gate name (the parser reuses the matrix of an identical name +
+    # parameter text) still get every check of their own
+    for text, kind in (("h q[0];\nh(", "PARSE"), ("rx(0.1) q[0];\nrx(0.1 q[0];", "PARSE"),
+                       ("rx(0.1) q[0];\nrx(0.1) q[0],q[1];", "INVALID_ARG"),
+                       ("h q[0];\nh(0.1) q[0];", "INVALID_ARG"), ("cx q[0],q[1];\ncx q[1],q[1];", "INVALID_ARG")):
+        with pytest.raises(q.QgpuError) as e:
+            q.Circuit("OPENQASM 2.0;\nqreg q[2];\n" + text + "\n")
+        assert e.value.kind == kind, text
     c = q.Circuit("OPENQASM 2.0;\nqreg a[2];\nqreg b[3];\ncreg c[5];\nh b;\ncx a[1],b[2];\n"
                   "rx(-pi/2^2 + 2*sin(pi/6)) a[0];\nbarrier a;\nmeasure a[0] -> c[0];\n")
     assert c.info() == (5, 5)
