@@ -672,8 +672,21 @@ qgpu_status apply_circuit_impl(qgpu_state* st, const qgpu_circuit* c, int meas_m
         CK(cudaMemsetAsync(st->d_meas, 0, size_t(8) << meas_m, st->stream));
         st->meas_pass = &hit->passes[size_t(last)];
         st->meas_m = meas_m;
+        // bucket bit order inside the kernel: requested lane bits first, in lane order, so the
+        // lanes of a warp add to consecutive shared-memory words (mode 2 without bank
+        // conflicts); meas_perm maps a kernel bucket bit back to the caller's bit
+        int jj = 0;
+        const Pass& lp = hit->passes[size_t(last)];
+        for (int k = 0; k < std::min(5, lp.b); ++k)
+          for (int j = 0; j < meas_m; ++j)
+            if (at.pos[meas_q[j]] == lp.spos[k]) st->meas_perm[jj++] = j;
         for (int j = 0; j < meas_m; ++j) {
-          const int pos = at.pos[meas_q[j]];
+          bool lane = false;
+          for (int k = 0; k < std::min(5, lp.b); ++k) lane = lane || at.pos[meas_q[j]] == lp.spos[k];
+          if (!lane) st->meas_perm[jj++] = j;
+        }
+        for (int j = 0; j < meas_m; ++j) {
+          const int pos = at.pos[meas_q[st->meas_perm[j]]];
           st->meas_pos[j] = pos < 0 ? 63 : pos;  // never involved: the bit is 0 everywhere
         }
       }
@@ -710,6 +723,16 @@ qgpu_status qgpu_apply_circuit_probabilities(qgpu_state* st, const qgpu_circuit*
   CK(cudaMemcpyAsync(out, st->d_meas, (size_t(8) << mq), cudaMemcpyDeviceToHost, st->stream));
   st->stats.d2h_bytes += size_t(8) << mq;
   CK(cudaStreamSynchronize(st->stream));
+  bool ident = true;
+  for (int j = 0; j < mq; ++j) ident = ident && st->meas_perm[j] == j;
+  if (!ident) {  // kernel bucket bit j' holds the caller's bit meas_perm[j']
+    std::vector<double> k(out, out + (size_t(1) << mq));
+    for (uint64_t y = 0; y < (uint64_t(1) << mq); ++y) {
+      uint64_t yk = 0;
+      for (int j = 0; j < mq; ++j) yk |= ((y >> st->meas_perm[j]) & 1) << j;
+      out[y] = k[yk];
+    }
+  }
   return drain_timing(st);
 }
 

@@ -179,7 +179,8 @@ bool jit_cubin_cached(const std::string& src, std::string* cubin, std::string* l
   return true;
 }
 
-std::string tile_jit_source(const Pass& p, bool hist) {
+std::string tile_jit_source(const Pass& p, int hist_mode) {
+  const bool hist = hist_mode >= 0;
   const TileProgram& P = p.prog;
   const int NR = P.nr;
   // compile-time slot tables of a mapping: tile-local offset J[r] and physical offset Pq[r]
@@ -263,6 +264,7 @@ std::string tile_jit_source(const Pass& p, bool hist) {
   hdr << "  static constexpr uint32_t kZW0 = " << zw_start << "u;\n";
   hdr << "  static constexpr bool kStatic = true;\n";
   hdr << "  static constexpr bool kHist = " << (hist ? "true" : "false") << ";\n";
+  hdr << "  static constexpr int kHistMode = " << (hist ? hist_mode : 0) << ";\n";
   {  // tile positions as runs of consecutive bits (tile index -> base address at compile time)
     std::vector<int> rp, rl;
     for (int i = 0; i < p.b;) {
@@ -597,11 +599,12 @@ cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, s
                             double* compile_ms) {
   if (!jit_available(nullptr)) return cudaErrorNotSupported;
   JitLib& L = lib();
-  const bool hist = a.hist != nullptr;  // fused measurement: its own variant, not cached in p
-  CUfunction fn = hist ? nullptr : static_cast<CUfunction>(p.jit_fn);
+  const bool hist = a.hist != nullptr;  // fused measurement: its own variant
+  const int hmode = hist ? std::clamp(a.hacc, 0, 2) : -1;
+  CUfunction fn = static_cast<CUfunction>(hist ? p.jit_fn_hist[hmode] : p.jit_fn);
   std::string src;
   if (!fn) {
-    src = tile_jit_source(p, hist);
+    src = tile_jit_source(p, hmode);
     std::lock_guard<std::mutex> g(L.mu);
     auto it = L.cache.find(src);
     if (it != L.cache.end()) fn = it->second;
@@ -625,7 +628,7 @@ cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, s
     std::lock_guard<std::mutex> g(L.mu);
     L.cache.emplace(src, fn);
   }
-  if (!hist) p.jit_fn = fn;
+  (hist ? p.jit_fn_hist[hmode] : p.jit_fn) = fn;  // later launches skip source generation and lookup
   const unsigned threads = 32u << a.nw;
   int bps = 1;
   if (L.occupancy(&bps, fn, int(threads), smem) != CUDA_SUCCESS || bps < 1) bps = 1;

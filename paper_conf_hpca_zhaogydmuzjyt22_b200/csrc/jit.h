@@ -11,7 +11,7 @@
 namespace qgpu {
 
 // CUDA source of the specialised kernel for one tile pass (host-only, deterministic).
-std::string tile_jit_source(const Pass& p, bool hist = false);  // hist: fused-measurement variant
+std::string tile_jit_source(const Pass& p, int hist_mode = -1);  // >= 0: fused-measurement variant (TileArgs::hacc)
 // Compile source to an sm_100a cubin with NVRTC (works without a GPU).
 bool jit_compile_cubin(const std::string& src, std::string* cubin, std::string* log);
 // Same, through the on-disk cubin cache ($QGPU_JIT_CACHE or <lib dir>/build/jitcache).

@@ -171,6 +171,7 @@ struct InterpBody {
   static constexpr uint32_t kZW0 = 0u;
   static constexpr bool kStatic = false;  // mappings read from the program at run time
   static constexpr bool kHist = true;     // fused measurement decided at run time (a.hist)
+  static constexpr int kHistMode = -1;    // its epilogue too (a.hacc)
   static constexpr int kNsrun = -1;       // tile positions read from the arguments
   static constexpr int kSrunPos[1] = {0};
   static constexpr int kSrunLen[1] = {0};

@@ -146,6 +146,7 @@ struct Pass {
   int swap_global[8], swap_local[8];
   int kg_from = 0;              // activation pass
   mutable void* jit_fn = nullptr;  // specialised kernel, resolved at the first launch
+  mutable void* jit_fn_hist[3] = {nullptr, nullptr, nullptr};  // fused-measurement variants, per mode
   uint64_t unfused_bytes = 0;   // bytes the pass's gates would move one gate per pass
   // zero-position skipping (tile passes): physical positions p whose bit-p = 1 half of the live
   // state is exactly zero and NOT materialised in memory -- on input (zin: loads read zeros

@@ -177,6 +177,7 @@ struct qgpu_state {
   const Pass* meas_pass = nullptr;     // the pass that accumulates the histogram
   int meas_m = 0;
   int meas_pos[30] = {};
+  int meas_perm[30] = {};              // kernel bucket bit j -> the caller's qubit index j
   int meas_hacc = 0;                   // TileArgs::hacc (see apply_circuit_impl)
   uint32_t meas_hlred = 0;             // TileArgs::hlred: lane bits not requested
   double* d_meas = nullptr;            // 2^kMeasMax doubles

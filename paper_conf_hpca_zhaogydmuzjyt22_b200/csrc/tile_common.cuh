@@ -722,9 +722,11 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   uint64_t* mbar = reinterpret_cast<uint64_t*>(Chw + (size_t(nthr) >> 5) * a.npat);
   if (threadIdx.x == 0) Body::init_mbar(mbar);
   double* hsm = reinterpret_cast<double*>(mbar + a.nmbar);  // fused-measurement histogram
+  // the fused-measurement epilogue: compile-time in NVRTC variants, else TileArgs::hacc
+  const int hmode = Body::kHistMode >= 0 ? Body::kHistMode : a.hacc;
   if constexpr (Body::kHist)
     if (a.hist) {
-      const int hn = (a.hacc == 2 ? (blockDim.x >> 5) : 1) << a.hm;
+      const int hn = (hmode == 2 ? (blockDim.x >> 5) : 1) << a.hm;
       for (int i = threadIdx.x; i < hn; i += blockDim.x) hsm[i] = 0.0;
     }
 
@@ -780,7 +782,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   uint64_t cur_hi = ~0ull;
   double hacc[1 << NR];   // fused measurement with a.hacc: per-slot sums over this thread's tiles
   Mapping mpf = mp0;      // the final mapping (the same after every tile)
-  uint32_t hbk[1 << NR];  // fused measurement with a.hacc == 2: bucket bits of each slot (base 0)
+  uint32_t hb0 = 0, hrb[4] = {0u, 0u, 0u, 0u};  // hmode == 2: bucket parts (thread, register bits)
   bool hbk_set = false;
   if constexpr (Body::kHist) {
 #pragma unroll
@@ -885,44 +887,75 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
 #pragma unroll
       for (int r = 0; r < (1 << NR); ++r) v[r] = cmul(v[r], sc);
     }
-    if constexpr (Body::kHist) if (a.hist && c.own && a.hacc == 1) {  // buckets fixed per slot
+    if constexpr (Body::kHist) if (a.hist && c.own && hmode == 1) {  // buckets fixed per slot
 #pragma unroll
       for (int r = 0; r < (1 << NR); ++r) hacc[r] += fma(v[r].x, v[r].x, v[r].y * v[r].y);
       mpf = mp;
     }
-    if constexpr (Body::kHist) if (a.hist && a.hacc == 2) {
-      // per-warp private histogram: a slot's bucket = its bits at base 0 (fixed per thread, the
-      // final mapping is the same in every tile) | the tile base's bits (uniform)
+    if constexpr (Body::kHist) if (a.hist && hmode == 2) {
+      // per-warp private histogram. Bucket extraction is linear in the index bits, so a slot's
+      // bucket = hb0 (thread part at tile base 0) | hrb[k] for each set register bit k of r |
+      // bt (the tile base's bits, uniform); the final mapping is the same in every tile
       if (!hbk_set) {
         hbk_set = true;
         uint64_t pbh = 0;
         SlotAddr sah{};
         if constexpr (Body::kStatic) pbh = (mp.base & lowmask) | hiOff[mp.base >> l];
         else sah = slot_addr<NR>(mp, hiOff, lowmask, l);
-#pragma unroll
-        for (int r = 0; r < (1 << NR); ++r) {
-          uint64_t idx;
-          if constexpr (Body::kStatic) idx = pbh + Body::kPF[r];
-          else idx = sah.at(r);
+        auto bkt = [&](uint64_t idx) {
           uint32_t bk = 0;
           for (int j = 0; j < a.hm; ++j) bk |= uint32_t(idx >> a.hpos[j] & 1) << j;
-          hbk[r] = bk;
+          return bk;
+        };
+        if constexpr (Body::kStatic) hb0 = bkt(pbh);
+        else hb0 = bkt(sah.pb);
+#pragma unroll
+        for (int k = 0; k < NR; ++k) {
+          if constexpr (Body::kStatic) hrb[k] = bkt(Body::kPF[1 << k]);
+          else hrb[k] = bkt(sah.prb[k]);
         }
       }
-      uint32_t bt = 0;
+      uint32_t bt = hb0;
       for (int j = 0; j < a.hm; ++j) bt |= uint32_t(gbase >> a.hpos[j] & 1) << j;
       double* hw = hsm + (size_t(warp) << a.hm);
       const bool writer = (uint32_t(lane) & a.hlred) == 0u;
+      double x[1 << NR];
 #pragma unroll
       for (int r = 0; r < (1 << NR); ++r) {
-        double x = fma(v[r].x, v[r].x, v[r].y * v[r].y);
+        x[r] = fma(v[r].x, v[r].x, v[r].y * v[r].y);
 #pragma unroll
         for (int k = 0; k < 5; ++k)
-          if (a.hlred >> k & 1) x += __shfl_xor_sync(0xffffffffu, x, 1 << k);
-        if (writer) hw[hbk[r] | bt] += x;
+          if (a.hlred >> k & 1) x[r] += __shfl_xor_sync(0xffffffffu, x[r], 1 << k);
+      }
+      // slots that differ only in unrequested register bits share a bucket: sum them first, so
+      // the remaining ("live") slots have distinct buckets and all their loads can be issued
+      // before any store (one shared-memory latency per tile instead of one per slot)
+      uint32_t dead = 0;
+#pragma unroll
+      for (int k = 0; k < NR; ++k)
+        if (hrb[k] == 0u) {
+          dead |= 1u << k;
+#pragma unroll
+          for (int r = 0; r < (1 << NR); ++r)
+            if (r >> k & 1) x[r & ~(1 << k)] += x[r];
+        }
+      if (writer) {
+        uint32_t bk[1 << NR];
+        double old[1 << NR];
+#pragma unroll
+        for (int r = 0; r < (1 << NR); ++r) {
+          bk[r] = bt;
+#pragma unroll
+          for (int k = 0; k < NR; ++k)
+            if (r >> k & 1) bk[r] |= hrb[k];
+          old[r] = ((uint32_t(r) & dead) == 0u) ? hw[bk[r]] : 0.0;
+        }
+#pragma unroll
+        for (int r = 0; r < (1 << NR); ++r)
+          if ((uint32_t(r) & dead) == 0u) hw[bk[r]] = old[r] + x[r];
       }
     }
-    if constexpr (Body::kHist) if (a.hist && c.own && a.hacc == 0) {  // fused measurement: final amplitudes in registers
+    if constexpr (Body::kHist) if (a.hist && c.own && hmode == 0) {  // fused measurement: final amplitudes in registers
       uint64_t pbh = 0;
       SlotAddr sah{};
       if constexpr (Body::kStatic) pbh = base | (mp.base & lowmask) | hiOff[mp.base >> l];
@@ -1001,7 +1034,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   if (a.bstore && warp == 0) bulk_wait_all();  // shared memory must outlive the bulk reads
   if constexpr (Body::kHist) {
     if (a.hist) {
-      if (a.hacc == 1 && c.own) {
+      if (hmode == 1 && c.own) {
         // bucket of slot r: its tile-local index under the final mapping (tile base bits are not
         // requested, so base = 0); one shared-memory add per slot and thread
         uint64_t pbh = 0;
@@ -1019,7 +1052,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
         }
       }
       __syncthreads();
-      const int hw = a.hacc == 2 ? int(blockDim.x >> 5) : 1;
+      const int hw = hmode == 2 ? int(blockDim.x >> 5) : 1;
       for (int i = threadIdx.x; i < (1 << a.hm); i += blockDim.x) {
         double t = 0.0;
         for (int w = 0; w < hw; ++w) t += hsm[(size_t(w) << a.hm) + i];
