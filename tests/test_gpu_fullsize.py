@@ -138,3 +138,28 @@ def test_host_tier_qft30_basis_state_sampled(q, comp):
     assert worst <= TOL
     assert abs(p[0] - 1) <= 1e-12
     assert st["host_runs"] >= 1
+
+
+def test_bench_e2e_fused_measurement_full_size(q):
+    """The bench's e2e call at full size: QFT_28 on |0> and on |x>, qubits 0..9 measured inside
+    the last pass (mode 2 epilogue). QFT of a basis state has |amplitude|^2 = 2^-n everywhere, so
+    every marginal over 10 qubits is 2^-10 (closed form); QAOA_28 marginals vs the oracle's."""
+    qs = list(range(10))
+    for name in ("C2", "C2x"):
+        c = wc.config_circuit(name)
+        with q.State(c.n) as s:
+            p = s.apply_circuit_probabilities(q.Circuit(c.qasm()), qs)
+            p2 = s.probabilities(qs)
+            mixed = s.probabilities([27, 0, 13, 5])
+        assert np.abs(p - 2.0 ** -10).max() <= 1e-12, name
+        assert np.abs(p - p2).max() <= 1e-12, name
+        assert np.abs(mixed - 2.0 ** -4).max() <= 1e-12, name
+    c = wc.qaoa(28, 2, seed=1)
+    text = c.qasm()
+    for sel in (qs, [27, 26, 0, 1, 14], [3, 17, 9]):
+        with q.State(c.n) as s:
+            p = s.apply_circuit_probabilities(q.Circuit(text), sel)
+        if sel is qs:
+            ref_psi = osv.simulate(text)
+        ref = osv.probabilities(ref_psi, c.n, sel)
+        assert np.abs(p - ref).max() <= 1e-12, sel
