@@ -165,12 +165,12 @@ __global__ void __launch_bounds__(kThreads) phase_kernel(PhaseArgs a) {
 // The generic (interpreted) fused-pass kernel: the pass program is walked op by op. The
 // persistent tile loop, loads, constants and store are tile_driver (tile_common.cuh); the JIT
 // path (jit.cpp) replaces this body by straight-line code specialised to one pass.
-template <int NR>
+template <int NR, bool H>
 struct InterpBody {
   static constexpr unsigned kZM0 = 0u;
   static constexpr uint32_t kZW0 = 0u;
   static constexpr bool kStatic = false;  // mappings read from the program at run time
-  static constexpr bool kHist = true;     // fused measurement decided at run time (a.hist)
+  static constexpr bool kHist = H;        // H: the instantiation launched for a fused measurement
   static constexpr int kHistMode = -1;    // its epilogue too (a.hacc)
   static constexpr int kNsrun = -1;       // tile positions read from the arguments
   static constexpr int kSrunPos[1] = {0};
@@ -248,9 +248,9 @@ struct InterpBody {
   }
 };
 
-template <int NR>
+template <int NR, bool H>
 __global__ void __launch_bounds__(NR >= 4 ? 256 : 512, 1) tile_kernel(TileArgs a) {
-  InterpBody<NR> body{a.nops};
+  InterpBody<NR, H> body{a.nops};
   tile_driver<NR>(a, body);
 }
 
@@ -581,21 +581,21 @@ cudaError_t launch_phase(cudaStream_t st, const PhaseArgs& a) {
   return cudaGetLastError();
 }
 
-template <int NR>
+template <int NR, bool H>
 cudaError_t launch_tile_nr(cudaStream_t st, const TileArgs& a, size_t smem) {
   static bool configured = false;
   if (!configured) {
-    cudaError_t e = cudaFuncSetAttribute(tile_kernel<NR>, cudaFuncAttributeMaxDynamicSharedMemorySize,
+    cudaError_t e = cudaFuncSetAttribute(tile_kernel<NR, H>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          227 * 1024);
     if (e != cudaSuccess) return e;
     configured = true;
   }
   const int threads = 32 << a.nw;
   int bps = 0;
-  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, tile_kernel<NR>, threads, smem);
+  cudaOccupancyMaxActiveBlocksPerMultiprocessor(&bps, tile_kernel<NR, H>, threads, smem);
   if (bps <= 0) bps = 1;
   const unsigned g = unsigned(std::min<uint64_t>(a.ntiles, uint64_t(num_sms()) * bps));
-  tile_kernel<NR><<<g, threads, smem, st>>>(a);
+  tile_kernel<NR, H><<<g, threads, smem, st>>>(a);
   return cudaGetLastError();
 }
 
@@ -603,12 +603,22 @@ cudaError_t launch_tile(cudaStream_t st, const TileArgs& a) {
   if (a.ntiles == 0) return cudaSuccess;
   const size_t smem = tile_smem_bytes(a);
   if (smem > 227 * 1024) return cudaErrorInvalidValue;
+  // the fused-measurement epilogues live only in the H instantiation: they cost registers
+  if (a.hist) {
+    switch (a.nr) {
+      case 0: return launch_tile_nr<0, true>(st, a, smem);
+      case 1: return launch_tile_nr<1, true>(st, a, smem);
+      case 2: return launch_tile_nr<2, true>(st, a, smem);
+      case 3: return launch_tile_nr<3, true>(st, a, smem);
+      default: return launch_tile_nr<4, true>(st, a, smem);
+    }
+  }
   switch (a.nr) {
-    case 0: return launch_tile_nr<0>(st, a, smem);
-    case 1: return launch_tile_nr<1>(st, a, smem);
-    case 2: return launch_tile_nr<2>(st, a, smem);
-    case 3: return launch_tile_nr<3>(st, a, smem);
-    default: return launch_tile_nr<4>(st, a, smem);
+    case 0: return launch_tile_nr<0, false>(st, a, smem);
+    case 1: return launch_tile_nr<1, false>(st, a, smem);
+    case 2: return launch_tile_nr<2, false>(st, a, smem);
+    case 3: return launch_tile_nr<3, false>(st, a, smem);
+    default: return launch_tile_nr<4, false>(st, a, smem);
   }
 }
 
