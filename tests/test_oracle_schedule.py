@@ -193,3 +193,66 @@ def test_refined_rule_delays_involvement_at_least_as_much():
         a = os_.involvement_trace(gates, rule=0)
         b = os_.involvement_trace(gates, rule=1)
         assert all((y & ~x) == 0 for x, y in zip(a, b))
+
+
+# ------------------------------------------------------ pins of the soundness-check helpers
+
+def test_zero_map_hand_states():
+    """sv_zero_map (the data zero map of the pruning-soundness checks) on hand-built
+    states whose map is obvious: z[j] = 1 iff every amplitude of chunk j is exactly 0.0.
+    A map that wrongly reports "all zero" would make every soundness check vacuous."""
+    n, c = 4, 2                                        # 4 chunks of 4 amplitudes
+    psi = np.zeros(1 << n, dtype=np.complex128)
+    psi[7] = 1e-300                                    # the LAST slot of chunk 1
+    psi[8] = complex(-0.0, -0.0)                       # -0.0 is zero (chunk 2 stays zero)
+    psi[12] = complex(0.0, 5e-324)                     # a denormal imaginary part is non-zero
+    assert osv.zero_map(psi, n, c).tolist() == [True, False, True, False]
+    psi[0] = complex(0.0, -2.0)                        # the FIRST slot, imaginary only
+    assert osv.zero_map(psi, n, c).tolist() == [False, False, True, False]
+    # c = 0: every amplitude is its own chunk
+    z0 = osv.zero_map(psi, n, 0)
+    assert z0.tolist() == [not (x.real != 0.0 or x.imag != 0.0) for x in psi]
+    assert z0.sum() == 16 - 3
+    # c = n: one chunk covering the whole state
+    assert osv.zero_map(psi, n, n).tolist() == [False]
+    assert osv.zero_map(np.zeros(1 << n, np.complex128), n, n).tolist() == [True]
+    neg = np.full(1 << n, complex(-0.0, -0.0))
+    assert osv.zero_map(neg, n, 1).tolist() == [True] * 8
+
+
+def test_zero_map_sees_the_nonzero_support():
+    """After H on qubits {0, 2} of |0000>, exactly the indices with bits 1 and 3 clear are
+    non-zero: with c = 1 the chunks j with (j << 1) & 0b1010 == 0 are the non-zero ones."""
+    n, c = 4, 1
+    psi = osv.zero_state(n)
+    H = np.array([[1, 1], [1, -1]]) / np.sqrt(2)
+    for q in (0, 2):
+        osv.apply_gate(psi, n, H, [q])
+    z = osv.zero_map(psi, n, c)
+    assert z.tolist() == [((j << c) & 0b1010) != 0 for j in range(1 << (n - c))]
+
+
+def test_ops_before_full_involvement_gs5():
+    """Table II statistic (reading Q17) fixed by the three published gs_5 profiles:
+    4 operations before full involvement in program order, 6 with the paper's greedy
+    picks, 8 with forward-looking reordering."""
+    g, gates = _gs5()
+    want = g["ops_before_full_involvement"]
+    assert os_.ops_before_full_involvement(gates, 5) == want["original"] == 4
+    gr = os_.reorder_greedy(gates, forced=g["greedy_forced_picks"])
+    assert os_.ops_before_full_involvement(gates, 5, gr) == want["greedy"] == 6
+    fw = os_.reorder_forward(gates)
+    assert os_.ops_before_full_involvement(gates, 5, fw) == want["forward"] == 8
+
+
+def test_ops_before_full_involvement_edge_cases():
+    """The first op involves everything -> 0; full involvement never reached -> the number of
+    operations; reached by the last op -> len - 1 (off-by-one checks of reading Q17)."""
+    one = [(0, 1, 2)]                                         # ccx-like: all 3 qubits at once
+    assert os_.ops_before_full_involvement(one, 3) == 0
+    never = [(0,), (1,), (0, 1)]
+    assert os_.ops_before_full_involvement(never, 3) == 3          # qubit 2 never touched
+    last = [(0,), (1,), (2,)]
+    assert os_.ops_before_full_involvement(last, 3) == 2
+    assert os_.ops_before_full_involvement(last, 3, order=[2, 1, 0]) == 2
+    assert os_.ops_before_full_involvement(last, 2) == 1           # n = 2: q2 is outside
