@@ -73,8 +73,10 @@ typedef struct {
   int timing;                 /* 1: time every launch with CUDA events into qgpu_stats     */
   uint64_t swap_slab_bytes;   /* staging bytes per all-to-all slab (sharded mode)          */
   int jit;                    /* fused passes: 0 = generic tile kernel only; 1 (default) = NVRTC-
-                                 specialised kernel for passes of >= 2^20 amplitudes; 2 = always.
-                                 Falls back to the generic kernel if NVRTC is unavailable   */
+                                 specialised kernel for passes whose live output range is >=
+                                 2^12 amplitudes (env QGPU_JIT_MIN_BITS overrides the 12);
+                                 2 = always. Falls back to the generic kernel if NVRTC is
+                                 unavailable                                               */
   int host_slice_bits;        /* h: host-memory tier (the paper's setting,
                                  P:185-191). 0 (default) = state resident in HBM. h > 0
                                  (world_size = 1 only): the 2^n amplitudes live in pinned host

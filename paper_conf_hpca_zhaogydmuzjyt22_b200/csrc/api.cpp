@@ -127,6 +127,20 @@ uint64_t plan_key(const qgpu_state* st, const qgpu_circuit* c) {
 
 PlanOptions plan_options(const qgpu_config& cfg, bool fuse);
 
+// Content equality of two circuits (everything the planner reads; the source line is not)
+bool same_circuit(const Circuit& a, const Circuit& b) {
+  if (a.n != b.n || a.gates.size() != b.gates.size()) return false;
+  for (size_t i = 0; i < a.gates.size(); ++i) {
+    const Gate& x = a.gates[i];
+    const Gate& y = b.gates[i];
+    if (x.nt != y.nt || x.t[0] != y.t[0] || (x.nt == 2 && x.t[1] != y.t[1]) || x.cmask != y.cmask ||
+        x.diag != y.diag || x.relabel != y.relabel)
+      return false;
+    if (std::memcmp(x.U, y.U, sizeof(cplx) << (2 * x.nt)) != 0) return false;
+  }
+  return true;
+}
+
 // Copy the programs of a plan's fused passes to a device buffer owned by the plan.
 qgpu_status upload_plan(qgpu_state* st, CachedPlan* cp) {
   size_t nbytes = 0;
@@ -308,8 +322,12 @@ qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out
       qgpu_state_destroy(st);
       return s;
     };
-    cudaError_t e = cudaSetDevice(cfg.device);
-    if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaSetDevice(%d): %s", cfg.device, cudaGetErrorString(e)));
+    int ndev = 0;
+    cudaError_t e = cudaGetDeviceCount(&ndev);
+    if (e != cudaSuccess) return bail(fail(QGPU_ERR_CUDA, "cudaGetDeviceCount: %s", cudaGetErrorString(e)));
+    if (cfg.device < 0 || cfg.device >= ndev)
+      return bail(fail(QGPU_ERR_INVALID_ARG, "device %d out of [0, %d)", cfg.device, ndev));
+    QGPU_ON_DEVICE(st);
     if (cfg.stream) {
       st->stream = static_cast<cudaStream_t>(cfg.stream);
     } else {
@@ -418,6 +436,7 @@ qgpu_status qgpu_state_create(int n, const qgpu_config* cfg_in, qgpu_state** out
 }
 
 qgpu_status qgpu_state_destroy(qgpu_state* st) {
+  QGPU_ON_DEVICE(st);
   if (!st) return QGPU_OK;
   if (st->stream) cudaStreamSynchronize(st->stream);
   for (auto& t : st->pending) {
@@ -461,6 +480,7 @@ qgpu_status qgpu_state_destroy(qgpu_state* st) {
 }
 
 qgpu_status qgpu_state_reset(qgpu_state* st) {
+  QGPU_ON_DEVICE(st);
   if (qgpu_status s = check_state(st)) return s;
   st->map.init(st->n, st->m);
   st->trace_order.clear();
@@ -477,6 +497,7 @@ qgpu_status qgpu_state_reset(qgpu_state* st) {
 }
 
 qgpu_status qgpu_set_amplitudes(qgpu_state* st, const double* amps) {
+  QGPU_ON_DEVICE(st);
   if (qgpu_status s = check_state(st)) return s;
   if (!amps) return fail(QGPU_ERR_INVALID_ARG, "amps is NULL");
   if (st->g > 0 && !st->host) return fail(QGPU_ERR_UNSUPPORTED, "set_amplitudes is single-GPU only");
@@ -505,6 +526,7 @@ qgpu_status qgpu_set_amplitudes(qgpu_state* st, const double* amps) {
 }
 
 qgpu_status qgpu_synchronize(qgpu_state* st) {
+  QGPU_ON_DEVICE(st);
   if (qgpu_status s = check_state(st)) return s;
   CK(cudaStreamSynchronize(st->stream));
   return drain_timing(st);
@@ -521,6 +543,7 @@ qgpu_status qgpu_state_info(const qgpu_state* st, int* n, int* nl, void** dev) {
 qgpu_status qgpu_apply_gate(qgpu_state* st, const double* U, int nt, const int* targets, int nc,
                             const int* controls) {
   try {
+    QGPU_ON_DEVICE(st);
     if (qgpu_status s = check_state(st)) return s;
     if (!U || !targets) return fail(QGPU_ERR_INVALID_ARG, "U/targets is NULL");
     if (nt < 1 || nt > 2) return fail(QGPU_ERR_INVALID_ARG, "n_targets must be 1 or 2");
@@ -569,16 +592,18 @@ bool hacc_enabled() {
 // qgpu_apply_circuit; meas_m >= 0 also asks the last fused pass to histogram qubits meas_q
 qgpu_status apply_circuit_impl(qgpu_state* st, const qgpu_circuit* c, int meas_m, const int* meas_q) {
   try {
+    QGPU_ON_DEVICE(st);
     if (qgpu_status s = check_state(st)) return s;
     if (!c) return fail(QGPU_ERR_INVALID_ARG, "circuit is NULL");
     if (c->c.n > st->n) return fail(QGPU_ERR_INVALID_ARG, "circuit has %d qubits, state %d", c->c.n, st->n);
     const uint64_t key = plan_key(st, c);
     CachedPlan* hit = nullptr;
     for (CachedPlan& cp : st->plans)
-      if (cp.key == key) hit = &cp;
+      if (cp.key == key && same_circuit(cp.circ, c->c)) hit = &cp;
     if (!hit) {
       CachedPlan cp;
       cp.key = key;
+      cp.circ = c->c;
       cp.order = reorder(c->c.gates, st->cfg.reorder, st->cfg.involve_rule);
       QubitMap map = st->map;
       plan_circuit(c->c.gates, cp.order, map, plan_options(st->cfg, st->cfg.fuse_bits > 0), &cp.passes, &cp.inv);
@@ -718,6 +743,7 @@ qgpu_status qgpu_apply_circuit_probabilities(qgpu_state* st, const qgpu_circuit*
     if (q < 0 || q >= st->n || (seen >> q & 1)) return fail(QGPU_ERR_INVALID_ARG, "bad qubit %d", q);
     seen |= 1ull << q;
   }
+  QGPU_ON_DEVICE(st);
   if (qgpu_status s = apply_circuit_impl(st, c, mq, qubits)) return s;
   if (!st->meas_done) return qgpu_probabilities(st, mq, qubits, out);  // not fusable: read the state
   CK(cudaMemcpyAsync(out, st->d_meas, (size_t(8) << mq), cudaMemcpyDeviceToHost, st->stream));
@@ -737,6 +763,7 @@ qgpu_status qgpu_apply_circuit_probabilities(qgpu_state* st, const qgpu_circuit*
 }
 
 qgpu_status qgpu_get_amplitudes_device(qgpu_state* st, uint64_t start, uint64_t count, double* dev_out) {
+  QGPU_ON_DEVICE(st);
   if (qgpu_status s = check_state(st)) return s;
   if (!dev_out && count) return fail(QGPU_ERR_INVALID_ARG, "dev_out is NULL");
   if (start + count > (1ull << st->n) || start + count < start)
@@ -773,6 +800,7 @@ qgpu_status qgpu_get_amplitudes_device(qgpu_state* st, uint64_t start, uint64_t 
 }
 
 qgpu_status qgpu_get_amplitudes(qgpu_state* st, uint64_t start, uint64_t count, double* out) {
+  QGPU_ON_DEVICE(st);
   if (qgpu_status s = check_state(st)) return s;
   if (!out && count) return fail(QGPU_ERR_INVALID_ARG, "out is NULL");
   const uint64_t chunk = std::min<uint64_t>(count, 1ull << 24);
@@ -794,6 +822,7 @@ qgpu_status qgpu_get_amplitudes(qgpu_state* st, uint64_t start, uint64_t count, 
 }
 
 qgpu_status qgpu_probabilities(qgpu_state* st, int mq, const int* qubits, double* out) {
+  QGPU_ON_DEVICE(st);
   if (qgpu_status s = check_state(st)) return s;
   if (mq < 0 || mq > 30) return fail(QGPU_ERR_INVALID_ARG, "m=%d out of [0, 30]", mq);
   if (!out || (mq > 0 && !qubits)) return fail(QGPU_ERR_INVALID_ARG, "NULL argument");
@@ -1051,6 +1080,7 @@ qgpu_status qgpu_get_qubit_map(qgpu_state* st, int* pos) {
 }
 
 qgpu_status qgpu_get_stats(qgpu_state* st, qgpu_stats* out) {
+  QGPU_ON_DEVICE(st);
   if (!st || !out) return fail(QGPU_ERR_INVALID_ARG, "NULL argument");
   if (!st->pending.empty()) {
     if (qgpu_status s = drain_timing(st)) return s;
@@ -1064,6 +1094,7 @@ qgpu_status qgpu_get_stats(qgpu_state* st, qgpu_stats* out) {
 }
 
 qgpu_status qgpu_reset_stats(qgpu_state* st) {
+  QGPU_ON_DEVICE(st);
   if (!st) return fail(QGPU_ERR_INVALID_ARG, "state is NULL");
   if (qgpu_status s = drain_timing(st)) return s;
   const int64_t obf = st->stats.ops_before_full_involvement;

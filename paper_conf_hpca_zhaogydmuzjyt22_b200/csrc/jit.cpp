@@ -161,6 +161,14 @@ void cache_write(const std::string& key, const std::string& cubin) {
   std::rename(tmp.c_str(), (d + "/" + key + ".cubin").c_str());
 }
 
+// loaded functions belong to the current device's primary context: the in-memory cache is
+// keyed by device ordinal + source (the caller has made the state's device current)
+std::string device_tag() {
+  int d = 0;
+  cudaGetDevice(&d);
+  return "dev" + std::to_string(d) + "|";
+}
+
 }  // namespace
 
 bool jit_cubin_cached(const std::string& src, std::string* cubin, std::string* log, bool* hit) {
@@ -552,11 +560,12 @@ int jit_prepare(const std::vector<const Pass*>& passes, double* compile_ms) {
   JitLib& L = lib();
   const auto t0 = std::chrono::steady_clock::now();
   std::vector<std::string> srcs;
+  const std::string dev = device_tag();
   {
     std::lock_guard<std::mutex> g(L.mu);
     for (const Pass* p : passes) {
       std::string src = tile_jit_source(*p);
-      if (!L.cache.count(src) && std::find(srcs.begin(), srcs.end(), src) == srcs.end()) srcs.push_back(std::move(src));
+      if (!L.cache.count(dev + src) && std::find(srcs.begin(), srcs.end(), src) == srcs.end()) srcs.push_back(std::move(src));
     }
   }
   if (srcs.empty()) return 0;
@@ -585,7 +594,7 @@ int jit_prepare(const std::vector<const Pass*>& passes, double* compile_ms) {
     if (L.moduleGetFunction(&fn, mod, "qgpu_tile_pass") != CUDA_SUCCESS) continue;
     if (L.funcSetAttribute(fn, CU_FUNC_ATTRIBUTE_MAX_DYNAMIC_SHARED_SIZE_BYTES, 227 * 1024) != CUDA_SUCCESS) continue;
     std::lock_guard<std::mutex> g(L.mu);
-    L.cache.emplace(srcs[i], fn);
+    L.cache.emplace(dev + srcs[i], fn);
     ++loaded;
   }
   if (compile_ms)
@@ -603,10 +612,11 @@ cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, s
   const int hmode = hist ? std::clamp(a.hacc, 0, 2) : -1;
   CUfunction fn = static_cast<CUfunction>(hist ? p.jit_fn_hist[hmode] : p.jit_fn);
   std::string src;
+  const std::string dev = device_tag();
   if (!fn) {
     src = tile_jit_source(p, hmode);
     std::lock_guard<std::mutex> g(L.mu);
-    auto it = L.cache.find(src);
+    auto it = L.cache.find(dev + src);
     if (it != L.cache.end()) fn = it->second;
   }
   if (!fn) {
@@ -626,7 +636,7 @@ cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, s
     const auto t1 = std::chrono::steady_clock::now();
     if (compile_ms) *compile_ms += std::max(1e-3, std::chrono::duration<double, std::milli>(t1 - t0).count());
     std::lock_guard<std::mutex> g(L.mu);
-    L.cache.emplace(src, fn);
+    L.cache.emplace(dev + src, fn);
   }
   (hist ? p.jit_fn_hist[hmode] : p.jit_fn) = fn;  // later launches skip source generation and lookup
   const unsigned threads = 32u << a.nw;

@@ -525,15 +525,21 @@ __global__ void add_kernel(double* out, const double* in, uint64_t count) {
 
 // --------------------------------------------------------------------------- launchers
 namespace {
-int g_num_sms = 0;
+constexpr int kMaxDevices = 64;
+int cur_device() {
+  int dev = 0;
+  cudaGetDevice(&dev);
+  return (dev >= 0 && dev < kMaxDevices) ? dev : 0;
+}
+int g_num_sms[kMaxDevices] = {};
 int num_sms() {
-  if (!g_num_sms) {
-    int dev = 0;
-    cudaGetDevice(&dev);
-    cudaDeviceGetAttribute(&g_num_sms, cudaDevAttrMultiProcessorCount, dev);
-    if (g_num_sms <= 0) g_num_sms = 148;
+  const int dev = cur_device();
+  if (!g_num_sms[dev]) {
+    int v = 0;
+    cudaDeviceGetAttribute(&v, cudaDevAttrMultiProcessorCount, dev);
+    g_num_sms[dev] = v > 0 ? v : 148;
   }
-  return g_num_sms;
+  return g_num_sms[dev];
 }
 unsigned grid_for(uint64_t work_items, int per_block, int blocks_per_sm) {
   const uint64_t need = (work_items + per_block - 1) / per_block;
@@ -583,12 +589,13 @@ cudaError_t launch_phase(cudaStream_t st, const PhaseArgs& a) {
 
 template <int NR, bool H>
 cudaError_t launch_tile_nr(cudaStream_t st, const TileArgs& a, size_t smem) {
-  static bool configured = false;
-  if (!configured) {
+  static bool configured[kMaxDevices] = {};  // function attributes are per device
+  const int dev = cur_device();
+  if (!configured[dev]) {
     cudaError_t e = cudaFuncSetAttribute(tile_kernel<NR, H>, cudaFuncAttributeMaxDynamicSharedMemorySize,
                                          227 * 1024);
     if (e != cudaSuccess) return e;
-    configured = true;
+    configured[dev] = true;
   }
   const int threads = 32 << a.nw;
   int bps = 0;
@@ -650,10 +657,11 @@ cudaError_t launch_probs(cudaStream_t st, ProbArgs a, double*) {
   }
   const int mode = a.m <= 10 ? 0 : (a.m <= 12 ? 1 : 2);
   const size_t smem = mode == 0 ? B * sizeof(double) * (kThreads / 32) : (mode == 1 ? B * sizeof(double) : 0);
-  static bool configured = false;
-  if (!configured) {
+  static bool configured[kMaxDevices] = {};
+  const int dev = cur_device();
+  if (!configured[dev]) {
     cudaFuncSetAttribute(probs_kernel, cudaFuncAttributeMaxDynamicSharedMemorySize, 96 * 1024);
-    configured = true;
+    configured[dev] = true;
   }
   const unsigned g = unsigned(num_sms()) * 2;
   probs_kernel<<<g, kThreads, smem, st>>>(a, mode);

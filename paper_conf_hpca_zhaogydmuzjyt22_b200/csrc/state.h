@@ -34,6 +34,7 @@ namespace qgpu_impl {
 // copy of a few KB that keeps each apply's inputs flowing like an uncached run.
 struct CachedPlan {
   uint64_t key = 0;
+  Circuit circ;  // the planned circuit: a key hit is reused only if the content matches too
   std::vector<int> order;
   std::vector<uint64_t> inv;
   std::vector<Pass> passes;
@@ -79,13 +80,11 @@ inline bool host_sweep_per_pass() {
   return ev && std::atoi(ev) != 0;
 }
 
-// jit=1: specialise fused passes whose live range is >= 2^jit_min_bits amplitudes
+// jit=1: specialise fused passes whose live range is >= 2^jit_min_bits amplitudes (default 12;
+// read per call, so a test can run the same circuits at the library default and above it)
 inline int jit_min_bits() {
-  static const int v = [] {
-    const char* ev = std::getenv("QGPU_JIT_MIN_BITS");
-    return ev ? std::atoi(ev) : 12;
-  }();
-  return v;
+  const char* ev = std::getenv("QGPU_JIT_MIN_BITS");
+  return ev ? std::atoi(ev) : 12;
 }
 
 extern thread_local std::string g_err;
@@ -184,6 +183,23 @@ struct qgpu_state {
   bool meas_done = false;
 };
 
+
+// Every entry point that touches a state runs on the state's device and restores the caller's
+// current device on return (a state may be used from a thread whose current device differs, or
+// next to states on other devices in the same process).
+struct DeviceGuard {
+  int prev = -1;
+  bool changed = false;
+  explicit DeviceGuard(int dev) {
+    if (cudaGetDevice(&prev) == cudaSuccess && prev != dev) changed = cudaSetDevice(dev) == cudaSuccess;
+  }
+  ~DeviceGuard() {
+    if (changed) cudaSetDevice(prev);
+  }
+  DeviceGuard(const DeviceGuard&) = delete;
+  DeviceGuard& operator=(const DeviceGuard&) = delete;
+};
+#define QGPU_ON_DEVICE(st) DeviceGuard qgpu_device_guard_((st) ? (st)->cfg.device : 0)
 
 #define CK(expr)                                                                        \
   do {                                                                                  \

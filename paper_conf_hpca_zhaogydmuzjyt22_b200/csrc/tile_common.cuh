@@ -835,7 +835,8 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       tile = next;
       // no barrier: a zero tile neither reads nor fills its buffer (its loads were skipped), so
       // running ahead through zero tiles cannot overwrite a buffer another warp still reads --
-      // the barrier after each live tile already orders every reuse of a buffer
+      // the barrier after each live tile (every program with remaps ends a live tile with one)
+      // already orders every reuse of a buffer
       continue;
     }
     // pattern constants of this tile, per warp (lane-strided; each lane owns the same patterns
@@ -1027,9 +1028,11 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     // the lanes of this warp are done reading this tile's pattern constants before the next
     // tile's constants are written
     __syncwarp();
-    // with two buffers the next prefetch refills the buffer other warps read during remaps;
-    // with warp-group remaps this is the one CTA barrier per tile that bounds warp drift
-    if ((nbuf < 3 || Body::kGroupRemap) && a.remaps) __syncthreads();
+    // programs with remaps read other threads' slots of this tile's buffer: no warp may run
+    // ahead and prefetch into it (two buffers: the next tile's; three: the tile after a skipped
+    // zero / zout tile, which has no barrier of its own) until every warp has finished reading
+    // it. With warp-group remaps this is also the one CTA barrier per tile bounding warp drift.
+    if (a.remaps) __syncthreads();
   }
   if (a.bstore && warp == 0) bulk_wait_all();  // shared memory must outlive the bulk reads
   if constexpr (Body::kHist) {
