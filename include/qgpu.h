@@ -70,7 +70,9 @@ typedef struct {
                                  2 forward-looking (Alg.3, default)            */
   int fuse_bits;              /* b: tile qubits per fused HBM pass (default 12);
                                  0 = one kernel per gate (pair/quad/diag kernels)          */
-  int timing;                 /* 1: time every launch with CUDA events into qgpu_stats     */
+  int timing;                 /* 1: time passes with CUDA events into the statistics (a run
+                                 of consecutive fused passes is one interval); 2: every pass its
+                                 own interval, recorded for qgpu_get_pass_profile          */
   uint64_t swap_slab_bytes;   /* staging bytes per all-to-all slab (sharded mode)          */
   int jit;                    /* fused passes: 0 = generic tile kernel only; 1 (default) = NVRTC-
                                  specialised kernel for passes whose live output range is >=
@@ -136,6 +138,18 @@ typedef struct {
   double host_ms;              /* timing=1: CUDA-event time of the streaming sweeps          */
 } qgpu_stats;
 
+/* One pass of the last qgpu_apply_circuit / qgpu_apply_gate call when cfg.timing = 2 (every
+ * pass timed by its own CUDA events): the per-pass roofline inputs. */
+typedef struct qgpu_pass_profile {
+  int32_t kind;                /* as qgpu_circuit_plan: 0 tile, 1 pair, 2 quad, 3 diag, 5 swap, 7 zero */
+  int32_t k_in, k_out;         /* log2 live local size before / after                          */
+  int32_t n_gates;             /* gates fused into the pass                                    */
+  double ms;                   /* CUDA-event time of the pass (all local shards)               */
+  uint64_t bytes;              /* algorithmic HBM bytes (live input read + output written)     */
+  uint64_t amps_computed;      /* amplitudes the program ran on (zero tiles excluded)          */
+  double fp64_ops;             /* FP64 pipe instructions (DFMA/DMUL/DADD) by the pass model    */
+} qgpu_pass_profile;
+
 /* ---- configuration and state ---------------------------------------------------------- */
 
 /* Fill *cfg with defaults (device 0, own stream, prune=1, reorder=2, chunk_bits=21,
@@ -161,6 +175,9 @@ qgpu_status qgpu_state_reset(qgpu_state* st);
  * logical index order. Marks every qubit involved (nothing left to prune). Synchronises.
  * Single-GPU or host tier (UNSUPPORTED when sharded over ranks). */
 qgpu_status qgpu_set_amplitudes(qgpu_state* st, const double* amps);
+
+/* Change cfg.timing (0 off, 1 grouped, 2 per pass) for the calls that follow. */
+qgpu_status qgpu_set_timing(qgpu_state* st, int mode);
 
 /* Block until all work enqueued on the state's stream is done; reports async errors. */
 qgpu_status qgpu_synchronize(qgpu_state* st);
@@ -276,6 +293,17 @@ qgpu_status qgpu_get_qubit_map(qgpu_state* st, int* pos);
 
 qgpu_status qgpu_get_stats(qgpu_state* st, qgpu_stats* out);
 qgpu_status qgpu_reset_stats(qgpu_state* st);
+
+/* Per-pass profile (cfg.timing = 2) of the passes executed since the last call of this
+ * function with out != NULL or qgpu_state_reset: out[0..min(cap, n)), *n = records available
+ * (out = NULL: size query, the records are kept). Synchronises.
+ * Diagnostic (bench.py's per-pass binding bound, max(bytes / HBM peak, FP64 / FP64 peak)). */
+qgpu_status qgpu_get_pass_profile(qgpu_state* st, qgpu_pass_profile* out, uint64_t cap, uint64_t* n);
+
+/* Measure this device's FP64 FMA throughput: a kernel of independent DFMA chains on every SM,
+ * timed with CUDA events (best of 3). *fma_per_s = thread-level DFMA per second (a DFMA is 2
+ * flops). The FP64 peak of the per-pass roofline. Synchronous; ~0.1 s. */
+qgpu_status qgpu_measure_fp64_peak(int device, double* fma_per_s);
 
 /* Host: a fresh 128-byte ncclUniqueId (rank 0 creates it, the caller broadcasts it, e.g. with
  * torch.distributed). UNSUPPORTED if libnccl.so.2 cannot be loaded ($QGPU_NCCL_LIB). */

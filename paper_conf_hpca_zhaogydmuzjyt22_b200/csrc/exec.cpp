@@ -32,6 +32,10 @@ qgpu_status drain_timing(qgpu_state* st) {
         st->stats.tile_algo_bytes += t.bytes;
       }
     }
+    if (t.prof) {
+      t.rec.ms = ms;
+      st->prof.push_back(t.rec);
+    }
     st->event_pool.push_back(t.a);
     st->event_pool.push_back(t.b);
   }
@@ -307,6 +311,21 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
   return QGPU_OK;
 }
 
+// Amplitudes a pass's program runs on in one shard: a fused pass skips the tiles whose base
+// lies in the zero region of an expansion (a non-tile position >= k_in set) or selects a
+// skipped zero half (zin / zout positions); the per-gate kernels touch the live range.
+uint64_t computed_amps(const qgpu_state* st, const Pass& p) {
+  const int kin = st->cfg.prune ? p.k_in : st->m, kout = st->cfg.prune ? p.k_out : st->m;
+  if (p.kind != PK_TILE) return 1ull << kout;
+  uint64_t S = 0;
+  for (int i = 0; i < p.b; ++i) S |= 1ull << p.spos[i];
+  const uint64_t z = st->cfg.prune ? (p.zin | p.zout) : 0;
+  int free_bits = 0;
+  for (int q = 0; q < kout; ++q)
+    if (!(S >> q & 1) && q < kin && !(z >> q & 1)) ++free_bits;
+  return 1ull << (free_bits + p.b);
+}
+
 // Execute one planned pass: compute passes on every active local shard (ranks >= 2^kg hold
 // only zeros and skip the work), swaps through the communicator, activations as memsets.
 qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops, bool own_timing = true,
@@ -361,6 +380,16 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops,
   if (timing) {
     CK(cudaEventRecord(tl.b, st->stream));
     tl.bytes = bytes;
+    if (st->cfg.timing == 2) {
+      tl.prof = true;
+      tl.rec.kind = p.kind;
+      tl.rec.k_in = kin;
+      tl.rec.k_out = kout;
+      tl.rec.n_gates = p.count;
+      tl.rec.bytes = bytes;
+      tl.rec.amps_computed = p.kind == PK_SWAP ? 0 : computed_amps(st, p);
+      tl.rec.fp64_ops = p.fp64_per_amp * double(tl.rec.amps_computed);
+    }
     st->pending.push_back(tl);
   }
   if (p.kind != PK_SWAP) {
@@ -699,7 +728,7 @@ qgpu_status exec_passes(qgpu_state* st, const std::vector<Pass>& passes,
     // timing=1: a run of consecutive fused passes on one shard is timed as ONE event interval
     // (events between back-to-back kernels cost a launch gap each); the interval's launches and
     // algorithmic bytes are recorded with it
-    const bool group = st->cfg.timing != 0 && st->shards.size() == 1;
+    const bool group = st->cfg.timing == 1 && st->shards.size() == 1;
     TimedLaunch grp{};
     bool open = false;
     auto close_group = [&]() -> qgpu_status {

@@ -700,6 +700,50 @@ cudaError_t launch_zero_where(cudaStream_t st, double2* psi, uint64_t L, uint64_
   return cudaGetLastError();
 }
 
+// FP64 roofline peak: independent DFMA chains (8 per thread, so the pipe, not the latency,
+// bounds the issue rate) on every SM; the result is stored so nothing is eliminated.
+__global__ void __launch_bounds__(256) fp64_probe_kernel(double* out, int iters, double a, double b) {
+  double x[8];
+#pragma unroll
+  for (int k = 0; k < 8; ++k) x[k] = double(threadIdx.x + k);
+  for (int i = 0; i < iters; ++i) {
+#pragma unroll
+    for (int k = 0; k < 8; ++k) x[k] = fma(x[k], a, b);
+  }
+  double s = 0.0;
+#pragma unroll
+  for (int k = 0; k < 8; ++k) s += x[k];
+  if (s == 12345.678) out[threadIdx.x] = s;  // practically never; keeps the chains live
+}
+
+cudaError_t probe_fp64(double* fma_per_s) {
+  double* out = nullptr;
+  cudaError_t e = cudaMalloc(&out, 256 * sizeof(double));
+  if (e != cudaSuccess) return e;
+  cudaEvent_t a, b;
+  cudaEventCreate(&a);
+  cudaEventCreate(&b);
+  const int iters = 1 << 14;
+  const unsigned grid = unsigned(num_sms()) * 8;
+  double best = 0.0;
+  fp64_probe_kernel<<<grid, 256>>>(out, iters, 0.999999, 1e-7);  // warm-up
+  for (int r = 0; r < 3 && e == cudaSuccess; ++r) {
+    cudaEventRecord(a);
+    fp64_probe_kernel<<<grid, 256>>>(out, iters, 0.999999, 1e-7);
+    cudaEventRecord(b);
+    e = cudaEventSynchronize(b);
+    float ms = 0;
+    if (e == cudaSuccess) e = cudaEventElapsedTime(&ms, a, b);
+    if (e == cudaSuccess && ms > 0) best = std::max(best, double(grid) * 256.0 * 8.0 * iters / (ms * 1e-3));
+  }
+  if (e == cudaSuccess) e = cudaGetLastError();
+  cudaEventDestroy(a);
+  cudaEventDestroy(b);
+  cudaFree(out);
+  *fma_per_s = best;
+  return e;
+}
+
 cudaError_t launch_set_amp(cudaStream_t st, double2* psi, uint64_t i, double re, double im) {
   set_amp_kernel<<<1, 1, 0, st>>>(psi, i, make_double2(re, im));
   return cudaGetLastError();

@@ -73,6 +73,8 @@ cudaError_t launch_tile(cudaStream_t st, const TileArgs& a);
 cudaError_t launch_gather(cudaStream_t st, const GatherArgs& a);
 cudaError_t launch_probs(cudaStream_t st, ProbArgs a, double* scratch);
 cudaError_t launch_set_amp(cudaStream_t st, double2* psi, uint64_t i, double re, double im);
+// FP64 peak probe (qgpu_measure_fp64_peak): thread-level DFMA per second on the current device
+cudaError_t probe_fp64(double* fma_per_s);
 cudaError_t launch_zero_where(cudaStream_t st, double2* psi, uint64_t L, uint64_t mask);
 // sharded swaps (a10)
 cudaError_t launch_swap_halves(cudaStream_t st, double2* a, double2* b, int lp, uint64_t half);

@@ -148,6 +148,8 @@ struct Pass {
   mutable void* jit_fn = nullptr;  // specialised kernel, resolved at the first launch
   mutable void* jit_fn_hist[3] = {nullptr, nullptr, nullptr};  // fused-measurement variants, per mode
   uint64_t unfused_bytes = 0;   // bytes the pass's gates would move one gate per pass
+  double fp64_per_amp = 0.0;    // FP64 pipe instructions per computed amplitude (roofline model,
+                                // fp64_model() in sched.cpp)
   // zero-position skipping (tile passes): physical positions p whose bit-p = 1 half of the live
   // state is exactly zero and NOT materialised in memory -- on input (zin: loads read zeros
   // instead) and on output (zout: those amplitudes are not stored); PK_ZERO materialises zmask
@@ -182,5 +184,8 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
 void build_tile_ops(Pass& p, int m, int reg_bits = 4);
 // Unfused byte model of one gate on live size 2^k.
 uint64_t unfused_gate_bytes(const PhysGate& g, int k_in, int k_out);
+// FP64 instructions per amplitude a pass's program executes (fused tile pass) or its single
+// gate needs (pair / quad / diagonal kernels): the FP64 side of the per-pass roofline.
+double fp64_model(const Pass& p);
 
 }  // namespace qgpu

@@ -24,6 +24,10 @@
 
 namespace qgpu {
 
+namespace {
+int mat_class(const cplx* U, int nt);
+}  // namespace
+
 // ----------------------------------------------------------------------------------- a2
 namespace {
 
@@ -182,6 +186,44 @@ uint64_t unfused_gate_bytes(const PhysGate& g, int k_in, int k_out) {
   const int nc = std::popcount(g.pc);
   if (k_out > k_in) return uint64_t(16.0 * double(1ull << k_in) + 16.0 * L);
   return uint64_t(32.0 * L / double(1ull << nc));
+}
+
+// FP64 pipe instructions per amplitude (each DFMA / DMUL / DADD counts 1):
+//  1-qubit U on a pair: generic complex 2x2 16 per pair (8 per amplitude), real or
+//  real-diagonal / imaginary-off-diagonal 8 per pair (4), X 0; 2-qubit U: 64 per quad (16);
+//  a run of phase patterns: one complex multiply per owned amplitude (4) plus its table built
+//  by doubling (2^NR - 1 complex multiplies per thread for 2^NR amplitudes, ~4) and one more
+//  complex multiply per general r-condition group on the amplitudes it selects; the
+//  tile-uniform scalar 4. Conditions scale an op by the fraction of amplitudes they select.
+double fp64_model(const Pass& p) {
+  auto cls_cost = [](int cls) { return cls == MAT_GENERIC ? 8.0 : cls == MAT_X ? 0.0 : 4.0; };
+  if (p.kind == PK_TILE) {
+    const TileProgram& P = p.prog;
+    double c = P.scalar.empty() ? 0.0 : 4.0;
+    for (size_t i = 1; i < P.ops.size(); ++i) {
+      const TileOp& o = P.ops[i];
+      const double frac = std::ldexp(1.0, -std::popcount(o.rmask) - std::popcount(o.tmask));
+      switch (o.kind) {
+        case OP_U1R: case OP_U1L: case OP_SMEM1: c += cls_cost(o.cls) * frac; break;
+        case OP_U2R: case OP_SMEM2: c += 16.0 * frac; break;
+        case OP_RUN: {
+          const uint32_t slots = uint32_t(o.a0 + o.a1 + o.cls) + o.tmask + o.tmatch;
+          if (slots) c += 4.0 + 4.0 * (1.0 - std::ldexp(1.0, -P.nr));
+          for (uint32_t e = o.moff + slots; e < o.moff + o.cnt; ++e)
+            if (P.entries[e].gend) c += 4.0 * std::ldexp(1.0, -std::popcount(uint32_t(P.entries[e].rmask)));
+          break;
+        }
+        default: break;
+      }
+    }
+    return c;
+  }
+  if (p.gates.empty()) return 0.0;
+  const PhysGate& g = p.gates[0];
+  if (p.kind == PK_PAIR) return cls_cost(mat_class(g.U, 1));
+  if (p.kind == PK_QUAD) return 16.0;
+  if (p.kind == PK_DIAG) return 4.0;
+  return 0.0;
 }
 
 namespace {
@@ -830,6 +872,7 @@ struct Builder {
       while (p.l < p.b && p.spos[p.l] == p.l) ++p.l;
       build_tile_ops(p, map.m, opt.reg_bits);
     }
+    p.fp64_per_amp = fp64_model(p);
     out->push_back(std::move(p));
     cur = Pass();
     open = false;

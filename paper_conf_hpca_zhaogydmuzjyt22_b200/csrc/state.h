@@ -34,7 +34,9 @@ namespace qgpu_impl {
 // copy of a few KB that keeps each apply's inputs flowing like an uncached run.
 struct CachedPlan {
   uint64_t key = 0;
-  Circuit circ;  // the planned circuit: a key hit is reused only if the content matches too
+  // the planned circuit: a key hit is reused only if the content matches too
+  int circ_n = 0;
+  std::vector<Gate> circ_gates;
   std::vector<int> order;
   std::vector<uint64_t> inv;
   std::vector<Pass> passes;
@@ -98,6 +100,9 @@ struct TimedLaunch {
   int kind;
   uint64_t bytes;
   int count = 1;  // launches between a and b (a run of consecutive fused passes: one interval)
+  // timing = 2: the pass this interval times (qgpu_get_pass_profile)
+  bool prof = false;
+  qgpu_pass_profile rec = {};
 };
 
 }  // namespace qgpu_impl
@@ -136,6 +141,7 @@ struct qgpu_state {
   double2* d_zero = nullptr;  // zero amplitudes: source of the expanded region in tile loads
   // timing
   std::vector<TimedLaunch> pending;
+  std::vector<qgpu_pass_profile> prof;  // timing = 2: completed per-pass records
   std::vector<cudaEvent_t> event_pool;
   Comm* comm = nullptr;
   std::vector<CachedPlan> plans;  // small LRU (kMaxPlans)

@@ -27,7 +27,8 @@ EXPORTS = [
     "qgpu_circuit_reorder", "qgpu_circuit_plan", "qgpu_circuit_plan_text", "qgpu_circuit_jit_check", "qgpu_get_involvement", "qgpu_get_chunk_bitmap",
     "qgpu_get_schedule", "qgpu_get_qubit_map", "qgpu_get_stats", "qgpu_reset_stats",
     "qgpu_nccl_unique_id", "qgpu_gfc_max_bytes", "qgpu_gfc_compress", "qgpu_gfc_decompress",
-    "qgpu_last_error", "qgpu_version",
+    "qgpu_last_error", "qgpu_version", "qgpu_get_pass_profile", "qgpu_measure_fp64_peak",
+    "qgpu_set_timing",
 ]
 
 
@@ -67,6 +68,15 @@ class Stats(ctypes.Structure):
         return {k: getattr(self, k) for k, _ in self._fields_}
 
 
+class PassProfile(ctypes.Structure):
+    _fields_ = [("kind", ctypes.c_int32), ("k_in", ctypes.c_int32), ("k_out", ctypes.c_int32),
+                ("n_gates", ctypes.c_int32), ("ms", ctypes.c_double), ("bytes", ctypes.c_uint64),
+                ("amps_computed", ctypes.c_uint64), ("fp64_ops", ctypes.c_double)]
+
+    def as_dict(self):
+        return {k: getattr(self, k) for k, _ in self._fields_}
+
+
 _lib = None
 
 
@@ -98,6 +108,8 @@ def load(path: str = LIB_PATH) -> ctypes.CDLL:
         "qgpu_gfc_max_bytes": [U64, ctypes.c_uint32, P],
         "qgpu_gfc_compress": [P, U64, ctypes.c_uint32, P, U64, P, P, P],
         "qgpu_gfc_decompress": [P, P, U64, ctypes.c_uint32, P, P],
+        "qgpu_get_pass_profile": [P, P, U64, P], "qgpu_measure_fp64_peak": [I, P],
+        "qgpu_set_timing": [P, I],
     }
     for name, args in sig.items():
         f = getattr(lib, name)
@@ -308,6 +320,17 @@ class State:
     def reset_stats(self):
         _check(load().qgpu_reset_stats(self._h))
 
+    def set_timing(self, mode: int):
+        _check(load().qgpu_set_timing(self._h, mode))
+
+    def pass_profile(self) -> list:
+        """Per-pass records (cfg timing=2) since the last call / reset (qgpu_get_pass_profile)."""
+        cnt = ctypes.c_uint64()
+        _check(load().qgpu_get_pass_profile(self._h, None, 0, ctypes.byref(cnt)))
+        arr = (PassProfile * max(cnt.value, 1))()
+        _check(load().qgpu_get_pass_profile(self._h, arr, cnt.value, ctypes.byref(cnt)))
+        return [arr[i].as_dict() for i in range(cnt.value)]
+
 
 def _nccl_lib_path():
     try:
@@ -350,6 +373,13 @@ def gfc_compress(d_in: int, n: int, seg_len: int, d_out: int, out_cap: int, d_of
 def gfc_decompress(d_in: int, d_offsets: int, n: int, seg_len: int, d_out: int, stream: int = 0) -> None:
     """Inverse of gfc_compress (device addresses; asynchronous on `stream`)."""
     _check(load().qgpu_gfc_decompress(d_in, d_offsets, n, seg_len, d_out, stream or None))
+
+
+def measure_fp64_peak(device: int = 0) -> float:
+    """Thread-level DFMA per second of `device` (qgpu_measure_fp64_peak)."""
+    out = ctypes.c_double()
+    _check(load().qgpu_measure_fp64_peak(device, ctypes.byref(out)))
+    return out.value
 
 
 def version() -> str:
