@@ -116,8 +116,8 @@ typedef struct {
   uint64_t chunks_skipped;     /* sum over passes of all-zero chunks skipped         */
   uint64_t algo_bytes;         /* algorithmic HBM bytes: reads of live input + writes        */
   uint64_t unfused_bytes;      /* bytes the same gates would move one gate per pass          */
-  uint64_t swaps;              /* global-local swaps (sharded mode)                          */
-  uint64_t swap_bytes;         /* bytes sent by this rank in swaps                           */
+  uint64_t swaps;              /* batched global-local swaps (sharded mode; one all-to-all each) */
+  uint64_t swap_bytes;         /* amplitude bytes sent by this rank in swaps                  */
   int64_t ops_before_full_involvement; /* Table II statistic, -1 if never    */
   double kernel_ms;            /* timing=1: summed CUDA-event time of pass kernels           */
   double tile_kernel_ms;       /* timing=1: time of fused tile kernels only                  */
@@ -136,6 +136,7 @@ typedef struct {
   uint64_t host_slice_skips;   /* slice visits skipped because the slice is all zero  */
   uint64_t host_runs;          /* runs of passes (one streaming sweep over the slices each)  */
   double host_ms;              /* timing=1: CUDA-event time of the streaming sweeps          */
+  uint64_t swap_bits;          /* rank bits exchanged by the swaps (sum of their widths s)   */
 } qgpu_stats;
 
 /* One pass of the last qgpu_apply_circuit / qgpu_apply_gate call when cfg.timing = 2 (every
@@ -255,7 +256,9 @@ qgpu_status qgpu_circuit_plan(const qgpu_circuit* c, int n_qubits, int world_siz
 /* Host-only (no GPU needed): the physical plan as text, for diagnostics and for executing the
  * sharded protocol independently in tests. One line per pass
  *   "P kind k_in k_out kg kg_from nswap g0 l0 g1 l1 ..." (kind as in qgpu_circuit_plan; 6 =
- *   activation of ranks [2^kg_from, 2^kg); 5 = swap of rank bit positions g with local l),
+ *   activation of ranks [2^kg_from, 2^kg): zeroed, or -- written as kg_from' = -1 - kg_from --
+ *   each receiving a copy of rank r - 2^kg_from's live prefix [0, 2^k_in) (cross-rank expand);
+ *   5 = ONE batched swap: rank bit position g_i <-> local position l_i for all i at once),
  * followed by one line per gate of the pass in physical positions at execution time
  *   "G nt p0 p1 control_mask diag re im re im ..." (the (2^nt)^2 matrix, row-major),
  * and a final "M pos_0 ... pos_{n-1}" with the final qubit map (-1 = never involved).

@@ -122,6 +122,8 @@ uint64_t plan_key(const qgpu_state* st, const qgpu_circuit* c) {
   if (const char* ev = std::getenv("QGPU_ZSKIP")) mix(uint64_t(std::atoi(ev) + 1) << 56);
   if (const char* ev = std::getenv("QGPU_LMIN")) mix(uint64_t(std::atoi(ev) + 1) << 60);
   if (const char* ev = std::getenv("QGPU_LRELAX")) mix(uint64_t(std::atoi(ev) + 1) << 52);
+  if (const char* ev = std::getenv("QGPU_GLOBAL_FIRST")) mix(uint64_t(std::atoi(ev) + 1) << 20);
+  if (const char* ev = std::getenv("QGPU_GLOBAL_MIN_LOCAL")) mix(uint64_t(std::atoi(ev) + 1) << 24);
   return h;
 }
 
@@ -186,11 +188,17 @@ void plan_env(PlanOptions* o) {
   if (const char* ev = std::getenv("QGPU_REGBITS")) o->reg_bits = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_MAX_UOPS")) o->max_u_ops = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_LOOKAHEAD")) o->lookahead = std::atoi(ev);
+  if (const char* ev = std::getenv("QGPU_GLOBAL_FIRST")) o->global_first = o->global_first && std::atoi(ev) != 0;
+  if (const char* ev = std::getenv("QGPU_GLOBAL_MIN_LOCAL")) o->global_min_local = std::atoi(ev);
 }
 
 PlanOptions plan_options(const qgpu_config& cfg, bool fuse) {
   PlanOptions o;
   o.fuse_bits = fuse ? cfg.fuse_bits : 0;
+  // sharded over ranks (NCCL or virtual): cross-rank first-touch expand; the host tier folds its
+  // swaps into streaming sweeps over <= 4 slices, so it keeps local-first placement, 2-bit swaps
+  o.global_first = cfg.world_size > 1 && cfg.host_slice_bits == 0;
+  if (cfg.host_slice_bits > 0) o.max_swap_bits = 2;
   plan_env(&o);
   o.prune = cfg.prune != 0;
   o.rule = cfg.involve_rule;
@@ -469,6 +477,8 @@ qgpu_status qgpu_state_destroy(qgpu_state* st) {
   if (st->h_ops) cudaFreeHost(st->h_ops);
   if (st->d_scratch) cudaFree(st->d_scratch);
   if (st->d_zero) cudaFree(st->d_zero);
+  for (double2* b : st->vstage)
+    if (b) cudaFree(b);
   if (st->d_meas) cudaFree(st->d_meas);
   for (CachedPlan& cp : st->plans) {
     if (cp.d_blob) cudaFree(cp.d_blob);
@@ -955,6 +965,7 @@ qgpu_status qgpu_circuit_plan(const qgpu_circuit* c, int n, int world, int reord
     map.init(n, n - g);
     PlanOptions o;
     o.fuse_bits = fuse_bits;
+    o.global_first = world > 1;
     plan_env(&o);
     o.rule = reorder_mode >> 2 & 1;
     std::vector<Pass> passes;
@@ -987,6 +998,7 @@ qgpu_status qgpu_circuit_plan_text(const qgpu_circuit* c, int n, int world, int 
     map.init(n, n - g);
     PlanOptions o;
     o.fuse_bits = fuse_bits;
+    o.global_first = world > 1;
     plan_env(&o);
     o.rule = reorder_mode >> 2 & 1;
     std::vector<Pass> passes;
@@ -994,7 +1006,8 @@ qgpu_status qgpu_circuit_plan_text(const qgpu_circuit* c, int n, int world, int 
     std::string t;
     char line[512];
     for (const Pass& p : passes) {
-      std::snprintf(line, sizeof(line), "P %d %d %d %d %d %d", p.kind, p.k_in, p.k_out, p.kg, p.kg_from, p.nswap);
+      std::snprintf(line, sizeof(line), "P %d %d %d %d %d %d", p.kind, p.k_in, p.k_out, p.kg,
+                    p.kind == PK_ACTIVATE && p.act_copy ? -1 - p.kg_from : p.kg_from, p.nswap);
       t += line;
       for (int i = 0; i < p.nswap; ++i) {
         std::snprintf(line, sizeof(line), " %d %d", p.swap_global[i], p.swap_local[i]);

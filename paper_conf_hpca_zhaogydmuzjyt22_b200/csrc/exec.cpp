@@ -67,38 +67,123 @@ qgpu_status zero_fill(qgpu_state* st, double2* psi, uint64_t from, uint64_t to) 
   return QGPU_OK;
 }
 
-// Global-local swap (a10): exchange rank bit (swap_global - m) with local position swap_local,
-// one pair at a time. Virtual ranks: in-device swap of the two halves; NCCL: pack, send/recv with
-// the partner rank in slabs through bounded staging, unpack (in place: the received half lands
-// in the slots of the half that was sent).
+// Global-local swap (a10): the pass's s pairs (rank bit swap_global - m <-> local position
+// swap_local) as ONE batched all-to-all inside each group of 2^s ranks, over the live prefix only
+// (amplitudes beyond 2^kl are zero on every rank and stay zero). NCCL: comm_swap (pipelined slabs,
+// two streams). Virtual ranks (every shard on this GPU): the same geometry, pack / unpack kernels
+// and slab loop, with device-to-device copies between the shards' staging as the transport.
 qgpu_status exec_swap(qgpu_state* st, const Pass& p, uint64_t* bytes) {
   const int m = st->m;
-  const uint64_t half = 1ull << (m - 1);
+  const uint64_t L = live(st, p.k_in);
   const uint64_t active = 1ull << p.kg;
+  int j[8], l[8];
   for (int i = 0; i < p.nswap; ++i) {
-    const int j = p.swap_global[i] - m, lp = p.swap_local[i];
-    if (st->virt) {
-      for (Shard& sh : st->shards) {
-        const uint64_t r = uint64_t(sh.rank);
-        if (r >= active || (r >> j & 1)) continue;
-        const uint64_t partner = r | (1ull << j);
-        CK(launch_swap_halves(st->stream, sh.psi, st->shards[partner].psi, lp, half));
-        st->stats.kernels_launched++;
-      }
-    } else {
-      for (Shard& sh : st->shards) {
-        if (uint64_t(sh.rank) >= active) continue;
-        qgpu_status s = comm_swap_bit(st->comm, sh.psi, m, sh.rank, j, lp, st->stream, &g_err);
-        if (s) {
-          st->poisoned = true;
-          return s;
-        }
+    j[i] = p.swap_global[i] - m;
+    l[i] = p.swap_local[i];
+  }
+  const uint64_t slab_req = std::max<uint64_t>(32, st->cfg.swap_slab_bytes / 16 / ((1ull << p.nswap) - 1));
+  uint64_t sent = 0;
+  if (!st->virt) {
+    for (Shard& sh : st->shards) {
+      if (uint64_t(sh.rank) >= active) continue;
+      SwapGeom g;
+      g.init(sh.rank, p.nswap, j, l, L);
+      qgpu_status s = comm_swap(st->comm, sh.psi, g, slab_req, st->stream, &sent, &g_err);
+      if (s) {
+        st->poisoned = true;
+        return s;
       }
     }
-    *bytes += 16 * half;
-    st->stats.swaps++;
-    st->stats.swap_bytes += 16 * half;
+  } else {
+    std::vector<SwapGeom> geo(st->shards.size());
+    for (Shard& sh : st->shards)
+      if (uint64_t(sh.rank) < active) geo[size_t(sh.rank)].init(sh.rank, p.nswap, j, l, L);
+    const SwapGeom& g0 = geo[0];
+    const uint64_t slab = std::max<uint64_t>(1, std::min(slab_req, g0.rest));
+    const size_t need = size_t(slab) * size_t(g0.nb);
+    if (need > st->vstage_cap) {
+      CK(cudaStreamSynchronize(st->stream));
+      for (double2* b : st->vstage) CK(cudaFree(b));
+      st->vstage.assign(2 * st->shards.size(), nullptr);
+      for (double2*& b : st->vstage) CK(cudaMalloc(&b, need * sizeof(double2)));
+      st->vstage_cap = need;
+    }
+    for (uint64_t t0 = 0; t0 < g0.rest; t0 += slab) {
+      const uint64_t cnt = std::min(slab, g0.rest - t0);
+      BlockArgs a{};
+      for (Shard& sh : st->shards) {  // pack every active shard's slab
+        if (uint64_t(sh.rank) >= active) continue;
+        const SwapGeom& g = geo[size_t(sh.rank)];
+        a.psi = sh.psi;
+        a.buf = st->vstage[2 * size_t(sh.rank)];
+        a.nins = g.nins;
+        for (int k = 0; k < g.nins; ++k) a.ins[k] = g.ins[k];
+        a.t0 = t0;
+        a.cnt = cnt;
+        a.nb = g.nb;
+        for (int b = 0; b < g.nb; ++b) a.pat[b] = g.pat[b];
+        CK(launch_pack_blocks(st->stream, a));
+        st->stats.kernels_launched++;
+      }
+      for (Shard& sh : st->shards) {  // transport: block b of rank r -> peer's slot for r's block
+        if (uint64_t(sh.rank) >= active) continue;
+        const SwapGeom& g = geo[size_t(sh.rank)];
+        for (int b = 0; b < g.nb; ++b) {
+          const SwapGeom& gp = geo[size_t(g.peer[b])];
+          double2* dst = st->vstage[2 * size_t(g.peer[b]) + 1] + size_t(gp.slot(g.e)) * cnt;
+          const double2* src = st->vstage[2 * size_t(sh.rank)] + size_t(b) * cnt;
+          CK(cudaMemcpyAsync(dst, src, cnt * sizeof(double2), cudaMemcpyDeviceToDevice, st->stream));
+        }
+        if (sh.rank == 0) sent += 16 * cnt * uint64_t(g.nb);
+      }
+      for (Shard& sh : st->shards) {  // unpack the received blocks in place
+        if (uint64_t(sh.rank) >= active) continue;
+        const SwapGeom& g = geo[size_t(sh.rank)];
+        a.psi = sh.psi;
+        a.buf = st->vstage[2 * size_t(sh.rank) + 1];
+        a.nins = g.nins;
+        for (int k = 0; k < g.nins; ++k) a.ins[k] = g.ins[k];
+        a.t0 = t0;
+        a.cnt = cnt;
+        a.nb = g.nb;
+        for (int b = 0; b < g.nb; ++b) a.pat[b] = g.pat[b];
+        CK(launch_unpack_blocks(st->stream, a));
+        st->stats.kernels_launched++;
+      }
+    }
   }
+  *bytes += sent;
+  st->stats.swaps++;
+  st->stats.swap_bits += uint64_t(p.nswap);
+  st->stats.swap_bytes += sent;
+  return QGPU_OK;
+}
+
+// Rank activation (PK_ACTIVATE): ranks [2^kg_from, 2^kg) start to hold live amplitudes. A copy
+// activation (a fresh qubit placed on a rank bit by an uncontrolled 1-qubit gate, §8e) gives each
+// new rank the live prefix of rank r - 2^kg_from; otherwise the new ranks are zeroed.
+qgpu_status exec_activate(qgpu_state* st, const Pass& p) {
+  const uint64_t active = 1ull << p.kg, from = 1ull << p.kg_from;
+  if (!p.act_copy) {
+    for (Shard& sh : st->shards)
+      if (uint64_t(sh.rank) >= from && uint64_t(sh.rank) < active) {
+        qgpu_status s = zero_fill(st, sh.psi, 0, 1ull << st->m);
+        if (s) return s;
+      }
+    return QGPU_OK;
+  }
+  const uint64_t L = live(st, p.k_in);
+  if (!st->virt) {
+    qgpu_status s = comm_activate_copy(st->comm, st->shards[0].psi, p.kg_from, p.kg, L, st->stream, &g_err);
+    if (s) st->poisoned = true;
+    // the rest of a newly active buffer is read as zeros only through the live prefix: with
+    // prune = 0 the copy covers the whole buffer (L = 2^m)
+    return s;
+  }
+  for (Shard& sh : st->shards)
+    if (uint64_t(sh.rank) >= from && uint64_t(sh.rank) < active)
+      CK(cudaMemcpyAsync(sh.psi, st->shards[size_t(sh.rank) - size_t(from)].psi, L * sizeof(double2),
+                         cudaMemcpyDeviceToDevice, st->stream));
   return QGPU_OK;
 }
 
@@ -346,14 +431,7 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops,
     }
     return QGPU_OK;
   }
-  if (p.kind == PK_ACTIVATE) {
-    for (Shard& sh : st->shards)
-      if (uint64_t(sh.rank) >= (1ull << p.kg_from) && uint64_t(sh.rank) < active) {
-        qgpu_status s = zero_fill(st, sh.psi, 0, 1ull << m);
-        if (s) return s;
-      }
-    return QGPU_OK;
-  }
+  if (p.kind == PK_ACTIVATE) return exec_activate(st, p);
   const bool timing = st->cfg.timing != 0 && own_timing;
   TimedLaunch tl{};
   if (timing) {
@@ -707,6 +785,7 @@ qgpu_status host_sweep(qgpu_state* st, const std::vector<const Pass*>& run,
   for (const HostSwap& x : sw) {
     (void)x;
     st->stats.swaps++;
+    st->stats.swap_bits++;
     st->stats.swap_bytes += 16 * (full / 2) * (nact >> 1);
   }
   st->stats.host_runs++;

@@ -507,16 +507,22 @@ __global__ void swap_halves_kernel(double2* a, double2* b, int lp, uint64_t half
     __stcs(b + i0, x);
   }
 }
-// a10 (NCCL): gather / scatter slab [t0, t0+count) of the half with local bit lp == bit
-__global__ void pack_half_kernel(const double2* psi, double2* buf, int lp, int bit, uint64_t t0, uint64_t count) {
+// a10 batched swap: gather / scatter one slab of every exchanged block (kernels.h BlockArgs).
+// blockIdx.y = block; x grid-strides over the slab's rest indices, so with swapped positions >= 5
+// every warp moves >= 512 contiguous bytes.
+__global__ void pack_blocks_kernel(BlockArgs a) {
+  const uint64_t pat = a.pat[blockIdx.y];
+  double2* out = a.buf + uint64_t(blockIdx.y) * a.cnt;
   const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
-  for (uint64_t t = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < count; t += stride)
-    buf[t] = __ldcs(psi + (insert0(t0 + t, lp) | (uint64_t(bit) << lp)));
+  for (uint64_t t = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < a.cnt; t += stride)
+    out[t] = __ldcs(a.psi + (deposit(a.t0 + t, a.ins, a.nins) | pat));
 }
-__global__ void unpack_half_kernel(double2* psi, const double2* buf, int lp, int bit, uint64_t t0, uint64_t count) {
+__global__ void unpack_blocks_kernel(BlockArgs a) {
+  const uint64_t pat = a.pat[blockIdx.y];
+  const double2* in = a.buf + uint64_t(blockIdx.y) * a.cnt;
   const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
-  for (uint64_t t = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < count; t += stride)
-    __stcs(psi + (insert0(t0 + t, lp) | (uint64_t(bit) << lp)), buf[t]);
+  for (uint64_t t = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; t < a.cnt; t += stride)
+    __stcs(a.psi + (deposit(a.t0 + t, a.ins, a.nins) | pat), in[t]);
 }
 __global__ void add_kernel(double* out, const double* in, uint64_t count) {
   const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
@@ -672,14 +678,16 @@ cudaError_t launch_swap_halves(cudaStream_t st, double2* a, double2* b, int lp, 
   swap_halves_kernel<<<grid_for(half, 256 * 4, 8), 256, 0, st>>>(a, b, lp, half);
   return cudaGetLastError();
 }
-cudaError_t launch_pack_half(cudaStream_t st, const double2* psi, double2* buf, int lp, int bit, uint64_t t0,
-                             uint64_t count) {
-  pack_half_kernel<<<grid_for(count, 256 * 4, 8), 256, 0, st>>>(psi, buf, lp, bit, t0, count);
+cudaError_t launch_pack_blocks(cudaStream_t st, const BlockArgs& a) {
+  if (!a.cnt || !a.nb) return cudaSuccess;
+  const unsigned gx = std::max(1u, grid_for(a.cnt * a.nb, 256 * 4, 8) / unsigned(a.nb));
+  pack_blocks_kernel<<<dim3(gx, unsigned(a.nb)), 256, 0, st>>>(a);
   return cudaGetLastError();
 }
-cudaError_t launch_unpack_half(cudaStream_t st, double2* psi, const double2* buf, int lp, int bit, uint64_t t0,
-                               uint64_t count) {
-  unpack_half_kernel<<<grid_for(count, 256 * 4, 8), 256, 0, st>>>(psi, buf, lp, bit, t0, count);
+cudaError_t launch_unpack_blocks(cudaStream_t st, const BlockArgs& a) {
+  if (!a.cnt || !a.nb) return cudaSuccess;
+  const unsigned gx = std::max(1u, grid_for(a.cnt * a.nb, 256 * 4, 8) / unsigned(a.nb));
+  unpack_blocks_kernel<<<dim3(gx, unsigned(a.nb)), 256, 0, st>>>(a);
   return cudaGetLastError();
 }
 cudaError_t launch_add(cudaStream_t st, double* out, const double* in, uint64_t count) {

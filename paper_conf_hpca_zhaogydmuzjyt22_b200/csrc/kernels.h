@@ -78,10 +78,24 @@ cudaError_t probe_fp64(double* fma_per_s);
 cudaError_t launch_zero_where(cudaStream_t st, double2* psi, uint64_t L, uint64_t mask);
 // sharded swaps (a10)
 cudaError_t launch_swap_halves(cudaStream_t st, double2* a, double2* b, int lp, uint64_t half);
-cudaError_t launch_pack_half(cudaStream_t st, const double2* psi, double2* buf, int lp, int bit, uint64_t t0,
-                             uint64_t count);
-cudaError_t launch_unpack_half(cudaStream_t st, double2* psi, const double2* buf, int lp, int bit, uint64_t t0,
-                               uint64_t count);
+// a10 batched global-local swap of s rank bits with s local positions: the live local amplitudes
+// split into 2^s blocks by their bits at the local positions; block d (all but the rank's own)
+// goes to the peer whose rank bits are d. A slab is the rest-index range [t0, t0 + cnt) of every
+// block (rest index = the live index with the swapped local positions removed); pack gathers it
+// into buf[b * cnt + t], unpack scatters buf back (in place: a received block lands in the slots
+// of the block that was sent to the same peer).
+constexpr int kMaxSwapBlocks = 63;  // 2^6 - 1: up to 64 ranks in one batched swap
+struct BlockArgs {
+  double2* psi;
+  double2* buf;
+  int nins;
+  int ins[8];       // the swapped local positions, ascending
+  uint64_t t0, cnt;
+  int nb;           // blocks in the slab
+  uint64_t pat[kMaxSwapBlocks];  // block b's bits at the swapped local positions
+};
+cudaError_t launch_pack_blocks(cudaStream_t st, const BlockArgs& a);
+cudaError_t launch_unpack_blocks(cudaStream_t st, const BlockArgs& a);
 cudaError_t launch_add(cudaStream_t st, double* out, const double* in, uint64_t count);
 
 // GFC compression (gfc.cu): per-segment padded sizes, encode at scanned offsets,

@@ -89,6 +89,7 @@ struct QubitMap {
   void touch(uint64_t mask);
   uint64_t phys_mask(uint64_t logical_mask) const;
   void swap_positions(int pa, int pb);  // exchange the logical qubits at two positions
+  void place_global(int q);             // place a never-involved qubit on the next rank bit
 };
 
 // --------------------------------------------------------------------------- device ops
@@ -126,7 +127,8 @@ struct PhysGate {
 
 enum PassKind : int {
   PK_TILE = 0, PK_PAIR = 1, PK_QUAD = 2, PK_DIAG = 3, PK_RELABEL = 4, PK_SWAP = 5,
-  PK_ACTIVATE = 6,  // ranks [2^kg_from, 2^kg) become active (their buffers are zeroed)
+  PK_ACTIVATE = 6,  // ranks [2^kg_from, 2^kg) become active: zeroed, or (act_copy) each receives a
+                    // copy of the live prefix of rank r - 2^kg_from (cross-rank first-touch expand)
   PK_ZERO = 7       // write zeros over the live amplitudes that have a bit of `zmask` set
 };
 
@@ -145,6 +147,7 @@ struct Pass {
   int nswap = 0;
   int swap_global[8], swap_local[8];
   int kg_from = 0;              // activation pass
+  int act_copy = 0;             // activation by copy (a fresh qubit placed on a rank bit, §8e)
   mutable void* jit_fn = nullptr;  // specialised kernel, resolved at the first launch
   mutable void* jit_fn_hist[3] = {nullptr, nullptr, nullptr};  // fused-measurement variants, per mode
   uint64_t unfused_bytes = 0;   // bytes the pass's gates would move one gate per pass
@@ -171,6 +174,12 @@ struct PlanOptions {
   // skip the halves of positions that a first touch left zero (placed by a diagonal gate or as
   // a control) until a non-diagonal op targets them; single resident state, fused passes only
   bool zskip = true;
+  // sharded (m < n): place fresh qubits first touched by an uncontrolled 1-qubit non-diagonal
+  // gate on the rank bits (up to log2 G of them) once >= global_min_local local positions are
+  // assigned, so every rank holds live amplitudes from early on (cross-rank expand, §8e)
+  bool global_first = false;
+  int global_min_local = 10;
+  int max_swap_bits = 8;  // rank bits per batched swap (the host tier's sweeps fold at most 2)
 };
 
 // Cut `gates` into passes, updating `map` (involvement, placement) exactly as the execution

@@ -161,6 +161,12 @@ uint64_t QubitMap::phys_mask(uint64_t lm) const {
   return r;
 }
 
+void QubitMap::place_global(int q) {
+  const int p = m + kg++;
+  pos[q] = p;
+  lq[p] = q;
+}
+
 void QubitMap::swap_positions(int pa, int pb) {
   const int qa = lq[pa], qb = lq[pb];
   lq[pa] = qb;
@@ -958,6 +964,25 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
   };
   int xi = 0;  // execution index: passes are consecutive runs of the execution order
 
+  // a10 swap planning: order positions at which each logical qubit is a non-diagonal target
+  // (the only use that needs it on a local position); next_use(q, k) = the first at or after k
+  std::vector<std::vector<int>> nd_uses(size_t(std::max(map.n, 1)));
+  if (map.m < map.n) {
+    for (int k = 0; k < G; ++k) {
+      if (peephole && absorbed[k]) continue;
+      const Gate& gg = (peephole && fused[k] >= 0) ? fgates[fused[k]] : gates[order[k]];
+      if (gg.diag || gg.relabel) continue;
+      for (int j = 0; j < gg.nt; ++j) nd_uses[size_t(gg.t[j])].push_back(k);
+    }
+  }
+  constexpr int kNever = std::numeric_limits<int>::max();
+  auto next_use = [&](int q, int k) {
+    if (q < 0) return kNever;
+    const auto& v = nd_uses[size_t(q)];
+    auto it = std::lower_bound(v.begin(), v.end(), k);
+    return it == v.end() ? kNever : *it;
+  };
+
   // execute order position k: placement, sharded activation / swaps, then the gate joins the
   // open fused pass or opens a new one
   Gate restricted;  // refined rule: a diagonal gate restricted to its involved operands
@@ -997,6 +1022,27 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
       }
       gp = &restricted;
     }
+    // cross-rank first-touch expand (§8e): a fresh qubit whose first touch is an uncontrolled
+    // 1-qubit non-diagonal gate U may go to the next rank bit: the newly active ranks receive a
+    // copy of the live prefix (PK_ACTIVATE with act_copy) and, because that bit was |0>
+    // everywhere, U acts as the diagonal diag(U00, U10) on the rank bit -- rank r with the bit
+    // set scales its copy by U10, the others by U00 (exact).
+    Gate gdiag;
+    int gfirst_q = -1;
+    if (opt.global_first && map.kg < map.n - map.m && map.kl >= std::min(map.m, opt.global_min_local) && !gp &&
+        !(peephole && absorbed[k])) {
+      const Gate& gg = gate_at(k);
+      if (!gg.diag && !gg.relabel && gg.nt == 1 && gg.cmask == 0 && (fresh >> gg.t[0] & 1)) {
+        gfirst_q = gg.t[0];
+        map.place_global(gfirst_q);
+        gdiag = gg;
+        gdiag.diag = true;
+        gdiag.U[0] = gg.U[0];
+        gdiag.U[3] = gg.U[2];
+        gdiag.U[1] = gdiag.U[2] = cplx{0.0, 0.0};
+        gp = &gdiag;
+      }
+    }
     map.touch(inv_g);
     const Gate& g = gp ? *gp : gate_at(k);
     if (zskip && fresh) {
@@ -1035,6 +1081,7 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
       B.start(PK_ACTIVATE, xi, k_before);
       B.cur.kg_from = kg_before;
       B.cur.kg = map.kg;
+      B.cur.act_copy = gfirst_q >= 0 ? 1 : 0;
       B.cur.k_out = map.kl;
       B.close();
     }
@@ -1074,15 +1121,48 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
         B.close();
         B.start(PK_SWAP, xi, map.kl);
         B.cur.count = 0;
-        int victim = m - 1;
-        for (int j = 0; j < ng; ++j) {
-          while (tloc >> victim & 1) --victim;
-          B.cur.swap_global[j] = gl[j];
-          B.cur.swap_local[j] = victim;
-          --victim;
+        // Victims: the assigned local positions whose qubits are needed (as non-diagonal
+        // targets) farthest in the future, preferring positions >= 5 (the swap's pack / unpack
+        // then move >= 512-byte runs). The rank bits needed now are swapped in; other rank-bit
+        // qubits join the same batched swap while they are needed sooner than the next victim
+        // (one s-bit all-to-all moves 1 - 2^-s of the live data; s one-bit swaps move s/2).
+        const int gbits = map.n - m;
+        std::vector<int> vic;
+        for (int pass_lo = 0; pass_lo < 2 && int(vic.size()) < ng; ++pass_lo) {
+          vic.clear();
+          for (int p = 0; p < map.kl; ++p)
+            if (!(tloc >> p & 1) && (pass_lo == 1 || p >= 5)) vic.push_back(p);
         }
-        B.cur.nswap = ng;
-        for (int j = 0; j < ng; ++j) map.swap_positions(B.cur.swap_global[j], B.cur.swap_local[j]);
+        std::stable_sort(vic.begin(), vic.end(), [&](int a, int b) {
+          const int na = next_use(map.lq[a], k), nb = next_use(map.lq[b], k);
+          if (na != nb) return na > nb;
+          return a > b;
+        });
+        int ns = 0;
+        for (int j = 0; j < ng; ++j) {
+          B.cur.swap_global[ns] = gl[j];
+          B.cur.swap_local[ns] = vic[size_t(j)];
+          ++ns;
+        }
+        std::vector<int> extra;
+        for (int j = 0; j < map.kg; ++j) {
+          const int P = m + j;
+          if (P == gl[0] || (ng > 1 && P == gl[1])) continue;
+          if (next_use(map.lq[P], k) != kNever) extra.push_back(P);
+        }
+        std::stable_sort(extra.begin(), extra.end(),
+                         [&](int a, int b) { return next_use(map.lq[a], k) < next_use(map.lq[b], k); });
+        for (int P : extra) {
+          if (ns >= gbits || ns >= opt.max_swap_bits || ns >= int(vic.size())) break;
+          if (next_use(map.lq[P], k) >= next_use(map.lq[vic[size_t(ns)]], k)) break;
+          B.cur.swap_global[ns] = P;
+          B.cur.swap_local[ns] = vic[size_t(ns)];
+          ++ns;
+        }
+        B.cur.nswap = ns;
+        const int ng_all = ns;
+        (void)ng_all;
+        for (int j = 0; j < B.cur.nswap; ++j) map.swap_positions(B.cur.swap_global[j], B.cur.swap_local[j]);
         B.cur.k_out = map.kl;
         B.close();
       }

@@ -144,6 +144,10 @@ struct qgpu_state {
   std::vector<qgpu_pass_profile> prof;  // timing = 2: completed per-pass records
   std::vector<cudaEvent_t> event_pool;
   Comm* comm = nullptr;
+  // virtual ranks: per shard a send and a receive staging buffer of vstage_cap amplitudes (the
+  // device-copy transport of the batched swap)
+  std::vector<double2*> vstage;
+  size_t vstage_cap = 0;
   std::vector<CachedPlan> plans;  // small LRU (kMaxPlans)
   uint64_t plan_clock = 0;
   // host-memory tier (cfg.host_slice_bits = h > 0, NEXT-2): 2^h slices of 2^m amplitudes in

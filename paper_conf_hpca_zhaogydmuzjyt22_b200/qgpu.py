@@ -62,7 +62,7 @@ class Stats(ctypes.Structure):
         ("jit_launches", ctypes.c_uint64), ("jit_compiles", ctypes.c_uint64), ("jit_ms", ctypes.c_double),
         ("host_h2d_bytes", ctypes.c_uint64), ("host_d2h_bytes", ctypes.c_uint64),
         ("host_slice_loads", ctypes.c_uint64), ("host_slice_skips", ctypes.c_uint64),
-        ("host_runs", ctypes.c_uint64), ("host_ms", ctypes.c_double)]
+        ("host_runs", ctypes.c_uint64), ("host_ms", ctypes.c_double), ("swap_bits", ctypes.c_uint64)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}

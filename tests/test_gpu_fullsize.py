@@ -15,6 +15,19 @@ pytestmark = [pytest.mark.gpu, pytest.mark.slow]
 TOL = 1e-10
 
 
+@pytest.fixture(autouse=True)
+def library_default_jit_threshold():
+    """Run these tests in exactly the configuration bench.py times: the library's default JIT
+    threshold (every fused pass of >= 2^12 amplitudes NVRTC-specialised), not the suite-wide
+    2^20 of conftest.py (the library reads QGPU_JIT_MIN_BITS per call)."""
+    import os
+    old = os.environ.get("QGPU_JIT_MIN_BITS")
+    os.environ.pop("QGPU_JIT_MIN_BITS", None)
+    yield
+    if old is not None:
+        os.environ["QGPU_JIT_MIN_BITS"] = old
+
+
 @pytest.fixture(scope="module")
 def q():
     import torch
@@ -45,16 +58,97 @@ def test_c2_qft28_basis_state_full_state(q):
     assert abs(p[0] - 1) <= 1e-12
 
 
-def test_c2_qft28_zero_state_and_stats(q):
+def test_c2_qft28_zero_state_full_state_and_stats(q):
+    """configs[1], the bench's QFT_28 on |0...0>: all 2^28 amplitudes vs the closed form
+    QFT|0> = 2^-14 everywhere (P3), read in 2^24-amplitude pieces; the fused passes of
+    >= 2^12 amplitudes ran NVRTC-specialised kernels (as in bench.py)."""
     c = wc.qft(28)
     with q.State(28, chunk_bits=21) as s:
         s.apply_circuit(q.Circuit(c.qasm()))
-        a = s.amplitudes(0, 1 << 20)
-        b = s.amplitudes((1 << 28) - (1 << 20), 1 << 20)
+        u = 1 / math.sqrt(1 << 28)
+        worst = 0.0
+        for start in range(0, 1 << 28, 1 << 24):
+            worst = max(worst, float(np.abs(s.amplitudes(start, 1 << 24) - u).max()))
         st = s.stats()
-    u = 1 / math.sqrt(1 << 28)
-    assert np.abs(a - u).max() <= TOL and np.abs(b - u).max() <= TOL
+    assert worst <= TOL
     assert st["chunks_skipped"] > 0 and st["ops_before_full_involvement"] > 300
+    plan = q.Circuit(c.qasm()).plan(28)
+    want = int(sum(1 for r in plan if r[2] == 0 and r[4] >= 12))
+    assert want >= 3 and st["jit_launches"] == want
+
+
+def test_c3_qaoa32_vs_oracle_full_state(q):
+    """configs[2] at full size: QAOA MaxCut p=2, 32 qubits, the bench's exact
+    configuration (reorder=2, prune=1, b=12, default JIT threshold) against the oracle's plain
+    program-order simulation of the same QASM (64 GiB on the host, all cores), every one of the
+    2^32 amplitudes compared in 2^24-amplitude pieces."""
+    import os
+    c = wc.config_circuit("C3")
+    text = c.qasm()
+    avail = 0
+    for line in open("/proc/meminfo"):
+        if line.startswith("MemAvailable"):
+            avail = int(line.split()[1]) * 1024
+    if avail < (16 << c.n) + (8 << 30):
+        pytest.skip(f"needs {16 << c.n} B of host memory for the oracle state, {avail} available")
+    ref = osv.simulate(text, threads=os.cpu_count())
+    with q.State(c.n) as s:
+        s.apply_circuit(q.Circuit(text))
+        worst = 0.0
+        for start in range(0, 1 << c.n, 1 << 24):
+            got = s.amplitudes(start, 1 << 24)
+            worst = max(worst, float(np.abs(got - ref[start:start + (1 << 24)]).max()))
+        p = s.probabilities([])
+    del ref
+    assert worst <= TOL
+    assert abs(p[0] - 1) <= 1e-12
+
+
+@pytest.mark.parametrize("n", [31, 32])
+def test_unfused_kernels_full_size_high_indices(q, n):
+    """a6/a7/a8 unfused kernels (fuse_bits=0, as the bench's microbenchmark) at n = 31, 32, i.e.
+    amplitude indices above 2^31: a random product state built gate by gate from |0> (first-touch
+    expansion of every qubit), then generic 1-qubit gates at low / middle / top positions with and
+    without controls on the top qubits, 2-qubit gates spanning bit 0 and the top bits, CX with
+    control 0, CP on (top, 0) and a 2-qubit diagonal; sampled amplitudes (contiguous ranges at the
+    bottom, middle and top of the index space) vs the oracle's light-cone evaluation."""
+    from oracle import qasm as oq
+    from lightcone import product_light_cone
+    rng = np.random.default_rng(100 + n)
+    top = n - 1
+    factors = []
+    prep = []
+    for t in range(n):
+        U = oq.u3(*rng.uniform(-3, 3, 3))
+        prep.append(U)
+        factors.append(U[:, 0].copy())            # U|0>
+    U4 = np.linalg.qr(rng.normal(size=(4, 4)) + 1j * rng.normal(size=(4, 4)))[0]
+    X = np.array([[0, 1], [1, 0]], dtype=complex)
+    gates = [(oq.u3(*rng.uniform(-3, 3, 3)), [0], []),
+             (oq.u3(*rng.uniform(-3, 3, 3)), [top], []),
+             (oq.u3(*rng.uniform(-3, 3, 3)), [17], [top]),
+             (oq.u3(*rng.uniform(-3, 3, 3)), [2], [top - 1, top]),
+             (U4, [top, 3], []),
+             (U4.conj().T @ np.diag(np.exp(1j * rng.uniform(-3, 3, 4))), [0, top - 1], []),
+             (X, [top], [0]),
+             (oq.phase(0.7), [0], [top]),
+             (np.diag(np.exp(1j * rng.uniform(-3, 3, 4))), [top, 1], [])]
+    with q.State(n, fuse_bits=0) as s:
+        for t in range(n):
+            s.apply_gate(prep[t], [t])
+        for U, t, cs in gates:
+            s.apply_gate(U, t, cs)
+        worst = 0.0
+        starts = [0, (1 << (n - 1)) - 2048, 1 << (n - 1), 3 << (n - 2), (1 << n) - 4096,
+                  int(rng.integers(1 << (n - 1), (1 << n) - 4096))]
+        for st_ in starts:
+            got = s.amplitudes(st_, 4096)
+            idx = np.arange(st_, st_ + 4096, dtype=np.int64)
+            exp = product_light_cone(n, factors, gates, idx)
+            worst = max(worst, float(np.abs(got - exp).max()))
+        p = s.probabilities([])
+    assert worst <= TOL
+    assert abs(p[0] - 1) <= 1e-12
 
 
 def test_qaoa28_vs_oracle_full(q):

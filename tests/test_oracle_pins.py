@@ -307,3 +307,24 @@ def test_parser_errors_and_broadcast():
     assert n == 5 and [x.targets for x in g[:3]] == [(2,), (3,), (4,)]
     assert g[3].controls == (1,) and g[3].targets == (4,)
     assert np.allclose(g[4].U, oq.rx(-math.pi / 4 + 1.0))
+
+
+def test_light_cone_helper_matches_full_simulation():
+    """The sampled-amplitude helper of the n = 31/32 GPU tests (tests/lightcone.py) equals the
+    oracle's full simulation of the same product preparation + gates, at n = 9 on every index."""
+    from lightcone import product_light_cone
+    n = 9
+    rng = np.random.default_rng(7)
+    prep = [oq.u3(*rng.uniform(-3, 3, 3)) for _ in range(n)]
+    factors = [U[:, 0].copy() for U in prep]
+    U4 = np.linalg.qr(rng.normal(size=(4, 4)) + 1j * rng.normal(size=(4, 4)))[0]
+    gates = [(oq.u3(*rng.uniform(-3, 3, 3)), [0], []), (oq.u3(1, 2, 3), [8], [7]),
+             (U4, [8, 3], []), (np.array([[0, 1], [1, 0]], dtype=complex), [8], [0]),
+             (oq.phase(0.7), [0], [8]), (np.diag(np.exp(1j * rng.uniform(-3, 3, 4))), [8, 1], [])]
+    psi = osv.zero_state(n)
+    for t in range(n):
+        osv.apply_gate(psi, n, prep[t], [t])
+    for U, t, cs in gates:
+        osv.apply_gate(psi, n, U, t, cs)
+    got = product_light_cone(n, factors, gates, np.arange(1 << n))
+    assert np.abs(got - psi).max() <= 1e-14

@@ -85,19 +85,52 @@ def _shard_main(rank, world, port, text, n, out):
     if rank == 0:
         psi[0] = 1.0
     passes, fmap = _parse_plan(text)
+    loc = np.arange(psi.size)
     for p in passes:
-        if p["kind"] == 5:  # global-local swap, one rank bit at a time
-            for gp, lp in p["swaps"]:
+        if p["kind"] == 6 and p["kg_from"] < 0:  # cross-rank expand: copy of rank r - 2^kg_from
+            kf, kg = -1 - p["kg_from"], p["kg"]
+            assert kg == kf + 1
+            lo = 1 << kf
+            if rank < lo and rank + lo < (1 << kg):
+                dist.send(torch.from_numpy(psi.view(np.float64).copy()), rank + lo)
+            elif lo <= rank < (1 << kg):
+                buf = torch.empty(2 * psi.size, dtype=torch.float64)
+                dist.recv(buf, rank - lo)
+                psi[:] = buf.numpy().view(np.complex128)
+        if p["kind"] == 5 and rank < (1 << p["kg"]):
+            # ONE batched swap: for every pair (g_i, l_i) the logical qubit on rank bit g_i - m
+            # trades places with the one on local position l_i. The amplitude at (rank r, local i)
+            # moves to the rank whose bits g_i - m equal i's bits l_i, at the local index whose
+            # bits l_i equal r's bits g_i - m (the rest of i unchanged): an all-to-all inside each
+            # group of ranks that differ only in the swapped rank bits.
+            pairs = p["swaps"]
+            dest_rank = np.full(psi.size, rank, dtype=np.int64)
+            dest_loc = loc.copy()
+            for gp, lp in pairs:
                 j = gp - m
-                b = (rank >> j) & 1
-                partner = rank ^ (1 << j)
-                idx = np.nonzero(((np.arange(psi.size) >> lp) & 1) == (1 - b))[0]
-                send = torch.from_numpy(psi[idx].view(np.float64).copy())
-                recv = torch.empty_like(send)
-                reqs = [dist.isend(send, partner), dist.irecv(recv, partner)]
-                for r in reqs:
-                    r.wait()
-                psi[idx] = recv.numpy().view(np.complex128)
+                bit_l = (loc >> lp) & 1
+                dest_rank = (dest_rank & ~(1 << j)) | (bit_l << j)
+                dest_loc = (dest_loc & ~(1 << lp)) | (((rank >> j) & 1) << lp)
+            peers = sorted(set(dest_rank.tolist()))
+            new = psi.copy()
+            mine = dest_rank == rank
+            new[dest_loc[mine]] = psi[mine]
+            reqs, bufs = [], {}
+            for pr in peers:
+                if pr == rank:
+                    continue
+                sel = dest_rank == pr
+                send = torch.from_numpy(np.ascontiguousarray(
+                    np.stack([dest_loc[sel].astype(np.float64), psi[sel].real, psi[sel].imag])).copy())
+                bufs[pr] = torch.empty_like(send)
+                reqs.append(dist.isend(send, pr))
+                reqs.append(dist.irecv(bufs[pr], pr))
+            for r_ in reqs:
+                r_.wait()
+            for pr, b in bufs.items():
+                a = b.numpy()
+                new[a[0].astype(np.int64)] = a[1] + 1j * a[2]
+            psi = new
         for (nt, targets, pc, diag, U) in p["gates"]:
             _apply(psi, rank, m, nt, targets, pc, U)
     t = torch.from_numpy(psi.view(np.float64).copy())
@@ -158,6 +191,25 @@ def test_sharded_protocol_vs_oracle(q, world, name):
     assert np.abs(got - ref).max() <= 1e-12
     if name in ("random", "rqc", "ghz"):
         assert "\nP 5 " in "\n" + text  # the plan exercised at least one global-local swap
+
+
+@pytest.mark.parametrize("world", [2, 4])
+@pytest.mark.parametrize("name", ["random", "qft", "rqc", "gs", "hlf"])
+def test_sharded_protocol_early_global_placement(q, world, name, monkeypatch):
+    """§8e cross-rank first-touch expand: with QGPU_GLOBAL_MIN_LOCAL=2 the first log2 G qubits
+    first touched by an uncontrolled 1-qubit gate go to rank bits while only 2 local positions
+    are assigned (copy activations), so later non-diagonal gates on them need batched swaps with
+    few assigned local positions; executed with gloo against the oracle."""
+    monkeypatch.setenv("QGPU_GLOBAL_MIN_LOCAL", "2")
+    c = {"random": lambda: wc.random_circuit(8, 90, seed=world + 10),
+         "qft": lambda: wc.qft(8, x=171),
+         "rqc": lambda: wc.rqc(8, 6, seed=3),
+         "gs": lambda: wc.gs(2, 4),
+         "hlf": lambda: wc.hlf(2, 4, seed=2)}[name]()
+    got, text = _run_sharded(q, c, world, fuse=12)
+    assert np.abs(got - osv.simulate(c.qasm())).max() <= 1e-12
+    lines = text.splitlines()
+    assert any(l.startswith("P 6 ") and int(l.split()[5]) < 0 for l in lines)  # a copy activation
 
 
 @pytest.mark.parametrize("world", [2, 4])
