@@ -123,6 +123,7 @@ uint64_t plan_key(const qgpu_state* st, const qgpu_circuit* c) {
   if (const char* ev = std::getenv("QGPU_LMIN")) mix(uint64_t(std::atoi(ev) + 1) << 60);
   if (const char* ev = std::getenv("QGPU_LRELAX")) mix(uint64_t(std::atoi(ev) + 1) << 52);
   if (const char* ev = std::getenv("QGPU_GLOBAL_FIRST")) mix(uint64_t(std::atoi(ev) + 1) << 20);
+  if (const char* ev = std::getenv("QGPU_AUTO_LANES")) mix(uint64_t(std::atoi(ev) + 1) << 28);
   if (const char* ev = std::getenv("QGPU_GLOBAL_MIN_LOCAL")) mix(uint64_t(std::atoi(ev) + 1) << 24);
   return h;
 }
@@ -183,8 +184,15 @@ void prepare_jit(qgpu_state* st, const std::vector<Pass>& passes) {
 // experiment overrides of the planner defaults (also part of the plan-cache key)
 void plan_env(PlanOptions* o) {
   if (const char* ev = std::getenv("QGPU_ZSKIP")) o->zskip = std::atoi(ev) != 0;
-  if (const char* ev = std::getenv("QGPU_LMIN")) o->l_min = std::atoi(ev);
-  if (const char* ev = std::getenv("QGPU_LRELAX")) o->l_relax = std::atoi(ev);
+  if (const char* ev = std::getenv("QGPU_LMIN")) {  // a fixed lane policy (experiments)
+    o->l_min = std::atoi(ev);
+    o->auto_lanes = false;
+  }
+  if (const char* ev = std::getenv("QGPU_LRELAX")) {
+    o->l_relax = std::atoi(ev);
+    o->auto_lanes = false;
+  }
+  if (const char* ev = std::getenv("QGPU_AUTO_LANES")) o->auto_lanes = o->auto_lanes && std::atoi(ev) != 0;
   if (const char* ev = std::getenv("QGPU_REGBITS")) o->reg_bits = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_MAX_UOPS")) o->max_u_ops = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_LOOKAHEAD")) o->lookahead = std::atoi(ev);
@@ -630,7 +638,7 @@ qgpu_status apply_circuit_impl(qgpu_state* st, const qgpu_circuit* c, int meas_m
       cp.circ_gates = c->c.gates;
       cp.order = reorder(c->c.gates, st->cfg.reorder, st->cfg.involve_rule);
       QubitMap map = st->map;
-      plan_circuit(c->c.gates, cp.order, map, plan_options(st->cfg, st->cfg.fuse_bits > 0), &cp.passes, &cp.inv);
+      plan_circuit_auto(c->c.gates, cp.order, map, plan_options(st->cfg, st->cfg.fuse_bits > 0), &cp.passes, &cp.inv);
       cp.map_after = map;
       for (const Gate& g : c->c.gates) cp.relabels += g.relabel ? 1 : 0;
       if (qgpu_status s = upload_plan(st, &cp)) return s;
@@ -786,6 +794,136 @@ qgpu_status qgpu_apply_circuit_probabilities(qgpu_state* st, const qgpu_circuit*
   return drain_timing(st);
 }
 
+namespace {
+// GatherArgs of rank `rank` for the logical range [start, start + count)
+GatherArgs gather_args(const qgpu_state* st, const double2* psi, uint64_t rank, uint64_t start, uint64_t count,
+                       double* dev_out) {
+  GatherArgs a{};
+  a.psi = psi;
+  a.out = reinterpret_cast<double2*>(dev_out);
+  a.start = start;
+  a.count = count;
+  a.n = st->n;
+  a.m = st->m;
+  a.rank = rank;
+  for (int q = 0; q < st->n; ++q) {
+    a.pos[q] = st->map.pos[q] < 0 ? 0 : st->map.pos[q];
+    if (st->map.pos[q] < 0) a.unassigned |= 1ull << q;
+  }
+  a.L = live(st, st->map.kl);
+  return a;
+}
+}  // namespace
+
+// Sharded readout, point to point: the owner of each logical index is the rank whose
+// bits the index has on the qubits at rank-bit positions. Every rank compacts the amplitudes it
+// owns in the range (owner flags -> inclusive scan -> slot), sends its compact list to every other
+// rank and receives theirs (grouped ncclSend / ncclRecv: each rank moves only what it owns, once
+// per peer), then scatters every list into the output. All ranks share the qubit map, so each
+// computes every rank's list length locally. Virtual ranks run the same kernels with the shards'
+// compact lists read in place.
+qgpu_status sharded_gather(qgpu_state* st, uint64_t start, uint64_t count, double* dev_out) {
+  const uint64_t nact = 1ull << st->map.kg;
+  const int world = int(uint64_t(1) << st->g);
+  uint64_t *pos = nullptr, *scr = nullptr;
+  double2 *own = nullptr, *rcv = nullptr;
+  cudaStream_t s = st->stream;
+  auto cleanup = [&]() {
+    for (void* p : {static_cast<void*>(pos), static_cast<void*>(scr), static_cast<void*>(own), static_cast<void*>(rcv)})
+      if (p) cudaFreeAsync(p, s);
+  };
+  cudaError_t e = cudaMallocAsync(reinterpret_cast<void**>(&pos), count * sizeof(uint64_t), s);
+  if (e == cudaSuccess)
+    e = cudaMallocAsync(reinterpret_cast<void**>(&scr), std::max<uint64_t>(1, gfc_scan_scratch_elems(count)) * sizeof(uint64_t), s);
+  if (e == cudaSuccess) e = cudaMallocAsync(reinterpret_cast<void**>(&own), count * sizeof(double2), s);
+  if (e != cudaSuccess) {
+    cleanup();
+    CK(e);
+  }
+  CK(cudaMemsetAsync(dev_out, 0, count * 2 * sizeof(double), s));
+  auto scan_for = [&](uint64_t r) -> cudaError_t {
+    GatherArgs a = gather_args(st, nullptr, r, start, count, dev_out);
+    cudaError_t x = launch_owner_flags(s, a, pos);
+    if (x == cudaSuccess) x = launch_scan_u64(s, pos, count, scr);
+    return x;
+  };
+  if (st->virt) {
+    for (Shard& sh : st->shards) {
+      if (uint64_t(sh.rank) >= nact) continue;  // inactive: all zero
+      GatherArgs a = gather_args(st, sh.psi, uint64_t(sh.rank), start, count, dev_out);
+      cudaError_t x = scan_for(uint64_t(sh.rank));
+      if (x == cudaSuccess) x = launch_owned_compact(s, a, pos, own);
+      if (x == cudaSuccess) x = launch_owned_scatter(s, a, pos, own);
+      if (x != cudaSuccess) {
+        cleanup();
+        CK(x);
+      }
+      st->stats.kernels_launched += 5;
+    }
+    cleanup();
+    return QGPU_OK;
+  }
+  // NCCL: list lengths of every rank (host), this rank's compact list, the exchange, the scatter
+  const Shard& me = st->shards[0];
+  std::vector<uint64_t> n_of(size_t(world), 0);
+  uint64_t* tot = nullptr;
+  CK(cudaMallocHost(&tot, sizeof(uint64_t) * size_t(world)));
+  for (int r = 0; r < world; ++r) {
+    if (uint64_t(r) >= nact) continue;
+    cudaError_t x = scan_for(uint64_t(r));
+    if (x == cudaSuccess) x = cudaMemcpyAsync(tot + r, pos + count - 1, sizeof(uint64_t), cudaMemcpyDeviceToHost, s);
+    if (x == cudaSuccess && r == me.rank)
+      x = launch_owned_compact(s, gather_args(st, me.psi, uint64_t(r), start, count, dev_out), pos, own);
+    if (x != cudaSuccess) {
+      cudaFreeHost(tot);
+      cleanup();
+      CK(x);
+    }
+  }
+  CK(cudaStreamSynchronize(s));
+  uint64_t recv_total = 0;
+  for (int r = 0; r < world; ++r) {
+    n_of[size_t(r)] = uint64_t(r) < nact ? tot[r] : 0;
+    if (r != me.rank) recv_total += n_of[size_t(r)];
+  }
+  cudaFreeHost(tot);
+  if (recv_total) CK(cudaMallocAsync(reinterpret_cast<void**>(&rcv), recv_total * sizeof(double2), s));
+  std::vector<int> peer;
+  std::vector<const double*> sb;
+  std::vector<double*> rb;
+  std::vector<size_t> sc, rc;
+  std::vector<uint64_t> roff(size_t(world), 0);
+  uint64_t off = 0;
+  for (int r = 0; r < world; ++r) {
+    if (r == me.rank) continue;
+    peer.push_back(r);
+    sb.push_back(reinterpret_cast<const double*>(own));
+    sc.push_back(size_t(2 * n_of[size_t(me.rank)]));
+    roff[size_t(r)] = off;
+    rb.push_back(reinterpret_cast<double*>(rcv + off));
+    rc.push_back(size_t(2 * n_of[size_t(r)]));
+    off += n_of[size_t(r)];
+  }
+  if (qgpu_status x = comm_exchange(st->comm, int(peer.size()), peer.data(), sb.data(), sc.data(), rb.data(), rc.data(),
+                                    s, &g_err)) {
+    st->poisoned = true;
+    cleanup();
+    return x;
+  }
+  for (int r = 0; r < world; ++r) {
+    if (!n_of[size_t(r)]) continue;
+    GatherArgs a = gather_args(st, nullptr, uint64_t(r), start, count, dev_out);
+    cudaError_t x = scan_for(uint64_t(r));
+    if (x == cudaSuccess) x = launch_owned_scatter(s, a, pos, r == me.rank ? own : rcv + roff[size_t(r)]);
+    if (x != cudaSuccess) {
+      cleanup();
+      CK(x);
+    }
+  }
+  cleanup();
+  return QGPU_OK;
+}
+
 qgpu_status qgpu_get_amplitudes_device(qgpu_state* st, uint64_t start, uint64_t count, double* dev_out) {
   QGPU_ON_DEVICE(st);
   if (qgpu_status s = check_state(st)) return s;
@@ -794,31 +932,16 @@ qgpu_status qgpu_get_amplitudes_device(qgpu_state* st, uint64_t start, uint64_t 
     return fail(QGPU_ERR_INVALID_ARG, "range [%llu, +%llu) outside 2^%d", (unsigned long long)start,
                 (unsigned long long)count, st->n);
   if (!count) return QGPU_OK;
-  const bool sharded = st->g > 0;
-  if (sharded) CK(cudaMemsetAsync(dev_out, 0, count * 2 * sizeof(double), st->stream));
+  if (st->g > 0 && !st->host) return sharded_gather(st, start, count, dev_out);
+  if (st->g > 0) CK(cudaMemsetAsync(dev_out, 0, count * 2 * sizeof(double), st->stream));  // host tier slices
   for (Shard& sh : st->shards) {
-    if (sharded && (uint64_t(sh.rank) >> st->map.kg) != 0) continue;  // inactive: all zero
-    GatherArgs a{};
-    a.psi = sh.psi;
+    if (st->g > 0 && (uint64_t(sh.rank) >> st->map.kg) != 0) continue;  // host tier: inactive slice
+    GatherArgs a = gather_args(st, sh.psi, uint64_t(sh.rank), start, count, dev_out);
     if (qgpu_status s = host_readable(st, size_t(sh.rank), &a.psi)) return s;
-    a.out = reinterpret_cast<double2*>(dev_out);
-    a.start = start;
-    a.count = count;
-    a.n = st->n;
-    a.m = st->m;
-    a.rank = uint64_t(sh.rank);
-    a.only_owned = sharded ? 1 : 0;
-    for (int q = 0; q < st->n; ++q) {
-      a.pos[q] = st->map.pos[q] < 0 ? 0 : st->map.pos[q];
-      if (st->map.pos[q] < 0) a.unassigned |= 1ull << q;
-    }
-    a.L = live(st, st->map.kl);
+    a.only_owned = st->g > 0 ? 1 : 0;
     if (st->host) a.L = std::min(a.L, st->hlive[size_t(sh.rank)]);  // zero-copy read of the slice
     CK(launch_gather(st->stream, a));
     st->stats.kernels_launched++;
-  }
-  if (sharded && st->comm) {  // every rank gets the full range (collective)
-    if (qgpu_status s = comm_allreduce_sum(st->comm, dev_out, count * 2, st->stream, &g_err)) return s;
   }
   return QGPU_OK;
 }
@@ -969,7 +1092,7 @@ qgpu_status qgpu_circuit_plan(const qgpu_circuit* c, int n, int world, int reord
     plan_env(&o);
     o.rule = reorder_mode >> 2 & 1;
     std::vector<Pass> passes;
-    plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode & 3, o.rule), map, o, &passes, nullptr);
+    plan_circuit_auto(c->c.gates, reorder(c->c.gates, reorder_mode & 3, o.rule), map, o, &passes, nullptr);
     if (n_passes) *n_passes = passes.size();
     for (uint64_t i = 0; info && i < std::min<uint64_t>(cap, passes.size()); ++i) {
       const Pass& p = passes[i];
@@ -1002,7 +1125,7 @@ qgpu_status qgpu_circuit_plan_text(const qgpu_circuit* c, int n, int world, int 
     plan_env(&o);
     o.rule = reorder_mode >> 2 & 1;
     std::vector<Pass> passes;
-    plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode & 3, o.rule), map, o, &passes, nullptr);
+    plan_circuit_auto(c->c.gates, reorder(c->c.gates, reorder_mode & 3, o.rule), map, o, &passes, nullptr);
     std::string t;
     char line[512];
     for (const Pass& p : passes) {
@@ -1053,7 +1176,7 @@ qgpu_status qgpu_circuit_jit_check(const qgpu_circuit* c, int n, int reorder_mod
     plan_env(&o);
     o.rule = reorder_mode >> 2 & 1;
     std::vector<Pass> passes;
-    plan_circuit(c->c.gates, reorder(c->c.gates, reorder_mode & 3, o.rule), map, o, &passes, nullptr);
+    plan_circuit_auto(c->c.gates, reorder(c->c.gates, reorder_mode & 3, o.rule), map, o, &passes, nullptr);
     std::string cubin, log;
     for (const Pass& p : passes) {
       if (p.kind != PK_TILE) continue;

@@ -1,8 +1,25 @@
 // Pass execution of libqgpu: resident fused / per-gate passes, global-local swaps (a10), and the
 // host-memory tier's streaming sweeps (NEXT-2, with the GFC link of NEXT-3). Called from api.cpp.
+#include <nvtx3/nvToolsExt.h>
+
 #include "state.h"
 
 namespace qgpu_impl {
+
+// NVTX range per pass / swap / sweep (visible in Nsight timelines; header-only NVTX3,
+// a no-op unless a tool is attached)
+struct PassRange {
+  explicit PassRange(const Pass& p) {
+    static const char* const kinds[] = {"tile", "pair", "quad", "diag", "relabel", "swap", "activate", "zero"};
+    char name[96];
+    if (p.kind == PK_SWAP)
+      std::snprintf(name, sizeof(name), "qgpu swap %d-bit k%d", p.nswap, p.k_in);
+    else
+      std::snprintf(name, sizeof(name), "qgpu %s k%d->%d gates %d", kinds[p.kind & 7], p.k_in, p.k_out, p.count);
+    nvtxRangePushA(name);
+  }
+  ~PassRange() { nvtxRangePop(); }
+};
 
 cudaEvent_t get_event(qgpu_state* st) {
   if (!st->event_pool.empty()) {
@@ -241,6 +258,9 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     // programs without remaps need one tile buffer (each thread only reads its own slots),
     // which lets two CTAs share an SM; otherwise triple (or double) buffering
     a.nbuf = a.remaps ? 3 : 1;
+    // QGPU_2CTA=1 (experiment): two single-buffered CTAs per SM at <= 128 registers (JIT only)
+    const bool two_cta = jit2cta() && (st->cfg.jit == 2 || (st->cfg.jit == 1 && p.k_out >= jit_min_bits()));
+    if (two_cta) a.nbuf = 1;
     // optional bulk stores (staged tile, async copies per run; QGPU_BSTORE)
     const int bs = bstore_mode();
     if (bs == 2 || (bs == 1 && a.remaps)) a.nbuf = 3;
@@ -415,6 +435,7 @@ uint64_t computed_amps(const qgpu_state* st, const Pass& p) {
 // only zeros and skip the work), swaps through the communicator, activations as memsets.
 qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops, bool own_timing = true,
                       uint64_t* bytes_out = nullptr) {
+  PassRange nvtx_range(p);
   const int m = st->m;
   const int kin = st->cfg.prune ? p.k_in : m, kout = st->cfg.prune ? p.k_out : m;
   const uint64_t L_in = 1ull << kin, L_out = 1ull << kout;
@@ -646,6 +667,10 @@ void host_account_stores(qgpu_state* st) {
 qgpu_status host_sweep(qgpu_state* st, const std::vector<const Pass*>& run,
                        const std::vector<const unsigned char*>& ops, const std::vector<HostSwap>& sw,
                        int kg_sw) {
+  nvtxRangePushA("qgpu host-tier sweep");
+  struct Pop {
+    ~Pop() { nvtxRangePop(); }
+  } pop;
   const int m = st->m;
   const uint64_t full = 1ull << m;
   int kg = sw.empty() ? 0 : kg_sw;

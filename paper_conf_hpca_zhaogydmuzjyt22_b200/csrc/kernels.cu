@@ -276,6 +276,38 @@ __global__ void gather_kernel(GatherArgs a) {
   }
 }
 
+// a11 sharded readout, point to point: ownership of a logical index (kernels.h)
+__device__ __forceinline__ bool owned_local(const GatherArgs& a, uint64_t X, uint64_t* local) {
+  if (X & a.unassigned) return false;
+  uint64_t phys = 0;
+  for (int q = 0; q < a.n; ++q)
+    if (X >> q & 1) phys |= 1ull << a.pos[q];
+  if ((phys >> a.m) != a.rank) return false;
+  *local = phys & ((1ull << a.m) - 1);
+  return true;
+}
+__global__ void owner_flags_kernel(GatherArgs a, uint64_t* flags) {
+  const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+  for (uint64_t x = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; x < a.count; x += stride) {
+    uint64_t loc;
+    flags[x] = owned_local(a, a.start + x, &loc) ? 1u : 0u;
+  }
+}
+__global__ void owned_compact_kernel(GatherArgs a, const uint64_t* pos, double2* compact) {
+  const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+  for (uint64_t x = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; x < a.count; x += stride) {
+    uint64_t loc;
+    if (owned_local(a, a.start + x, &loc)) compact[pos[x] - 1] = loc < a.L ? a.psi[loc] : make_double2(0, 0);
+  }
+}
+__global__ void owned_scatter_kernel(GatherArgs a, const uint64_t* pos, const double2* compact) {
+  const uint64_t stride = uint64_t(gridDim.x) * blockDim.x;
+  for (uint64_t x = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; x < a.count; x += stride) {
+    uint64_t loc;
+    if (owned_local(a, a.start + x, &loc)) a.out[x] = compact[pos[x] - 1];
+  }
+}
+
 // a11 probabilities. Each warp owns a contiguous range of the live prefix and walks it 32
 // amplitudes at a time (lane bits = index bits 0..4). The bucket index splits into a part
 // given by requested positions < 5 (per lane) and a part given by positions >= 5 (uniform over
@@ -633,6 +665,22 @@ cudaError_t launch_tile(cudaStream_t st, const TileArgs& a) {
     case 3: return launch_tile_nr<3, false>(st, a, smem);
     default: return launch_tile_nr<4, false>(st, a, smem);
   }
+}
+
+cudaError_t launch_owner_flags(cudaStream_t st, const GatherArgs& a, uint64_t* flags) {
+  if (a.count == 0) return cudaSuccess;
+  owner_flags_kernel<<<grid_for(a.count, 256, 8), 256, 0, st>>>(a, flags);
+  return cudaGetLastError();
+}
+cudaError_t launch_owned_compact(cudaStream_t st, const GatherArgs& a, const uint64_t* pos, double2* compact) {
+  if (a.count == 0) return cudaSuccess;
+  owned_compact_kernel<<<grid_for(a.count, 256, 8), 256, 0, st>>>(a, pos, compact);
+  return cudaGetLastError();
+}
+cudaError_t launch_owned_scatter(cudaStream_t st, const GatherArgs& a, const uint64_t* pos, const double2* compact) {
+  if (a.count == 0) return cudaSuccess;
+  owned_scatter_kernel<<<grid_for(a.count, 256, 8), 256, 0, st>>>(a, pos, compact);
+  return cudaGetLastError();
 }
 
 cudaError_t launch_gather(cudaStream_t st, const GatherArgs& a) {

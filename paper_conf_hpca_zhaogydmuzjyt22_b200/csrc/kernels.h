@@ -53,6 +53,15 @@ struct GatherArgs {
   int only_owned;          // sharded: write only the amplitudes this rank owns
 };
 
+// Sharded readout by point-to-point exchange (qgpu_get_amplitudes): for the logical
+// range [start, start + count), flags[x] = 1 where rank `rank` owns x (x's bits on the qubits at
+// rank-bit positions equal the rank, no bit on a never-involved qubit); after an inclusive scan
+// flags[x] - 1 is x's slot in that rank's compact list. compact: the owner writes its amplitudes
+// (psi, live prefix L) to their slots; scatter: a receiver places a rank's compact list.
+cudaError_t launch_owner_flags(cudaStream_t st, const GatherArgs& a, uint64_t* flags);
+cudaError_t launch_owned_compact(cudaStream_t st, const GatherArgs& a, const uint64_t* pos, double2* compact);
+cudaError_t launch_owned_scatter(cudaStream_t st, const GatherArgs& a, const uint64_t* pos, const double2* compact);
+
 struct ProbArgs {
   const double2* psi;
   uint64_t L;

@@ -180,6 +180,9 @@ struct PlanOptions {
   bool global_first = false;
   int global_min_local = 10;
   int max_swap_bits = 8;  // rank bits per batched swap (the host tier's sweeps fold at most 2)
+  // plan_circuit_auto: try the lane-bit policies (l_min, l_relax) = (5, 0) (5, 4) (5, 3) (4, 0)
+  // (3, 0) and keep the plan with the lowest modelled time
+  bool auto_lanes = true;
 };
 
 // Cut `gates` into passes, updating `map` (involvement, placement) exactly as the execution
@@ -189,6 +192,15 @@ struct PlanOptions {
 void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order, QubitMap& map,
                   const PlanOptions& opt, std::vector<Pass>* passes,
                   std::vector<uint64_t>* inv_after);
+// plan_circuit over candidate lane-bit policies (opt.l_min / opt.l_relax) when opt.auto_lanes:
+// every candidate is planned from a copy of `map`, its passes costed by pass_cost_model(), and the
+// cheapest plan is kept (map, passes, inv_after as plan_circuit leaves them).
+void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& order, QubitMap& map,
+                       const PlanOptions& opt, std::vector<Pass>* passes, std::vector<uint64_t>* inv_after);
+// Modelled seconds of one pass on one B200: max(HBM bytes / (copy peak x efficiency of its
+// contiguous run length 16 * 2^l B), modelled FP64 instructions / (FP64 peak x issue efficiency))
+// plus a launch gap.
+double pass_cost_model(const Pass& p, int m);
 // Build the device ops of a tile pass from its gates and tile positions.
 void build_tile_ops(Pass& p, int m, int reg_bits = 4);
 // Unfused byte model of one gate on live size 2^k.

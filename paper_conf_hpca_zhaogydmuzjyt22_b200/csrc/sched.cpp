@@ -1272,3 +1272,75 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
 }
 
 }  // namespace qgpu
+
+namespace qgpu {
+
+double pass_cost_model(const Pass& p, int m) {
+  // measured on B200 (profiles/r02): a pass whose warp accesses are 512-byte runs (l >= 5) streams
+  // at ~0.93 of the copy peak, 256-byte runs ~0.87, 128-byte runs ~0.82; fused programs issue
+  // FP64 at ~0.6 of the DFMA peak
+  constexpr double kHbm = 6.5e12, kFp64 = 16.0e12, kFpEff = 0.6, kLaunch = 4e-6;
+  const int kin = p.k_in, kout = p.k_out;
+  if (p.kind == PK_RELABEL || p.kind == PK_ACTIVATE) return 0.0;
+  if (p.kind == PK_SWAP) return 16.0 * std::ldexp(1.0, kin) / 7.0e11;
+  if (p.kind == PK_ZERO) return 16.0 * std::ldexp(1.0, kout) / kHbm + kLaunch;
+  double bytes = 16.0 * (std::ldexp(1.0, kin - std::popcount(p.zin & ((1ull << kin) - 1))) +
+                         std::ldexp(1.0, kout - std::popcount(p.zout & ((1ull << kout) - 1))));
+  double eff = 0.93, amps = std::ldexp(1.0, kout);
+  if (p.kind == PK_TILE) {
+    eff = p.l >= 5 ? 0.93 : p.l == 4 ? 0.87 : p.l == 3 ? 0.82 : 0.6;
+    uint64_t S = 0;
+    for (int i = 0; i < p.b; ++i) S |= 1ull << p.spos[i];
+    int free_bits = 0;
+    for (int q = 0; q < kout; ++q)
+      if (!(S >> q & 1) && q < kin && !((p.zin | p.zout) >> q & 1)) ++free_bits;
+    amps = std::ldexp(1.0, free_bits + p.b);
+  }
+  (void)m;
+  return std::max(bytes / (kHbm * eff), p.fp64_per_amp * amps / (kFp64 * kFpEff)) + kLaunch;
+}
+
+void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& order, QubitMap& map,
+                       const PlanOptions& opt, std::vector<Pass>* passes, std::vector<uint64_t>* inv_after) {
+  if (!opt.auto_lanes || opt.fuse_bits <= 0) {
+    plan_circuit(gates, order, map, opt, passes, inv_after);
+    return;
+  }
+  static const int cand[][2] = {{5, 0}, {5, 4}, {5, 3}, {4, 0}, {3, 0}};
+  double best = 0.0;
+  bool have = false;
+  QubitMap best_map;
+  std::vector<Pass> best_passes;
+  std::vector<uint64_t> best_inv;
+  for (const auto& c : cand) {
+    if (have && !best_passes.empty()) {
+      // other lane policies can only merge passes that run at the full live size; with at most
+      // one such pass in the first plan (e.g. QFT: every pass expands) the first plan is kept
+      int kmax = 0, steady = 0;
+      for (const Pass& p : best_passes) kmax = std::max(kmax, p.k_out);
+      for (const Pass& p : best_passes) steady += (p.kind == PK_TILE && p.k_in == kmax && p.k_out == kmax);
+      if (steady <= 1) break;
+    }
+    PlanOptions o = opt;
+    o.l_min = std::min(opt.l_min, c[0]);
+    o.l_relax = c[1];
+    QubitMap mp = map;
+    std::vector<Pass> ps;
+    std::vector<uint64_t> inv;
+    plan_circuit(gates, order, mp, o, &ps, inv_after ? &inv : nullptr);
+    double t = 0.0;
+    for (const Pass& p : ps) t += pass_cost_model(p, mp.m);
+    if (!have || t < best * 0.995) {  // ties keep the earlier (longer-run) policy
+      have = true;
+      best = t;
+      best_map = mp;
+      best_passes = std::move(ps);
+      best_inv = std::move(inv);
+    }
+  }
+  map = best_map;
+  *passes = std::move(best_passes);
+  if (inv_after) *inv_after = std::move(best_inv);
+}
+
+}  // namespace qgpu

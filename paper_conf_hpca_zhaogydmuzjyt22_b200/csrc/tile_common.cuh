@@ -91,7 +91,7 @@ struct TileArgs {
                            // read as zero; tiles with a zout bit are neither loaded nor stored
   uint64_t rank_base;      // rank << m (global bits for tile-uniform conditions)
   const double2* zero;     // >= 2^kMaxTileBits zero amplitudes (source of the expanded region)
-  int nbuf;                // tile buffers in shared memory (2 or 3)
+  int nbuf;                // tile buffers in shared memory (1, 2 or 3)
   int bstore;              // 1: results staged in the tile buffer and written by bulk async
                            // copies (needs nbuf == 3), 0: per-thread stores from registers
   int remaps;              // the program contains REMAP / shared-memory ops
@@ -880,10 +880,18 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       else j = mp0.j(r);
       v[r] = (c.own && !((zm0 >> r) & 1)) ? s[j] : make_double2(0.0, 0.0);
     }
-    if (more && nbuf == 1) issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
+    // nbuf == 1 without remaps: each thread reads only its own slots, so the next tile's loads
+    // can go into the buffer right after this reload; with remaps (two CTAs per SM, each single-
+    // buffered: the other CTA's compute covers this one's load latency) the buffer is free only
+    // once every thread of the CTA has finished the program's remaps
+    if (more && nbuf == 1 && !a.remaps) issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
     c.mpar = nexec & 1u;
     ++nexec;
     body(v, mp, c);
+    if (more && nbuf == 1 && a.remaps) {
+      __syncthreads();
+      issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
+    }
     if (Body::kHasScalar && !(sc.x == 1.0 && sc.y == 0.0)) {
 #pragma unroll
       for (int r = 0; r < (1 << NR); ++r) v[r] = cmul(v[r], sc);

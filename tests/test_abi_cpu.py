@@ -127,7 +127,9 @@ def test_plan_invariants(q, name, fuse):
                 S = int(slo) | (int(shi) << 32)
                 assert bin(S).count("1") == b <= fuse
                 assert b == min(fuse, kout)
-                lm = min(5, kout)
+                # the lane-bit policies the planner may pick (plan_circuit_auto) keep
+                # at least the 3 lowest positions (128-byte runs per warp access) in every tile
+                lm = min(3, kout)
                 assert S & ((1 << lm) - 1) == (1 << lm) - 1
                 assert S >> kout == 0
     assert pos == ng

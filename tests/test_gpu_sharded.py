@@ -76,7 +76,7 @@ def test_virtual_ranks_gate_stream_and_prune_neutrality(q, world):
 
 EARLY = {
     "rqc": lambda: wc.rqc(16, 8, seed=3),
-    "qaoa": lambda: wc.qaoa(15, 2, seed=5),
+    "qaoa": lambda: wc.qaoa(16, 2, seed=5),
     "gs": lambda: wc.gs(3, 5),
     "random": lambda: wc.random_circuit(15, 300, seed=78),
     "grqc": lambda: wc.grqc(3, 5, 40, seed=5),
