@@ -498,8 +498,7 @@ std::string tile_jit_source(const Pass& p, int hist_mode) {
   o << body.str() << "};\n";
   // one CTA per SM with up to 255 registers: measured faster than 2 CTAs/SM at <= 128
   // registers even for the single-buffer (remap-free) programs
-  int minb = 1;  // CTAs per SM the register budget is cut for (QGPU_2CTA / QGPU_JIT_MINBLOCKS)
-  if (const char* ev = std::getenv("QGPU_2CTA")) minb = std::atoi(ev) ? 2 : 1;
+  int minb = pass_two_cta(p) ? 2 : 1;  // CTAs per SM the register budget is cut for
   if (const char* ev = std::getenv("QGPU_JIT_MINBLOCKS")) minb = std::max(1, std::atoi(ev));
   o << "extern \"C\" __global__ void __launch_bounds__(" << (NR >= 4 ? 256 : 512) << ", " << minb
     << ") qgpu_tile_pass(const TileArgs a) {\n";

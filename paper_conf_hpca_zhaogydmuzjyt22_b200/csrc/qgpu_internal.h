@@ -201,6 +201,10 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
 // contiguous run length 16 * 2^l B), modelled FP64 instructions / (FP64 peak x issue efficiency))
 // plus a launch gap.
 double pass_cost_model(const Pass& p, int m);
+// Two single-buffered CTAs per SM at <= 128 registers for this pass's NVRTC kernel (instead of
+// one triple-buffered CTA at <= 255): QGPU_2CTA=1 every pass, 2 passes whose program runs
+// >= 40 FP64 instructions per amplitude (the latency-bound ones), 0 none (read per call).
+bool pass_two_cta(const Pass& p);
 // Build the device ops of a tile pass from its gates and tile positions.
 void build_tile_ops(Pass& p, int m, int reg_bits = 4);
 // Unfused byte model of one gate on live size 2^k.

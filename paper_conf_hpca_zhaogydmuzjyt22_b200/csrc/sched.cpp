@@ -1344,3 +1344,12 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
 }
 
 }  // namespace qgpu
+
+namespace qgpu {
+bool pass_two_cta(const Pass& p) {
+  const char* ev = std::getenv("QGPU_2CTA");
+  const int mode = ev ? std::atoi(ev) : 0;
+  if (p.kind != PK_TILE || mode == 0) return false;
+  return mode == 1 || p.fp64_per_amp >= 40.0;
+}
+}  // namespace qgpu

@@ -89,11 +89,6 @@ inline int jit_min_bits() {
   return ev ? std::atoi(ev) : 12;
 }
 
-// QGPU_2CTA=1 (experiment, read per call): NVRTC pass kernels with two single-buffered CTAs per SM
-inline bool jit2cta() {
-  const char* ev = std::getenv("QGPU_2CTA");
-  return ev && std::atoi(ev) != 0;
-}
 
 extern thread_local std::string g_err;
 
