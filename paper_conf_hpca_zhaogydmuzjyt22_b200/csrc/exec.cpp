@@ -244,6 +244,21 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
       i = j + 1;
     }
     a.ntiles = 1ull << (kout - p.b);
+    // tiles whose base selects a skipped zero half (zout) do no work: leave them out of the tile
+    // enumeration (tile-index bit i <-> the i-th non-tile position below k_out)
+    a.nzs = 0;
+    const char* zd = std::getenv("QGPU_ZOUT_DEAL");  // 0: enumerate (and skip) them (A/B)
+    if (st->cfg.prune && p.zout && !(zd && zd[0] == '0')) {
+      uint64_t S = 0;
+      for (int i = 0; i < p.b; ++i) S |= 1ull << p.spos[i];
+      int ti = 0;
+      for (int q = 0; q < kout; ++q) {
+        if (S >> q & 1) continue;
+        if (p.zout >> q & 1) a.zs_pos[a.nzs++] = ti;
+        ++ti;
+      }
+      a.ntiles >>= a.nzs;
+    }
     a.L_in = L_in;
     a.zin = st->cfg.prune ? p.zin : 0;
     a.zout = st->cfg.prune ? p.zout : 0;

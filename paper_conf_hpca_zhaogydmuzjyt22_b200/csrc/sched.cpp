@@ -879,6 +879,7 @@ struct Builder {
       build_tile_ops(p, map.m, opt.reg_bits);
     }
     p.fp64_per_amp = fp64_model(p);
+    if (std::getenv("QGPU_DEBUG_PLAN")) std::fprintf(stderr, "  pass fp64/amp %.2f\n", p.fp64_per_amp);
     out->push_back(std::move(p));
     cur = Pass();
     open = false;
@@ -1277,9 +1278,12 @@ namespace qgpu {
 
 double pass_cost_model(const Pass& p, int m) {
   // measured on B200 (profiles/r02): a pass whose warp accesses are 512-byte runs (l >= 5) streams
-  // at ~0.93 of the copy peak, 256-byte runs ~0.87, 128-byte runs ~0.82; fused programs issue
-  // FP64 at ~0.6 of the DFMA peak
-  constexpr double kHbm = 6.5e12, kFp64 = 16.0e12, kFpEff = 0.6, kLaunch = 4e-6;
+  // at ~0.93 of the copy peak, 256-byte runs ~0.87, 128-byte runs ~0.82. The program's SM time
+  // per amplitude, in SM clocks: FP64 instructions / 64 per clock, plus the shared-memory / shuffle
+  // (MIO) pipe: a lane-bit op is 4 32-bit shuffles per amplitude at 32 per clock, a remap stores
+  // and reloads 32 B per amplitude at 128 B per clock; the two pipes overlap only partly, so they
+  // add, at ~0.6 issue efficiency
+  constexpr double kHbm = 6.5e12, kClk = 1.9e9 * 148.0, kFpEff = 0.6, kLaunch = 4e-6;
   const int kin = p.k_in, kout = p.k_out;
   if (p.kind == PK_RELABEL || p.kind == PK_ACTIVATE) return 0.0;
   if (p.kind == PK_SWAP) return 16.0 * std::ldexp(1.0, kin) / 7.0e11;
@@ -1297,7 +1301,15 @@ double pass_cost_model(const Pass& p, int m) {
     amps = std::ldexp(1.0, free_bits + p.b);
   }
   (void)m;
-  return std::max(bytes / (kHbm * eff), p.fp64_per_amp * amps / (kFp64 * kFpEff)) + kLaunch;
+  double mio = 0.0;
+  if (p.kind == PK_TILE) {
+    for (size_t i = 1; i < p.prog.ops.size(); ++i) {
+      const int k = p.prog.ops[i].kind;
+      mio += k == OP_U1L ? 4.0 / 32.0 : (k == OP_REMAP || k == OP_SMEM1 || k == OP_SMEM2) ? 32.0 / 128.0 : 0.0;
+    }
+  }
+  const double sm_clk_per_amp = p.fp64_per_amp / 64.0 + mio;
+  return std::max(bytes / (kHbm * eff), sm_clk_per_amp * amps / (kClk * kFpEff)) + kLaunch;
 }
 
 void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& order, QubitMap& map,
@@ -1330,6 +1342,9 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
     plan_circuit(gates, order, mp, o, &ps, inv_after ? &inv : nullptr);
     double t = 0.0;
     for (const Pass& p : ps) t += pass_cost_model(p, mp.m);
+    if (std::getenv("QGPU_DEBUG_AUTO"))
+      std::fprintf(stderr, "plan_circuit_auto: l_min %d l_relax %d: %zu passes, modelled %.3f ms\n", o.l_min, o.l_relax,
+                   ps.size(), t * 1e3);
     if (!have || t < best * 0.995) {  // ties keep the earlier (longer-run) policy
       have = true;
       best = t;

@@ -85,7 +85,10 @@ struct TileArgs {
   int spos[kMaxTileBits];
   int nsrun;                      // maximal runs of consecutive tile positions (for deposit)
   int srun_pos[kMaxTileBits], srun_len[kMaxTileBits];
-  uint64_t ntiles;
+  uint64_t ntiles;          // tiles the kernel visits (tiles selecting a zout half excluded)
+  int nzs;                  // tile-index bits of the zout positions: visited tile j is the real
+  int zs_pos[32];            // tile deposit(j, zs_pos) -- the skipped halves are never dealt out,
+                            // so every CTA receives an equal share of the tiles that do work
   uint64_t L_in;
   uint64_t zin, zout;      // zero-position skipping (Pass::zin / zout): amplitudes with a zin bit
                            // read as zero; tiles with a zout bit are neither loaded nor stored
@@ -775,8 +778,9 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     if (it < nfull) return ((it >> a.lb) * G + blockIdx.x) * CH + (it & (CH - 1));
     return rem0 + blockIdx.x + (it - nfull) * G;
   };
+  auto real = [&](uint64_t j) -> uint64_t { return a.nzs ? deposit(j, a.zs_pos, a.nzs) : j; };
   uint64_t tile = tile_at(0);
-  uint64_t base_next = tile_base_t<Body>(tile, a);  // base of `tile`, carried across iterations
+  uint64_t base_next = tile_base_t<Body>(real(tile), a);  // base of `tile`, carried across iterations
   if (tile < a.ntiles) issue_own_loads<NR, Body>(bufs, a, mp0, sa0, base_next, zm0, c.own);
   int k = 0;
   uint64_t cur_hi = ~0ull;
@@ -795,7 +799,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     const uint64_t gbase = a.rank_base | base;
     const uint64_t next = tile_at(it + 1);
     const bool more = next < a.ntiles;
-    base_next = tile_base_t<Body>(next, a);
+    base_next = tile_base_t<Body>(real(next), a);
     // nbuf >= 2: prefetch into the next buffer now; nbuf == 1 (programs without remaps, every
     // thread reads only its own slots): prefetch into the same buffer right after the reload
     if (more && nbuf > 1) issue_own_loads<NR, Body>(bufs + kn * T, a, mp0, sa0, base_next, zm0, c.own);
@@ -842,8 +846,9 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     // pattern constants of this tile, per warp (lane-strided; each lane owns the same patterns
     // in Chw and Cw): high-bit part once per run of 2^lb tiles, then table x loose terms
     {
-      const uint64_t hi = tile >> a.lb;
-      const uint32_t lo = uint32_t(tile) & uint32_t(CH - 1);
+      const uint64_t treal = real(tile);
+      const uint64_t hi = treal >> a.lb;
+      const uint32_t lo = uint32_t(treal) & uint32_t(CH - 1);
       double2* cw = Cw + size_t(warp) * a.npat;
       double2* chw = Chw + size_t(warp) * a.npat;
       if (hi != cur_hi) {
