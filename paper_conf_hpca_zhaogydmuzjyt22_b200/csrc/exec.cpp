@@ -231,6 +231,9 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     a.off_pool = int(P.off_pool);
     a.nr = P.nr;
     a.nw = P.nw;
+    a.umat_n = int(std::min(P.pool.size(), size_t(kUmatParam)));
+    if (P.pool.size() <= size_t(kUmatParam))
+      for (size_t i = 0; i < P.pool.size(); ++i) a.umat[i] = make_double2(P.pool[i].re, P.pool[i].im);
     a.b = p.b;
     a.l = p.l;
     for (int i = 0; i < p.b; ++i) a.spos[i] = p.spos[i];

@@ -296,7 +296,7 @@ std::string tile_jit_source(const Pass& p, int hist_mode) {
   hdr << "  static constexpr uint64_t kP0[kRegAmps] = " << ptab(R) << ";\n";
   hdr << "  static constexpr uint64_t kPF[kRegAmps] = " << ptab(RF) << ";\n";
   hdr << "  static constexpr uint32_t kJF[kRegAmps] = " << jtab(RF) << ";\n";
-  o << "  __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c) const {\n";
+  o << "  __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c, const TileArgs& a) const {\n";
   o << "    const TileOp* ops = c.ops;\n";
   {
     const unsigned zm = zmask();
@@ -307,6 +307,23 @@ std::string tile_jit_source(const Pass& p, int hist_mode) {
       o << " }\n";
     }
   }
+  // U matrices: from the kernel-parameter pool at compile-time offsets when the pool fits
+  // (TileArgs::umat), else from the program blob in shared memory
+  const bool upar = P.pool.size() <= size_t(kUmatParam);
+  auto umat = [&](const TileOp& op) {
+    return upar ? "a.umat + " + std::to_string(op.moff) : std::string("c.pool + op.moff");
+  };
+  // conditions as compile-time constants (they are structural: positions, not values)
+  auto active = [&](const TileOp& op) {
+    std::ostringstream t;
+    t << "((c.gbase & " << op.omask << "ull) == " << op.omatch << "ull)";
+    return t.str();
+  };
+  auto thrc = [&](const TileOp& op) {
+    std::ostringstream t;
+    t << "((mp.base & " << op.tmask << "u) == " << op.tmatch << "u)";
+    return t.str();
+  };
   for (size_t i = 1; i < P.ops.size(); ++i) {
     const TileOp& op = P.ops[i];
     const bool uni = op.omask != 0;       // tile-uniform condition present
@@ -407,8 +424,11 @@ std::string tile_jit_source(const Pass& p, int hist_mode) {
             break;
           }
         }
+        // QGPU_RUN_SPLIT=0: one 16-entry factor table (run_apply_ptab_z) instead of two 4-entry
+        const char* rs_env = std::getenv("QGPU_RUN_SPLIT");
+        const bool split_tab = NR == 4 && !(rs_env && rs_env[0] == '0');
         if (used)
-          o << "      run_apply_ptab_z<" << NR << ", " << (used & 1 ? "true" : "false") << ", "
+          o << "      " << (split_tab ? "run_apply_split_z<" : "run_apply_ptab_z<") << NR << ", " << (used & 1 ? "true" : "false") << ", "
             << ((used >> 1) & 1 ? "true" : "false") << ", " << ((used >> 2) & 1 ? "true" : "false") << ", "
             << ((used >> 3) & 1 ? "true" : "false") << ", " << ((used >> 4) & 1 ? "true" : "false") << ", " << zm
             << "u>(v, t0, e0, e1, e2, e3);\n";
@@ -424,20 +444,20 @@ std::string tile_jit_source(const Pass& p, int hist_mode) {
         break;
       }
       case OP_U1R:
-        o << "      if (" << (uni ? "op_active(op, c.gbase)" : "true") << (thr ? " && (mp.base & op.tmask) == op.tmatch" : "")
-          << ") op_u1r_z<" << NR << ", " << op.a0 << ", " << op.cls << ", " << zm << "u>(v, c.pool + op.moff, "
+        o << "      if (" << (uni ? active(op) : "true") << (thr ? " && " + thrc(op) : "")
+          << ") op_u1r_z<" << NR << ", " << op.a0 << ", " << op.cls << ", " << zm << "u>(v, " << umat(op) << ", "
           << op.rmask << "u, " << op.rmatch << "u);\n";
         zpos &= ~(1u << R[op.a0]);
         break;
       case OP_U1L:
-        o << "      if (" << (uni ? "op_active(op, c.gbase)" : "true") << ") op_u1l_z<" << NR << ", " << op.cls
-          << ", " << zm << "u>(v, c.pool + op.moff, " << op.a0 << ", c.lane, "
-          << (thr ? "(mp.base & op.tmask) == op.tmatch" : "true") << ", " << op.rmask << "u, " << op.rmatch << "u);\n";
+        o << "      if (" << (uni ? active(op) : "true") << ") op_u1l_z<" << NR << ", " << op.cls
+          << ", " << zm << "u>(v, " << umat(op) << ", " << op.a0 << ", c.lane, "
+          << (thr ? thrc(op) : "true") << ", " << op.rmask << "u, " << op.rmatch << "u);\n";
         zpos &= ~(1u << op.a0);
         break;
       case OP_U2R:
-        o << "      if (" << (uni ? "op_active(op, c.gbase)" : "true") << (thr ? " && (mp.base & op.tmask) == op.tmatch" : "")
-          << ") op_u2r_z<" << NR << ", " << op.a0 << ", " << op.a1 << ", " << zm << "u>(v, c.pool + op.moff, "
+        o << "      if (" << (uni ? active(op) : "true") << (thr ? " && " + thrc(op) : "")
+          << ") op_u2r_z<" << NR << ", " << op.a0 << ", " << op.a1 << ", " << zm << "u>(v, " << umat(op) << ", "
           << op.rmask << "u, " << op.rmatch << "u);\n";
         zpos &= ~((1u << R[op.a0]) | (1u << R[op.a1]));
         break;
@@ -472,7 +492,7 @@ std::string tile_jit_source(const Pass& p, int hist_mode) {
       }
       case OP_SMEM1:
       case OP_SMEM2:
-        o << "      if (" << (uni ? "op_active(op, c.gbase)" : "true") << ") { constexpr uint32_t Jc[kRegAmps] = "
+        o << "      if (" << (uni ? active(op) : "true") << ") { constexpr uint32_t Jc[kRegAmps] = "
           << jtab(R) << ";\n        tile_spill_j<" << NR << ">(v, c, mp.base, Jc); ";
         if (op.kind == OP_SMEM2) o << "op_smem2(c, op); ";
         else o << "op_smem1<" << op.cls << ">(c, op); ";

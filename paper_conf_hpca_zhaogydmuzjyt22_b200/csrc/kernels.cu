@@ -161,6 +161,42 @@ __global__ void __launch_bounds__(kThreads) phase_kernel(PhaseArgs a) {
   }
 }
 
+// Single-term diagonal with position 0 fixed (e.g. CP / CZ / CX-type phases on qubit 0): the
+// affected amplitudes are every other 16-byte slot, i.e. half of each 32-byte DRAM sector. Each
+// thread reads and writes the whole sector (the affected amplitude and its bit-0 partner,
+// unchanged), so no sector is written partially (a partial write costs a fill read).
+template <int APT>
+__global__ void __launch_bounds__(kThreads) phase_sector_kernel(PhaseArgs a) {
+  const uint64_t stride = uint64_t(gridDim.x) * kThreads * APT;
+  for (uint64_t v0 = uint64_t(blockIdx.x) * kThreads * APT + threadIdx.x; v0 < a.count;
+       v0 += stride) {
+    double2 x0[APT], x1[APT];
+    uint64_t idx[APT];
+#pragma unroll
+    for (int r = 0; r < APT; ++r) {
+      const uint64_t v = v0 + uint64_t(r) * kThreads;
+      idx[r] = (deposit(v, a.ins, a.nins) | a.fixed) & ~1ull;
+      const bool ok = v < a.count;
+      x0[r] = ok ? ld_stream(a.psi + idx[r]) : make_double2(0, 0);
+      x1[r] = ok ? ld_stream(a.psi + idx[r] + 1) : make_double2(0, 0);
+    }
+    const bool odd = a.fixed & 1;
+#pragma unroll
+    for (int r = 0; r < APT; ++r) {
+      const uint64_t v = v0 + uint64_t(r) * kThreads;
+      if (v >= a.count) break;
+      const uint64_t i = idx[r] | (odd ? 1 : 0);
+      int sel = 0;
+      if (a.nt >= 1) sel |= int(i >> a.t0 & 1);
+      if (a.nt >= 2) sel |= int(i >> a.t1 & 1) << 1;
+      if (odd) x1[r] = cmul(x1[r], a.d[sel]);
+      else x0[r] = cmul(x0[r], a.d[sel]);
+      st_stream(a.psi + idx[r], x0[r]);
+      st_stream(a.psi + idx[r] + 1, x1[r]);
+    }
+  }
+}
+
 // ------------------------------------------------------------------------------ a9 tile
 // The generic (interpreted) fused-pass kernel: the pass program is walked op by op. The
 // persistent tile loop, loads, constants and store are tile_driver (tile_common.cuh); the JIT
@@ -183,7 +219,8 @@ struct InterpBody {
   static constexpr uint64_t kPF[kRegAmps] = {};
   static constexpr uint32_t kJF[kRegAmps] = {};
   int nops;
-  __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c) const {
+  __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c,
+                                             const TileArgs&) const {
     for (int i = 1; i < nops; ++i) {
       const TileOp& op = c.ops[i];
       switch (op.kind) {
@@ -621,7 +658,11 @@ cudaError_t launch_phase(cudaStream_t st, const PhaseArgs& a) {
   if (a.count == 0) return cudaSuccess;
   constexpr int APT = 4;
   const unsigned g = grid_for(a.count, kThreads * APT, 8);
-  phase_kernel<APT><<<g, kThreads, 0, st>>>(a);
+  // position 0 among the fixed (enumerated) positions: whole 32-byte sectors
+  bool sector = false;
+  for (int i = 0; i < a.nins; ++i) sector = sector || a.ins[i] == 0;
+  if (sector) phase_sector_kernel<APT><<<g, kThreads, 0, st>>>(a);
+  else phase_kernel<APT><<<g, kThreads, 0, st>>>(a);
   return cudaGetLastError();
 }
 

@@ -202,8 +202,8 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
 // plus a launch gap.
 double pass_cost_model(const Pass& p, int m);
 // Two single-buffered CTAs per SM at <= 128 registers for this pass's NVRTC kernel (instead of
-// one triple-buffered CTA at <= 255): QGPU_2CTA=1 every pass, 2 passes whose program runs
-// >= 40 FP64 instructions per amplitude (the latency-bound ones), 0 none (read per call).
+// one triple-buffered CTA at <= 255): QGPU_2CTA=1 every pass, 2 (default) passes whose program
+// runs >= 40 FP64 instructions per amplitude (the latency-bound ones), 0 none (read per call).
 bool pass_two_cta(const Pass& p);
 // Build the device ops of a tile pass from its gates and tile positions.
 void build_tile_ops(Pass& p, int m, int reg_bits = 4);

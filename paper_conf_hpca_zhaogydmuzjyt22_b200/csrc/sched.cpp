@@ -1362,8 +1362,10 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
 
 namespace qgpu {
 bool pass_two_cta(const Pass& p) {
+  // default 2 (profiles/r02 A/B, same box: QAOA_32 175.9 -> 166.5 ms fixed lanes and 178.4 ->
+  // 158.8 auto lanes, rqc_30 146.9 -> 139.5, grqc_32 8.43 -> 8.20 s, QFT_28 1.13 -> 1.10 ms)
   const char* ev = std::getenv("QGPU_2CTA");
-  const int mode = ev ? std::atoi(ev) : 0;
+  const int mode = ev ? std::atoi(ev) : 2;
   if (p.kind != PK_TILE || mode == 0) return false;
   return mode == 1 || p.fp64_per_amp >= 40.0;
 }

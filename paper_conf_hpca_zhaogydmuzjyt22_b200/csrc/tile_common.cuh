@@ -22,6 +22,7 @@ namespace qgpu {
 
 constexpr int kMaxTileBits = 13;
 constexpr int kRegAmps = 16;
+constexpr int kUmatParam = 512;  // complex entries of the U-matrix pool passed as a kernel parameter
 
 enum OpKind : int {
   OP_REMAP = 0,  // a0: packed register bits (4 bits each), a1: packed warp bits
@@ -113,6 +114,10 @@ struct TileArgs {
   // differ -- add without atomics. 0: requested bits uniform across a warp's slots.
   int hacc;
   uint32_t hlred;
+  // the pass's U matrices as a kernel parameter (constant bank), when they fit: the NVRTC bodies
+  // read them at compile-time offsets (no shared-memory loads, no registers held across tiles)
+  int umat_n;
+  double2 umat[kUmatParam];
 };
 
 __device__ __forceinline__ double2 cmul(double2 a, double2 b) {
@@ -562,6 +567,44 @@ __device__ __forceinline__ void run_apply_ptab_z(double2 (&v)[kRegAmps], double2
   for (int r = 0; r < (1 << NR); ++r)
     if (!((ZM >> r) & 1) && !id[r]) v[r] = cmul(v[r], P[r]);
 }
+// Same product as run_apply_ptab_z with two 4-entry tables instead of one 16-entry table: A over
+// register bits 0-1 (t0, e0, e1), B over bits 2-3 (e2, e3), v[r] *= A[r & 3] * B[r >> 2] applied
+// as two multiplies. About the same FP64 count (16 + 12 multiplies + 4 for the tables vs 16 + 15)
+// but 8 complex table registers instead of 16 at the program's register peak.
+template <int NR, bool T0, bool E0, bool E1, bool E2, bool E3, unsigned ZM>
+__device__ __forceinline__ void run_apply_split_z(double2 (&v)[kRegAmps], double2 t0, double2 e0, double2 e1,
+                                                  double2 e2, double2 e3) {
+  double2 A[4], B[4];
+  bool ia[4], ib[4];
+  A[0] = t0;
+  ia[0] = !T0;
+  A[1] = ia[0] ? e0 : cmul(A[0], e0);
+  ia[1] = ia[0] && !E0;
+  if (!E0) A[1] = A[0];
+  A[2] = ia[0] ? e1 : cmul(A[0], e1);
+  ia[2] = ia[0] && !E1;
+  if (!E1) A[2] = A[0];
+  A[3] = ia[1] ? e1 : cmul(A[1], e1);
+  ia[3] = ia[1] && !E1;
+  if (!E1) A[3] = A[1];
+  B[0] = make_double2(1.0, 0.0);
+  ib[0] = true;
+  B[1] = e2;
+  ib[1] = !E2;
+  B[2] = e3;
+  ib[2] = !E3;
+  B[3] = E2 ? (E3 ? cmul(e2, e3) : e2) : e3;
+  ib[3] = !E2 && !E3;
+#pragma unroll
+  for (int r = 0; r < (1 << NR); ++r) {
+    if ((ZM >> r) & 1) continue;
+    const int ra = r & 3, rb = r >> 2;
+    const bool use_a = !ia[ra] && (NR >= 1) && (ra < (1 << (NR < 2 ? NR : 2)));
+    const bool use_b = NR > 2 && !ib[rb];
+    if (use_a) v[r] = cmul(v[r], A[ra]);
+    if (use_b) v[r] = cmul(v[r], B[rb]);
+  }
+}
 template <int NR, unsigned RM, unsigned RT, unsigned ZM>
 __device__ __forceinline__ void run_apply_group_z(double2 (&v)[kRegAmps], double2 acc) {
 #pragma unroll
@@ -702,7 +745,7 @@ __device__ __forceinline__ void bulk_store_tile(double2* s, const TileArgs& a, u
 // (lane bits = physical positions 0..4: each warp store writes 512 contiguous bytes). Pattern
 // constants are computed per warp and the tile-uniform phase per lane, so a tile without
 // remaps runs with no CTA-wide barrier.
-// Body: void operator()(double2 (&v)[16], Mapping& mp, const TileCtx& c); Body::kZM0 = slots
+// Body: void operator()(double2 (&v)[16], Mapping& mp, const TileCtx& c, const TileArgs& a); Body::kZM0 = slots
 // known zero at the start of the pass, Body::kZW0 = warp bits whose warps hold only zeros.
 template <int NR, class Body>
 __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
@@ -892,7 +935,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     if (more && nbuf == 1 && !a.remaps) issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
     c.mpar = nexec & 1u;
     ++nexec;
-    body(v, mp, c);
+    body(v, mp, c, a);
     if (more && nbuf == 1 && a.remaps) {
       __syncthreads();
       issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);

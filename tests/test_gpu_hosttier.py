@@ -62,9 +62,11 @@ def test_host_tier_vs_oracle(q, h, name, fuse, comp):
 
 
 @pytest.mark.parametrize("name", ["random", "qaoa", "grqc"])
-def test_host_tier_bit_identical_to_resident_virtual_ranks(q, name):
+def test_host_tier_bit_identical_to_resident_virtual_ranks(q, name, monkeypatch):
     """Same plan and kernels as 2^h HBM-resident virtual ranks: the streamed result is the same
-    bits (the host tier only changes where the slices live between runs)."""
+    bits (the host tier only changes where the slices live between runs). The host tier keeps
+    local-first placement, so the virtual ranks are planned without the cross-rank expand."""
+    monkeypatch.setenv("QGPU_GLOBAL_FIRST", "0")
     c = CIRCS[name]()
     text = c.qasm()
     with q.State(c.n, host_slice_bits=2, fuse_bits=9) as s:
