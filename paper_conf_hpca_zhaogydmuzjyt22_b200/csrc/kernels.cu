@@ -230,12 +230,15 @@ struct InterpBody {
         case OP_U1R: {
           if (!op_active(op, c.gbase) || (mp.base & op.tmask) != op.tmatch) break;
           const double2* u = c.pool + op.moff;
-          switch (op.a0 * 4 + op.cls) {
+          switch (op.a0 * 8 + op.cls) {
 #define QGPU_U1R(K, CL) \
-  case K * 4 + CL: op_u1r<NR, K, CL>(v, u, op.rmask, op.rmatch); break;
+  case K * 8 + CL: op_u1r<NR, K, CL>(v, u, op.rmask, op.rmatch); break;
             QGPU_U1R(0, 0) QGPU_U1R(0, 1) QGPU_U1R(0, 2) QGPU_U1R(0, 3) QGPU_U1R(1, 0) QGPU_U1R(1, 1)
             QGPU_U1R(1, 2) QGPU_U1R(1, 3) QGPU_U1R(2, 0) QGPU_U1R(2, 1) QGPU_U1R(2, 2) QGPU_U1R(2, 3)
             QGPU_U1R(3, 0) QGPU_U1R(3, 1) QGPU_U1R(3, 2) QGPU_U1R(3, 3)
+            QGPU_U1R(0, 4) QGPU_U1R(0, 5) QGPU_U1R(0, 6) QGPU_U1R(0, 7) QGPU_U1R(1, 4) QGPU_U1R(1, 5)
+            QGPU_U1R(1, 6) QGPU_U1R(1, 7) QGPU_U1R(2, 4) QGPU_U1R(2, 5) QGPU_U1R(2, 6) QGPU_U1R(2, 7)
+            QGPU_U1R(3, 4) QGPU_U1R(3, 5) QGPU_U1R(3, 6) QGPU_U1R(3, 7)
 #undef QGPU_U1R
             default: break;
           }
@@ -245,10 +248,14 @@ struct InterpBody {
           if (!op_active(op, c.gbase)) break;
           const bool tc = (mp.base & op.tmask) == op.tmatch;
           const double2* u = c.pool + op.moff;
-          if (op.cls == MAT_X) op_u1l<NR, MAT_X>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch);
-          else if (op.cls == MAT_RI) op_u1l<NR, MAT_RI>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch);
-          else if (op.cls == MAT_REAL) op_u1l<NR, MAT_REAL>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch);
-          else op_u1l<NR, MAT_GENERIC>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch);
+          switch (op.cls) {
+#define QGPU_U1L(CL) \
+  case CL: op_u1l<NR, CL>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch); break;
+            QGPU_U1L(MAT_X) QGPU_U1L(MAT_RI) QGPU_U1L(MAT_REAL) QGPU_U1L(MAT_RU) QGPU_U1L(MAT_RUN)
+            QGPU_U1L(MAT_IU) QGPU_U1L(MAT_IUN)
+#undef QGPU_U1L
+            default: op_u1l<NR, MAT_GENERIC>(v, u, op.a0, c.lane, tc, op.rmask, op.rmatch); break;
+          }
           break;
         }
         case OP_U2R: {
@@ -273,10 +280,14 @@ struct InterpBody {
           if (!op_active(op, c.gbase)) break;
           tile_spill<NR>(v, c, mp);
           if (op.kind == OP_SMEM2) op_smem2(c, op);
-          else if (op.cls == MAT_X) op_smem1<MAT_X>(c, op);
-          else if (op.cls == MAT_RI) op_smem1<MAT_RI>(c, op);
-          else if (op.cls == MAT_REAL) op_smem1<MAT_REAL>(c, op);
-          else op_smem1<MAT_GENERIC>(c, op);
+          else switch (op.cls) {
+#define QGPU_SM1(CL) \
+  case CL: op_smem1<CL>(c, op); break;
+            QGPU_SM1(MAT_X) QGPU_SM1(MAT_RI) QGPU_SM1(MAT_REAL) QGPU_SM1(MAT_RU) QGPU_SM1(MAT_RUN)
+            QGPU_SM1(MAT_IU) QGPU_SM1(MAT_IUN)
+#undef QGPU_SM1
+            default: op_smem1<MAT_GENERIC>(c, op); break;
+          }
           tile_reload<NR>(v, c, mp);
           break;
         }

@@ -202,7 +202,7 @@ uint64_t unfused_gate_bytes(const PhysGate& g, int k_in, int k_out) {
 //  complex multiply per general r-condition group on the amplitudes it selects; the
 //  tile-uniform scalar 4. Conditions scale an op by the fraction of amplitudes they select.
 double fp64_model(const Pass& p) {
-  auto cls_cost = [](int cls) { return cls == MAT_GENERIC ? 8.0 : cls == MAT_X ? 0.0 : 4.0; };
+  auto cls_cost = [](int cls) { return cls == MAT_GENERIC ? 8.0 : cls == MAT_X ? 0.0 : mat_unit(cls) ? 2.0 : 4.0; };
   if (p.kind == PK_TILE) {
     const TileProgram& P = p.prog;
     double c = P.scalar.empty() ? 0.0 : 4.0;
@@ -615,6 +615,9 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
   }
 
   // 3. mapping
+  double pass_scale = 1.0;  // deferred real factor of the unit-diagonal ops
+  const char* uf_env = std::getenv("QGPU_UNIT_FORMS");  // 0: keep the plain classes (A/B)
+  const bool unit_forms = !(uf_env && uf_env[0] == '0');
   const int b = p.b;
   const int lanes = std::min(5, b);
   const int nonlane = b - lanes;
@@ -749,7 +752,27 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
     op.omatch = o.omatch;
     op.moff = uint32_t(P.pool.size());
     const int dim = o.kind == 0 ? 2 : 4;
-    for (int e = 0; e < dim * dim; ++e) P.pool.push_back(o.U[e]);
+    cplx Un[16];
+    std::memcpy(Un, o.U, sizeof(Un));
+    // unit-diagonal form (MAT_RU / RUN / IU / IUN): an unconditional real or RX-type 1-qubit op
+    // with |U00| = |U11| >= its off-diagonal magnitudes is divided by U00 (U11 / U00 is then +1 or
+    // -1 exactly); the factor U00 joins the pass's deferred scale, applied once per amplitude with
+    // the tile-uniform scalar. Every amplitude of the tile passes through every such op, so the
+    // product of the factors is one constant of the pass.
+    if (unit_forms && o.kind == 0 && o.lmask == 0 && o.omask == 0 && (op.cls == MAT_REAL || op.cls == MAT_RI)) {
+      const bool ri = op.cls == MAT_RI;
+      const double a = o.U[0].re, d = o.U[3].re;
+      const double b = ri ? o.U[1].im : o.U[1].re, c = ri ? o.U[2].im : o.U[2].re;
+      if (a != 0.0 && std::fabs(a) == std::fabs(d) && std::fabs(a) >= std::fabs(b) && std::fabs(a) >= std::fabs(c)) {
+        const bool neg = (d / a) < 0.0;
+        for (int e = 0; e < 4; ++e) Un[e] = cplx{o.U[e].re / a, o.U[e].im / a};
+        Un[0] = cplx{1.0, 0.0};
+        Un[3] = cplx{neg ? -1.0 : 1.0, 0.0};
+        op.cls = ri ? (neg ? MAT_IUN : MAT_IU) : (neg ? MAT_RUN : MAT_RU);
+        pass_scale *= a;
+      }
+    }
+    for (int e = 0; e < dim * dim; ++e) P.pool.push_back(Un[e]);
     if (o.kind == 0) {
       const int t = o.t[0];
       if (t < lanes) {
@@ -785,6 +808,7 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
     P.ops.push_back(op);
     ++i;
   }
+  if (pass_scale != 1.0) P.scalar.push_back(PhaseTerm{0, 0, pass_scale, 0.0});
   split_patterns(P, p, m);
   P.layout();
   if (std::getenv("QGPU_DEBUG_PLAN")) {

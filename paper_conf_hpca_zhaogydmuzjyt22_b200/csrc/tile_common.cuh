@@ -37,8 +37,24 @@ enum MatClass : int {
   MAT_GENERIC = 0,  // complex 2x2: 16 FP64 per pair
   MAT_REAL = 1,     // real entries (H, RY): 8 per pair
   MAT_X = 2,        // exactly X: a swap, no arithmetic
-  MAT_RI = 3        // real diagonal, imaginary off-diagonal (RX, SX up to phase...): 8 per pair
+  MAT_RI = 3,       // real diagonal, imaginary off-diagonal (RX, SX up to phase...): 8 per pair
+  // Unit-diagonal forms of REAL / RI: an unconditional op's matrix divided by its U00 (|U00| =
+  // |U11| >= the off-diagonal magnitudes, U11 / U00 = +1 or -1), the factor U00 deferred into the
+  // pass's tile-uniform scalar. 4 FP64 per pair (one DFMA per output component): H, RX, RY, SX,
+  // SY and the real rotation of a split generic gate.
+  MAT_RU = 4,       // [[1, b], [c, 1]] real b, c
+  MAT_RUN = 5,      // [[1, b], [c, -1]]
+  MAT_IU = 6,       // [[1, i b], [i c, 1]] real b, c
+  MAT_IUN = 7       // [[1, i b], [i c, -1]]
 };
+#if defined(__CUDACC__)
+#define QGPU_HD __host__ __device__
+#else
+#define QGPU_HD
+#endif
+QGPU_HD constexpr bool mat_unit(int c) { return c >= MAT_RU; }
+QGPU_HD constexpr bool mat_unit_neg(int c) { return c == MAT_RUN || c == MAT_IUN; }
+QGPU_HD constexpr bool mat_unit_imag(int c) { return c == MAT_IU || c == MAT_IUN; }
 
 struct TileOp {
   int kind;
@@ -222,6 +238,20 @@ __device__ __forceinline__ void apply2(double2& x0, double2& x1, const double2 (
     const double2 y1 = make_double2(fma(d, x1.x, -c * x0.y), fma(d, x1.y, c * x0.x));
     x0 = y0;
     x1 = y1;
+  } else if (CLS == MAT_RU || CLS == MAT_RUN) {  // [[1, b], [c, +-1]]
+    const double bq = u[1].x, c = u[2].x;
+    const double2 x1s = CLS == MAT_RUN ? make_double2(-x1.x, -x1.y) : x1;
+    const double2 y0 = make_double2(fma(bq, x1.x, x0.x), fma(bq, x1.y, x0.y));
+    const double2 y1 = make_double2(fma(c, x0.x, x1s.x), fma(c, x0.y, x1s.y));
+    x0 = y0;
+    x1 = y1;
+  } else if (CLS == MAT_IU || CLS == MAT_IUN) {  // [[1, i b], [i c, +-1]]
+    const double bq = u[1].y, c = u[2].y;
+    const double2 x1s = CLS == MAT_IUN ? make_double2(-x1.x, -x1.y) : x1;
+    const double2 y0 = make_double2(fma(-bq, x1.y, x0.x), fma(bq, x1.x, x0.y));
+    const double2 y1 = make_double2(fma(-c, x0.y, x1s.x), fma(c, x0.x, x1s.y));
+    x0 = y0;
+    x1 = y1;
   } else {
     const double2 y0 = cfma(u[0], x0, cmul(u[1], x1));
     const double2 y1 = cfma(u[2], x0, cmul(u[3], x1));
@@ -353,6 +383,16 @@ __device__ __forceinline__ void op_u1l(double2 (&v)[kRegAmps], const double2* up
       const double2 own = hi ? a1 : a0, oth = hi ? a0 : a1;
       const double dg = hi ? up[3].x : up[0].x, od = hi ? up[2].y : up[1].y;
       y = make_double2(fma(dg, own.x, -od * oth.y), fma(dg, own.y, od * oth.x));
+    } else if (mat_unit(CLS)) {  // own coefficient +-1: one DFMA per component
+      const double2 own = v[r];
+      const double2 owns = (mat_unit_neg(CLS) && hi) ? make_double2(-own.x, -own.y) : own;
+      if (mat_unit_imag(CLS)) {
+        const double od = hi ? up[2].y : up[1].y;
+        y = make_double2(fma(-od, pv.y, owns.x), fma(od, pv.x, owns.y));
+      } else {
+        const double od = hi ? up[2].x : up[1].x;
+        y = make_double2(fma(od, pv.x, owns.x), fma(od, pv.y, owns.y));
+      }
     } else {
       y = cfma(c0, a0, cmul(c1, a1));
     }
@@ -439,6 +479,10 @@ __device__ __forceinline__ void apply2_x1zero(double2& x0, double2& x1, const do
   } else if (CLS == MAT_REAL) {
     x1 = make_double2(u[2].x * x0.x, u[2].x * x0.y);
     x0 = make_double2(u[0].x * x0.x, u[0].x * x0.y);
+  } else if (CLS == MAT_RU || CLS == MAT_RUN) {  // (x0, 0) -> (x0, c x0)
+    x1 = make_double2(u[2].x * x0.x, u[2].x * x0.y);
+  } else if (CLS == MAT_IU || CLS == MAT_IUN) {  // (x0, 0) -> (x0, i c x0)
+    x1 = make_double2(-u[2].y * x0.y, u[2].y * x0.x);
   } else {
     x1 = cmul(u[2], x0);
     x0 = cmul(u[0], x0);
@@ -453,6 +497,12 @@ __device__ __forceinline__ void apply2_x0zero(double2& x0, double2& x1, const do
   } else if (CLS == MAT_REAL) {
     x0 = make_double2(u[1].x * x1.x, u[1].x * x1.y);
     x1 = make_double2(u[3].x * x1.x, u[3].x * x1.y);
+  } else if (CLS == MAT_RU || CLS == MAT_RUN) {  // (0, x1) -> (b x1, +-x1)
+    x0 = make_double2(u[1].x * x1.x, u[1].x * x1.y);
+    if (CLS == MAT_RUN) x1 = make_double2(-x1.x, -x1.y);
+  } else if (CLS == MAT_IU || CLS == MAT_IUN) {  // (0, x1) -> (i b x1, +-x1)
+    x0 = make_double2(-u[1].y * x1.y, u[1].y * x1.x);
+    if (CLS == MAT_IUN) x1 = make_double2(-x1.x, -x1.y);
   } else {
     x0 = cmul(u[1], x1);
     x1 = cmul(u[3], x1);
@@ -495,6 +545,16 @@ __device__ __forceinline__ void op_u1l_z(double2 (&v)[kRegAmps], const double2* 
       const double2 own = hi ? a1 : a0, oth = hi ? a0 : a1;
       const double dg = hi ? up[3].x : up[0].x, od = hi ? up[2].y : up[1].y;
       y = make_double2(fma(dg, own.x, -od * oth.y), fma(dg, own.y, od * oth.x));
+    } else if (mat_unit(CLS)) {  // own coefficient +-1: one DFMA per component
+      const double2 own = v[r];
+      const double2 owns = (mat_unit_neg(CLS) && hi) ? make_double2(-own.x, -own.y) : own;
+      if (mat_unit_imag(CLS)) {
+        const double od = hi ? up[2].y : up[1].y;
+        y = make_double2(fma(-od, pv.y, owns.x), fma(od, pv.x, owns.y));
+      } else {
+        const double od = hi ? up[2].x : up[1].x;
+        y = make_double2(fma(od, pv.x, owns.x), fma(od, pv.y, owns.y));
+      }
     } else {
       y = cfma(c0, a0, cmul(c1, a1));
     }
