@@ -231,15 +231,6 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     a.off_pool = int(P.off_pool);
     a.nr = P.nr;
     a.nw = P.nw;
-    a.bigmask = 0;
-    a.nbig = 0;
-    const char* bp_env = std::getenv("QGPU_BIGPAT");  // 0: every pattern by one lane (A/B)
-    const bool bigpat = !(bp_env && bp_env[0] == '0');
-    for (size_t pi = 0; bigpat && pi < P.patterns.size() && pi < 64 && a.nbig < 16; ++pi)
-      if (P.patterns[pi].count > 6) {
-        a.bigmask |= 1ull << pi;
-        a.big[a.nbig++] = int(pi);
-      }
     a.umat_n = int(std::min(P.pool.size(), size_t(kUmatParam)));
     if (P.pool.size() <= size_t(kUmatParam))
       for (size_t i = 0; i < P.pool.size(); ++i) a.umat[i] = make_double2(P.pool[i].re, P.pool[i].im);

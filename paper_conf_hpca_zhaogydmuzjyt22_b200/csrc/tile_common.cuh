@@ -133,12 +133,6 @@ struct TileArgs {
   // the pass's U matrices as a kernel parameter (constant bank), when they fit: the NVRTC bodies
   // read them at compile-time offsets (no shared-memory loads, no registers held across tiles)
   int umat_n;
-  // patterns with many terms (the tile-uniform scalar of a phase-heavy pass collects dozens):
-  // their per-tile products are evaluated by the whole warp (lane-strided terms, butterfly
-  // product) instead of by one lane while the others wait
-  uint64_t bigmask;        // bit pi: pattern pi (< 64) is in big[]
-  int nbig;
-  int big[16];
   double2 umat[kUmatParam];
 };
 
@@ -960,51 +954,22 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       const uint32_t lo = uint32_t(treal) & uint32_t(CH - 1);
       double2* cw = Cw + size_t(warp) * a.npat;
       double2* chw = Chw + size_t(warp) * a.npat;
-      // product of the matching terms [q0, q1) of a big pattern over the whole warp
-      auto warp_product = [&](uint32_t q0, uint32_t q1) {
-        double2 cc = make_double2(1.0, 0.0);
-        for (uint32_t q = q0 + uint32_t(lane); q < q1; q += 32)
-          if ((gbase & terms[q].omask) == terms[q].omatch) cc = cmul(cc, make_double2(terms[q].re, terms[q].im));
-#pragma unroll
-        for (int o = 16; o > 0; o >>= 1) {
-          double2 oc;
-          oc.x = __shfl_xor_sync(0xffffffffu, cc.x, o);
-          oc.y = __shfl_xor_sync(0xffffffffu, cc.y, o);
-          cc = cmul(cc, oc);
-        }
-        return cc;
-      };
-      auto is_big = [&](int pi) { return pi < 64 && ((a.bigmask >> pi) & 1ull); };
       if (hi != cur_hi) {
         cur_hi = hi;
         for (int pi = lane; pi < a.npat; pi += 32) {
-          if (is_big(pi)) continue;
           double2 cc = make_double2(1.0, 0.0);
           const Pattern pt = pats[pi];
           for (uint32_t q = pt.first; q < pt.first + pt.nhi; ++q)
             if ((gbase & terms[q].omask) == terms[q].omatch) cc = cmul(cc, make_double2(terms[q].re, terms[q].im));
           chw[pi] = cc;
         }
-        for (int bi = 0; bi < a.nbig; ++bi) {
-          const Pattern pt = pats[a.big[bi]];
-          const double2 cc = warp_product(pt.first, pt.first + pt.nhi);
-          if (lane == 0) chw[a.big[bi]] = cc;
-        }
-        __syncwarp();
       }
       for (int pi = lane; pi < a.npat; pi += 32) {
-        if (is_big(pi)) continue;
         double2 cc = cmul(chw[pi], tlo[(size_t(pi) << a.lb) + lo]);
         const Pattern pt = pats[pi];
         for (uint32_t q = pt.first + pt.nhi; q < pt.first + pt.count; ++q)
           if ((gbase & terms[q].omask) == terms[q].omatch) cc = cmul(cc, make_double2(terms[q].re, terms[q].im));
         cw[pi] = cc;
-      }
-      for (int bi = 0; bi < a.nbig; ++bi) {
-        const int pi = a.big[bi];
-        const Pattern pt = pats[pi];
-        const double2 cl = warp_product(pt.first + pt.nhi, pt.first + pt.count);
-        if (lane == 0) cw[pi] = cmul(cmul(chw[pi], tlo[(size_t(pi) << a.lb) + lo]), cl);
       }
     }
     if (more && nbuf > 1) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
