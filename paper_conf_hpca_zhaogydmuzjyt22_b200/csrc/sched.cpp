@@ -644,7 +644,13 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
       if (ux != uy) return ux < uy;
       return x > y;
     });
+    int oldR[4] = {R[0], R[1], R[2], R[3]};
     for (int k = 0; k < nr; ++k) R[k] = cand[k];
+    if (std::getenv("QGPU_DEBUG_REMAP") && !P.ops.empty()) {
+      int chg = 0;
+      for (int k = 0; k < nr; ++k) chg += std::find(oldR, oldR + nr, R[k]) == oldR + nr;
+      std::fprintf(stderr, "remap k%d->%d: %d of %d register bits change\n", p.k_in, p.k_out, chg, nr);
+    }
     std::vector<int> w(cand.begin() + nr, cand.end());
     std::sort(w.begin(), w.end());
     if (P.ops.empty()) {
