@@ -532,6 +532,16 @@ def measure_workload(q, torch, device, stream, args, text, n, steps, warmup, wor
     return st, c, times, stats, (clk.summary() if clk else None)
 
 
+def ncu_traffic(key: str):
+    """DRAM bytes per tile launch from the committed ncu launch list of this workload (or None)."""
+    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+    try:
+        t = json.load(open(tp)).get(key)
+        return (t.get("dram_bytes_per_launch"), t.get("source")) if t else (None, None)
+    except Exception:
+        return None, None
+
+
 def tile_roofline(stats, ms, peak, peak_src):
     """Roofline of the dominant kernel (fused tile pass): algorithmic bytes / CUDA-event time."""
     tile_ms = statistics.mean(x["tile_kernel_ms"] for x in stats)
@@ -605,15 +615,7 @@ def run_ours(args):
     kernel_ms = statistics.mean(x["kernel_ms"] for x in stats)
     algo_bytes = statistics.mean(x["algo_bytes"] for x in stats)
     unfused = statistics.mean(x["unfused_bytes"] for x in stats)
-    tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
-    if os.path.exists(tp):
-        try:
-            t = json.load(open(tp)).get(f"{args.workload}_{n}")
-            if t:
-                roof["traffic"] = t.get("dram_bytes_per_launch")
-                roof["traffic_source"] = t.get("source")
-        except Exception:
-            pass
+    roof["traffic"], roof["traffic_source"] = ncu_traffic(f"{args.workload}_{n}")
     s0 = stats[-1]
     launches = s0["kernels_launched"]
 
@@ -748,7 +750,8 @@ def run_ours(args):
             ems = allreduce_max(statistics.mean(et), world, device)
             extras[key] = {"workload": edesc, "value": ems / 1e3, "unit": "s", "ms_per_step": ems,
                            "ms_per_step_best": min(et), "gates": len(ec.ops),
-                           "roofline": tile_roofline(estats, ems, peak, peak_src),
+                           "roofline": dict(tile_roofline(estats, ems, peak, peak_src),
+                                            **dict(zip(("traffic", "traffic_source"), ncu_traffic(f"{key}_{ec.n}")))),
                            "passes": estats[-1]["passes"],
                            "ops_before_full_involvement": estats[-1]["ops_before_full_involvement"]}
             if key == "qft28" and args.gfc:
