@@ -591,7 +591,8 @@ def run_ours(args):
     q.load()
 
     sharded = args.sharded and world > 1
-    circ, desc = workload(args.workload, args.n, world if sharded else 1)
+    vr = args.virtual_ranks if not sharded else 0
+    circ, desc = workload(args.workload, args.n, world if sharded else (vr or 1))
     text = circ.qasm()
     n = circ.n
     stream = torch.cuda.Stream(device=device)
@@ -603,6 +604,11 @@ def run_ours(args):
         obj = [q.nccl_unique_id() if rank == 0 else None]
         dist.broadcast_object_list(obj, src=0)
         cfg_extra = dict(world_size=world, rank=rank, nccl_unique_id=obj[0])
+    elif vr > 1:
+        # the sharded plan on ONE GPU: 2^g shards in this process, rank-bit conditions, copy
+        # activations and batched swaps through the same pack / unpack slab loop, with device
+        # copies between the shards' staging as the transport instead of NVLink
+        cfg_extra = dict(world_size=vr)
     flush = torch.empty(64 << 20, dtype=torch.float32, device=device)  # 256 MiB > 126 MB L2
     peak, peak_src = peaks()
 
@@ -698,6 +704,13 @@ def run_ours(args):
         "gpu_launches_per_step": launches,
         "clocks": clocks,
     }
+    if vr > 1:
+        sb = statistics.mean(x["swap_bytes"] for x in stats)
+        sms = statistics.mean(x["swap_ms"] for x in stats)
+        line["config"]["parallelism"] = f"1 GPU, {vr} virtual ranks (sharded plan, device-copy transport)"
+        line["swap"] = {"transport": "device copies between the shards' staging (virtual ranks, one GPU)",
+                        "swaps_per_step": s0["swaps"], "swap_bits_per_step": s0["swap_bits"],
+                        "bytes_moved_per_step": sb, "swap_ms_per_step": sms}
     if sharded:
         # global-local swap throughput per GPU (bytes this rank sent / CUDA-event time
         # of its swap passes on the state's stream), against NVLink 5's 900 GB/s per direction
@@ -810,6 +823,8 @@ def main():
                     help="h > 0: host-memory tier, state in pinned host memory as 2^h slices (NEXT-2)")
     ap.add_argument("--host-compress", type=int, default=0,
                     help="1: host tier slices cross the link GFC-compressed (NEXT-3 on the NEXT-2 link)")
+    ap.add_argument("--virtual-ranks", type=int, default=0,
+                    help="G > 1 (N = 1): plan and run the sharded path with G shards on this one GPU")
     ap.add_argument("--sharded", action="store_true",
                     help="N>1: shard one state over the ranks (NCCL swaps) instead of N replicas")
     args = ap.parse_args()

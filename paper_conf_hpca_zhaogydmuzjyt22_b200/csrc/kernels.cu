@@ -659,7 +659,14 @@ cudaError_t launch_pair(cudaStream_t st, const PairArgs& a, bool shfl) {
 
 cudaError_t launch_quad(cudaStream_t st, const QuadArgs& a) {
   if (a.nquads == 0) return cudaSuccess;
-  constexpr int QPT = 1;
+  // two quads (8 loads of 16 B) in flight per thread (QGPU_QPT=1: one, A/B)
+  const char* qe = std::getenv("QGPU_QPT");
+  if (qe && qe[0] == '1') {
+    const unsigned g1 = grid_for(a.nquads, kThreads, 8);
+    quad_kernel<1><<<g1, kThreads, 0, st>>>(a);
+    return cudaGetLastError();
+  }
+  constexpr int QPT = 2;
   const unsigned g = grid_for(a.nquads, kThreads * QPT, 8);
   quad_kernel<QPT><<<g, kThreads, 0, st>>>(a);
   return cudaGetLastError();
