@@ -557,23 +557,34 @@ def tile_roofline(stats, ms, peak, peak_src):
 
 def per_pass_binding(prof, hbm_gbs, fp64_fma_per_s):
     """SURVEY §8d / P:401 roofline per pass: bound = max(bytes / HBM peak, FP64 instructions /
-    FP64 peak); frac = bound / measured time. Also the step total."""
+    FP64 peak); frac = bound / measured time. Also the step total. Supplementary `sm_bound`: the
+    SM side of the same pass with the shared-memory / shuffle (MIO) pipe the kernel design adds
+    (4 shuffles per amplitude per lane-bit op, 32 B per amplitude per remap, at one MIO op per
+    clock per SM) on top of the FP64 instructions: max(HBM, FP64 + MIO)."""
     rows = []
-    tb = tm = 0.0
+    tb = tm = tsm = 0.0
+    clk = fp64_fma_per_s / (148 * 64.0) if fp64_fma_per_s else 1.9e9  # SM clock implied by the FP64 probe
     kinds = {0: "tile", 1: "pair", 2: "quad", 3: "diag", 5: "swap", 7: "zero"}
     for r in prof:
         t_hbm = r["bytes"] / (hbm_gbs * 1e9) * 1e3
         t_fp = r["fp64_ops"] / fp64_fma_per_s * 1e3 if fp64_fma_per_s else 0.0
         bound = max(t_hbm, t_fp)
+        mio_clk = r.get("lane_ops", 0) * 4.0 / 32.0 + r.get("remaps", 0) * 32.0 / 128.0
+        t_mio = r["amps_computed"] * mio_clk / (148 * clk) * 1e3
+        tsm += max(t_hbm, t_fp + t_mio)
         rows.append({"kind": kinds.get(r["kind"], r["kind"]), "k": f"{r['k_in']}->{r['k_out']}",
                      "gates": r["n_gates"], "ms": round(r["ms"], 4), "bytes": r["bytes"],
                      "fp64_per_amp": round(r["fp64_ops"] / r["amps_computed"], 2) if r["amps_computed"] else 0.0,
                      "hbm_ms": round(t_hbm, 4), "fp64_ms": round(t_fp, 4),
-                     "binding": "fp64" if t_fp > t_hbm else "hbm",
+                     "binding": "fp64" if t_fp > t_hbm else "hbm", "lane_ops": r.get("lane_ops"),
+                     "remaps": r.get("remaps"), "mio_ms": round(t_mio, 4),
                      "frac_of_binding": round(bound / r["ms"], 3) if r["ms"] > 0 else None})
         tb += bound
         tm += r["ms"]
-    return {"passes": rows, "bound_ms": tb, "measured_ms": tm, "frac": tb / tm if tm else None}
+    return {"passes": rows, "bound_ms": tb, "measured_ms": tm, "frac": tb / tm if tm else None,
+            "sm_bound": {"bound_ms": tsm, "frac": tsm / tm if tm else None,
+                         "model": "per pass max(HBM, FP64 + MIO); MIO = shuffles of lane-bit ops and "
+                                  "shared-memory remaps at one op per clock per SM"}}
 
 
 def run_ours(args):

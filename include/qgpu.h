@@ -149,6 +149,8 @@ typedef struct qgpu_pass_profile {
   uint64_t bytes;              /* algorithmic HBM bytes (live input read + output written)     */
   uint64_t amps_computed;      /* amplitudes the program ran on (zero tiles excluded)          */
   double fp64_ops;             /* FP64 pipe instructions (DFMA/DMUL/DADD) by the pass model    */
+  int32_t lane_ops;            /* fused pass: 1-qubit ops on lane bits (4 warp shuffles per amplitude) */
+  int32_t remaps;              /* fused pass: remaps / shared-memory ops (32 B of shared memory per amplitude) */
 } qgpu_pass_profile;
 
 /* ---- configuration and state ---------------------------------------------------------- */

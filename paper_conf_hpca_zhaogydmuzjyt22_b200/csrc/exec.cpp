@@ -506,6 +506,12 @@ qgpu_status exec_pass(qgpu_state* st, const Pass& p, const unsigned char* d_ops,
       tl.rec.bytes = bytes;
       tl.rec.amps_computed = p.kind == PK_SWAP ? 0 : computed_amps(st, p);
       tl.rec.fp64_ops = p.fp64_per_amp * double(tl.rec.amps_computed);
+      if (p.kind == PK_TILE)
+        for (size_t i = 1; i < p.prog.ops.size(); ++i) {
+          const int k = p.prog.ops[i].kind;
+          tl.rec.lane_ops += k == OP_U1L;
+          tl.rec.remaps += k == OP_REMAP || k == OP_SMEM1 || k == OP_SMEM2;
+        }
     }
     st->pending.push_back(tl);
   }

@@ -71,7 +71,8 @@ class Stats(ctypes.Structure):
 class PassProfile(ctypes.Structure):
     _fields_ = [("kind", ctypes.c_int32), ("k_in", ctypes.c_int32), ("k_out", ctypes.c_int32),
                 ("n_gates", ctypes.c_int32), ("ms", ctypes.c_double), ("bytes", ctypes.c_uint64),
-                ("amps_computed", ctypes.c_uint64), ("fp64_ops", ctypes.c_double)]
+                ("amps_computed", ctypes.c_uint64), ("fp64_ops", ctypes.c_double),
+                ("lane_ops", ctypes.c_int32), ("remaps", ctypes.c_int32)]
 
     def as_dict(self):
         return {k: getattr(self, k) for k, _ in self._fields_}
