@@ -724,6 +724,9 @@ qgpu_status apply_circuit_impl(qgpu_state* st, const qgpu_circuit* c, int meas_m
           }
         }
       }
+      if (std::getenv("QGPU_DEBUG_HIST"))
+        std::fprintf(stderr, "fused measurement: last fused pass %d, mode %d, unrequested lane bits %x\n", last,
+                     st->meas_hacc, st->meas_hlred);
       if (last >= 0) {
         if (!st->d_meas) CK(cudaMalloc(&st->d_meas, (size_t(8) << kMeasMax)));
         CK(cudaMemsetAsync(st->d_meas, 0, size_t(8) << meas_m, st->stream));
