@@ -1019,7 +1019,10 @@ qgpu_status qgpu_probabilities(qgpu_state* st, int mq, const int* qubits, double
     if (i > 0) CK(launch_add(st->stream, acc, tmp, B));
   }
   if (st->comm) {
-    if (qgpu_status s = comm_allreduce_sum(st->comm, acc, B, st->stream, &g_err)) return s;
+    if (qgpu_status s = comm_allreduce_sum(st->comm, acc, B, st->stream, &g_err)) {
+      st->poisoned = true;  // an NCCL failure leaves the communicator unusable
+      return s;
+    }
   }
   CK(cudaMemcpyAsync(out, acc, B * sizeof(double), cudaMemcpyDeviceToHost, st->stream));
   st->stats.d2h_bytes += B * sizeof(double);
