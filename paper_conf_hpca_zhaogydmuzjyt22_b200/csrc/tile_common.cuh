@@ -891,46 +891,6 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   Mapping mpf = mp0;      // the final mapping (the same after every tile)
   uint32_t hb0 = 0, hrb[4] = {0u, 0u, 0u, 0u};  // hmode == 2: bucket parts (thread, register bits)
   bool hbk_set = false;
-  uint32_t h_btile = ~0u;  // hmode == 2: the tile-base bucket bits hacc currently accumulates
-  // hmode == 2: add the accumulated per-slot sums x (destroyed) with tile-base bucket bits bt to
-  // this warp's histogram: sum the slots that differ only in unrequested register bits (same
-  // bucket), reduce the remaining slots over the unrequested lane bits (butterfly), then the lanes
-  // whose unrequested lane bits are 0 -- distinct buckets for every slot -- add without atomics
-  auto hist_flush = [&](double (&x)[1 << NR], uint32_t bt) {
-    double* hw = hsm + (size_t(warp) << a.hm);
-    uint32_t dead = 0;
-#pragma unroll
-    for (int k = 0; k < NR; ++k)
-      if (hrb[k] == 0u) {
-        dead |= 1u << k;
-#pragma unroll
-        for (int r = 0; r < (1 << NR); ++r)
-          if (r >> k & 1) x[r & ~(1 << k)] += x[r];
-      }
-#pragma unroll
-    for (int r = 0; r < (1 << NR); ++r) {
-      if (uint32_t(r) & dead) continue;
-#pragma unroll
-      for (int k = 0; k < 5; ++k)
-        if (a.hlred >> k & 1) x[r] += __shfl_xor_sync(0xffffffffu, x[r], 1 << k);
-    }
-    if ((uint32_t(lane) & a.hlred) == 0u) {
-      uint32_t bk[1 << NR];
-      double old[1 << NR];
-#pragma unroll
-      for (int r = 0; r < (1 << NR); ++r) {
-        bk[r] = bt | hb0;
-#pragma unroll
-        for (int k = 0; k < NR; ++k)
-          if (r >> k & 1) bk[r] |= hrb[k];
-        old[r] = ((uint32_t(r) & dead) == 0u) ? hw[bk[r]] : 0.0;
-      }
-#pragma unroll
-      for (int r = 0; r < (1 << NR); ++r)
-        if ((uint32_t(r) & dead) == 0u) hw[bk[r]] = old[r] + x[r];
-    }
-  };
-  (void)hist_flush;
   if constexpr (Body::kHist) {
 #pragma unroll
     for (int r = 0; r < (1 << NR); ++r) hacc[r] = 0.0;
@@ -1052,10 +1012,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     if constexpr (Body::kHist) if (a.hist && hmode == 2) {
       // per-warp private histogram. Bucket extraction is linear in the index bits, so a slot's
       // bucket = hb0 (thread part at tile base 0) | hrb[k] for each set register bit k of r |
-      // the tile base's bits (uniform); the final mapping is the same in every tile. A slot's
-      // |psi|^2 accumulates in registers over consecutive tiles whose base gives the same bucket
-      // bits (a CTA walks runs of 2^lb consecutive tiles) and is added to the histogram when they
-      // change and at the end of the kernel (hist_flush)
+      // bt (the tile base's bits, uniform); the final mapping is the same in every tile
       if (!hbk_set) {
         hbk_set = true;
         uint64_t pbh = 0;
@@ -1075,16 +1032,45 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
           else hrb[k] = bkt(sah.prb[k]);
         }
       }
-      uint32_t btile = 0;
-      for (int j = 0; j < a.hm; ++j) btile |= uint32_t(gbase >> a.hpos[j] & 1) << j;
-      if (btile != h_btile) {
-        if (h_btile != ~0u) hist_flush(hacc, h_btile);
-        h_btile = btile;
+      uint32_t bt = hb0;
+      for (int j = 0; j < a.hm; ++j) bt |= uint32_t(gbase >> a.hpos[j] & 1) << j;
+      double* hw = hsm + (size_t(warp) << a.hm);
+      const bool writer = (uint32_t(lane) & a.hlred) == 0u;
+      double x[1 << NR];
 #pragma unroll
-        for (int r = 0; r < (1 << NR); ++r) hacc[r] = 0.0;
+      for (int r = 0; r < (1 << NR); ++r) {
+        x[r] = fma(v[r].x, v[r].x, v[r].y * v[r].y);
+#pragma unroll
+        for (int k = 0; k < 5; ++k)
+          if (a.hlred >> k & 1) x[r] += __shfl_xor_sync(0xffffffffu, x[r], 1 << k);
       }
+      // slots that differ only in unrequested register bits share a bucket: sum them first, so
+      // the remaining ("live") slots have distinct buckets and all their loads can be issued
+      // before any store (one shared-memory latency per tile instead of one per slot)
+      uint32_t dead = 0;
 #pragma unroll
-      for (int r = 0; r < (1 << NR); ++r) hacc[r] += fma(v[r].x, v[r].x, v[r].y * v[r].y);
+      for (int k = 0; k < NR; ++k)
+        if (hrb[k] == 0u) {
+          dead |= 1u << k;
+#pragma unroll
+          for (int r = 0; r < (1 << NR); ++r)
+            if (r >> k & 1) x[r & ~(1 << k)] += x[r];
+        }
+      if (writer) {
+        uint32_t bk[1 << NR];
+        double old[1 << NR];
+#pragma unroll
+        for (int r = 0; r < (1 << NR); ++r) {
+          bk[r] = bt;
+#pragma unroll
+          for (int k = 0; k < NR; ++k)
+            if (r >> k & 1) bk[r] |= hrb[k];
+          old[r] = ((uint32_t(r) & dead) == 0u) ? hw[bk[r]] : 0.0;
+        }
+#pragma unroll
+        for (int r = 0; r < (1 << NR); ++r)
+          if ((uint32_t(r) & dead) == 0u) hw[bk[r]] = old[r] + x[r];
+      }
     }
     if constexpr (Body::kHist) if (a.hist && c.own && hmode == 0) {  // fused measurement: final amplitudes in registers
       uint64_t pbh = 0;
@@ -1167,7 +1153,6 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   if (a.bstore && warp == 0) bulk_wait_all();  // shared memory must outlive the bulk reads
   if constexpr (Body::kHist) {
     if (a.hist) {
-      if (hmode == 2 && h_btile != ~0u) hist_flush(hacc, h_btile);
       if (hmode == 1 && c.own) {
         // bucket of slot r: its tile-local index under the final mapping (tile base bits are not
         // requested, so base = 0); one shared-memory add per slot and thread
