@@ -1401,6 +1401,7 @@ bool pass_two_cta(const Pass& p) {
   const char* ev = std::getenv("QGPU_2CTA");
   const int mode = ev ? std::atoi(ev) : 2;
   if (p.kind != PK_TILE || mode == 0) return false;
+  if (mode == 3) return p.fp64_per_amp >= 40.0 || p.k_in == p.k_out;  // + steady-state passes
   return mode == 1 || p.fp64_per_amp >= 40.0;
 }
 }  // namespace qgpu
