@@ -283,6 +283,8 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     const int bs = bstore_mode();
     if (bs == 2 || (bs == 1 && a.remaps)) a.nbuf = 3;
     if (tile_smem_bytes(a) > 227 * 1024) a.nbuf = 2;
+    if (const char* nb = std::getenv("QGPU_NBUF"))  // experiments: fewer tile buffers
+      if (a.remaps && !two_cta) a.nbuf = std::max(1, std::min(a.nbuf, std::atoi(nb)));
     a.bstore = (a.nbuf == 3 && (bs == 2 || (bs == 1 && a.remaps))) ? 1 : 0;
     if (st->meas_pass == &p && !a.bstore) {  // fused measurement, if its histogram fits in smem
       TileArgs h = a;
