@@ -276,7 +276,8 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     // programs without remaps need one tile buffer (each thread only reads its own slots),
     // which lets two CTAs share an SM; otherwise triple (or double) buffering
     a.nbuf = a.remaps ? 3 : 1;
-    // QGPU_2CTA=1 (experiment): two single-buffered CTAs per SM at <= 128 registers (JIT only)
+    // FP64-heavy passes (pass_two_cta, default on): two single-buffered CTAs per SM at <= 128
+    // registers (NVRTC kernels only)
     const bool two_cta = pass_two_cta(p) && (st->cfg.jit == 2 || (st->cfg.jit == 1 && p.k_out >= jit_min_bits()));
     if (two_cta) a.nbuf = 1;
     // optional bulk stores (staged tile, async copies per run; QGPU_BSTORE)

@@ -459,6 +459,7 @@ __global__ void __launch_bounds__(kThreads) probs_kernel(ProbArgs a, int mode) {
 // non-requested lane bits and one atomic per bucket and warp adds into the output. Needs the
 // live range to be a power of two (it always is) and >= 2^5.
 struct ProbMap {
+  uint64_t fixed;                 // positions < k not enumerated by the loop (lanes, warps, CTAs, e)
   int wbits, cbits, ebits;
   int wpos[4], cpos[16], epos[3];
   int nfrun;                      // runs of fixed (non-loop) positions, ascending
@@ -493,15 +494,16 @@ __global__ void __launch_bounds__(512) probs_mapped_kernel(ProbArgs a, ProbMap m
   for (int e = 0; e < NE; ++e) acc[e] = 0.0;
   constexpr int U = NE >= 8 ? 1 : 8 / NE;  // loads in flight per thread: U * NE = 8
   const uint64_t nouter = 1ull << mp.obits;
+  // the loop's index bits, enumerated by a masked increment: with every fixed position set, +1
+  // carries straight through them to the next loop bit (t_{o+1} = ((t_o | fixed) + 1) & ~fixed)
+  const uint64_t fixed = mp.fixed;
+  uint64_t tnext = 0;
   for (uint64_t o = 0; o < nouter; o += U) {
     double2 v[U][NE];
 #pragma unroll
     for (int u = 0; u < U; ++u) {
-      uint64_t t = o + u;
-      for (int i = 0; i < mp.nfrun; ++i) {
-        const int p = mp.frun_pos[i];
-        t = ((t >> p) << (p + mp.frun_len[i])) | (t & ((1ull << p) - 1));
-      }
+      const uint64_t t = tnext;
+      tnext = ((tnext | fixed) + 1) & ~fixed;
       const bool ok = o + u < nouter;
 #pragma unroll
       for (int e = 0; e < NE; ++e) v[u][e] = ok ? __ldcs(a.psi + (tb | t | eoff[e])) : make_double2(0.0, 0.0);
@@ -558,6 +560,7 @@ bool plan_probs_map(const ProbArgs& a, int k, ProbMap* mp) {
     fixed |= 1ull << mp->epos[i];
   }
   mp->obits = k - 5 - mp->wbits - mp->cbits - mp->ebits;
+  mp->fixed = fixed;
   mp->nfrun = 0;
   for (int p = 0; p < k;) {
     if (!((fixed >> p) & 1)) {
