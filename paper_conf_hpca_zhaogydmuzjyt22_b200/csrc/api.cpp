@@ -607,7 +607,8 @@ qgpu_status qgpu_apply_gate(qgpu_state* st, const double* U, int nt, const int* 
 
 namespace {
 constexpr int kMeasMax = 12;
-// QGPU_HACC=0 turns the per-slot fused measurement off (A/B against the separate readout)
+// QGPU_HACC=0 turns the per-slot fused measurement off (A/B against the separate readout);
+// QGPU_HACC=2 fuses mode 2 even when lane bits need the butterfly
 bool hacc_enabled() {
   static const bool on = [] {
     const char* e = std::getenv("QGPU_HACC");
@@ -719,6 +720,13 @@ qgpu_status apply_circuit_impl(qgpu_state* st, const qgpu_circuit* c, int meas_m
               for (int j = 0; j < meas_m; ++j) req = req || at.pos[meas_q[j]] == lp.spos[k];
               if (!req) st->meas_hlred |= 1u << k;
             }
+            // an unrequested lane bit costs every stored slot a shuffle butterfly and halves the
+            // lanes that add: measured on QAOA_32 (one such bit) the epilogue added 15 ms to a
+            // 23 ms pass while the separate readout reads the 64 GiB state in 9.4 ms; with every
+            // lane bit requested (QFT_28, qubits 0..9) it adds 0.11 ms against a 0.66 ms readout.
+            // So mode 2 is fused only without the butterfly (QGPU_HACC=2 forces it)
+            const char* he = std::getenv("QGPU_HACC");
+            if (st->meas_hlred != 0u && !(he && he[0] == '2')) last = -1;
           } else {
             last = -1;
           }

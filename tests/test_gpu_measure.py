@@ -10,6 +10,18 @@ from workloads import circuits as wc
 pytestmark = pytest.mark.gpu
 
 
+@pytest.fixture(autouse=True, params=["default", "force_mode2"])
+def hacc_mode(request, monkeypatch):
+    """Every test runs with the library's choice (mode 2 is fused only when no lane bit needs the
+    shuffle butterfly; otherwise the separate readout) and with QGPU_HACC=2 (the mode-2 epilogue
+    with the butterfly forced), so both the fused kernels and the fallback stay covered."""
+    if request.param == "force_mode2":
+        monkeypatch.setenv("QGPU_HACC", "2")
+    else:
+        monkeypatch.delenv("QGPU_HACC", raising=False)
+    return request.param
+
+
 @pytest.fixture(scope="module")
 def q():
     import torch
