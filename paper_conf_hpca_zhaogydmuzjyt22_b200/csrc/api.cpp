@@ -124,6 +124,8 @@ uint64_t plan_key(const qgpu_state* st, const qgpu_circuit* c) {
   if (const char* ev = std::getenv("QGPU_LRELAX")) mix(uint64_t(std::atoi(ev) + 1) << 52);
   if (const char* ev = std::getenv("QGPU_GLOBAL_FIRST")) mix(uint64_t(std::atoi(ev) + 1) << 20);
   if (const char* ev = std::getenv("QGPU_AUTO_LANES")) mix(uint64_t(std::atoi(ev) + 1) << 28);
+  if (const char* ev = std::getenv("QGPU_PASS_SCHED")) mix(uint64_t(std::atoi(ev) + 1) << 16);
+  if (const char* ev = std::getenv("QGPU_SCHED_ROLLOUT")) mix(uint64_t(std::atoi(ev) + 1) << 12);
   if (const char* ev = std::getenv("QGPU_GLOBAL_MIN_LOCAL")) mix(uint64_t(std::atoi(ev) + 1) << 24);
   return h;
 }
@@ -193,6 +195,16 @@ void plan_env(PlanOptions* o) {
     o->auto_lanes = false;
   }
   if (const char* ev = std::getenv("QGPU_AUTO_LANES")) o->auto_lanes = o->auto_lanes && std::atoi(ev) != 0;
+  if (const char* ev = std::getenv("QGPU_SCHED_ROLLOUT")) o->sched_rollout = std::atoi(ev) != 0;
+  // pass-aware execution order: 0 off, 1 tried by plan_circuit_auto (default), 2 always (no auto)
+  if (const char* ev = std::getenv("QGPU_PASS_SCHED")) {
+    const int v = std::atoi(ev);
+    o->auto_sched = v == 1;
+    if (v == 2) {
+      o->pass_sched = true;
+      o->auto_lanes = false;
+    }
+  }
   if (const char* ev = std::getenv("QGPU_REGBITS")) o->reg_bits = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_MAX_UOPS")) o->max_u_ops = std::atoi(ev);
   if (const char* ev = std::getenv("QGPU_LOOKAHEAD")) o->lookahead = std::atoi(ev);

@@ -169,6 +169,11 @@ struct PlanOptions {
   int reg_bits = 4;     // register bits per thread (2^reg_bits amplitudes in registers)
   bool peephole = true; // fuse CX . D . CX into a diagonal (exact)
   int lookahead = 192;  // fusion lookahead window (gates); 0: passes are runs of `order`
+  // pass-aware execution order (pass_schedule in sched.cpp): the gates are re-ordered, within
+  // the commutation DAG, pass by pass -- each pass takes the closure of the ready gates over a
+  // tile set chosen greedily by gain; single resident state, involvement rule 0, no relabels
+  bool pass_sched = false;
+  bool sched_rollout = true;  // near the full live size, choose each pass's kmax by a rollout
   bool prune = true;
   int rule = 0;         // involvement rule (see involving())
   // skip the halves of positions that a first touch left zero (placed by a diagonal gate or as
@@ -183,6 +188,8 @@ struct PlanOptions {
   // plan_circuit_auto: try the lane-bit policies (l_min, l_relax) = (5, 0) (5, 4) (5, 3) (4, 0)
   // (3, 0) and keep the plan with the lowest modelled time
   bool auto_lanes = true;
+  // plan_circuit_auto also tries pass_sched = true (QGPU_PASS_SCHED=0 turns it off)
+  bool auto_sched = true;
 };
 
 // Cut `gates` into passes, updating `map` (involvement, placement) exactly as the execution

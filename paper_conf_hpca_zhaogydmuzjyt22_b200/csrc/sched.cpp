@@ -18,6 +18,7 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <functional>
 #include <limits>
 
 #include "qgpu_internal.h"
@@ -957,6 +958,311 @@ struct Builder {
   }
 };
 
+// ------------------------------------------------------------------------------------------
+// Pass-aware execution order (opt.pass_sched; DESIGN.md §4 "Pass scheduling").
+//
+// Alg.3 fixes when each qubit becomes involved; the Builder above cuts that order
+// into consecutive runs (plus a lookahead over gates sharing no qubit), so a pass closes as soon
+// as the next gate in order needs a 13th tile position, although many later gates could still
+// run on the tile positions at hand. Here the execution order is chosen pass by pass over the
+// commutation DAG of the units (the gates after the CX.D.CX peephole). Two units commute when
+// neither's non-diagonal targets touch the other's qubits (diagonal gates commute with each other
+// and with controls), so every topological order of the DAG yields the same state up to rounding.
+// A pass, for a candidate bound kmax on the live size, is the closure of the ready units whose
+// non-diagonal targets lie in an allowed qubit set A, under exactly the Builder's budget
+// (fits()); A starts as the lane qubits and grows greedily by the number of units each added
+// qubit unlocks. Of the candidate kmax the one with the most units per byte the pass moves
+// (16 * (2^k_in + 2^k_out) plus a launch gap) is kept. Units are taken in Alg.3 order among the ready ones, so the
+// involvement still follows Alg.3's priorities within each pass.
+//
+// units[u] = the gate of the u-th unit, in Alg.3 order. Returns false (no plan) when the DAG
+// model does not apply (relabels move qubits between positions).
+bool pass_schedule(const std::vector<const Gate*>& units, const QubitMap& map0, const PlanOptions& opt,
+                   std::vector<int>* seq, std::vector<char>* brk) {
+  const int N = int(units.size());
+  const int Bt = opt.fuse_bits;
+  std::vector<uint64_t> T(units.size()), Q(units.size());
+  std::vector<int> ops(units.size());
+  for (int u = 0; u < N; ++u) {
+    const Gate& g = *units[size_t(u)];
+    if (g.relabel) return false;
+    Q[size_t(u)] = g.qmask();
+    T[size_t(u)] = g.diag ? 0 : g.tmask();
+    ops[size_t(u)] = g.diag ? (1 << g.nt) : 1;
+  }
+  // DAG: u after the last unit with a non-diagonal target on each of its qubits, and, on its own
+  // non-diagonal targets, after every unit touching them since (edges may repeat: indeg counts
+  // them, and each is released once)
+  std::vector<std::vector<int>> succ(units.size());
+  std::vector<int> indeg(units.size(), 0);
+  {
+    std::vector<int> lastT(kMaxQubits, -1);
+    std::vector<std::vector<int>> qonly(kMaxQubits);
+    for (int u = 0; u < N; ++u) {
+      for (uint64_t r = Q[size_t(u)]; r; r &= r - 1) {
+        const int q = std::countr_zero(r);
+        auto edge = [&](int v) {
+          succ[size_t(v)].push_back(u);
+          ++indeg[size_t(u)];
+        };
+        if (lastT[size_t(q)] >= 0) edge(lastT[size_t(q)]);
+        if (T[size_t(u)] >> q & 1) {
+          for (int v : qonly[size_t(q)]) edge(v);
+          qonly[size_t(q)].clear();
+          lastT[size_t(q)] = u;
+        } else {
+          qonly[size_t(q)].push_back(u);
+        }
+      }
+    }
+  }
+  std::vector<char> done(units.size(), 0);
+  QubitMap mp = map0;
+  // the open pass
+  uint64_t used = 0;
+  int n_est = 0, n_u = 0, kin = mp.kl;
+  std::vector<int> exec, declog, blocked, heap;
+  struct Ck {
+    QubitMap mp;
+    uint64_t used;
+    int n_est, n_u;
+    size_t nexec, ndec, nblk;
+  };
+  auto ckpt = [&]() { return Ck{mp, used, n_est, n_u, exec.size(), declog.size(), blocked.size()}; };
+  auto undo = [&](const Ck& c) {
+    while (declog.size() > c.ndec) {
+      ++indeg[size_t(declog.back())];
+      declog.pop_back();
+    }
+    while (exec.size() > c.nexec) {
+      done[size_t(exec.back())] = 0;
+      exec.pop_back();
+    }
+    blocked.resize(c.nblk);
+    mp = c.mp;
+    used = c.used;
+    n_est = c.n_est;
+    n_u = c.n_u;
+  };
+  auto fits = [&](uint64_t need, int o, int kcur) {
+    if (n_est + o > opt.max_ops) return false;
+    if (need && n_u + 1 > opt.max_u_ops) return false;
+    auto fits_l = [&](int lmin) {
+      const int lm = std::min(lmin, std::max(kcur, 0));
+      const uint64_t S = used | need | ((lm > 0) ? ((1ull << lm) - 1) : 0);
+      return std::popcount(S) <= Bt;
+    };
+    return fits_l(opt.l_min) || (opt.l_relax > 0 && fits_l(opt.l_relax));
+  };
+  // closure of the units in `heap` (and those they release) over A within kmax
+  auto run = [&](uint64_t A, int kmax) {
+    std::make_heap(heap.begin(), heap.end(), std::greater<int>());
+    while (!heap.empty()) {
+      std::pop_heap(heap.begin(), heap.end(), std::greater<int>());
+      const int u = heap.back();
+      heap.pop_back();
+      if (done[size_t(u)]) continue;
+      const uint64_t fresh = Q[size_t(u)] & ~mp.involvement;
+      bool ok = (T[size_t(u)] & ~A) == 0 && mp.kl + std::popcount(fresh) <= kmax;
+      uint64_t need = 0;
+      if (ok) {
+        for (uint64_t r = T[size_t(u)]; r; r &= r - 1) {
+          const int q = std::countr_zero(r);
+          const int p = mp.pos[q] >= 0 ? mp.pos[q] : mp.kl + std::popcount(fresh & ((1ull << q) - 1));
+          need |= 1ull << p;
+        }
+        ok = exec.size() == 0 || fits(need, ops[size_t(u)], mp.kl);  // (a pass's first gate always opens it)
+      }
+      if (!ok) {
+        blocked.push_back(u);
+        continue;
+      }
+      mp.touch(Q[size_t(u)]);
+      used |= need;
+      n_est += ops[size_t(u)];
+      if (need) ++n_u;
+      done[size_t(u)] = 1;
+      exec.push_back(u);
+      for (int s : succ[size_t(u)]) {
+        declog.push_back(s);
+        if (--indeg[size_t(s)] == 0) {
+          heap.push_back(s);
+          std::push_heap(heap.begin(), heap.end(), std::greater<int>());
+        }
+      }
+    }
+  };
+  // drop executed and repeated entries of `blocked` (a unit re-blocked after a resume is listed again)
+  std::vector<int> stamp(units.size(), -1);
+  int stamp_id = 0;
+  auto compact = [&]() {
+    ++stamp_id;
+    size_t w = 0;
+    for (int u : blocked)
+      if (!done[size_t(u)] && stamp[size_t(u)] != stamp_id) {
+        stamp[size_t(u)] = stamp_id;
+        blocked[w++] = u;
+      }
+    blocked.resize(w);
+  };
+  const int L = std::max(opt.l_min, 0);
+  // build one candidate pass from the (empty) open pass; `adds` receives the qubits added to A
+  // in order, so that replaying them reproduces the pass exactly
+  auto build = [&](int kmax, const std::vector<int>& ready, std::vector<int>* adds, bool replay) {
+    uint64_t A = 0;
+    for (int p = 0; p < std::min(L, mp.kl); ++p) A |= 1ull << mp.lq[p];
+    heap = ready;
+    run(A, kmax);
+    if (replay) {
+      for (int q : *adds) {
+        A |= 1ull << q;
+        compact();
+        heap.clear();
+        for (int u : blocked)
+          if (!done[size_t(u)] && (T[size_t(u)] >> q & 1)) heap.push_back(u);
+        run(A, kmax);
+      }
+      return;
+    }
+    std::vector<std::vector<int>> byq(kMaxQubits);
+    for (int round = 0; round < kMaxQubits; ++round) {
+      compact();
+      for (auto& v : byq) v.clear();
+      for (int u : blocked)
+        if (!done[size_t(u)])
+          for (uint64_t r = T[size_t(u)] & ~A; r; r &= r - 1) byq[size_t(std::countr_zero(r))].push_back(u);
+      int bq = -1;
+      size_t bgain = 0, bcnt = 0;
+      for (int q = 0; q < kMaxQubits; ++q) {
+        if (byq[size_t(q)].empty()) continue;
+        const Ck c = ckpt();
+        heap = byq[size_t(q)];
+        run(A | (1ull << q), kmax);
+        const size_t gain = exec.size() - c.nexec;
+        undo(c);
+        if (bq < 0 || gain > bgain || (gain == bgain && byq[size_t(q)].size() > bcnt)) {
+          bq = q;
+          bgain = gain;
+          bcnt = byq[size_t(q)].size();
+        }
+      }
+      if (bq < 0) break;
+      A |= 1ull << bq;
+      adds->push_back(bq);
+      heap = byq[size_t(bq)];
+      run(A, kmax);
+    }
+  };
+  auto pass_cost = [&](int kin_, int kk) {
+    // bytes moved plus a launch gap (~4 us at the copy peak ~ 26 MB) per pass
+    return 16.0 * (std::ldexp(1.0, kin_) + std::ldexp(1.0, kk)) + 2.6e7;
+  };
+  size_t lo = 0;  // lowest unit not done
+  auto all_done = [&]() {
+    while (lo < size_t(N) && done[lo]) ++lo;
+    return lo >= size_t(N);
+  };
+  // plan and commit one pass; with rollout, every candidate kmax is scored by the cost of the
+  // whole rest of the plan (this pass, then greedy passes to the end) instead of units per byte
+  int depth = 0;  // nested plan_pass calls (rollouts) record nothing
+  std::function<bool(bool, double*)> plan_pass = [&](bool rollout, double* cost_out) {
+    struct Depth {
+      int& d;
+      explicit Depth(int& x) : d(++x) {}
+      ~Depth() { --d; }
+    } guard(depth);
+    std::vector<int> ready;
+    for (size_t u = lo; u < size_t(N); ++u)
+      if (!done[u] && indeg[u] == 0) ready.push_back(int(u));
+    kin = mp.kl;
+    const Ck c0 = ckpt();
+    double best = -1.0, best_total = 0.0;
+    int bk = -1;
+    std::vector<int> badds, adds;
+    for (int kmax = std::max(kin, 1); kmax <= mp.m; ++kmax) {
+      adds.clear();
+      build(kmax, ready, &adds, false);
+      const size_t cnt = exec.size();
+      const int kk = mp.kl;
+      undo(c0);
+      if (cnt == 0) continue;
+      const double cost = pass_cost(kin, kk);
+      const double score = double(cnt) / cost;
+      if (rollout) {
+        // the rest of the plan from this candidate, then restore everything
+        const std::vector<char> done0 = done;
+        const std::vector<int> indeg0 = indeg;
+        const QubitMap mp0 = mp;
+        const size_t lo0 = lo;
+        build(kmax, ready, &adds, true);
+        exec.clear();
+        declog.clear();
+        blocked.clear();
+        used = 0;
+        n_est = 0;
+        n_u = 0;
+        // up to kHorizon greedy passes, the rest estimated at their cost per unit
+        constexpr int kHorizon = 6;
+        double total = cost, hcost = 0.0;
+        size_t hunits = 0;
+        for (int h = 0; h < kHorizon && !all_done(); ++h) {
+          double c = 0.0;
+          const size_t before = size_t(std::count(done.begin(), done.end(), char(1)));
+          if (!plan_pass(false, &c)) break;
+          hcost += c;
+          hunits += size_t(std::count(done.begin(), done.end(), char(1))) - before;
+        }
+        total += hcost;
+        if (!all_done() && hunits > 0)
+          total += hcost / double(hunits) * double(std::count(done.begin(), done.end(), char(0)));
+        done = done0;
+        indeg = indeg0;
+        mp = mp0;
+        lo = lo0;
+        kin = mp.kl;
+        if (bk < 0 || total < best_total) {
+          best_total = total;
+          bk = kmax;
+          badds = adds;
+        }
+      } else if (score > best) {
+        best = score;
+        bk = kmax;
+        badds = adds;
+      }
+      if (kk < kmax) break;  // the window is not the limit: a larger kmax plans the same pass
+      // a pass that moves 4x the bytes of the best one so far would need 4x its units
+      if (!rollout && cost > 4.0 * double(cnt) / best && 16.0 * std::ldexp(1.0, kk) > 1e8) break;
+    }
+    if (bk < 0) return false;
+    build(bk, ready, &badds, true);
+    if (cost_out) *cost_out = pass_cost(kin, mp.kl);
+    if (depth == 1) {
+      for (size_t i = 0; i < exec.size(); ++i) {
+        seq->push_back(exec[i]);
+        brk->push_back(i == 0);
+      }
+    }
+    // commit: the pass's state stays, its logs are dropped
+    exec.clear();
+    declog.clear();
+    blocked.clear();
+    used = 0;
+    n_est = 0;
+    n_u = 0;
+    return true;
+  };
+  seq->clear();
+  brk->clear();
+  while (!all_done()) {
+    // rollout only where passes are expensive (live size within 4 qubits of the full state)
+    // (at the full live size there is one candidate, nothing to choose)
+    const bool rollout = opt.sched_rollout && mp.kl >= mp.m - 4 && mp.kl < mp.m;
+    if (!plan_pass(rollout, nullptr)) return false;
+  }
+  return true;
+}
+
 }  // namespace
 
 void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order, QubitMap& map,
@@ -1267,6 +1573,28 @@ void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order,
   std::vector<std::array<int, 2>> part_of(size_t(G), {-1, -1});
   for (int k = 0; k < G; ++k)
     if (peephole && fused[k] >= 0) part_of[size_t(k)] = parts[size_t(fused[k])];
+  // pass-aware execution order (see pass_schedule): single resident state, the paper's
+  // involvement rule (the refined rule rewrites gates at emission), fused passes
+  if (opt.pass_sched && fuse && m == map.n && opt.rule == 0) {
+    std::vector<const Gate*> units;
+    for (int k : pend) units.push_back(&gate_at(k));
+    std::vector<int> seq;
+    std::vector<char> brk;
+    if (pass_schedule(units, map, opt, &seq, &brk)) {
+      for (size_t i = 0; i < seq.size(); ++i) {
+        if (brk[i]) B.close();
+        const int k = pend[size_t(seq[i])];
+        emit(k);
+        if (part_of[size_t(k)][0] >= 0) {
+          emit(part_of[size_t(k)][0]);
+          emit(part_of[size_t(k)][1]);
+        }
+      }
+      B.close();
+      B.materialise(xi);
+      return;
+    }
+  }
   const int W = fuse ? opt.lookahead : 0;
   size_t head = 0;
   std::vector<char> done(size_t(G), 0);
@@ -1351,25 +1679,33 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
   }
   // (l_min, l_relax, max_u_ops) candidates (smaller op budgets were modelled and measured no
   // better on QAOA / rqc and are not tried)
-  static const int cand[][3] = {{5, 0, 32}, {5, 4, 32}, {5, 3, 32}, {4, 0, 32}, {3, 0, 32}};
+  // (pass_sched candidates last: on ties the consecutive-run plan is kept)
+  static const int cand[][4] = {{5, 0, 32, 0}, {5, 4, 32, 0}, {5, 3, 32, 0}, {4, 0, 32, 0}, {3, 0, 32, 0},
+                                {5, 0, 32, 1}, {4, 0, 32, 1}, {3, 0, 32, 1}};
   double best = 0.0;
   bool have = false;
   QubitMap best_map;
   std::vector<Pass> best_passes;
   std::vector<uint64_t> best_inv;
+  const bool try_sched = opt.auto_sched && map.m == map.n && opt.rule == 0;
+  bool first_only = false;
   for (const auto& c : cand) {
-    if (have && !best_passes.empty()) {
+    if (c[3] && !try_sched) continue;
+    if (!c[3] && first_only) continue;
+    if (!c[3] && have && !best_passes.empty()) {
       // other lane policies can only merge passes that run at the full live size; with at most
       // one such pass in the first plan (e.g. QFT: every pass expands) the first plan is kept
       int kmax = 0, steady = 0;
       for (const Pass& p : best_passes) kmax = std::max(kmax, p.k_out);
       for (const Pass& p : best_passes) steady += (p.kind == PK_TILE && p.k_in == kmax && p.k_out == kmax);
-      if (steady <= 1) break;
+      if (steady <= 1) first_only = true;
+      if (first_only) continue;
     }
     PlanOptions o = opt;
     o.l_min = std::min(opt.l_min, c[0]);
     o.l_relax = c[1];
     o.max_u_ops = std::min(opt.max_u_ops, c[2]);
+    o.pass_sched = c[3] != 0;
     QubitMap mp = map;
     std::vector<Pass> ps;
     std::vector<uint64_t> inv;
@@ -1377,8 +1713,8 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
     double t = 0.0;
     for (const Pass& p : ps) t += pass_cost_model(p, mp.m);
     if (std::getenv("QGPU_DEBUG_AUTO"))
-      std::fprintf(stderr, "plan_circuit_auto: l_min %d l_relax %d max_u_ops %d: %zu passes, modelled %.3f ms\n", o.l_min,
-                   o.l_relax, o.max_u_ops, ps.size(), t * 1e3);
+      std::fprintf(stderr, "plan_circuit_auto: l_min %d l_relax %d max_u_ops %d sched %d: %zu passes, modelled %.3f ms\n",
+                   o.l_min, o.l_relax, o.max_u_ops, int(o.pass_sched), ps.size(), t * 1e3);
     if (!have || t < best * 0.995) {  // ties keep the earlier (longer-run) policy
       have = true;
       best = t;

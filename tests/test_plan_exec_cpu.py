@@ -61,7 +61,14 @@ CIRCS = {
 @pytest.mark.parametrize("fuse", [0, 7, 9])
 @pytest.mark.parametrize("mode", [0, 1, 2])
 @pytest.mark.parametrize("rule", [0, 1])
-def test_physical_plan_executes_to_the_oracle(q, name, fuse, mode, rule):
+@pytest.mark.parametrize("sched", ["1", "0", "2"])
+def test_physical_plan_executes_to_the_oracle(q, name, fuse, mode, rule, sched, monkeypatch):
+    """sched: QGPU_PASS_SCHED -- 1 the default (plan_circuit_auto picks), 0 consecutive runs of
+    the execution order only, 2 the pass-aware execution order always. 0 and 2 only where they
+    differ from the default: fused passes under the paper's involvement rule."""
+    if sched != "1" and (rule == 1 or fuse == 0 or (sched == "0" and fuse != 9)):
+        pytest.skip("same plan as the default")
+    monkeypatch.setenv("QGPU_PASS_SCHED", sched)
     for seed in (1, 2):
         c = CIRCS[name](seed)
         text = c.qasm()
