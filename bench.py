@@ -532,14 +532,23 @@ def measure_workload(q, torch, device, stream, args, text, n, steps, warmup, wor
     return st, c, times, stats, (clk.summary() if clk else None)
 
 
-def ncu_traffic(key: str):
-    """DRAM bytes per tile launch from the committed ncu launch list of this workload (or None)."""
+def ncu_traffic(key: str, roof: dict):
+    """DRAM bytes per tile launch from the committed ncu launch list of this workload (or None).
+    The entry is used only if it was taken on the same pass plan: its launch count and its
+    algorithmic bytes per launch (recorded from the profiled run's stats) must match this run's
+    (a plan change leaves a stale entry, reported as such instead of a wrong traffic figure)."""
     tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
     try:
         t = json.load(open(tp)).get(key)
-        return (t.get("dram_bytes_per_launch"), t.get("source")) if t else (None, None)
     except Exception:
         return None, None
+    if not t:
+        return None, None
+    algo = t.get("algo_bytes_per_launch")
+    if (algo is None or t.get("launches_per_circuit") != roof["launches_per_step"]
+            or abs(algo - roof["algo_bytes_per_launch"]) > 0.01 * roof["algo_bytes_per_launch"]):
+        return None, f"stale: {t.get('source')} was taken on another pass plan"
+    return t.get("dram_bytes_per_launch"), t.get("source")
 
 
 def tile_roofline(stats, ms, peak, peak_src):
@@ -632,7 +641,7 @@ def run_ours(args):
     kernel_ms = statistics.mean(x["kernel_ms"] for x in stats)
     algo_bytes = statistics.mean(x["algo_bytes"] for x in stats)
     unfused = statistics.mean(x["unfused_bytes"] for x in stats)
-    roof["traffic"], roof["traffic_source"] = ncu_traffic(f"{args.workload}_{n}")
+    roof["traffic"], roof["traffic_source"] = ncu_traffic(f"{args.workload}_{n}", roof)
     s0 = stats[-1]
     launches = s0["kernels_launched"]
 
@@ -775,10 +784,11 @@ def run_ours(args):
             ems = allreduce_max(statistics.mean(et), world, device)
             extras[key] = {"workload": edesc, "value": ems / 1e3, "unit": "s", "ms_per_step": ems,
                            "ms_per_step_best": min(et), "gates": len(ec.ops),
-                           "roofline": dict(tile_roofline(estats, ems, peak, peak_src),
-                                            **dict(zip(("traffic", "traffic_source"), ncu_traffic(f"{key}_{ec.n}")))),
+                           "roofline": tile_roofline(estats, ems, peak, peak_src),
                            "passes": estats[-1]["passes"],
                            "ops_before_full_involvement": estats[-1]["ops_before_full_involvement"]}
+            er = extras[key]["roofline"]
+            er["traffic"], er["traffic_source"] = ncu_traffic(f"{key}_{ec.n}", er)
             if key == "qft28" and args.gfc:
                 extras[key]["gfc_compression"] = gfc_measure(q, torch, est)
             est.close()

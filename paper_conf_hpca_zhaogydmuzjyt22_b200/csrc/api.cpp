@@ -620,7 +620,8 @@ qgpu_status qgpu_apply_gate(qgpu_state* st, const double* U, int nt, const int* 
 namespace {
 constexpr int kMeasMax = 12;
 // QGPU_HACC=0 turns the per-slot fused measurement off (A/B against the separate readout);
-// QGPU_HACC=2 fuses mode 2 even when lane bits need the butterfly
+// QGPU_HACC=2 fuses mode 2 even when lane bits need the run-time butterfly, 3: mode 2 never with
+// unrequested lane bits (the round-2 rule, A/B)
 bool hacc_enabled() {
   static const bool on = [] {
     const char* e = std::getenv("QGPU_HACC");
@@ -732,13 +733,16 @@ qgpu_status apply_circuit_impl(qgpu_state* st, const qgpu_circuit* c, int meas_m
               for (int j = 0; j < meas_m; ++j) req = req || at.pos[meas_q[j]] == lp.spos[k];
               if (!req) st->meas_hlred |= 1u << k;
             }
-            // an unrequested lane bit costs every stored slot a shuffle butterfly and halves the
-            // lanes that add: measured on QAOA_32 (one such bit) the epilogue added 15 ms to a
-            // 23 ms pass while the separate readout reads the 64 GiB state in 9.4 ms; with every
-            // lane bit requested (QFT_28, qubits 0..9) it adds 0.11 ms against a 0.66 ms readout.
-            // So mode 2 is fused only without the butterfly (QGPU_HACC=2 forces it)
+            // an unrequested lane bit cost the run-time epilogue a shuffle butterfly on every
+            // stored slot, with one lane in 2^u adding: measured on QAOA_32 (one such bit) it
+            // added 15 ms to a 23 ms pass while the separate readout reads the 64 GiB state in
+            // 9.4 ms. The NVRTC variants compile the masks in and reduce-scatter instead
+            // (tile_driver, Body::kHistRS): mode 2 is fused with unrequested lane bits only when
+            // the last pass runs an NVRTC kernel (QGPU_HACC=2 forces it, QGPU_HACC=3 never)
             const char* he = std::getenv("QGPU_HACC");
-            if (st->meas_hlred != 0u && !(he && he[0] == '2')) last = -1;
+            const bool jit_last = (st->cfg.jit == 2 || (st->cfg.jit == 1 && lp.k_out >= jit_min_bits())) &&
+                                  jit_available(nullptr);
+            if (st->meas_hlred != 0u && !(he && he[0] == '2') && (!jit_last || (he && he[0] == '3'))) last = -1;
           } else {
             last = -1;
           }
@@ -1211,6 +1215,23 @@ qgpu_status qgpu_circuit_jit_check(const qgpu_circuit* c, int n, int reorder_mod
         return fail(QGPU_ERR_CUDA, "NVRTC: %s\n--- source ---\n%s", log.c_str(), tile_jit_source(p).c_str());
       }
       if (n_compiled) (*n_compiled)++;
+    }
+    // QGPU_JIT_CHECK_HIST=<key>: also the fused-measurement variants of the last tile pass (modes
+    // 0 and 1, mode 2 with run-time masks, and mode 2 with the compile-time masks `key`, see
+    // hist_rs_key: low 8 bits unrequested lane bits, bits 8..11 dead register bits)
+    if (const char* ev = std::getenv("QGPU_JIT_CHECK_HIST")) {
+      const uint32_t key = uint32_t(std::strtoul(ev, nullptr, 0));
+      for (int i = int(passes.size()) - 1; i >= 0; --i) {
+        const Pass& p = passes[size_t(i)];
+        if (p.kind != PK_TILE) continue;
+        for (int v = 0; v < 4; ++v) {
+          const std::string src = tile_jit_source(p, v < 3 ? v : 2, v < 3 ? ~0u : key);
+          if (!jit_cubin_cached(src, &cubin, &log, nullptr))
+            return fail(QGPU_ERR_CUDA, "NVRTC: %s\n--- source ---\n%s", log.c_str(), src.c_str());
+          if (n_compiled) (*n_compiled)++;
+        }
+        break;
+      }
     }
     return QGPU_OK;
   } catch (const std::exception& ex) {

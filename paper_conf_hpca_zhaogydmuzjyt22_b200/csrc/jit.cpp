@@ -187,7 +187,7 @@ bool jit_cubin_cached(const std::string& src, std::string* cubin, std::string* l
   return true;
 }
 
-std::string tile_jit_source(const Pass& p, int hist_mode) {
+std::string tile_jit_source(const Pass& p, int hist_mode, uint32_t hist_key) {
   const bool hist = hist_mode >= 0;
   const TileProgram& P = p.prog;
   const int NR = P.nr;
@@ -273,6 +273,13 @@ std::string tile_jit_source(const Pass& p, int hist_mode) {
   hdr << "  static constexpr bool kStatic = true;\n";
   hdr << "  static constexpr bool kHist = " << (hist ? "true" : "false") << ";\n";
   hdr << "  static constexpr int kHistMode = " << (hist ? hist_mode : 0) << ";\n";
+  {
+    const bool rs = hist && hist_mode == 2 && hist_key != ~0u;
+    hdr << "  static constexpr bool kHistRS = " << (rs ? "true" : "false") << ";\n";
+    hdr << "  static constexpr uint32_t kHlred = " << (rs ? (hist_key & 0xffu) : 0u) << "u;\n";
+    hdr << "  static constexpr uint32_t kDead = " << (rs ? (hist_key >> 8 & 0xfu) : 0u) << "u;\n";
+    hdr << "  static constexpr bool kHistGlob = " << (rs && (hist_key >> 12 & 1u) ? "true" : "false") << ";\n";
+  }
   {  // tile positions as runs of consecutive bits (tile index -> base address at compile time)
     std::vector<int> rp, rl;
     for (int i = 0; i < p.b;) {
@@ -296,7 +303,28 @@ std::string tile_jit_source(const Pass& p, int hist_mode) {
   hdr << "  static constexpr uint64_t kP0[kRegAmps] = " << ptab(R) << ";\n";
   hdr << "  static constexpr uint64_t kPF[kRegAmps] = " << ptab(RF) << ";\n";
   hdr << "  static constexpr uint32_t kJF[kRegAmps] = " << jtab(RF) << ";\n";
-  o << "  __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c, const TileArgs& a) const {\n";
+  // the last op that touches the tile buffer (remap, shared-memory op): after it the program
+  // runs from registers, so the driver's prefetch of the next tile into the single buffer of a
+  // two-CTA pass can be issued there (pf) instead of after the whole program
+  size_t last_smem = 0;
+  for (size_t i = 1; i < P.ops.size(); ++i)
+    if (P.ops[i].kind == OP_REMAP || P.ops[i].kind == OP_SMEM1 || P.ops[i].kind == OP_SMEM2) last_smem = i;
+  // only for programs with at most two remaps and >= 3 compute ops after the last one (A/B,
+  // profiles/r03: QAOA_32, one or two remaps mid-program, 49.0 -> 48.0 ms; rqc_30, many remaps,
+  // 111.2 -> 112.2 ms with it on every pass, also when gated on the ops after the last remap only)
+  {
+    int after = 0, nremap = 0;
+    for (size_t i = 1; i < P.ops.size(); ++i) nremap += P.ops[i].kind == OP_REMAP;
+    for (size_t i = last_smem + 1; i < P.ops.size() && last_smem > 0; ++i)
+      after += (P.ops[i].kind == OP_RUN || P.ops[i].kind == OP_U1R || P.ops[i].kind == OP_U1L ||
+                P.ops[i].kind == OP_U2R);
+    const char* ev = std::getenv("QGPU_EARLY_PF");  // 0: prefetch after the program, 2: always
+    const int mode = ev ? std::atoi(ev) : 1;
+    if (mode == 0 || (mode == 1 && (after < 3 || nremap > 2))) last_smem = 0;
+  }
+  hdr << "  static constexpr bool kEarlyPrefetch = " << (last_smem > 0 ? "true" : "false") << ";\n";
+  o << "  template <class PF>\n";
+  o << "  __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c, const TileArgs& a, PF&& pf) const {\n";
   o << "    const TileOp* ops = c.ops;\n";
   {
     const unsigned zm = zmask();
@@ -505,6 +533,7 @@ std::string tile_jit_source(const Pass& p, int hist_mode) {
     }
     if (wguard) o << "      }\n";
     o << "    }\n";
+    if (i == last_smem) o << "    pf();  // the tile buffer is free from here on\n";
   }
   o << "  }\n";
   }
@@ -625,6 +654,25 @@ int jit_prepare(const std::vector<const Pass*>& passes, double* compile_ms) {
   return loaded;
 }
 
+// Compile-time masks of the mode-2 measurement epilogue: the unrequested lane bits (a.hlred,
+// low 8 bits) and the register bits of the pass's final mapping whose positions are not
+// requested ("dead": their slots share buckets, bits 8..11), bit 12 = a.hglob
+uint32_t hist_rs_key(const Pass& p, const TileArgs& a) {
+  const TileProgram& P = p.prog;
+  int RF[4] = {0, 0, 0, 0};
+  for (const TileOp& op : P.ops)
+    if (op.kind == OP_REMAP)
+      for (int k = 0; k < 4; ++k) RF[k] = (op.a0 >> (4 * k)) & 15;
+  uint32_t dead = 0;
+  for (int k = 0; k < P.nr; ++k) {
+    const int pos = p.spos[RF[k]];
+    bool req = false;
+    for (int j = 0; j < a.hm; ++j) req = req || a.hpos[j] == pos;
+    if (!req) dead |= 1u << k;
+  }
+  return (a.hlred & 0xffu) | (dead << 8) | (a.hglob ? 1u << 12 : 0u);
+}
+
 // Compile (or fetch from the cache) and launch the specialised kernel of pass p.
 // Returns cudaErrorNotSupported when the JIT is unavailable (caller falls back).
 cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, size_t smem, int num_sms,
@@ -633,11 +681,13 @@ cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, s
   JitLib& L = lib();
   const bool hist = a.hist != nullptr;  // fused measurement: its own variant
   const int hmode = hist ? std::clamp(a.hacc, 0, 2) : -1;
+  const uint32_t hkey = hmode == 2 ? hist_rs_key(p, a) : ~0u;
   CUfunction fn = static_cast<CUfunction>(hist ? p.jit_fn_hist[hmode] : p.jit_fn);
+  if (hmode == 2 && p.jit_hist_key != hkey) fn = nullptr;  // another measured-qubit set
   std::string src;
   const std::string dev = device_tag();
   if (!fn) {
-    src = tile_jit_source(p, hmode);
+    src = tile_jit_source(p, hmode, hkey);
     std::lock_guard<std::mutex> g(L.mu);
     auto it = L.cache.find(dev + src);
     if (it != L.cache.end()) fn = it->second;
@@ -662,6 +712,7 @@ cudaError_t launch_tile_jit(cudaStream_t st, const Pass& p, const TileArgs& a, s
     L.cache.emplace(dev + src, fn);
   }
   (hist ? p.jit_fn_hist[hmode] : p.jit_fn) = fn;  // later launches skip source generation and lookup
+  if (hmode == 2) p.jit_hist_key = hkey;
   const unsigned threads = 32u << a.nw;
   int bps = 1;
   if (L.occupancy(&bps, fn, int(threads), smem) != CUDA_SUCCESS || bps < 1) bps = 1;

@@ -11,7 +11,10 @@
 namespace qgpu {
 
 // CUDA source of the specialised kernel for one tile pass (host-only, deterministic).
-std::string tile_jit_source(const Pass& p, int hist_mode = -1);  // >= 0: fused-measurement variant (TileArgs::hacc)
+// hist_mode >= 0: fused-measurement variant (TileArgs::hacc); mode 2 with hist_key != ~0u: the
+// compile-time reduce-scatter epilogue for unrequested lane bits (hist_key & 0xff) and dead
+// register bits (hist_key >> 8), see hist_rs_key()
+std::string tile_jit_source(const Pass& p, int hist_mode = -1, uint32_t hist_key = ~0u);
 // Compile source to an sm_100a cubin with NVRTC (works without a GPU).
 bool jit_compile_cubin(const std::string& src, std::string* cubin, std::string* log);
 // Same, through the on-disk cubin cache ($QGPU_JIT_CACHE or <lib dir>/build/jitcache).

@@ -208,6 +208,9 @@ struct InterpBody {
   static constexpr bool kStatic = false;  // mappings read from the program at run time
   static constexpr bool kHist = H;        // H: the instantiation launched for a fused measurement
   static constexpr int kHistMode = -1;    // its epilogue too (a.hacc)
+  static constexpr bool kHistRS = false;  // mode 2 with run-time masks (a.hlred, a.hrb)
+  static constexpr uint32_t kHlred = 0u, kDead = 0u;
+  static constexpr bool kHistGlob = false;  // (a.hglob at run time)
   static constexpr int kNsrun = -1;       // tile positions read from the arguments
   static constexpr int kSrunPos[1] = {0};
   static constexpr int kSrunLen[1] = {0};
@@ -219,8 +222,10 @@ struct InterpBody {
   static constexpr uint64_t kPF[kRegAmps] = {};
   static constexpr uint32_t kJF[kRegAmps] = {};
   int nops;
+  static constexpr bool kEarlyPrefetch = false;  // the driver prefetches after the program
+  template <class PF>
   __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c,
-                                             const TileArgs&) const {
+                                             const TileArgs&, PF&&) const {
     for (int i = 1; i < nops; ++i) {
       const TileOp& op = c.ops[i];
       switch (op.kind) {
@@ -643,7 +648,7 @@ size_t tile_smem_bytes(const TileArgs& a) {
   const size_t nh = size_t(1) << (a.b - a.l);
   const size_t nwarps = size_t(1) << a.nw;
   return size_t(a.nbuf) * (size_t(1) << a.b) * 16 + ((nh + 1) & ~size_t(1)) * 8 + size_t(a.blob_bytes) +
-         2 * nwarps * size_t(a.npat) * 16 + size_t(a.nmbar) * 8 + 16 + (a.hist ? (size_t(8) << a.hm) * (a.hacc == 2 ? nwarps : 1) : 0);
+         2 * nwarps * size_t(a.npat) * 16 + size_t(a.nmbar) * 8 + 16 + (a.hist ? (size_t(8) << a.hm) * (a.hacc == 2 ? (a.hglob ? 0 : nwarps) : 1) : 0);
 }
 
 cudaError_t launch_pair(cudaStream_t st, const PairArgs& a, bool shfl) {

@@ -150,6 +150,7 @@ struct Pass {
   int act_copy = 0;             // activation by copy (a fresh qubit placed on a rank bit, §8e)
   mutable void* jit_fn = nullptr;  // specialised kernel, resolved at the first launch
   mutable void* jit_fn_hist[3] = {nullptr, nullptr, nullptr};  // fused-measurement variants, per mode
+  mutable uint32_t jit_hist_key = ~0u;  // the mode-2 variant's compile-time masks (hist_rs_key)
   uint64_t unfused_bytes = 0;   // bytes the pass's gates would move one gate per pass
   double fp64_per_amp = 0.0;    // FP64 pipe instructions per computed amplitude (roofline model,
                                 // fp64_model() in sched.cpp)

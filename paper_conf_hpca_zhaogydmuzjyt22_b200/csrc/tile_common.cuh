@@ -130,6 +130,9 @@ struct TileArgs {
   // differ -- add without atomics. 0: requested bits uniform across a warp's slots.
   int hacc;
   uint32_t hlred;
+  // mode 2 without private histograms: the lanes add straight to hist (global f64 reductions,
+  // no shared memory), used when per-warp histograms would cost the pass CTAs per SM
+  int hglob;
   // the pass's U matrices as a kernel parameter (constant bank), when they fit: the NVRTC bodies
   // read them at compile-time offsets (no shared-memory loads, no registers held across tiles)
   int umat_n;
@@ -832,7 +835,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   const int hmode = Body::kHistMode >= 0 ? Body::kHistMode : a.hacc;
   if constexpr (Body::kHist)
     if (a.hist) {
-      const int hn = (hmode == 2 ? (blockDim.x >> 5) : 1) << a.hm;
+      const int hn = (hmode == 2 ? (a.hglob ? 0 : (blockDim.x >> 5)) : 1) << a.hm;
       for (int i = threadIdx.x; i < hn; i += blockDim.x) hsm[i] = 0.0;
     }
 
@@ -995,8 +998,18 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     if (more && nbuf == 1 && !a.remaps) issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
     c.mpar = nexec & 1u;
     ++nexec;
-    body(v, mp, c, a);
-    if (more && nbuf == 1 && a.remaps) {
+    // nbuf == 1 with remaps: the next tile's loads go into the buffer once every thread is past
+    // the program's last remap / shared-memory op -- at that op when the body marks it
+    // (Body::kEarlyPrefetch, NVRTC bodies: the rest of the program overlaps the load latency),
+    // else after the program. Bulk stores read the buffer at the end: no early prefetch then.
+    const bool early = Body::kEarlyPrefetch && more && nbuf == 1 && a.remaps && !a.bstore;
+    body(v, mp, c, a, [&]() {
+      if (early) {
+        __syncthreads();
+        issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
+      }
+    });
+    if (more && nbuf == 1 && a.remaps && !early) {
       __syncthreads();
       issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
     }
@@ -1035,6 +1048,86 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
       uint32_t bt = hb0;
       for (int j = 0; j < a.hm; ++j) bt |= uint32_t(gbase >> a.hpos[j] & 1) << j;
       double* hw = hsm + (size_t(warp) << a.hm);
+      if constexpr (Body::kHistRS) {
+        // compile-time epilogue (NVRTC variants, masks Body::kHlred / kDead): slots that differ
+        // only in unrequested register bits are summed first; then, per unrequested lane bit,
+        // a reduce-scatter step (recursive halving): the two lanes exchange half of their live
+        // slot sums and each keeps the half selected by its lane bit, so s steps cost
+        // 2^NL (1 - 2^-s) shuffled doubles instead of a butterfly on every slot, and afterwards
+        // every lane adds its own 2^(NL - s) buckets (all distinct across the warp)
+        constexpr uint32_t kLB = ((1u << NR) - 1u) & ~Body::kDead;
+        constexpr int kNL = int(kLB & 1u) + int(kLB >> 1 & 1u) + int(kLB >> 2 & 1u) + int(kLB >> 3 & 1u);
+        double x[1 << NR];
+#pragma unroll
+        for (int r = 0; r < (1 << NR); ++r) x[r] = fma(v[r].x, v[r].x, v[r].y * v[r].y);
+#pragma unroll
+        for (int k = 0; k < NR; ++k)
+          if (Body::kDead >> k & 1u) {
+#pragma unroll
+            for (int r = 0; r < (1 << NR); ++r)
+              if (r >> k & 1) x[r & ~(1 << k)] += x[r];
+          }
+        // y[i]: the live slot whose live register bits are the bits of i (compile-time deposit)
+        double y[1 << NR];
+        uint32_t lbk[4] = {0u, 0u, 0u, 0u};  // bucket part of index bit t of y
+        {
+          int t = 0;
+#pragma unroll
+          for (int k = 0; k < NR; ++k)
+            if (kLB >> k & 1u) lbk[t++] = hrb[k];
+        }
+#pragma unroll
+        for (int i = 0; i < (1 << kNL); ++i) {
+          int r = 0, t = 0;
+#pragma unroll
+          for (int k = 0; k < NR; ++k)
+            if (kLB >> k & 1u) r |= ((i >> t++) & 1) << k;
+          y[i] = x[r];
+        }
+        uint32_t bb = bt;
+        uint32_t tail = 0u;  // unrequested lane bits left after the halving steps (butterfly)
+        int size_log = kNL;
+#pragma unroll
+        for (int k = 0; k < 5; ++k) {
+          if (!(Body::kHlred >> k & 1u)) continue;
+          if (size_log == 0) {
+            tail |= 1u << k;
+            y[0] += __shfl_xor_sync(0xffffffffu, y[0], 1 << k);
+            continue;
+          }
+          const bool h = (lane >> k) & 1;
+          const int half = 1 << (size_log - 1);
+#pragma unroll
+          for (int i = 0; i < (1 << kNL) / 2; ++i) {
+            if (i >= half) continue;
+            const double lo = y[i], hi = y[i + half];
+            const double send = h ? lo : hi;
+            const double keep = h ? hi : lo;
+            y[i] = keep + __shfl_xor_sync(0xffffffffu, send, 1 << k);
+          }
+          if (h) bb |= lbk[size_log - 1];
+          --size_log;
+        }
+        if ((uint32_t(lane) & tail) == 0u) {
+          double old[1 << NR];
+          uint32_t bk[1 << NR];
+#pragma unroll
+          for (int i = 0; i < (1 << kNL); ++i) {
+            if (i >= (1 << size_log)) continue;
+            bk[i] = bb;
+#pragma unroll
+            for (int t = 0; t < 4; ++t)
+              if (t < size_log && (i >> t & 1)) bk[i] |= lbk[t];
+            if constexpr (!Body::kHistGlob) old[i] = hw[bk[i]];
+          }
+#pragma unroll
+          for (int i = 0; i < (1 << kNL); ++i)
+            if (i < (1 << size_log)) {
+              if constexpr (Body::kHistGlob) atomicAdd(a.hist + bk[i], y[i]);  // RED.ADD.F64, no return
+              else hw[bk[i]] = old[i] + y[i];
+            }
+        }
+      } else {
       const bool writer = (uint32_t(lane) & a.hlred) == 0u;
       double x[1 << NR];
 #pragma unroll
@@ -1065,11 +1158,15 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
 #pragma unroll
           for (int k = 0; k < NR; ++k)
             if (r >> k & 1) bk[r] |= hrb[k];
-          old[r] = ((uint32_t(r) & dead) == 0u) ? hw[bk[r]] : 0.0;
+          old[r] = ((uint32_t(r) & dead) == 0u && !a.hglob) ? hw[bk[r]] : 0.0;
         }
 #pragma unroll
         for (int r = 0; r < (1 << NR); ++r)
-          if ((uint32_t(r) & dead) == 0u) hw[bk[r]] = old[r] + x[r];
+          if ((uint32_t(r) & dead) == 0u) {
+            if (a.hglob) atomicAdd(a.hist + bk[r], x[r]);
+            else hw[bk[r]] = old[r] + x[r];
+          }
+      }
       }
     }
     if constexpr (Body::kHist) if (a.hist && c.own && hmode == 0) {  // fused measurement: final amplitudes in registers
@@ -1171,8 +1268,8 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
         }
       }
       __syncthreads();
-      const int hw = hmode == 2 ? int(blockDim.x >> 5) : 1;
-      for (int i = threadIdx.x; i < (1 << a.hm); i += blockDim.x) {
+      const int hw = hmode == 2 ? (a.hglob ? 0 : int(blockDim.x >> 5)) : 1;
+      for (int i = threadIdx.x; i < (hw ? (1 << a.hm) : 0); i += blockDim.x) {
         double t = 0.0;
         for (int w = 0; w < hw; ++w) t += hsm[(size_t(w) << a.hm) + i];
         if (t != 0.0) atomicAdd(a.hist + i, t);

@@ -64,6 +64,7 @@ def main():
     ap.add_argument("--tag", default="r01")
     ap.add_argument("--workload", default="qft28")
     ap.add_argument("--n", type=int, default=28)
+    ap.add_argument("--stats", help="profile_step.py --stats-out of the profiled run (plan fingerprint)")
     args = ap.parse_args()
     out = os.path.join(ROOT, "profiles", args.tag)
     os.makedirs(out, exist_ok=True)
@@ -86,11 +87,28 @@ def main():
                 tile.append((ms, rd + wr))
         open(os.path.join(out, f"{args.workload}_launches.csv"), "w").write("\n".join(lines) + "\n")
         if tile:
-            tr = {"workload": args.workload, "n": args.n, "source": f"profiles/{args.tag}/{args.workload}_launches.csv",
+            # keyed "<workload>_<n>" entries read by bench.py (roofline.traffic), with the plan's
+            # fingerprint (tile launches and algorithmic bytes per launch of the profiled circuit)
+            tp = os.path.join(ROOT, "profiles", "ncu_traffic.json")
+            allt = json.load(open(tp)) if os.path.exists(tp) else {}
+            tr = {"workload": args.workload, "n": args.n,
                   "dram_bytes_per_launch": sum(t[1] for t in tile) / len(tile),
-                  "tile_launches": len(tile), "tile_share_of_step": sum(t[0] for t in tile) / tot if tot else None,
-                  "note": "ncu --clock-control none, cold-cache serialised launches; shares, not absolutes"}
-            json.dump(tr, open(os.path.join(ROOT, "profiles", "ncu_traffic.json"), "w"), indent=1)
+                  "launches_per_circuit": len(tile), "dram_bytes_per_circuit": sum(t[1] for t in tile),
+                  "tile_share_of_step": sum(t[0] for t in tile) / tot if tot else None,
+                  "source": f"profiles/{args.tag}/{args.workload}_launches.csv (ncu --metrics gpu__time_duration.sum,"
+                            "dram__bytes_read.sum,dram__bytes_write.sum --clock-control none, "
+                            "scripts/profile_step.py: second circuit)"}
+            if args.stats:
+                st = json.load(open(args.stats))["stats"]
+                if st["tile_kernel_launches"]:  # (filled when the profiled run had timing on)
+                    nl, ab = st["tile_kernel_launches"], st["tile_algo_bytes"]
+                else:  # every launched kernel a tile pass (QAOA / QFT): the totals are the tile ones
+                    assert st["kernels_launched"] == st["jit_launches"] == len(tile), st
+                    nl, ab = st["kernels_launched"], st["algo_bytes"]
+                tr["algo_bytes_per_launch"] = ab / nl
+                tr["launches_per_circuit_stats"] = nl
+            allt[f"{args.workload}_{args.n}"] = tr
+            json.dump(allt, open(tp, "w"), indent=1)
         print("\n".join(lines))
     if args.full:
         txt = subprocess.run(["ncu", "-i", args.full, "--page", "raw", "--csv"], capture_output=True, text=True).stdout

@@ -15,6 +15,7 @@ ap.add_argument("--n", type=int, default=None)
 ap.add_argument("--fuse-bits", type=int, default=12)
 ap.add_argument("--steps", type=int, default=1)
 ap.add_argument("--single", type=int, default=None, help="instead: one 1-qubit gate at this target on a full state")
+ap.add_argument("--stats-out", default=None, help="write the last circuit's qgpu_stats as JSON here")
 args = ap.parse_args()
 
 import numpy as np  # noqa: E402
@@ -34,8 +35,14 @@ if args.single is not None:
 circ, desc = bench.workload(args.workload, args.n)
 c = q.Circuit(circ.qasm())
 s = q.State(circ.n, fuse_bits=args.fuse_bits)
-for _ in range(1 + args.steps):
+for i in range(1 + args.steps):
     s.reset()
+    if i == args.steps:
+        s.reset_stats()
     s.apply_circuit(c)
 s.synchronize()
-print(desc, s.stats())
+st = s.stats()
+print(desc, st)
+if args.stats_out:
+    import json
+    json.dump({"workload": args.workload, "n": circ.n, "desc": desc, "stats": st}, open(args.stats_out, "w"), indent=1)

@@ -10,15 +10,23 @@ from workloads import circuits as wc
 pytestmark = pytest.mark.gpu
 
 
-@pytest.fixture(autouse=True, params=["default", "force_mode2"])
+@pytest.fixture(autouse=True, params=["default", "force_mode2", "global_hist", "round2_rule"])
 def hacc_mode(request, monkeypatch):
-    """Every test runs with the library's choice (mode 2 is fused only when no lane bit needs the
-    shuffle butterfly; otherwise the separate readout) and with QGPU_HACC=2 (the mode-2 epilogue
-    with the butterfly forced), so both the fused kernels and the fallback stay covered."""
+    """Every test runs with the library's choice (mode 2 with unrequested lane bits is fused when
+    the last pass is an NVRTC kernel -- compile-time reduce-scatter epilogue -- else the separate
+    readout), with QGPU_HACC=2 (mode 2 forced, the interpreted kernel's run-time butterfly too),
+    with QGPU_HGLOB=2 (mode 2 adds straight to the global histogram instead of per-warp shared-
+    memory histograms) and with QGPU_HACC=3 (never fused with unrequested lane bits), so the fused
+    kernels and the fallback stay covered."""
+    for k in ("QGPU_HACC", "QGPU_HGLOB"):
+        monkeypatch.delenv(k, raising=False)
     if request.param == "force_mode2":
         monkeypatch.setenv("QGPU_HACC", "2")
-    else:
-        monkeypatch.delenv("QGPU_HACC", raising=False)
+    elif request.param == "global_hist":
+        monkeypatch.setenv("QGPU_HACC", "2")
+        monkeypatch.setenv("QGPU_HGLOB", "2")
+    elif request.param == "round2_rule":
+        monkeypatch.setenv("QGPU_HACC", "3")
     return request.param
 
 
@@ -125,3 +133,29 @@ def test_fused_measurement_lane_register_bits_read_no_state(q, jit):
     assert k_fused < k_plain
     assert np.abs(p - p2).max() <= 1e-12
     assert np.abs(p - 2.0 ** -10).max() <= 1e-12  # QFT|0> is uniform: every marginal is 2^-10
+
+
+@pytest.mark.parametrize("name", ["qaoa", "rqc", "hlf"])
+def test_fused_measurement_unrequested_lane_bits_jit(q, name, hacc_mode):
+    """A requested set that leaves lane bits of the last pass unrequested (the qubit on position 0
+    plus qubits on high positions): with NVRTC kernels (jit=2) the library fuses it (compile-time
+    reduce-scatter epilogue; per-warp or global histogram) and launches no readout kernel (with
+    QGPU_HACC=3 it may take the separate readout). Both match the oracle."""
+    c = CIRCS[name]()
+    text = c.qasm()
+    plan = q.Circuit(text).plan_text(c.n)
+    fmap = [int(x) for x in plan.strip().splitlines()[-1].split()[1:]]
+    at = {p: lq for lq, p in enumerate(fmap) if p >= 0}
+    qubits = [at[0]] + [at[p] for p in sorted(at)[-3:]]
+    with q.State(c.n, fuse_bits=12, jit=2) as s:
+        p = s.apply_circuit_probabilities(q.Circuit(text), qubits)
+        k_fused = s.stats()["kernels_launched"]
+        s.reset()
+        s.apply_circuit(q.Circuit(text))
+        p2 = s.probabilities(qubits)
+        k_plain = s.stats()["kernels_launched"]
+    ref = osv.probabilities(osv.simulate(text), c.n, qubits)
+    assert np.abs(p - ref).max() <= 1e-12
+    assert np.abs(p - p2).max() <= 1e-12
+    if hacc_mode != "round2_rule":
+        assert k_fused < k_plain

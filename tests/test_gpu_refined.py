@@ -73,6 +73,8 @@ def test_refined_rule_shrinks_qft_on_zero(q, zskip, monkeypatch):
     paper's rule; with it (the default) the paper's rule already skips the same zero halves at the
     data level, so the bytes are at most equal while the involvement traces still differ."""
     monkeypatch.setenv("QGPU_ZSKIP", zskip)
+    # both rules under the consecutive-run planner (the pass-aware order applies to rule 0 only)
+    monkeypatch.setenv("QGPU_PASS_SCHED", "0")
     c = wc.qft(20)
     text = c.qasm()
     out = {}
