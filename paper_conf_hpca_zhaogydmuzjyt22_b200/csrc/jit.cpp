@@ -310,7 +310,7 @@ std::string tile_jit_source(const Pass& p, int hist_mode, uint32_t hist_key) {
   for (size_t i = 1; i < P.ops.size(); ++i)
     if (P.ops[i].kind == OP_REMAP || P.ops[i].kind == OP_SMEM1 || P.ops[i].kind == OP_SMEM2) last_smem = i;
   // only for programs with at most two remaps and >= 3 compute ops after the last one (A/B,
-  // profiles/r03: QAOA_32, one or two remaps mid-program, 49.0 -> 48.0 ms; rqc_30, many remaps,
+  // profiles/r02b: QAOA_32, one or two remaps mid-program, 49.0 -> 48.0 ms; rqc_30, many remaps,
   // 111.2 -> 112.2 ms with it on every pass, also when gated on the ops after the last remap only)
   {
     int after = 0, nremap = 0;
