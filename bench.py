@@ -572,6 +572,7 @@ def per_pass_binding(prof, hbm_gbs, fp64_fma_per_s):
     clock per SM) on top of the FP64 instructions: max(HBM, FP64 + MIO)."""
     rows = []
     tb = tm = tsm = 0.0
+    by = {"hbm": [0.0, 0.0], "fp64": [0.0, 0.0]}  # binding -> [bound ms, measured ms]
     clk = fp64_fma_per_s / (148 * 64.0) if fp64_fma_per_s else 1.9e9  # SM clock implied by the FP64 probe
     kinds = {0: "tile", 1: "pair", 2: "quad", 3: "diag", 5: "swap", 7: "zero"}
     for r in prof:
@@ -590,7 +591,11 @@ def per_pass_binding(prof, hbm_gbs, fp64_fma_per_s):
                      "frac_of_binding": round(bound / r["ms"], 3) if r["ms"] > 0 else None})
         tb += bound
         tm += r["ms"]
+        by[rows[-1]["binding"]][0] += bound
+        by[rows[-1]["binding"]][1] += r["ms"]
     return {"passes": rows, "bound_ms": tb, "measured_ms": tm, "frac": tb / tm if tm else None,
+            "by_binding": {k: {"bound_ms": v[0], "measured_ms": v[1], "frac": v[0] / v[1] if v[1] else None}
+                           for k, v in by.items()},
             "sm_bound": {"bound_ms": tsm, "frac": tsm / tm if tm else None,
                          "model": "per pass max(HBM, FP64 + MIO); MIO = shuffles of lane-bit ops and "
                                   "shared-memory remaps at one op per clock per SM"}}

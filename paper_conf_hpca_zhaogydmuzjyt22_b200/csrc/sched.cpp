@@ -20,6 +20,7 @@
 #include <cstring>
 #include <functional>
 #include <limits>
+#include <thread>
 
 #include "qgpu_internal.h"
 
@@ -1125,6 +1126,7 @@ bool pass_schedule(const std::vector<const Gate*>& units, const QubitMap& map0, 
       return;
     }
     std::vector<std::vector<int>> byq(kMaxQubits);
+    int zero_adds = 0;  // qubits admitted although they unlock nothing alone (2-qubit targets)
     for (int round = 0; round < kMaxQubits; ++round) {
       compact();
       for (auto& v : byq) v.clear();
@@ -1147,6 +1149,7 @@ bool pass_schedule(const std::vector<const Gate*>& units, const QubitMap& map0, 
         }
       }
       if (bq < 0) break;
+      if (bgain == 0 && ++zero_adds > 2) break;
       A |= 1ull << bq;
       adds->push_back(bq);
       heap = byq[size_t(bq)];
@@ -1689,38 +1692,56 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
   std::vector<uint64_t> best_inv;
   const bool try_sched = opt.auto_sched && map.m == map.n && opt.rule == 0;
   bool first_only = false;
-  for (const auto& c : cand) {
-    if (c[3] && !try_sched) continue;
-    if (!c[3] && first_only) continue;
-    if (!c[3] && have && !best_passes.empty()) {
-      // other lane policies can only merge passes that run at the full live size; with at most
-      // one such pass in the first plan (e.g. QFT: every pass expands) the first plan is kept
-      int kmax = 0, steady = 0;
-      for (const Pass& p : best_passes) kmax = std::max(kmax, p.k_out);
-      for (const Pass& p : best_passes) steady += (p.kind == PK_TILE && p.k_in == kmax && p.k_out == kmax);
-      if (steady <= 1) first_only = true;
-      if (first_only) continue;
-    }
+  struct Result {
+    double t = 0.0;
+    QubitMap mp;
+    std::vector<Pass> ps;
+    std::vector<uint64_t> inv;
+  };
+  auto run = [&](const int* c, Result* r) {
     PlanOptions o = opt;
     o.l_min = std::min(opt.l_min, c[0]);
     o.l_relax = c[1];
     o.max_u_ops = std::min(opt.max_u_ops, c[2]);
     o.pass_sched = c[3] != 0;
-    QubitMap mp = map;
-    std::vector<Pass> ps;
-    std::vector<uint64_t> inv;
-    plan_circuit(gates, order, mp, o, &ps, inv_after ? &inv : nullptr);
-    double t = 0.0;
-    for (const Pass& p : ps) t += pass_cost_model(p, mp.m);
+    r->mp = map;
+    plan_circuit(gates, order, r->mp, o, &r->ps, inv_after ? &r->inv : nullptr);
+    for (const Pass& p : r->ps) r->t += pass_cost_model(p, r->mp.m);
     if (std::getenv("QGPU_DEBUG_AUTO"))
       std::fprintf(stderr, "plan_circuit_auto: l_min %d l_relax %d max_u_ops %d sched %d: %zu passes, modelled %.3f ms\n",
-                   o.l_min, o.l_relax, o.max_u_ops, int(o.pass_sched), ps.size(), t * 1e3);
-    if (!have || t < best * 0.995) {  // ties keep the earlier (longer-run) policy
+                   o.l_min, o.l_relax, o.max_u_ops, int(o.pass_sched), r->ps.size(), r->t * 1e3);
+  };
+  // the first candidate decides which others can matter; those are planned concurrently (the
+  // planner has no shared mutable state) and compared in candidate order, so the choice does
+  // not depend on the threads
+  constexpr int kCand = int(sizeof(cand) / sizeof(cand[0]));
+  std::vector<Result> res(kCand);
+  run(cand[0], &res[0]);
+  {
+    int kmax = 0, steady = 0;
+    for (const Pass& p : res[0].ps) kmax = std::max(kmax, p.k_out);
+    for (const Pass& p : res[0].ps) steady += (p.kind == PK_TILE && p.k_in == kmax && p.k_out == kmax);
+    // other lane policies can only merge passes that run at the full live size; with at most
+    // one such pass in the first plan (e.g. QFT: every pass expands) they are not tried
+    first_only = steady <= 1;
+  }
+  std::vector<int> todo;
+  for (int ci = 1; ci < kCand; ++ci)
+    if (cand[ci][3] ? try_sched : !first_only) todo.push_back(ci);
+  {
+    std::vector<std::thread> th;
+    for (int ci : todo) th.emplace_back(run, cand[ci], &res[size_t(ci)]);
+    for (auto& t : th) t.join();
+  }
+  for (int ci = 0; ci < kCand; ++ci) {
+    if (ci > 0 && std::find(todo.begin(), todo.end(), ci) == todo.end()) continue;
+    Result& r = res[size_t(ci)];
+    if (!have || r.t < best * 0.995) {  // ties keep the earlier (longer-run) policy
       have = true;
-      best = t;
-      best_map = mp;
-      best_passes = std::move(ps);
-      best_inv = std::move(inv);
+      best = r.t;
+      best_map = r.mp;
+      best_passes = std::move(r.ps);
+      best_inv = std::move(r.inv);
     }
   }
   map = best_map;
