@@ -266,6 +266,7 @@ std::string tile_jit_source(const Pass& p, int hist_mode, uint32_t hist_key) {
     if (op.kind == OP_REMAP)
       for (int k = 0; k < 4; ++k) RF[k] = (op.a0 >> (4 * k)) & 15;
   std::ostringstream body, hdr;
+  bool fold_scalar = false;  // the tile-uniform scalar joins the first run (see below)
   {
     std::ostringstream& o = body;  // the program body is generated first (it fixes the barriers)
   hdr << "  static constexpr unsigned kZM0 = " << zm_start << "u;\n";
@@ -352,6 +353,20 @@ std::string tile_jit_source(const Pass& p, int hist_mode, uint32_t hist_key) {
     t << "((mp.base & " << op.tmask << "u) == " << op.tmatch << "u)";
     return t.str();
   };
+  // the tile-uniform scalar (phase terms on bits outside the tile and the deferred factors of
+  // the unit-diagonal matrix forms) commutes with the whole program: it joins the first run's
+  // t0 (every owned non-zero amplitude passes through it; by linearity the amplitudes that are
+  // still zero there carry it once they are formed) instead of a separate multiply of every
+  // amplitude at the end of the tile (QGPU_FOLD_SCALAR=0: A/B)
+  fold_scalar = !P.scalar.empty() && P.spat >= 0;
+  if (const char* ev = std::getenv("QGPU_FOLD_SCALAR"))
+    if (std::atoi(ev) == 0) fold_scalar = false;
+  {
+    bool has_run = false;
+    for (size_t i = 1; i < P.ops.size(); ++i) has_run = has_run || P.ops[i].kind == OP_RUN;
+    fold_scalar = fold_scalar && has_run;
+  }
+  bool scalar_pending = fold_scalar;
   for (size_t i = 1; i < P.ops.size(); ++i) {
     const TileOp& op = P.ops[i];
     const bool uni = op.omask != 0;       // tile-uniform condition present
@@ -403,6 +418,11 @@ std::string tile_jit_source(const Pass& p, int hist_mode, uint32_t hist_key) {
           if (ns[sl]) used |= 1 << sl;
           product(acc[sl], e, e + uint32_t(ns[sl]));
           e += uint32_t(ns[sl]);
+        }
+        if (scalar_pending) {
+          o << "      t0 = cmul(t0, c.C[" << P.spat << "]);  // the tile-uniform scalar\n";
+          used |= 1;
+          scalar_pending = false;
         }
         // general groups (compile-time r condition). Phase factors have modulus 1, so a factor
         // a on "r bit k clear" is a on all slots times conj(a) on "r bit k set" (two doubling
@@ -538,6 +558,7 @@ std::string tile_jit_source(const Pass& p, int hist_mode, uint32_t hist_key) {
   o << "  }\n";
   }
   o << "struct JitBody {\n" << hdr.str();
+  o << "  static constexpr bool kScalarFolded = " << (fold_scalar ? "true" : "false") << ";\n";
   o << "  static constexpr bool kGroupRemap = true;\n";
   o << "  __device__ static void init_mbar(uint64_t* mb) {\n";
   for (const auto& g : groups)

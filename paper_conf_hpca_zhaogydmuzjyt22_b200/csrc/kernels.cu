@@ -223,6 +223,7 @@ struct InterpBody {
   static constexpr uint32_t kJF[kRegAmps] = {};
   int nops;
   static constexpr bool kEarlyPrefetch = false;  // the driver prefetches after the program
+  static constexpr bool kScalarFolded = false;   // the driver applies the tile-uniform scalar
   template <class PF>
   __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c,
                                              const TileArgs&, PF&&) const {
