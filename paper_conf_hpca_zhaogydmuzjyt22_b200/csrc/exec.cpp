@@ -287,10 +287,6 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     if (const char* nb = std::getenv("QGPU_NBUF"))  // experiments: fewer tile buffers
       if (a.remaps && !two_cta) a.nbuf = std::max(1, std::min(a.nbuf, std::atoi(nb)));
     a.bstore = (a.nbuf == 3 && (bs == 2 || (bs == 1 && a.remaps))) ? 1 : 0;
-    {
-      const char* pf = std::getenv("QGPU_L2PF");  // 0: off (A/B)
-      a.l2pf = (a.nbuf == 1 && !(pf && pf[0] == '0')) ? 1 : 0;
-    }
     if (st->meas_pass == &p && !a.bstore) {  // fused measurement, if its histogram fits in smem
       TileArgs h = a;
       h.hist = st->d_meas;

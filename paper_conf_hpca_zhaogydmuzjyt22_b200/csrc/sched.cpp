@@ -1690,7 +1690,9 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
   QubitMap best_map;
   std::vector<Pass> best_passes;
   std::vector<uint64_t> best_inv;
-  const bool try_sched = opt.auto_sched && map.m == map.n && opt.rule == 0;
+  // (deep circuits, e.g. grqc_32's 7238 gates, keep planning cheap: their passes run at the full
+  // live size almost throughout, where the scheduler and the consecutive runs plan alike)
+  const bool try_sched = opt.auto_sched && map.m == map.n && opt.rule == 0 && gates.size() <= 4096;
   bool first_only = false;
   struct Result {
     double t = 0.0;

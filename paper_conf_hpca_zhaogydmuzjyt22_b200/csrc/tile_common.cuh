@@ -133,8 +133,6 @@ struct TileArgs {
   // mode 2 without private histograms: the lanes add straight to hist (global f64 reductions,
   // no shared memory), used when per-warp histograms would cost the pass CTAs per SM
   int hglob;
-  // single-buffered passes: bulk-prefetch the next tile's live runs into L2 at the start of a tile
-  int l2pf;
   // the pass's U matrices as a kernel parameter (constant bank), when they fit: the NVRTC bodies
   // read them at compile-time offsets (no shared-memory loads, no registers held across tiles)
   int umat_n;
@@ -189,10 +187,6 @@ __device__ __forceinline__ void cp_async16(void* smem, const void* gmem, int src
                : "memory");
 }
 __device__ __forceinline__ void cp_async_wait_all() { asm volatile("cp.async.wait_all;\n" ::: "memory"); }
-// bulk L2 prefetch of [p, p + bytes) (bytes a multiple of 16), no destination, no completion
-__device__ __forceinline__ void prefetch_l2_bulk(const void* p, uint32_t bytes) {
-  asm volatile("cp.async.bulk.prefetch.L2.global [%0], %1;\n" ::"l"(p), "r"(bytes) : "memory");
-}
 
 // ---- bulk asynchronous copies (TMA bulk path, SASS UBLKCP) with an mbarrier per buffer
 __device__ __forceinline__ uint32_t smem_u32(const void* p) {
@@ -912,15 +906,6 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     const uint64_t next = tile_at(it + 1);
     const bool more = next < a.ntiles;
     base_next = tile_base_t<Body>(real(next), a);
-    // single-buffered passes (two CTAs per SM) load the next tile only after this tile's program
-    // is done with the buffer: pull its live runs into L2 now, so those loads hit L2 (a.l2pf)
-    if (a.l2pf && more && nbuf == 1 && base_next < a.L_in && !(base_next & (a.zin | a.zout))) {
-      const uint32_t run = 16u << l;
-      for (int h = threadIdx.x; h < nh; h += nthr) {
-        const uint64_t idx = base_next | hiOff[h];
-        if (idx < a.L_in && !(idx & a.zin)) prefetch_l2_bulk(a.psi + idx, run);
-      }
-    }
     // nbuf >= 2: prefetch into the next buffer now; nbuf == 1 (programs without remaps, every
     // thread reads only its own slots): prefetch into the same buffer right after the reload
     if (more && nbuf > 1) issue_own_loads<NR, Body>(bufs + kn * T, a, mp0, sa0, base_next, zm0, c.own);

@@ -240,6 +240,41 @@ def test_jit_sources_compile_without_gpu(q):
         assert k == n_tile
 
 
+def test_jit_sources_specialise_the_fp64_bound_passes(q, monkeypatch, tmp_path):
+    """Round-2 NVRTC specialisations, checked in the generated sources of QAOA_16 (whose plan has
+    the same structure as QAOA_32's) and compiled for sm_100a on the CPU box: the tile-uniform
+    scalar joins the first phase run (kScalarFolded), programs with <= 2 remaps hand the buffer
+    to the next tile's loads after their last remap (pf()), and the fused-measurement variants
+    -- modes 0/1/2 and mode 2 with compile-time reduce-scatter masks and global reductions
+    (QGPU_JIT_CHECK_HIST key 0x131f: lane bits 0-4 unrequested, register bits 0-1 dead) --
+    compile."""
+    c = wc.qaoa(16, 2, seed=1)
+    monkeypatch.setenv("QGPU_JIT_DUMP", str(tmp_path))
+    monkeypatch.setenv("QGPU_JIT_CACHE", str(tmp_path / "cache"))
+    monkeypatch.setenv("QGPU_JIT_CHECK_HIST", "0x131f")
+    qc = q.Circuit(c.qasm())
+    try:
+        k = qc.jit_check(c.n, 2, 12)
+    except q.QgpuError as e:
+        if e.kind == "UNSUPPORTED":
+            pytest.skip("NVRTC not available")
+        raise
+    n_tile = sum(1 for r in qc.plan(c.n, 1, 2, 12) if r[2] == 0)
+    assert k == n_tile + 4
+    srcs = [p.read_text() for p in tmp_path.glob("qgpu_pass_*.cu")]
+    plain = [t for t in srcs if "kHist = false" in t]
+    assert len(plain) == n_tile
+    assert any("kScalarFolded = true" in t for t in plain)
+    for t in plain:  # the scalar is folded exactly when the program has a phase run
+        if "kHasScalar = true" in t:
+            assert ("kScalarFolded = true" in t) == ("run_apply_" in t)
+        assert t.count("pf();") <= 1
+        if "pf();" in t:
+            assert "kEarlyPrefetch = true" in t and t.count("tile_reload_j") <= 2 + 1
+    rs = [t for t in srcs if "kHistRS = true" in t]
+    assert len(rs) == 1 and "kHlred = 31u" in rs[0] and "kDead = 3u" in rs[0] and "kHistGlob = true" in rs[0]
+
+
 def test_fusion_lookahead_cuts_hbm_passes(q, monkeypatch):
     """Fusion lookahead (planner): commuting later gates join the open tile pass, so a depth-20
     random circuit needs far fewer full-state passes than cutting the reordered list in runs;
