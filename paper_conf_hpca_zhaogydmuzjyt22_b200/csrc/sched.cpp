@@ -18,8 +18,10 @@
 #include <cstdio>
 #include <cstdlib>
 #include <cstring>
+#include <exception>
 #include <functional>
 #include <limits>
+#include <system_error>
 #include <thread>
 
 #include "qgpu_internal.h"
@@ -1699,8 +1701,9 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
     QubitMap mp;
     std::vector<Pass> ps;
     std::vector<uint64_t> inv;
+    std::exception_ptr err;  // an exception thrown on a planner thread, rethrown by the caller
   };
-  auto run = [&](const int* c, Result* r) {
+  auto run_unsafe = [&](const int* c, Result* r) {
     PlanOptions o = opt;
     o.l_min = std::min(opt.l_min, c[0]);
     o.l_relax = c[1];
@@ -1712,6 +1715,13 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
     if (std::getenv("QGPU_DEBUG_AUTO"))
       std::fprintf(stderr, "plan_circuit_auto: l_min %d l_relax %d max_u_ops %d sched %d: %zu passes, modelled %.3f ms\n",
                    o.l_min, o.l_relax, o.max_u_ops, int(o.pass_sched), r->ps.size(), r->t * 1e3);
+  };
+  auto run = [&](const int* c, Result* r) {
+    try {
+      run_unsafe(c, r);
+    } catch (...) {
+      r->err = std::current_exception();
+    }
   };
   // the first candidate decides which others can matter; those are planned concurrently (the
   // planner has no shared mutable state) and compared in candidate order, so the choice does
@@ -1732,12 +1742,19 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
     if (cand[ci][3] ? try_sched : !first_only) todo.push_back(ci);
   {
     std::vector<std::thread> th;
-    for (int ci : todo) th.emplace_back(run, cand[ci], &res[size_t(ci)]);
+    for (int ci : todo) {
+      try {
+        th.emplace_back(run, cand[ci], &res[size_t(ci)]);
+      } catch (const std::system_error&) {  // no thread available: plan this candidate inline
+        run(cand[ci], &res[size_t(ci)]);
+      }
+    }
     for (auto& t : th) t.join();
   }
   for (int ci = 0; ci < kCand; ++ci) {
     if (ci > 0 && std::find(todo.begin(), todo.end(), ci) == todo.end()) continue;
     Result& r = res[size_t(ci)];
+    if (r.err) std::rethrow_exception(r.err);
     if (!have || r.t < best * 0.995) {  // ties keep the earlier (longer-run) policy
       have = true;
       best = r.t;
