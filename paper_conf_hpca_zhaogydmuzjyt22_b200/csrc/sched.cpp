@@ -571,6 +571,93 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
       }
     }
   }
+  // 1b. order the ops within their commutation DAG so that the U ops on non-lane tile bits come
+  //     in clusters that fit the register bits (each change of the register bits is a remap:
+  //     the tile is stored to and reloaded from shared memory). Two ops commute unless one's
+  //     targets touch the other's targets or tile-local conditions (phase terms are diagonal:
+  //     they commute with each other and with U ops on other bits). Greedy: run every ready op
+  //     whose non-lane targets are in the current register set (lowest index first, so the
+  //     given order is kept where it costs nothing); when none is left, switch the set to the
+  //     non-lane bits most wanted by the ready ops. Step 3 then assigns the register bits per
+  //     segment on the new order (QGPU_PASS_REORDER=0: the gate order, A/B).
+  {
+    const char* ev = std::getenv("QGPU_PASS_REORDER");
+    const int lanes_ = std::min(5, p.b);
+    const int nr_ = std::min(std::min(4, std::max(reg_bits, 3)), p.b - lanes_);
+    const size_t N = raw.size();
+    if (!(ev && ev[0] == '0') && nr_ > 0 && N > 2) {
+      const uint32_t lanemask = (1u << lanes_) - 1u;
+      std::vector<uint32_t> tb(N), cb(N);
+      for (size_t i = 0; i < N; ++i) {
+        const RawOp& o = raw[i];
+        tb[i] = o.kind == 2 ? 0u : ((1u << o.t[0]) | (o.kind == 1 ? 1u << o.t[1] : 0u));
+        cb[i] = o.lmask;
+      }
+      std::vector<std::vector<int>> succ(N);
+      std::vector<int> indeg(N, 0);
+      for (size_t j = 0; j < N; ++j)
+        for (size_t i = 0; i < j; ++i)
+          if ((tb[i] & (tb[j] | cb[j])) || (tb[j] & cb[i])) {
+            succ[i].push_back(int(j));
+            ++indeg[j];
+          }
+      std::vector<char> done(N, 0);
+      std::vector<int> order;
+      order.reserve(N);
+      uint32_t Rset = 0;
+      while (order.size() < N) {
+        bool progress = true;
+        while (progress) {
+          progress = false;
+          for (size_t u = 0; u < N; ++u) {
+            if (done[u] || indeg[u] != 0 || (tb[u] & ~lanemask & ~Rset)) continue;
+            done[u] = 1;
+            order.push_back(int(u));
+            for (int v : succ[u]) --indeg[size_t(v)];
+            progress = true;
+            break;
+          }
+        }
+        if (order.size() == N) break;
+        // the non-lane bits the ready ops wait for (then all remaining ops, then the lowest)
+        int want[32] = {0}, later[32] = {0};
+        for (size_t u = 0; u < N; ++u) {
+          if (done[u]) continue;
+          for (uint32_t r = tb[u] & ~lanemask; r; r &= r - 1) {
+            const int bit = std::countr_zero(r);
+            ++later[bit];
+            if (indeg[u] == 0) ++want[bit];
+          }
+        }
+        std::vector<int> bits;
+        for (int bit = lanes_; bit < p.b; ++bit) bits.push_back(bit);
+        std::stable_sort(bits.begin(), bits.end(), [&](int x, int y) {
+          if (want[x] != want[y]) return want[x] > want[y];
+          return later[x] > later[y];
+        });
+        Rset = 0;
+        for (int k = 0; k < nr_ && k < int(bits.size()); ++k) Rset |= 1u << bits[size_t(k)];
+        // a ready op that needs more non-lane bits than the register set holds (cannot happen
+        // for nr >= 2) would stall the loop: take the lowest ready op as it is
+        bool any = false;
+        for (size_t u = 0; u < N && !any; ++u)
+          any = !done[u] && indeg[u] == 0 && !(tb[u] & ~lanemask & ~Rset);
+        if (!any) {
+          for (size_t u = 0; u < N; ++u)
+            if (!done[u] && indeg[u] == 0) {
+              done[u] = 1;
+              order.push_back(int(u));
+              for (int v : succ[u]) --indeg[size_t(v)];
+              break;
+            }
+        }
+      }
+      std::vector<RawOp> re;
+      re.reserve(N);
+      for (int u : order) re.push_back(raw[size_t(u)]);
+      raw.swap(re);
+    }
+  }
   // 2. place phase terms. A term commutes with every U op that does not target one of its tile
   //    bits, so it may sit in any slot between the last U op before it and the first U op after
   //    it that targets one of its bits (slot s = just before U op s). Each distinct slot used is
