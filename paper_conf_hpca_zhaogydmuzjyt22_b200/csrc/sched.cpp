@@ -14,6 +14,7 @@
 #include <algorithm>
 #include <array>
 #include <bit>
+#include <climits>
 #include <cmath>
 #include <cstdio>
 #include <cstdlib>
@@ -652,10 +653,41 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
             }
         }
       }
-      std::vector<RawOp> re;
-      re.reserve(N);
-      for (int u : order) re.push_back(raw[size_t(u)]);
-      raw.swap(re);
+      // keep the new order only if it needs fewer register-set changes than the gate order
+      // (step 3's rule: when a U op's non-lane target is not a register bit, the register bits
+      // become the nr non-lane bits used soonest from there); on ties the gate order stays
+      // (QAOA_32's passes: one remap either way, and the gate order was measured faster)
+      auto remaps = [&](const std::vector<int>& ord) {
+        uint32_t R = 0;
+        int cnt = 0;
+        for (size_t i = 0; i < ord.size(); ++i) {
+          const uint32_t need = tb[size_t(ord[i])] & ~lanemask;
+          if (!need || !(need & ~R)) continue;
+          ++cnt;
+          int first[32];
+          for (int bit = 0; bit < 32; ++bit) first[bit] = INT32_MAX;
+          for (size_t j = ord.size(); j-- > i;)
+            for (uint32_t r = tb[size_t(ord[j])] & ~lanemask; r; r &= r - 1) first[std::countr_zero(r)] = int(j);
+          std::vector<int> bits;
+          for (int bit = lanes_; bit < p.b; ++bit) bits.push_back(bit);
+          std::stable_sort(bits.begin(), bits.end(), [&](int x, int y) {
+            const bool nx = need >> x & 1, ny = need >> y & 1;
+            if (nx != ny) return nx;
+            return first[x] < first[y];
+          });
+          R = 0;
+          for (int k = 0; k < nr_ && k < int(bits.size()); ++k) R |= 1u << bits[size_t(k)];
+        }
+        return cnt;
+      };
+      std::vector<int> given(N);
+      for (size_t i = 0; i < N; ++i) given[i] = int(i);
+      if (remaps(order) < remaps(given)) {
+        std::vector<RawOp> re;
+        re.reserve(N);
+        for (int u : order) re.push_back(raw[size_t(u)]);
+        raw.swap(re);
+      }
     }
   }
   // 2. place phase terms. A term commutes with every U op that does not target one of its tile
