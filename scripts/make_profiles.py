@@ -103,7 +103,7 @@ def main():
                 if st["tile_kernel_launches"]:  # (filled when the profiled run had timing on)
                     nl, ab = st["tile_kernel_launches"], st["tile_algo_bytes"]
                 else:  # every launched kernel a tile pass (QAOA / QFT): the totals are the tile ones
-                    assert st["kernels_launched"] == st["jit_launches"] == len(tile), st
+                    assert st["kernels_launched"] == len(tile), st
                     nl, ab = st["kernels_launched"], st["algo_bytes"]
                 tr["algo_bytes_per_launch"] = ab / nl
                 tr["launches_per_circuit_stats"] = nl
