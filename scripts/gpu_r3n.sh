@@ -1,0 +1,7 @@
+set -x
+O=gpurun_out/r3n; mkdir -p $O
+python -c "import __graft_entry__ as g; g.build()" > $O/build.log 2>&1
+timeout 1500 python -m pytest tests/test_gpu_measure.py tests/test_gpu_fullsize.py -m gpu -q -x -k "not c3_qaoa32_vs_oracle" > $O/pytest_a.log 2>&1; echo "rc=$?" >> $O/pytest_a.log
+bash scripts/gpu_ab.sh r3n/ab scripts/ab_variants15.txt
+python scripts/meas_profile.py qaoa32 > $O/meas_profile.log 2>&1
+tail -n 2 $O/pytest_a.log
