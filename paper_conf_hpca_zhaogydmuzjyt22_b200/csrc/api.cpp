@@ -500,7 +500,6 @@ qgpu_status qgpu_state_destroy(qgpu_state* st) {
   for (double2* b : st->vstage)
     if (b) cudaFree(b);
   if (st->d_meas) cudaFree(st->d_meas);
-  if (st->d_meas_priv) cudaFree(st->d_meas_priv);
   for (CachedPlan& cp : st->plans) {
     if (cp.d_blob) cudaFree(cp.d_blob);
     if (cp.h_blob) cudaFreeHost(cp.h_blob);

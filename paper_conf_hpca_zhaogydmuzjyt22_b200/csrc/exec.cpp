@@ -304,20 +304,6 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
         h.hglob = (hgm == 2 || (hgm == 1 && tile_smem_bytes(h) > cap)) ? 1 : 0;
       }
       if (tile_smem_bytes(h) > 227 * 1024 && h.nbuf == 3) h.nbuf = 2;  // make room: double buffering
-      if (h.hglob) {
-        // one private copy per resident CTA (<= 4 per SM), zeroed here, summed into d_meas after
-        h.hcopies = 4 * device_num_sms();
-        const size_t need = size_t(h.hcopies) << (h.hm + 3);
-        if (st->meas_priv_bytes < need) {
-          if (st->d_meas_priv) CK(cudaFree(st->d_meas_priv));
-          st->d_meas_priv = nullptr;
-          st->meas_priv_bytes = 0;
-          CK(cudaMalloc(&st->d_meas_priv, need));
-          st->meas_priv_bytes = need;
-        }
-        CK(cudaMemsetAsync(st->d_meas_priv, 0, need, st->stream));
-        h.hist = st->d_meas_priv;
-      }
       if (tile_smem_bytes(h) <= 227 * 1024) {
         a = h;
         st->meas_done = true;
@@ -334,10 +320,6 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     if (e == cudaErrorNotSupported) e = launch_tile(st->stream, a);
     CK(e);
     st->stats.kernels_launched++;
-    if (a.hist && a.hglob) {  // the private histograms -> the pass's measurement result
-      CK(launch_hist_reduce(st->stream, st->d_meas, a.hist, a.hcopies, 1u << a.hm));
-      st->stats.kernels_launched++;
-    }
     // live input / output amplitudes: a skipped zero position halves the part that moves
     bytes = 16 * ((L_in >> std::popcount(a.zin & (L_in - 1))) + (L_out >> std::popcount(a.zout & (L_out - 1))));
   } else if (p.kind == PK_ZERO) {

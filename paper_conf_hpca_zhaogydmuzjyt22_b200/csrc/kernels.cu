@@ -818,22 +818,6 @@ __global__ void zero_where_kernel(double2* psi, uint64_t L, uint64_t mask) {
   for (uint64_t i = uint64_t(blockIdx.x) * blockDim.x + threadIdx.x; i < L; i += stride)
     if (i & mask) __stcs(psi + i, make_double2(0.0, 0.0));
 }
-// out[i] = sum over the ncopies private histograms of bucket i (fused measurement, hglob)
-__global__ void hist_reduce_kernel(double* __restrict__ out, const double* __restrict__ priv, int ncopies,
-                                   uint32_t nb) {
-  for (uint32_t i = blockIdx.x * blockDim.x + threadIdx.x; i < nb; i += gridDim.x * blockDim.x) {
-    double t = 0.0;
-    for (int c = 0; c < ncopies; ++c) t += priv[size_t(c) * nb + i];
-    out[i] = t;
-  }
-}
-
-cudaError_t launch_hist_reduce(cudaStream_t st, double* out, const double* priv, int ncopies, uint32_t nb) {
-  const unsigned g = std::max(1u, std::min(148u, (nb + kThreads - 1) / kThreads));
-  hist_reduce_kernel<<<g, kThreads, 0, st>>>(out, priv, ncopies, nb);
-  return cudaGetLastError();
-}
-
 cudaError_t launch_zero_where(cudaStream_t st, double2* psi, uint64_t L, uint64_t mask) {
   if (!L || !mask) return cudaSuccess;
   zero_where_kernel<<<grid_for(L, 256 * 4, 8), 256, 0, st>>>(psi, L, mask);

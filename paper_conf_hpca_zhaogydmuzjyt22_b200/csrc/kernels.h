@@ -85,8 +85,6 @@ cudaError_t launch_set_amp(cudaStream_t st, double2* psi, uint64_t i, double re,
 // FP64 peak probe (qgpu_measure_fp64_peak): thread-level DFMA per second on the current device
 cudaError_t probe_fp64(double* fma_per_s);
 cudaError_t launch_zero_where(cudaStream_t st, double2* psi, uint64_t L, uint64_t mask);
-// fused measurement with private global histograms: out[i] = sum_c priv[c * nb + i]
-cudaError_t launch_hist_reduce(cudaStream_t st, double* out, const double* priv, int ncopies, uint32_t nb);
 // sharded swaps (a10)
 cudaError_t launch_swap_halves(cudaStream_t st, double2* a, double2* b, int lp, uint64_t half);
 // a10 batched global-local swap of s rank bits with s local positions: the live local amplitudes

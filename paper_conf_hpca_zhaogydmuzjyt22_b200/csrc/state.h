@@ -191,8 +191,6 @@ struct qgpu_state {
   int meas_hacc = 0;                   // TileArgs::hacc (see apply_circuit_impl)
   uint32_t meas_hlred = 0;             // TileArgs::hlred: lane bits not requested
   double* d_meas = nullptr;            // 2^kMeasMax doubles
-  double* d_meas_priv = nullptr;       // fused measurement, hglob: private per-CTA histograms
-  size_t meas_priv_bytes = 0;
   bool meas_done = false;
 };
 

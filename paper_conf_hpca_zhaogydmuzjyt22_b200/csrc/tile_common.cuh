@@ -130,13 +130,9 @@ struct TileArgs {
   // differ -- add without atomics. 0: requested bits uniform across a warp's slots.
   int hacc;
   uint32_t hlred;
-  // mode 2 without private histograms: the lanes add straight to a global histogram (f64
-  // reductions, no shared memory), used when per-warp histograms would cost the pass CTAs per
-  // SM. hist then holds hcopies private copies of 2^hm doubles; CTA i adds to copy i % hcopies
-  // (distinct addresses per CTA instead of every SM hammering the same 2^hm words), and a
-  // reduction kernel sums the copies after the pass
+  // mode 2 without private histograms: the lanes add straight to hist (global f64 reductions,
+  // no shared memory), used when per-warp histograms would cost the pass CTAs per SM
   int hglob;
-  int hcopies;
   // the pass's U matrices as a kernel parameter (constant bank), when they fit: the NVRTC bodies
   // read them at compile-time offsets (no shared-memory loads, no registers held across tiles)
   int umat_n;
@@ -1127,8 +1123,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
 #pragma unroll
           for (int i = 0; i < (1 << kNL); ++i)
             if (i < (1 << size_log)) {
-              if constexpr (Body::kHistGlob)  // RED.ADD.F64 (no return) to this CTA's copy
-                atomicAdd(a.hist + (size_t(blockIdx.x % unsigned(a.hcopies)) << a.hm) + bk[i], y[i]);
+              if constexpr (Body::kHistGlob) atomicAdd(a.hist + bk[i], y[i]);  // RED.ADD.F64, no return
               else hw[bk[i]] = old[i] + y[i];
             }
         }
@@ -1168,7 +1163,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
 #pragma unroll
         for (int r = 0; r < (1 << NR); ++r)
           if ((uint32_t(r) & dead) == 0u) {
-            if (a.hglob) atomicAdd(a.hist + (size_t(blockIdx.x % unsigned(a.hcopies)) << a.hm) + bk[r], x[r]);
+            if (a.hglob) atomicAdd(a.hist + bk[r], x[r]);
             else hw[bk[r]] = old[r] + x[r];
           }
       }

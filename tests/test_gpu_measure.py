@@ -118,11 +118,9 @@ def test_fused_measurement_jit_vs_oracle(q, name, qsel):
 
 
 @pytest.mark.parametrize("jit", [0, 2])
-def test_fused_measurement_lane_register_bits_read_no_state(q, jit, hacc_mode):
+def test_fused_measurement_lane_register_bits_read_no_state(q, jit):
     """Qubits 0..9 of QFT_18 sit on lane, register and tile-index bits of the last pass: per-warp
-    private histograms (or per-slot register sums) in the pass, so no readout kernel is launched.
-    (With the global histograms -- QGPU_HGLOB=2 -- a reduction over the per-CTA copies replaces
-    the readout kernel: as many launches, none of which reads the state.)"""
+    private histograms (or per-slot register sums) in the pass, so no readout kernel is launched."""
     text = wc.qft(18).qasm()
     qubits = list(range(10))
     with q.State(18, jit=jit) as s:
@@ -132,7 +130,7 @@ def test_fused_measurement_lane_register_bits_read_no_state(q, jit, hacc_mode):
         s.apply_circuit(q.Circuit(text))
         p2 = s.probabilities(qubits)
         k_plain = s.stats()["kernels_launched"]
-    assert k_fused <= k_plain if hacc_mode == "global_hist" else k_fused < k_plain
+    assert k_fused < k_plain
     assert np.abs(p - p2).max() <= 1e-12
     assert np.abs(p - 2.0 ** -10).max() <= 1e-12  # QFT|0> is uniform: every marginal is 2^-10
 
@@ -159,7 +157,5 @@ def test_fused_measurement_unrequested_lane_bits_jit(q, name, hacc_mode):
     ref = osv.probabilities(osv.simulate(text), c.n, qubits)
     assert np.abs(p - ref).max() <= 1e-12
     assert np.abs(p - p2).max() <= 1e-12
-    if hacc_mode == "global_hist":
-        assert k_fused <= k_plain  # the per-CTA histogram reduction replaces the readout kernel
-    elif hacc_mode != "round2_rule":
+    if hacc_mode != "round2_rule":
         assert k_fused < k_plain
