@@ -297,13 +297,13 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
       // mode 2's per-warp private histograms (2^m doubles per warp) must not cost the pass CTAs
       // per SM: a two-CTA pass (<= 113 KiB each) or one that would not fit at all adds straight
       // to the global histogram instead (QGPU_HGLOB=0: never, 2: always)
+      if (tile_smem_bytes(h) > 227 * 1024 && h.nbuf == 3) h.nbuf = 2;  // make room: double buffering
       if (h.hacc == 2) {
         const char* hg = std::getenv("QGPU_HGLOB");
         const int hgm = hg ? std::atoi(hg) : 1;
         const size_t cap = two_cta ? 113 * 1024 : 227 * 1024;
         h.hglob = (hgm == 2 || (hgm == 1 && tile_smem_bytes(h) > cap)) ? 1 : 0;
       }
-      if (tile_smem_bytes(h) > 227 * 1024 && h.nbuf == 3) h.nbuf = 2;  // make room: double buffering
       if (tile_smem_bytes(h) <= 227 * 1024) {
         a = h;
         st->meas_done = true;
