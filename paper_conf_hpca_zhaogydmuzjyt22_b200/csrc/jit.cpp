@@ -319,8 +319,9 @@ std::string tile_jit_source(const Pass& p, int hist_mode, uint32_t hist_key) {
     for (size_t i = last_smem + 1; i < P.ops.size() && last_smem > 0; ++i)
       after += (P.ops[i].kind == OP_RUN || P.ops[i].kind == OP_U1R || P.ops[i].kind == OP_U1L ||
                 P.ops[i].kind == OP_U2R);
-    const char* ev = std::getenv("QGPU_EARLY_PF");  // 0: prefetch after the program, 2: always
-    const int mode = ev ? std::atoi(ev) : 1;
+    const char* ev = std::getenv("QGPU_EARLY_PF");  // 0: after the program, 1: gated, 2: always
+    const int mode = ev ? std::atoi(ev) : 0;  // default off since the scalar folding (r3o: 46.0
+                                               // vs 46.7 ms with it on QAOA_32, one-table runs)
     if (mode == 0 || (mode == 1 && (after < 3 || nremap > 2))) last_smem = 0;
   }
   hdr << "  static constexpr bool kEarlyPrefetch = " << (last_smem > 0 ? "true" : "false") << ";\n";
@@ -472,9 +473,11 @@ std::string tile_jit_source(const Pass& p, int hist_mode, uint32_t hist_key) {
             break;
           }
         }
-        // QGPU_RUN_SPLIT=0: one 16-entry factor table (run_apply_ptab_z) instead of two 4-entry
+        // one 16-entry factor table (run_apply_ptab_z); QGPU_RUN_SPLIT=1: two 4-entry tables
+        // (fewer live registers; measured slower once the scalar was folded into the first run:
+        // profiles/r02b ab r3o, QAOA_32 46.8 -> 46.0 ms, rqc_30 96.4 -> 93.6 ms with one table)
         const char* rs_env = std::getenv("QGPU_RUN_SPLIT");
-        const bool split_tab = NR == 4 && !(rs_env && rs_env[0] == '0');
+        const bool split_tab = NR == 4 && (rs_env && rs_env[0] == '1');
         if (used)
           o << "      " << (split_tab ? "run_apply_split_z<" : "run_apply_ptab_z<") << NR << ", " << (used & 1 ? "true" : "false") << ", "
             << ((used >> 1) & 1 ? "true" : "false") << ", " << ((used >> 2) & 1 ? "true" : "false") << ", "
