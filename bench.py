@@ -794,6 +794,18 @@ def run_ours(args):
                            "ops_before_full_involvement": estats[-1]["ops_before_full_involvement"]}
             er = extras[key]["roofline"]
             er["traffic"], er["traffic_source"] = ncu_traffic(f"{key}_{ec.n}", er)
+            # per-pass binding bound of this circuit too (its middle passes are FP64-bound)
+            est.set_timing(2)
+            est.pass_profile()
+            eprof = None
+            for _ in range(3):
+                est.reset()
+                est.apply_circuit(q.Circuit(ec.qasm()))
+                eprof = est.pass_profile()
+            est.set_timing(1)
+            eb = per_pass_binding(eprof, peak, fp64)
+            er["binding"] = {"passes": eb["passes"], "bound_ms": eb["bound_ms"], "measured_ms": eb["measured_ms"],
+                             "frac": eb["frac"], "by_binding": eb["by_binding"]}
             if key == "qft28" and args.gfc:
                 extras[key]["gfc_compression"] = gfc_measure(q, torch, est)
             est.close()
