@@ -280,9 +280,6 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     // registers (NVRTC kernels only)
     const bool two_cta = pass_two_cta(p) && (st->cfg.jit == 2 || (st->cfg.jit == 1 && p.k_out >= jit_min_bits()));
     if (two_cta) a.nbuf = 1;
-    // split remaps: the NVRTC body decides (pass_split_remap); the extra half-size buffer is
-    // allocated whenever that kernel may run
-    a.psplit = (two_cta && pass_split_remap(p)) ? 1 : 0;
     // optional bulk stores (staged tile, async copies per run; QGPU_BSTORE)
     const int bs = bstore_mode();
     if (bs == 2 || (bs == 1 && a.remaps)) a.nbuf = 3;

@@ -368,7 +368,6 @@ std::string tile_jit_source(const Pass& p, int hist_mode, uint32_t hist_key) {
     fold_scalar = fold_scalar && has_run;
   }
   bool scalar_pending = fold_scalar;
-  const bool split_remap = pass_split_remap(p);
   for (size_t i = 1; i < P.ops.size(); ++i) {
     const TileOp& op = P.ops[i];
     const bool uni = op.omask != 0;       // tile-uniform condition present
@@ -514,16 +513,6 @@ std::string tile_jit_source(const Pass& p, int hist_mode, uint32_t hist_key) {
         zpos &= ~((1u << R[op.a0]) | (1u << R[op.a1]));
         break;
       case OP_REMAP: {
-        if (split_remap) {  // half-size remap buffer, two rounds (remap_split)
-          o << "      { constexpr uint32_t Jo[kRegAmps] = " << jtab(R) << ";\n";
-          decode(op);
-          decode_w(op);
-          o << "        constexpr uint32_t Jn[kRegAmps] = " << jtab(R) << ";\n";
-          o << "        const uint32_t nb = " << base_expr(op) << ";\n";
-          o << "        remap_split<" << NR << ">(v, c, mp.base, Jo, nb, Jn);\n";
-          o << "        mp.base = nb; }\n";
-          break;
-        }
         int Wold[4] = {W[0], W[1], W[2], W[3]};
         o << "      { constexpr uint32_t Jo[kRegAmps] = " << jtab(R) << ";\n";
         o << "        tile_store_j<" << NR << ">(v, c, mp.base, Jo); }\n";
@@ -573,7 +562,6 @@ std::string tile_jit_source(const Pass& p, int hist_mode, uint32_t hist_key) {
   }
   o << "struct JitBody {\n" << hdr.str();
   o << "  static constexpr bool kScalarFolded = " << (fold_scalar ? "true" : "false") << ";\n";
-  o << "  static constexpr bool kSplitRemap = " << (pass_split_remap(p) ? "true" : "false") << ";\n";
   o << "  static constexpr bool kGroupRemap = true;\n";
   o << "  __device__ static void init_mbar(uint64_t* mb) {\n";
   for (const auto& g : groups)

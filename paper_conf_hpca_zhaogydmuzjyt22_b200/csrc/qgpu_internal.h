@@ -213,10 +213,6 @@ double pass_cost_model(const Pass& p, int m);
 // one triple-buffered CTA at <= 255): QGPU_2CTA=1 every pass, 2 (default) passes whose program
 // runs >= 40 FP64 instructions per amplitude (the latency-bound ones), 0 none (read per call).
 bool pass_two_cta(const Pass& p);
-// Split remaps for this pass's NVRTC kernel (TileArgs::psplit, Body::kSplitRemap): two-CTA passes
-// with remaps and no shared-memory ops; the tile buffer then only takes loads (the next tile's
-// right after the reload) and remaps use a half-size buffer in two rounds.
-bool pass_split_remap(const Pass& p);
 // Build the device ops of a tile pass from its gates and tile positions.
 void build_tile_ops(Pass& p, int m, int reg_bits = 4);
 // Unfused byte model of one gate on live size 2^k.

@@ -1890,20 +1890,6 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
 }  // namespace qgpu
 
 namespace qgpu {
-bool pass_split_remap(const Pass& p) {
-  // two-CTA NVRTC passes with remaps and no shared-memory ops (QGPU_PSPLIT=0: off, A/B)
-  const char* ev = std::getenv("QGPU_PSPLIT");
-  if (ev && ev[0] == '0') return false;
-  if (p.kind != PK_TILE || !pass_two_cta(p) || p.b < 6) return false;
-  bool remap = false;
-  for (size_t i = 1; i < p.prog.ops.size(); ++i) {
-    const int k = p.prog.ops[i].kind;
-    if (k == OP_SMEM1 || k == OP_SMEM2) return false;
-    remap = remap || k == OP_REMAP;
-  }
-  return remap;
-}
-
 bool pass_two_cta(const Pass& p) {
   // default 2 (profiles/r02 A/B, same box: QAOA_32 175.9 -> 166.5 ms fixed lanes and 178.4 ->
   // 158.8 auto lanes, rqc_30 146.9 -> 139.5, grqc_32 8.43 -> 8.20 s, QFT_28 1.13 -> 1.10 ms)

@@ -133,11 +133,6 @@ struct TileArgs {
   // mode 2 without private histograms: the lanes add straight to hist (global f64 reductions,
   // no shared memory), used when per-warp histograms would cost the pass CTAs per SM
   int hglob;
-  // split remaps (two-CTA NVRTC passes, Body::kSplitRemap): the tile buffer only receives this
-  // thread's own loads, and remaps go through a separate half-size buffer in two rounds (one per
-  // value of lane bit 0), so the next tile's loads are issued right after the reload at the
-  // start of each tile; smem = 1.5 tiles per CTA
-  int psplit;
   // the pass's U matrices as a kernel parameter (constant bank), when they fit: the NVRTC bodies
   // read them at compile-time offsets (no shared-memory loads, no registers held across tiles)
   int umat_n;
@@ -352,30 +347,6 @@ __device__ __forceinline__ void tile_store_j(const double2 (&v)[kRegAmps], const
 __device__ __forceinline__ void group_sync(const TileCtx& c, int idx) {
   mbar_arrive(c.mbar + idx);
   mbar_wait(c.mbar + idx, c.mpar);
-}
-// Split remap (Body::kSplitRemap): c.s is a half-size buffer indexed by the tile index without
-// bit 0. Tile bit 0 is lane bit 0 under every mapping, so the threads with lane bit 0 = h hold
-// exactly the half of the tile with bit 0 = h before and after the remap: two rounds, each
-// stores that half, meets, reloads it; the barriers also keep the rounds (and consecutive
-// remaps) from overwriting a half that is still being read.
-template <int NR>
-__device__ __forceinline__ void remap_split(double2 (&v)[kRegAmps], const TileCtx& c, uint32_t ob,
-                                            const uint32_t (&Jo)[kRegAmps], uint32_t nb,
-                                            const uint32_t (&Jn)[kRegAmps]) {
-  const int h = c.lane & 1;
-#pragma unroll
-  for (int round = 0; round < 2; ++round) {
-    __syncthreads();
-    if (h == round) {
-#pragma unroll
-      for (int r = 0; r < (1 << NR); ++r) c.s[(ob + Jo[r]) >> 1] = v[r];
-    }
-    __syncthreads();
-    if (h == round) {
-#pragma unroll
-      for (int r = 0; r < (1 << NR); ++r) v[r] = c.s[(nb + Jn[r]) >> 1];
-    }
-  }
 }
 
 __device__ __forceinline__ bool op_active(const TileOp& op, uint64_t gbase) {
@@ -846,9 +817,8 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   const uint32_t T = 1u << b;
   const int nh = 1 << (b - l);
   const int nthr = blockDim.x, nwarps = nthr >> 5;
-  double2* bufs = reinterpret_cast<double2*>(smem_raw);  // nbuf x T (+ T / 2: split remaps)
-  uint64_t* hiOff = reinterpret_cast<uint64_t*>(bufs + nbuf * T + (a.psplit ? T / 2 : 0));
-  double2* const remap_buf = bufs + nbuf * T;  // Body::kSplitRemap: the half-size remap buffer
+  double2* bufs = reinterpret_cast<double2*>(smem_raw);  // nbuf x T
+  uint64_t* hiOff = reinterpret_cast<uint64_t*>(bufs + nbuf * T);
   unsigned char* blob = reinterpret_cast<unsigned char*>(hiOff + ((nh + 1) & ~1));
   const TileOp* ops = reinterpret_cast<const TileOp*>(blob);
   const RunEntry* ents = reinterpret_cast<const RunEntry*>(blob + a.off_entries);
@@ -1010,7 +980,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     __syncwarp();
     // tile-uniform phase (the scalar pattern)
     const double2 sc = (Body::kHasScalar && a.spat >= 0) ? Cw[size_t(warp) * a.npat + a.spat] : make_double2(1.0, 0.0);
-    c.s = Body::kSplitRemap ? remap_buf : s;
+    c.s = s;
     c.gbase = gbase;
     double2 v[kRegAmps];
     Mapping mp = mp0;
@@ -1025,22 +995,21 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     // can go into the buffer right after this reload; with remaps (two CTAs per SM, each single-
     // buffered: the other CTA's compute covers this one's load latency) the buffer is free only
     // once every thread of the CTA has finished the program's remaps
-    if (more && nbuf == 1 && (!a.remaps || Body::kSplitRemap))
-      issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
+    if (more && nbuf == 1 && !a.remaps) issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
     c.mpar = nexec & 1u;
     ++nexec;
     // nbuf == 1 with remaps: the next tile's loads go into the buffer once every thread is past
     // the program's last remap / shared-memory op -- at that op when the body marks it
     // (Body::kEarlyPrefetch, NVRTC bodies: the rest of the program overlaps the load latency),
     // else after the program. Bulk stores read the buffer at the end: no early prefetch then.
-    const bool early = Body::kEarlyPrefetch && !Body::kSplitRemap && more && nbuf == 1 && a.remaps && !a.bstore;
+    const bool early = Body::kEarlyPrefetch && more && nbuf == 1 && a.remaps && !a.bstore;
     body(v, mp, c, a, [&]() {
       if (early) {
         __syncthreads();
         issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
       }
     });
-    if (more && nbuf == 1 && a.remaps && !early && !Body::kSplitRemap) {
+    if (more && nbuf == 1 && a.remaps && !early) {
       __syncthreads();
       issue_own_loads<NR, Body>(s, a, mp0, sa0, base_next, zm0, c.own);
     }
