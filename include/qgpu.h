@@ -202,18 +202,22 @@ qgpu_status qgpu_apply_gate(qgpu_state* st, const double* U, int n_targets, cons
                             int n_controls, const int* controls);
 
 /* Apply a parsed circuit: reorder (cfg.reorder: Alg.2/Alg.3), update involvement and qubit
- * placement per gate, cut the order into consecutive fused passes (cfg.fuse_bits), execute
- * SWAP gates as qubit relabels, and launch. The result equals program-order application up to
- * floating-point rounding. The circuit must have n_qubits <= the state's n.
- * Errors: INVALID_ARG, STATE, CUDA, NCCL. Asynchronous. */
+ * placement per gate, cut the order into consecutive fused passes (cfg.fuse_bits) -- or, when
+ * the pass cost model prefers it (single resident state, involve_rule 0, no SWAP gates), plan
+ * the passes over the commutation DAG, keeping Alg.3's priority among ready gates (DESIGN.md
+ * §4 "Pass scheduling") -- execute SWAP gates as qubit relabels, and launch. The result equals
+ * program-order application up to floating-point rounding; the schedule and the
+ * involvement trace reported by qgpu_get_schedule follow Alg.3's order exactly. The circuit
+ * must have n_qubits <= the state's n. Errors: INVALID_ARG, STATE, CUDA, NCCL. Asynchronous. */
 qgpu_status qgpu_apply_circuit(qgpu_state* st, const qgpu_circuit* c);
 
 /* Apply a circuit and measure at its end (marginal probabilities as in
  * qgpu_probabilities, Eq.1): out[y] = sum over i with bits_Q(i) = y of |psi_i|^2 after the
  * circuit, qubits[0] <-> bit 0 of y, 0 <= m <= 30, out = 2^m doubles (host). When the plan ends
- * with a fused pass over the whole live state (single resident state, m <= 12, the histogram
- * fits in shared memory) that pass accumulates the histogram from the amplitudes it stores
- * (no extra read of the state); otherwise this is qgpu_apply_circuit + qgpu_probabilities.
+ * with a fused pass over the whole live state (single resident state, m <= 12) that pass
+ * accumulates the histogram from the amplitudes it stores (no extra read of the state; in
+ * shared memory, or with global f64 reductions when per-warp histograms would not fit beside
+ * the tile buffers); otherwise this is qgpu_apply_circuit + qgpu_probabilities.
  * The state is left as qgpu_apply_circuit leaves it. Synchronises. Errors as both calls. */
 qgpu_status qgpu_apply_circuit_probabilities(qgpu_state* st, const qgpu_circuit* c, int m,
                                              const int* qubits, double* out);
