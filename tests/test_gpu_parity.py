@@ -355,3 +355,30 @@ def test_jit_pruning_neutrality_exact(q):
     a = gpu_run(q, text, fuse_bits=12, prune=1, jit=2)
     b = gpu_run(q, text, fuse_bits=12, prune=0, jit=2)
     assert np.array_equal(a, b)
+
+
+SCHED_CIRCS = {
+    "qaoa": lambda: wc.qaoa(20, 2, seed=5),
+    "hlf": lambda: wc.hlf(4, 5, seed=3),
+    "rqc": lambda: wc.rqc(18, 8, seed=4),
+    "randdiag": lambda: wc.random_circuit(16, 240, seed=21, names=["cp", "cz", "rz", "cx", "crx", "ccx", "t",
+                                                                     "h", "rzz", "x", "u1", "crz", "s", "sx"]),
+}
+
+
+@pytest.mark.parametrize("name", sorted(SCHED_CIRCS))
+@pytest.mark.parametrize("sched", ["0", "2"])
+@pytest.mark.parametrize("reorder", ["1", "0"])
+def test_pass_schedule_and_op_clustering_vs_oracle(q, name, sched, reorder, monkeypatch):
+    """The pass-aware execution order forced on (QGPU_PASS_SCHED=2) and off (0), each with the
+    intra-pass op clustering on and off (QGPU_PASS_REORDER), on the NVRTC kernels at the
+    library's default threshold: every amplitude against the oracle (commuting
+    reorders change rounding only)."""
+    monkeypatch.setenv("QGPU_PASS_SCHED", sched)
+    monkeypatch.setenv("QGPU_PASS_REORDER", reorder)
+    monkeypatch.setenv("QGPU_JIT_MIN_BITS", "12")
+    c = SCHED_CIRCS[name]()
+    got = gpu_run(q, c.qasm())
+    ref = oracle_run(c.qasm())
+    assert np.abs(got - ref).max() <= TOL
+    assert abs(1.0 - float(np.sum(np.abs(got) ** 2))) <= NORM_TOL
