@@ -195,13 +195,15 @@ struct PlanOptions {
 
 // Cut `gates` into passes, updating `map` (involvement, placement) exactly as the execution
 // will. The execution order is `order` with fusion lookahead (later commuting gates that join
-// the open tile pass are pulled forward); passes are consecutive runs of that execution order.
+// the open tile pass are pulled forward) and passes are consecutive runs of it -- or, with
+// opt.pass_sched, the pass-aware order of pass_schedule (sched.cpp) cut at its pass boundaries.
 // inv_after[k] = involvement after the k-th gate of `order` (the paper's trace).
 void plan_circuit(const std::vector<Gate>& gates, const std::vector<int>& order, QubitMap& map,
                   const PlanOptions& opt, std::vector<Pass>* passes,
                   std::vector<uint64_t>* inv_after);
-// plan_circuit over candidate lane-bit policies (opt.l_min / opt.l_relax) when opt.auto_lanes:
-// every candidate is planned from a copy of `map`, its passes costed by pass_cost_model(), and the
+// plan_circuit over candidate lane-bit policies (opt.l_min / opt.l_relax), with and without the
+// pass-aware order (opt.auto_sched), when opt.auto_lanes: every candidate is planned from a copy
+// of `map` (concurrently, on host threads), its passes costed by pass_cost_model(), and the
 // cheapest plan is kept (map, passes, inv_after as plan_circuit leaves them).
 void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& order, QubitMap& map,
                        const PlanOptions& opt, std::vector<Pass>* passes, std::vector<uint64_t>* inv_after);
@@ -210,8 +212,9 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
 // plus a launch gap.
 double pass_cost_model(const Pass& p, int m);
 // Two single-buffered CTAs per SM at <= 128 registers for this pass's NVRTC kernel (instead of
-// one triple-buffered CTA at <= 255): QGPU_2CTA=1 every pass, 2 (default) passes whose program
-// runs >= 40 FP64 instructions per amplitude (the latency-bound ones), 0 none (read per call).
+// one triple-buffered CTA at <= 255): QGPU_2CTA=1 every pass, 2 passes whose program runs >= 40
+// FP64 instructions per amplitude (the latency-bound ones), 4 (default) those and the passes
+// whose program remaps at >= 20 FP64 per amplitude, 0 none (read per call).
 bool pass_two_cta(const Pass& p);
 // Build the device ops of a tile pass from its gates and tile positions.
 void build_tile_ops(Pass& p, int m, int reg_bits = 4);

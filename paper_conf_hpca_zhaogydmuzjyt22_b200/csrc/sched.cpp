@@ -1893,10 +1893,20 @@ namespace qgpu {
 bool pass_two_cta(const Pass& p) {
   // default 2 (profiles/r02 A/B, same box: QAOA_32 175.9 -> 166.5 ms fixed lanes and 178.4 ->
   // 158.8 auto lanes, rqc_30 146.9 -> 139.5, grqc_32 8.43 -> 8.20 s, QFT_28 1.13 -> 1.10 ms)
+  // default 4 = 2 plus passes whose program remaps (the tile goes through shared memory mid-
+  // program) at >= 20 FP64 per amplitude: gs_33's 26->33 expansion (28 FP64 per amplitude, one
+  // remap) 32.3 -> 26.5 ms with two CTAs, while remap-free HBM-bound passes (QFT_28's and
+  // hlf_33's last) are faster as one triple-buffered CTA (profiles/r02b ab r3v)
   const char* ev = std::getenv("QGPU_2CTA");
-  const int mode = ev ? std::atoi(ev) : 2;
+  const int mode = ev ? std::atoi(ev) : 4;
   if (p.kind != PK_TILE || mode == 0) return false;
   if (mode == 3) return p.fp64_per_amp >= 40.0 || p.k_in == p.k_out;  // + steady-state passes
+  if (mode == 4) {
+    if (p.fp64_per_amp >= 40.0) return true;
+    bool remap = false;
+    for (size_t i = 1; i < p.prog.ops.size(); ++i) remap = remap || p.prog.ops[i].kind == OP_REMAP;
+    return remap && p.fp64_per_amp >= 20.0;
+  }
   return mode == 1 || p.fp64_per_amp >= 40.0;
 }
 }  // namespace qgpu
