@@ -210,18 +210,45 @@ double fp64_model(const Pass& p) {
   auto cls_cost = [](int cls) { return cls == MAT_GENERIC ? 8.0 : cls == MAT_X ? 0.0 : mat_unit(cls) ? 2.0 : 4.0; };
   if (p.kind == PK_TILE) {
     const TileProgram& P = p.prog;
-    double c = P.scalar.empty() ? 0.0 : 4.0;
+    // the tile-uniform scalar costs a multiply only when no phase run can absorb it (folding)
+    static const bool zmodel = [] {  // QGPU_FP64_MODEL=0: the round-2 model (A/B)
+      const char* ev = std::getenv("QGPU_FP64_MODEL");
+      return !(ev && ev[0] == '0');
+    }();
+    bool has_run = false;
+    for (size_t i = 1; i < P.ops.size(); ++i) has_run = has_run || P.ops[i].kind == OP_RUN;
+    double c = (P.scalar.empty() || (has_run && zmodel)) ? 0.0 : 4.0;
+    // compile-time zero tracking of the NVRTC bodies (first-touch expansion inside the pass): a
+    // non-lane tile bit whose position is >= k_in (or a skipped zero half) holds zeros until a
+    // non-diagonal op targets it, and ops skip those slots (register bits) and warps (warp bits)
+    const int lanes = std::min(5, p.b);
+    const uint32_t lanemask = (1u << lanes) - 1u;
+    uint32_t zpos = 0;
+    for (int i = 0; i < p.b && zmodel; ++i)
+      if (p.spos[i] >= p.k_in || (p.zin >> p.spos[i] & 1)) zpos |= 1u << i;
+    int R[4] = {0, 0, 0, 0};
+    if (!P.ops.empty())
+      for (int k = 0; k < 4; ++k) R[k] = (P.ops[0].a0 >> (4 * k)) & 15;
     for (size_t i = 1; i < P.ops.size(); ++i) {
       const TileOp& o = P.ops[i];
-      const double frac = std::ldexp(1.0, -std::popcount(o.rmask) - std::popcount(o.tmask));
+      const double live = std::ldexp(1.0, -std::popcount(zpos & ~lanemask));
+      const double frac = live * std::ldexp(1.0, -std::popcount(o.rmask) - std::popcount(o.tmask));
+      switch (o.kind) {
+        case OP_REMAP: for (int k = 0; k < 4; ++k) R[k] = (o.a0 >> (4 * k)) & 15; break;
+        case OP_U1R: zpos &= ~(1u << R[o.a0 & 3]); break;
+        case OP_U1L: case OP_SMEM1: zpos &= ~(1u << (o.a0 & 31)); break;
+        case OP_U2R: zpos &= ~((1u << R[o.a0 & 3]) | (1u << R[o.a1 & 3])); break;
+        case OP_SMEM2: zpos &= ~((1u << (o.a0 & 31)) | (1u << (o.a1 & 31))); break;
+        default: break;
+      }
       switch (o.kind) {
         case OP_U1R: case OP_U1L: case OP_SMEM1: c += cls_cost(o.cls) * frac; break;
         case OP_U2R: case OP_SMEM2: c += 16.0 * frac; break;
         case OP_RUN: {
           const uint32_t slots = uint32_t(o.a0 + o.a1 + o.cls) + o.tmask + o.tmatch;
-          if (slots) c += 4.0 + 4.0 * (1.0 - std::ldexp(1.0, -P.nr));
+          if (slots) c += (4.0 + 4.0 * (1.0 - std::ldexp(1.0, -P.nr))) * live;
           for (uint32_t e = o.moff + slots; e < o.moff + o.cnt; ++e)
-            if (P.entries[e].gend) c += 4.0 * std::ldexp(1.0, -std::popcount(uint32_t(P.entries[e].rmask)));
+            if (P.entries[e].gend) c += 4.0 * std::ldexp(1.0, -std::popcount(uint32_t(P.entries[e].rmask))) * live;
           break;
         }
         default: break;
