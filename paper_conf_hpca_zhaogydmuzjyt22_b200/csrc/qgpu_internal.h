@@ -154,6 +154,7 @@ struct Pass {
   uint64_t unfused_bytes = 0;   // bytes the pass's gates would move one gate per pass
   double fp64_per_amp = 0.0;    // FP64 pipe instructions per computed amplitude (roofline model,
                                 // fp64_model() in sched.cpp)
+  double fp64_dense = 0.0;      // the same without zero-slot skipping / scalar folding (two-CTA rule)
   // zero-position skipping (tile passes): physical positions p whose bit-p = 1 half of the live
   // state is exactly zero and NOT materialised in memory -- on input (zin: loads read zeros
   // instead) and on output (zout: those amplitudes are not stored); PK_ZERO materialises zmask
@@ -222,6 +223,8 @@ void build_tile_ops(Pass& p, int m, int reg_bits = 4);
 uint64_t unfused_gate_bytes(const PhysGate& g, int k_in, int k_out);
 // FP64 instructions per amplitude a pass's program executes (fused tile pass) or its single
 // gate needs (pair / quad / diagonal kernels): the FP64 side of the per-pass roofline.
-double fp64_model(const Pass& p);
+// zero_aware: count what the NVRTC body executes (zero slots of a first-touch expansion skipped,
+// the tile-uniform scalar folded into a run); else the dense count (the two-CTA thresholds)
+double fp64_model(const Pass& p, bool zero_aware = true);
 
 }  // namespace qgpu

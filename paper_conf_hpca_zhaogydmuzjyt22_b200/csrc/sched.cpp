@@ -206,15 +206,16 @@ uint64_t unfused_gate_bytes(const PhysGate& g, int k_in, int k_out) {
 //  by doubling (2^NR - 1 complex multiplies per thread for 2^NR amplitudes, ~4) and one more
 //  complex multiply per general r-condition group on the amplitudes it selects; the
 //  tile-uniform scalar 4. Conditions scale an op by the fraction of amplitudes they select.
-double fp64_model(const Pass& p) {
+double fp64_model(const Pass& p, bool zero_aware) {
   auto cls_cost = [](int cls) { return cls == MAT_GENERIC ? 8.0 : cls == MAT_X ? 0.0 : mat_unit(cls) ? 2.0 : 4.0; };
   if (p.kind == PK_TILE) {
     const TileProgram& P = p.prog;
     // the tile-uniform scalar costs a multiply only when no phase run can absorb it (folding)
-    static const bool zmodel = [] {  // QGPU_FP64_MODEL=0: the round-2 model (A/B)
+    static const bool zmodel_env = [] {  // QGPU_FP64_MODEL=0: the dense model everywhere (A/B)
       const char* ev = std::getenv("QGPU_FP64_MODEL");
       return !(ev && ev[0] == '0');
     }();
+    const bool zmodel = zero_aware && zmodel_env;
     bool has_run = false;
     for (size_t i = 1; i < P.ops.size(); ++i) has_run = has_run || P.ops[i].kind == OP_RUN;
     double c = (P.scalar.empty() || (has_run && zmodel)) ? 0.0 : 4.0;
@@ -1058,7 +1059,8 @@ struct Builder {
       while (p.l < p.b && p.spos[p.l] == p.l) ++p.l;
       build_tile_ops(p, map.m, opt.reg_bits);
     }
-    p.fp64_per_amp = fp64_model(p);
+    p.fp64_per_amp = fp64_model(p, true);
+    p.fp64_dense = fp64_model(p, false);
     if (std::getenv("QGPU_DEBUG_PLAN")) std::fprintf(stderr, "  pass fp64/amp %.2f\n", p.fp64_per_amp);
     out->push_back(std::move(p));
     cur = Pass();
@@ -1927,13 +1929,14 @@ bool pass_two_cta(const Pass& p) {
   const char* ev = std::getenv("QGPU_2CTA");
   const int mode = ev ? std::atoi(ev) : 4;
   if (p.kind != PK_TILE || mode == 0) return false;
-  if (mode == 3) return p.fp64_per_amp >= 40.0 || p.k_in == p.k_out;  // + steady-state passes
+  // (thresholds on the dense FP64 count, as they were measured: fp64_dense)
+  if (mode == 3) return p.fp64_dense >= 40.0 || p.k_in == p.k_out;  // + steady-state passes
   if (mode == 4) {
-    if (p.fp64_per_amp >= 40.0) return true;
+    if (p.fp64_dense >= 40.0) return true;
     bool remap = false;
     for (size_t i = 1; i < p.prog.ops.size(); ++i) remap = remap || p.prog.ops[i].kind == OP_REMAP;
-    return remap && p.fp64_per_amp >= 20.0;
+    return remap && p.fp64_dense >= 20.0;
   }
-  return mode == 1 || p.fp64_per_amp >= 40.0;
+  return mode == 1 || p.fp64_dense >= 40.0;
 }
 }  // namespace qgpu
