@@ -155,7 +155,15 @@ __device__ __forceinline__ uint64_t deposit(uint64_t v, const int* ins, int nins
   for (int i = 0; i < nins; ++i) v = insert0(v, ins[i]);
   return v;
 }
+// tile stores: streaming (evict-first) by default; QGPU_JIT_OPTS="-DQGPU_STORE_WB" / "-DQGPU_STORE_CG"
+// compile the NVRTC bodies with write-back / L2-only stores instead (A/B of write-heavy passes)
+#if defined(QGPU_STORE_WB)
+__device__ __forceinline__ void st_stream(double2* p, double2 v) { *p = v; }
+#elif defined(QGPU_STORE_CG)
+__device__ __forceinline__ void st_stream(double2* p, double2 v) { __stcg(p, v); }
+#else
 __device__ __forceinline__ void st_stream(double2* p, double2 v) { __stcs(p, v); }
+#endif
 
 // tile index -> base amplitude index: insert the tile positions (as runs of consecutive bits)
 __device__ __forceinline__ uint64_t tile_base(uint64_t t, const TileArgs& a) {
