@@ -312,17 +312,8 @@ qgpu_status exec_compute(qgpu_state* st, const Pass& p, const unsigned char* d_o
     const int jit = st->cfg.jit;
     cudaError_t e = cudaErrorNotSupported;
     if (jit == 2 || (jit == 1 && p.k_out >= jit_min_bits())) {
-      TileArgs aj = a;
-      if (!aj.hist) {  // the stage ring of the NVRTC body (pass_stage_ring decides for both)
-        int stage_amps = 0;
-        const int D = pass_stage_ring(p, &stage_amps);
-        if (D > 0) {
-          aj.nbuf = 0;
-          aj.ring_amps = D * stage_amps;
-        }
-      }
       double ms = 0;
-      e = launch_tile_jit(st->stream, p, aj, tile_smem_bytes(aj), device_num_sms(), &ms);
+      e = launch_tile_jit(st->stream, p, a, tile_smem_bytes(a), device_num_sms(), &ms);
       if (e == cudaSuccess) st->stats.jit_launches++;
       st->stats.jit_ms += ms;
     }

@@ -304,30 +304,6 @@ std::string tile_jit_source(const Pass& p, int hist_mode, uint32_t hist_key) {
   hdr << "  static constexpr uint64_t kP0[kRegAmps] = " << ptab(R) << ";\n";
   hdr << "  static constexpr uint64_t kPF[kRegAmps] = " << ptab(RF) << ";\n";
   hdr << "  static constexpr uint32_t kJF[kRegAmps] = " << jtab(RF) << ";\n";
-  {  // stage ring (pass_stage_ring; not for the fused-measurement variants)
-    int stage_amps = 1;
-    const int D = hist ? 0 : pass_stage_ring(p, &stage_amps);
-    uint32_t live = 0;
-    for (int i = 0; i < p.b; ++i)
-      if (!(p.spos[i] >= p.k_in || (p.zin >> p.spos[i] & 1))) live |= 1u << i;
-    std::ostringstream t;
-    t << "{";
-    for (int r = 0; r < 16; ++r) {
-      uint32_t j = 0;
-      for (int k = 0; k < NR; ++k)
-        if (r >> k & 1) j |= 1u << R[k];
-      uint32_t c = 0;
-      int o = 0;
-      for (int bit = 0; bit < 13; ++bit)
-        if (live >> bit & 1u) c |= ((j >> bit) & 1u) << o++;
-      t << (r ? ", " : "") << (D ? c : 0u) << "u";
-    }
-    t << "}";
-    hdr << "  static constexpr int kStages = " << D << ";\n";
-    hdr << "  static constexpr uint32_t kStageAmps = " << (D ? stage_amps : 1) << "u;\n";
-    hdr << "  static constexpr uint32_t kLiveMask = " << (D ? live : 0u) << "u;\n";
-    hdr << "  static constexpr uint32_t kJ0c[kRegAmps] = " << t.str() << ";\n";
-  }
   // the last op that touches the tile buffer (remap, shared-memory op): after it the program
   // runs from registers, so the driver's prefetch of the next tile into the single buffer of a
   // two-CTA pass can be issued there (pf) instead of after the whole program

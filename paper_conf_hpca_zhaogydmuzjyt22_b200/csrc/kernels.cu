@@ -224,9 +224,6 @@ struct InterpBody {
   int nops;
   static constexpr bool kEarlyPrefetch = false;  // the driver prefetches after the program
   static constexpr bool kScalarFolded = false;   // the driver applies the tile-uniform scalar
-  static constexpr int kStages = 0;              // tile buffers, no stage ring
-  static constexpr uint32_t kStageAmps = 1u, kLiveMask = 0u;
-  static constexpr uint32_t kJ0c[kRegAmps] = {};
   template <class PF>
   __device__ __forceinline__ void operator()(double2 (&v)[kRegAmps], Mapping& mp, const TileCtx& c,
                                              const TileArgs&, PF&&) const {
@@ -651,8 +648,7 @@ int device_num_sms() { return num_sms(); }
 size_t tile_smem_bytes(const TileArgs& a) {
   const size_t nh = size_t(1) << (a.b - a.l);
   const size_t nwarps = size_t(1) << a.nw;
-  return size_t(a.nbuf) * (size_t(1) << a.b) * 16 + size_t(a.ring_amps) * 16 + ((nh + 1) & ~size_t(1)) * 8 +
-         size_t(a.blob_bytes) +
+  return size_t(a.nbuf) * (size_t(1) << a.b) * 16 + ((nh + 1) & ~size_t(1)) * 8 + size_t(a.blob_bytes) +
          2 * nwarps * size_t(a.npat) * 16 + size_t(a.nmbar) * 8 + 16 + (a.hist ? (size_t(8) << a.hm) * (a.hacc == 2 ? (a.hglob ? 0 : nwarps) : 1) : 0);
 }
 

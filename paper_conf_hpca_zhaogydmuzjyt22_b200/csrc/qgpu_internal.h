@@ -217,11 +217,6 @@ double pass_cost_model(const Pass& p, int m);
 // FP64 instructions per amplitude (the latency-bound ones), 4 (default) those and the passes
 // whose program remaps at >= 20 FP64 per amplitude, 0 none (read per call).
 bool pass_two_cta(const Pass& p);
-// Stage ring for this pass's NVRTC kernel (Body::kStages, TileArgs::ring_amps): one-CTA expansion
-// passes without remaps load only their live input slots into min(16, 3 * 2^z) compact stages of
-// 2^(b - z) amplitudes (z = tile bits on zero positions), loads running that many tiles ahead.
-// Returns the stage count (0: off) and the stage size.
-int pass_stage_ring(const Pass& p, int* stage_amps);
 // Build the device ops of a tile pass from its gates and tile positions.
 void build_tile_ops(Pass& p, int m, int reg_bits = 4);
 // Unfused byte model of one gate on live size 2^k.

@@ -1919,25 +1919,6 @@ void plan_circuit_auto(const std::vector<Gate>& gates, const std::vector<int>& o
 }  // namespace qgpu
 
 namespace qgpu {
-int pass_stage_ring(const Pass& p, int* stage_amps) {
-  // one-CTA NVRTC expansion passes without remaps / shared-memory ops (QGPU_RING=0: off, A/B)
-  const char* ev = std::getenv("QGPU_RING");
-  if (ev && ev[0] == '0') return 0;
-  const char* bs = std::getenv("QGPU_BSTORE");  // bulk stores stage the tile in its buffer
-  if (bs && bs[0] != '0') return 0;
-  if (p.kind != PK_TILE || pass_two_cta(p) || p.b < 6) return 0;
-  for (size_t i = 1; i < p.prog.ops.size(); ++i) {
-    const int k = p.prog.ops[i].kind;
-    if (k == OP_REMAP || k == OP_SMEM1 || k == OP_SMEM2) return 0;
-  }
-  int z = 0;
-  for (int i = 0; i < p.b; ++i) z += (p.spos[i] >= p.k_in || (p.zin >> p.spos[i] & 1)) ? 1 : 0;
-  if (z < 1) return 0;
-  if (stage_amps) *stage_amps = 1 << (p.b - z);
-  // at most 128 KiB of stages (the program blob and tables need the rest of shared memory)
-  return std::max(0, std::min({16, 3 << z, 8192 >> (p.b - z)}));
-}
-
 bool pass_two_cta(const Pass& p) {
   // default 2 (profiles/r02 A/B, same box: QAOA_32 175.9 -> 166.5 ms fixed lanes and 178.4 ->
   // 158.8 auto lanes, rqc_30 146.9 -> 139.5, grqc_32 8.43 -> 8.20 s, QFT_28 1.13 -> 1.10 ms)

@@ -133,11 +133,6 @@ struct TileArgs {
   // mode 2 without private histograms: the lanes add straight to hist (global f64 reductions,
   // no shared memory), used when per-warp histograms would cost the pass CTAs per SM
   int hglob;
-  // stage ring (Body::kStages > 0, NVRTC bodies of one-CTA expansion passes without remaps): the
-  // tile buffers are replaced by kStages compact stages holding only a tile's live input slots
-  // (the tile bits on zero positions dropped), so loads run kStages - 1 tiles ahead; ring_amps =
-  // kStages x stage size in amplitudes (shared-memory sizing)
-  int ring_amps;
   // the pass's U matrices as a kernel parameter (constant bank), when they fit: the NVRTC bodies
   // read them at compile-time offsets (no shared-memory loads, no registers held across tiles)
   int umat_n;
@@ -798,27 +793,6 @@ __device__ __forceinline__ void issue_own_loads(double2* buf, const TileArgs& a,
   asm volatile("cp.async.commit_group;\n" ::: "memory");
 }
 
-// Stage-ring loads (Body::kStages): as issue_own_loads, into the compact stage `stage` at
-// cb + kJ0c[r] (the slot's tile index with the zero-position bits removed); always one group.
-template <int NR, class Body>
-__device__ __forceinline__ void issue_stage_loads(double2* stage, const TileArgs& a, uint32_t cb, const SlotAddr& sa0,
-                                                  uint64_t base, unsigned zm, bool own, bool valid) {
-  if (valid && own && base < a.L_in && !(base & a.zin)) {
-#pragma unroll
-    for (int r = 0; r < (1 << NR); ++r) {
-      if ((zm >> r) & 1) continue;
-      const uint64_t idx = (base | sa0.pb) + Body::kP0[r];
-      const bool live = idx < a.L_in && !(idx & a.zin);
-      cp_async16(stage + cb + Body::kJ0c[r], a.psi + (live ? idx : 0), live ? 16 : 0);
-    }
-  }
-  asm volatile("cp.async.commit_group;\n" ::: "memory");
-}
-template <int N>
-__device__ __forceinline__ void cp_async_wait_group_n() {
-  asm volatile("cp.async.wait_group %0;\n" ::"n"(N) : "memory");
-}
-
 // Bulk store of a staged tile: the tile buffer holds the results at their tile index; runs of
 // 2^l consecutive tile indices are contiguous in HBM. The lanes of warp 0 first wait until the
 // previous tile's bulk reads of shared memory are done (that buffer is the next prefetch target),
@@ -852,7 +826,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   const int nh = 1 << (b - l);
   const int nthr = blockDim.x, nwarps = nthr >> 5;
   double2* bufs = reinterpret_cast<double2*>(smem_raw);  // nbuf x T
-  uint64_t* hiOff = reinterpret_cast<uint64_t*>(bufs + nbuf * T + a.ring_amps);
+  uint64_t* hiOff = reinterpret_cast<uint64_t*>(bufs + nbuf * T);
   unsigned char* blob = reinterpret_cast<unsigned char*>(hiOff + ((nh + 1) & ~1));
   const TileOp* ops = reinterpret_cast<const TileOp*>(blob);
   const RunEntry* ents = reinterpret_cast<const RunEntry*>(blob + a.off_entries);
@@ -921,23 +895,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
   auto real = [&](uint64_t j) -> uint64_t { return a.nzs ? deposit(j, a.zs_pos, a.nzs) : j; };
   uint64_t tile = tile_at(0);
   uint64_t base_next = tile_base_t<Body>(real(tile), a);  // base of `tile`, carried across iterations
-  constexpr int kD = Body::kStages;
-  constexpr uint32_t kStageAmps = kD > 0 ? Body::kStageAmps : 1u;
-  uint32_t cb = 0;  // stage ring: this thread's base slot index with the zero-position bits removed
-  if constexpr (kD > 0) {
-    int o = 0;
-#pragma unroll
-    for (int t = 0; t < 13; ++t)
-      if (Body::kLiveMask >> t & 1u) cb |= ((mp0.base >> t) & 1u) << o++;
-    for (int d = 0; d + 1 < kD; ++d) {
-      const uint64_t td = tile_at(uint64_t(d));
-      const bool ok = td < a.ntiles;
-      issue_stage_loads<NR, Body>(bufs + size_t(d) * kStageAmps, a, cb, sa0,
-                                  ok ? tile_base_t<Body>(real(td), a) : 0ull, zm0, c.own, ok);
-    }
-  } else {
-    if (tile < a.ntiles) issue_own_loads<NR, Body>(bufs, a, mp0, sa0, base_next, zm0, c.own);
-  }
+  if (tile < a.ntiles) issue_own_loads<NR, Body>(bufs, a, mp0, sa0, base_next, zm0, c.own);
   int k = 0;
   uint64_t cur_hi = ~0ull;
   double hacc[1 << NR];   // fused measurement with a.hacc: per-slot sums over this thread's tiles
@@ -959,13 +917,6 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
     // nbuf >= 2: prefetch into the next buffer now; nbuf == 1 (programs without remaps, every
     // thread reads only its own slots): prefetch into the same buffer right after the reload
     if (more && nbuf > 1) issue_own_loads<NR, Body>(bufs + kn * T, a, mp0, sa0, base_next, zm0, c.own);
-    if constexpr (kD > 0) {  // stage ring: tile it + kD - 1 into its stage, one group per tile
-      s = bufs + size_t(it % uint64_t(kD)) * kStageAmps;
-      const uint64_t ta = tile_at(it + uint64_t(kD - 1));
-      const bool ok = ta < a.ntiles;
-      issue_stage_loads<NR, Body>(bufs + size_t((it + uint64_t(kD - 1)) % uint64_t(kD)) * kStageAmps, a, cb, sa0,
-                                  ok ? tile_base_t<Body>(real(ta), a) : 0ull, zm0, c.own, ok);
-    }
     if (base & a.zout) {
       // zero-position skipping: a non-tile bit of this tile selects a half that is zero and is
       // not materialised in memory -> nothing to load, compute or store
@@ -1032,8 +983,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
         cw[pi] = cc;
       }
     }
-    if constexpr (kD > 0) cp_async_wait_group_n<(kD > 1 ? kD - 1 : 0)>();
-    else if (more && nbuf > 1) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
+    if (more && nbuf > 1) asm volatile("cp.async.wait_group 1;\n" ::: "memory");
     else cp_async_wait_all();
     __syncwarp();
     // tile-uniform phase (the scalar pattern)
@@ -1045,8 +995,7 @@ __device__ __forceinline__ void tile_driver(const TileArgs& a, Body& body) {
 #pragma unroll
     for (int r = 0; r < (1 << NR); ++r) {
       uint32_t j;
-      if constexpr (kD > 0) j = cb + Body::kJ0c[r];
-      else if constexpr (Body::kStatic) j = mp0.base + Body::kJ0[r];
+      if constexpr (Body::kStatic) j = mp0.base + Body::kJ0[r];
       else j = mp0.j(r);
       v[r] = (c.own && !((zm0 >> r) & 1)) ? s[j] : make_double2(0.0, 0.0);
     }
