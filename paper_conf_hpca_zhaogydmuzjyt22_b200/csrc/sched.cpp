@@ -965,18 +965,6 @@ void build_tile_ops(Pass& p, int m, int reg_bits) {
     P.ops.push_back(op);
     ++i;
   }
-  // store remap (QGPU_STORE_REMAP=1, experiment): in a write-dominated expansion pass, a final
-  // remap puts the register bits on the lowest non-lane tile positions, so each warp's 16 stores
-  // cover one contiguous 2^(lanes + nr)-amplitude block instead of 16 scattered runs
-  if (const char* ev = std::getenv("QGPU_STORE_REMAP")) {
-    if (ev[0] == '1' && nr > 0 && p.k_out - p.k_in >= 2 && lanes + nr <= b) {
-      uint32_t want = 0;
-      for (int k = 0; k < nr; ++k) want |= 1u << (lanes + k);
-      uint32_t have = 0;
-      for (int k = 0; k < nr; ++k) have |= 1u << R[k];
-      if (have != want) choose(want, seq.size());
-    }
-  }
   if (pass_scale != 1.0) P.scalar.push_back(PhaseTerm{0, 0, pass_scale, 0.0});
   split_patterns(P, p, m);
   P.layout();
@@ -1945,8 +1933,8 @@ bool pass_two_cta(const Pass& p) {
   if (mode == 3) return p.fp64_dense >= 40.0 || p.k_in == p.k_out;  // + steady-state passes
   if (mode == 4) {
     if (p.fp64_dense >= 40.0) return true;
-    bool remap = false;  // (a trailing remap is a store remap, not a mid-program one)
-    for (size_t i = 1; i + 1 < p.prog.ops.size(); ++i) remap = remap || p.prog.ops[i].kind == OP_REMAP;
+    bool remap = false;
+    for (size_t i = 1; i < p.prog.ops.size(); ++i) remap = remap || p.prog.ops[i].kind == OP_REMAP;
     return remap && p.fp64_dense >= 20.0;
   }
   return mode == 1 || p.fp64_dense >= 40.0;
